@@ -1,0 +1,216 @@
+/*
+ * tsmv.h -- C ABI of libtsmv.so: tiled sparse matrix - sparse vector
+ * multiplication (TileSpMSpV) and direction-optimising TileBFS on NVIDIA B200
+ * (sm_100a).
+ *
+ * Method: Ji, Song, Lu, Jin, Tan, Liu, "TileSpMSpV: A Tiled Algorithm for
+ * Sparse Matrix-Sparse Vector Multiplication on GPUs", ICPP '22.
+ * "P:n" = line n of the paper text; "R<k>" = reading k in DESIGN.md.
+ *
+ * Conventions for every entry point
+ *  - No C++ exception crosses the ABI; every call returns a tsmv_status.  On a
+ *    non-OK status a thread-local message is available from tsmv_last_error().
+ *  - Pointers marked "host or device" are classified per call with
+ *    cudaPointerGetAttributes: device (or managed) memory is used in place,
+ *    host memory (pageable or pinned) is staged through ctx-owned device
+ *    buffers with the copies enqueued on the caller's stream.
+ *  - A context is bound to one CUDA device and is not thread-safe.  All work
+ *    is enqueued on the `cuda_stream` argument (a cudaStream_t; NULL = the
+ *    legacy default stream).
+ *  - Index types: row pointers int64, column / row / vertex ids int32 (so
+ *    n < 2^31), counts int64.
+ */
+#ifndef TSMV_H
+#define TSMV_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct tsmv_ctx tsmv_ctx; /* opaque */
+
+typedef enum {
+    TSMV_OK = 0,
+    TSMV_EINVAL = 1,      /* bad argument (sizes, NULL, unsorted/duplicate x, source range) */
+    TSMV_ENOMEM = 2,      /* device or host allocation failed */
+    TSMV_ECUDA = 3,       /* a CUDA runtime error (message in tsmv_last_error) */
+    TSMV_ENCCL = 4,       /* reserved: collective failure (exchange is done by the caller) */
+    TSMV_ECAPACITY = 5,   /* y_cap < y_nnz: *y_nnz holds the required size */
+    TSMV_EUNSUPPORTED = 6 /* valid request this build does not support */
+} tsmv_status;
+
+typedef enum { TSMV_F64 = 0, TSMV_F32 = 1, TSMV_PATTERN = 2 } tsmv_dtype;
+
+/* Semirings of y = A x (P:157-160 problem statement; Boolean AND = x, OR = +).
+ *  PLUS_TIMES : y_i = sum_j a_ij * x_j.  F32 matrices: fp32 storage, fp64
+ *               accumulation, one rounding at the end (R3).  PATTERN: a_ij = 1.
+ *  OR_AND     : structural product only; y_val is not written (may be NULL).
+ *  MIN_SECOND : y_i = min_j x_j over stored a_ij (a_ij ignored); with x_j = j
+ *               this yields the minimum-id parent of BFS. */
+typedef enum { TSMV_PLUS_TIMES = 0, TSMV_OR_AND = 1, TSMV_MIN_SECOND = 2 } tsmv_semiring;
+
+/* TileBFS kernels (Sec 3.4): Push-CSC (Alg 5), Push-CSR (Alg 6),
+ * Pull-CSC (Alg 7); AUTO applies the per-level rule of reading R9. */
+typedef enum {
+    TSMV_DIR_AUTO = 0,
+    TSMV_DIR_PUSH_CSC = 1,
+    TSMV_DIR_PUSH_CSR = 2,
+    TSMV_DIR_PULL_CSC = 3
+} tsmv_dir;
+
+typedef struct {
+    int32_t device;              /* CUDA ordinal the context lives on */
+    int32_t tile_dim;            /* nt in {16, 32, 64}; default 16 */
+    int32_t sparse_tile_max_nnz; /* tiles with <= this many nonzeros go to the side
+                                    matrix (R12); default 2; 0 = none */
+    int32_t build_bfs;           /* 1 = also build the TileBFS bitmask tiles (square A);
+                                    default 1 when nrows == ncols and nranks == 1 */
+    double push_csr_density;     /* |F|/n threshold Push-CSC -> Push-CSR; default 0.01 */
+    double pull_alpha;           /* Pull-CSC when m_f > m_u / alpha (R9); default 14 */
+    int32_t force_dir;           /* tsmv_dir; AUTO = rule of R9 (tests / ablation) */
+    int32_t rank, nranks;        /* row-block partition: this rank / number of ranks (1 = single GPU) */
+    int64_t row_begin;           /* global id of local row 0 (multiple of 64 when nranks > 1) */
+    const int64_t *row_splits;   /* host, nranks+1 global row boundaries (NULL when nranks == 1);
+                                    copied by tsmv_create */
+} tsmv_options;
+
+/* Per-call counters of the last tsmv_spmspv (read from device on request). */
+typedef struct {
+    int64_t x_nnz;          /* k */
+    int64_t x_segments;     /* non-empty nt-segments of x */
+    int64_t tile_items;     /* tiles in the tile columns of non-empty segments (a3) */
+    int64_t side_items;     /* side-matrix nonzeros in the columns of x (a5) */
+    int64_t y_nnz;
+} tsmv_call_stats;
+
+/* Built-format census. */
+typedef struct {
+    int64_t nrows, ncols, nnz;
+    int32_t tile_dim;
+    int32_t symmetric;          /* pattern symmetric (detected; BFS then keeps one bitmask copy) */
+    int64_t n_tiles;            /* non-empty tiles (before extraction) */
+    int64_t n_dense_tiles;      /* tiles kept in tile format (> sparse_tile_max_nnz nnz) */
+    int64_t dense_nnz;          /* nonzeros in tile format */
+    int64_t side_nnz;           /* nonzeros in the side matrix */
+    int64_t bytes_spmspv;       /* device bytes of the SpMSpV structures */
+    int64_t bytes_bfs;          /* device bytes of the BFS bitmask structures */
+    int64_t bytes_workspace;    /* accumulators, bitmaps, scratch */
+    double build_ms;            /* device time of tsmv_create's builder */
+} tsmv_info;
+
+#define TSMV_MAX_LEVELS 65536
+typedef struct {
+    int32_t nlevels;                 /* number of non-empty levels (source level counts) */
+    int64_t reached;                 /* vertices with level >= 0 (global) */
+    int64_t edges_traversed;         /* sum of out-degrees of reached vertices (R16) */
+    double ms;                       /* device time source-init -> last level */
+    int32_t dir_per_level[TSMV_MAX_LEVELS];       /* tsmv_dir used to expand level L */
+    int64_t frontier_per_level[TSMV_MAX_LEVELS];  /* |F| of level L */
+} tsmv_bfs_stats;
+
+/* Fill *opt with the defaults documented above.  Never fails for non-NULL opt. */
+tsmv_status tsmv_default_options(tsmv_options *opt);
+
+/* Build the tiled representation of A (Sec 3.2.1; BFS bitmasks
+ * Sec 3.2.3) on opt->device.
+ *   nrows, ncols : local rows (rows of this rank's block) and global columns.
+ *   row_ptr      : int64[nrows+1], host or device; row_ptr[0] must be 0.
+ *   col_idx      : int32[nnz], host or device; ascending and unique within each row,
+ *                  in [0, ncols).
+ *   values       : nnz values (double for F64, float for F32), host or device;
+ *                  must be NULL iff dtype == TSMV_PATTERN.
+ *   opt          : NULL = defaults.
+ * The ctx deep-copies everything; the caller may free its inputs on return.
+ * Errors: EINVAL (sizes, tile_dim, unsorted/duplicate/out-of-range columns),
+ * ENOMEM, ECUDA.  *out is NULL on failure. */
+tsmv_status tsmv_create(tsmv_ctx **out, int64_t nrows, int64_t ncols, const int64_t *row_ptr,
+                        const int32_t *col_idx, const void *values, tsmv_dtype dtype,
+                        const tsmv_options *opt);
+
+/* y = A x over `sr` (Sec 3.3, Fig 4).
+ *   x_nnz, x_idx, x_val : the sparse x; x_idx int32 STRICTLY ASCENDING global column
+ *                  ids (R18), host or device; x_val double (F64/PATTERN) or float
+ *                  (F32), host or device, may be NULL for OR_AND.
+ *   y_cap, y_idx, y_val : caller-owned outputs (host or device).  y_idx int32
+ *                  ascending GLOBAL row ids; y_val same type as x_val (not written
+ *                  for OR_AND; may then be NULL).  y_cap >= nrows always suffices.
+ *   y_nnz        : host out; set even on ECAPACITY (contents of y then unspecified).
+ * The call synchronises `cuda_stream` once (to return y_nnz).
+ * Errors: EINVAL (unsorted / duplicate / out-of-range x, semiring/dtype mismatch),
+ * ECAPACITY, ECUDA.  On EINVAL the ctx workspaces stay clean. */
+tsmv_status tsmv_spmspv(tsmv_ctx *c, tsmv_semiring sr, int64_t x_nnz, const int32_t *x_idx,
+                        const void *x_val, int64_t y_cap, int32_t *y_idx, void *y_val,
+                        int64_t *y_nnz, void *cuda_stream);
+
+/* Counters of the last tsmv_spmspv on this ctx (synchronous D2H read). */
+tsmv_status tsmv_last_call_stats(tsmv_ctx *c, tsmv_call_stats *s);
+
+/* TileBFS from `source` (Alg 3 P:418-430 with the three kernels of Sec 3.4,
+ * P:1417-1628).  Single-GPU contexts only (nranks == 1; distributed BFS uses
+ * the tsmv_bfs_dist_* calls).  Requires a square A built with build_bfs.
+ *   levels : int32[nrows] host or device out: hop count from source, -1 if
+ *            unreachable (R15).
+ *   stats  : host, may be NULL.
+ * Returns after the traversal (stream synchronised).  Errors: EINVAL (source
+ * out of range, not square, no BFS structures), ECUDA. */
+tsmv_status tsmv_bfs(tsmv_ctx *c, int64_t source, int32_t *levels, tsmv_bfs_stats *stats,
+                     void *cuda_stream);
+
+/* ---- distributed TileBFS (row-block partition, Sec 8(e) of SURVEY / DESIGN.md) ----
+ * Each rank owns global rows [row_splits[rank], row_splits[rank+1]).  Per level:
+ *   tsmv_bfs_dist_expand  -> this rank's newly discovered owned vertices as a bitmap
+ *                            segment (uint32 words, bit v%32 of word (v-row_begin)/32);
+ *   caller all-gathers the segments (torch.distributed / NCCL), each padded to
+ *   `stride_words` words, in rank order;
+ *   tsmv_bfs_dist_merge   -> OR the gathered frontier into the replicated visited
+ *                            bitmap, rebuild the frontier, return its size.
+ * begin / merge return out_stats[3] = { |F| (global: same on every rank),
+ * m_f local (sum over F of this block's column counts), m_u local (sum of the
+ * in-degrees of this rank's unvisited rows) }; the caller all-reduces m_f and
+ * m_u and passes tsmv_choose_dir(...) of the global numbers as `dir` (1..3) to
+ * expand, so every rank takes the same decision.  levels: device memory,
+ * int32[local rows].  All ranks make the same calls in the same order. */
+tsmv_status tsmv_bfs_dist_begin(tsmv_ctx *c, int64_t source, int32_t *levels, int64_t *out_stats,
+                                void *cuda_stream);
+tsmv_status tsmv_bfs_dist_expand(tsmv_ctx *c, int32_t dir, uint32_t *owned_words_out, void *cuda_stream);
+tsmv_status tsmv_bfs_dist_merge(tsmv_ctx *c, const uint32_t *gathered, int64_t stride_words,
+                                int64_t *out_stats, void *cuda_stream);
+/* Words of this rank's owned segment = ceil((row_splits[r+1]-row_splits[r])/32). */
+int64_t tsmv_owned_words(const tsmv_ctx *c);
+
+/* Direction rule of reading R9: PULL_CSC if m_f > m_u / pull_alpha,
+ * else PUSH_CSR if frontier / n >= push_csr_density, else PUSH_CSC; force_dir wins
+ * when not AUTO.  opt NULL = defaults. */
+int32_t tsmv_choose_dir(const tsmv_options *opt, int64_t n, int64_t frontier, int64_t m_f, int64_t m_u);
+
+/* Census of the built format (host out). */
+tsmv_status tsmv_get_info(const tsmv_ctx *c, tsmv_info *info);
+
+/* Rebuild CSR from the tiled structures (tiles + side matrix), host outputs:
+ * row_ptr int64[nrows+1], col_idx int32[nnz], values (type of the ctx; NULL
+ * allowed).  Used by the round-trip test of the builder. */
+tsmv_status tsmv_export_csr(tsmv_ctx *c, int64_t *row_ptr, int32_t *col_idx, void *values);
+
+/* Export the TileBFS bitmask tiles in the paper's presentation (Fig 5,
+ * P:770-788): orient 0 = A1 column words, 1 = A2 row words, MSB-first bits,
+ * tiles listed in (J, I) order for A1 and (I, J) for A2, side-matrix entries
+ * folded back in.  Host outputs of capacity max_tiles (EINVAL if exceeded). */
+tsmv_status tsmv_export_bitmask_tiles(tsmv_ctx *c, int32_t orient, int64_t max_tiles,
+                                      int64_t *tile_I, int64_t *tile_J, uint64_t *words,
+                                      int64_t *n_tiles);
+
+/* Free everything the ctx owns.  NULL-safe. */
+tsmv_status tsmv_destroy(tsmv_ctx *c);
+
+/* Thread-local message for the last non-OK status ("" if none). */
+const char *tsmv_last_error(void);
+
+/* ABI version, (major << 16) | minor. */
+int32_t tsmv_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* TSMV_H */

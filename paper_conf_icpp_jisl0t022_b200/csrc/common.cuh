@@ -1,0 +1,218 @@
+// common.cuh -- internal definitions of libtsmv.so (not part of the ABI).
+//
+// Layout of the tiled matrix in HBM (DESIGN.md §"Data layout"):
+//   TileSet = one "tile-CSC": non-empty nt x nt tiles grouped by tile column
+//   (P:481-503 stores them "in the CSR format" by tile row; we keep the
+//   column-grouped twin because the vector-driven kernels walk tile columns,
+//   P:1439-1457), structure-of-arrays so that the intersection step reads only
+//   the 2..8-byte column masks of the tiles it tests.
+#pragma once
+#include <cstdint>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <vector>
+#include <cuda_runtime.h>
+#include "../../include/tsmv.h"
+
+#define TSMV_VERSION ((1 << 16) | 0)
+
+namespace tsmv {
+
+// ------------------------------------------------------------------ errors
+void set_error(const char *fmt, ...);
+
+struct Err {
+    tsmv_status st;
+};
+
+#define TSMV_CUDA(call)                                                                 \
+    do {                                                                                \
+        cudaError_t _e = (call);                                                        \
+        if (_e != cudaSuccess) {                                                        \
+            ::tsmv::set_error("%s:%d %s: %s", __FILE__, __LINE__, #call,                \
+                              cudaGetErrorString(_e));                                  \
+            throw ::tsmv::Err{_e == cudaErrorMemoryAllocation ? TSMV_ENOMEM : TSMV_ECUDA}; \
+        }                                                                               \
+    } while (0)
+
+#define TSMV_REQUIRE(cond, ...)                 \
+    do {                                        \
+        if (!(cond)) {                          \
+            ::tsmv::set_error(__VA_ARGS__);     \
+            throw ::tsmv::Err{TSMV_EINVAL};     \
+        }                                       \
+    } while (0)
+
+// ------------------------------------------------------------------ tile traits
+template <int NT> struct Tr;
+template <> struct Tr<16> { using word_t = uint16_t; using idx_t = uint8_t;  static constexpr int LOG = 4; };
+template <> struct Tr<32> { using word_t = uint32_t; using idx_t = uint16_t; static constexpr int LOG = 5; };
+template <> struct Tr<64> { using word_t = unsigned long long; using idx_t = uint16_t; static constexpr int LOG = 6; };
+
+inline int log2_nt(int nt) { return nt == 16 ? 4 : nt == 32 ? 5 : 6; }
+inline int idx_bytes(int nt) { return nt == 16 ? 1 : 2; }
+inline int word_bytes(int nt) { return nt / 8; }
+
+// ------------------------------------------------------------------ device memory
+struct DevBuf {
+    void *p = nullptr;
+    size_t bytes = 0;
+    void alloc(size_t b) {
+        release();
+        if (b == 0) b = 16;
+        TSMV_CUDA(cudaMalloc(&p, b));
+        bytes = b;
+    }
+    void ensure(size_t b) {
+        if (b > bytes) alloc(b);
+    }
+    void release() {
+        if (p) cudaFree(p);
+        p = nullptr;
+        bytes = 0;
+    }
+    template <class T> T *as() const { return static_cast<T *>(p); }
+};
+
+// One tile-CSC ("TileSet") built from a set of (row, col[, val]) entries of a
+// dimR x dimC matrix.  For A itself (push / SpMSpV) rows are A's rows; for the
+// pull structure of a directed graph it is built from A^T.
+struct TileSet {
+    int64_t dimR = 0, dimC = 0, nTR = 0, nTC = 0;
+    int64_t n_tiles_all = 0;  // non-empty tiles before extraction
+    int64_t T = 0;            // tiles kept (dense)
+    int64_t dense_nnz = 0, side_nnz = 0;
+    DevBuf ptr;      // int64[nTC+1]: tiles of tile column J are [ptr[J], ptr[J+1])
+    DevBuf trow;     // int32[T]: tile row I of each tile
+    DevBuf tgrp;     // int32[T]: tile column J of each tile (group id)
+    DevBuf mask;     // word_t[T]: column-occupancy mask (bit c = column c non-empty)
+    DevBuf off;      // int64[T+1]: first in-tile nonzero of each tile
+    DevBuf idx;      // idx_t[dense_nnz]: (c << LOG) | r, column-major inside a tile
+    DevBuf val;      // double/float[dense_nnz] (absent for pattern)
+    DevBuf planes;   // word_t[NT][T]: plane c holds column word c of every tile (bit r = row r)
+    DevBuf sptr;     // int64[dimC+1]: side matrix (very sparse tiles), CSC
+    DevBuf srow;     // int32[side_nnz]
+    DevBuf sval;     // double/float[side_nnz]
+    bool has_vals = false, has_planes = false, has_list = false;
+    size_t bytes() const {
+        return ptr.bytes + trow.bytes + tgrp.bytes + mask.bytes + off.bytes + idx.bytes + val.bytes +
+               planes.bytes + sptr.bytes + srow.bytes + sval.bytes;
+    }
+    void release() {
+        for (DevBuf *b : {&ptr, &trow, &tgrp, &mask, &off, &idx, &val, &planes, &sptr, &srow, &sval})
+            b->release();
+    }
+};
+
+// Device counters shared by the kernels of one call (one cache line each group).
+struct Counters {
+    // x / frontier scan results
+    long long nLt, Wt, nLs, Ws;    // segment list size, tile work, side list size, side work
+    long long nCt, nCs;            // chunk counts
+    long long fsize, mf, din;      // BFS: |F|, sum outdeg(F), sum indeg(new owned)
+    long long y_nnz;
+    int err;                       // 1 = x not strictly ascending / out of range
+    int pad0;
+    unsigned int bid_scan;         // dynamic block-id counters (reset by the next kernel)
+    unsigned int bid_compact;
+    unsigned int chunk_next;       // work-queue head of the expand kernel
+    unsigned int pad1;
+    long long reached, edges;      // BFS totals
+};
+
+template <int K> struct LBDesc {
+    long long agg[K];
+    long long inc[K];
+    unsigned int status;  // (epoch << 2) | flag ; flag 1 = aggregate, 2 = inclusive prefix
+    unsigned int pad;
+};
+
+// Per-call list workspace (capacity grows on demand).
+struct Lists {
+    int64_t cap_seg = 0, cap_ent = 0, cap_ct = 0, cap_cs = 0, cap_blk = 0;
+    DevBuf Lt_seg, Lt_mask, Lt_first, Lt_tbeg, Lt_wpre;  // per non-empty segment with tiles
+    DevBuf Ls_beg, Ls_wpre, Ls_x, Ls_col;                // per x entry / vertex with side work
+    DevBuf Ct, Cs;                                        // chunk -> first list index
+    DevBuf xv;                                            // x values as double
+    DevBuf desc_scan;                                     // LBDesc<4>[blocks]
+    size_t bytes() const {
+        return Lt_seg.bytes + Lt_mask.bytes + Lt_first.bytes + Lt_tbeg.bytes + Lt_wpre.bytes +
+               Ls_beg.bytes + Ls_wpre.bytes + Ls_x.bytes + Ls_col.bytes + Ct.bytes + Cs.bytes +
+               xv.bytes + desc_scan.bytes;
+    }
+    void release() {
+        for (DevBuf *b : {&Lt_seg, &Lt_mask, &Lt_first, &Lt_tbeg, &Lt_wpre, &Ls_beg, &Ls_wpre, &Ls_x,
+                          &Ls_col, &Ct, &Cs, &xv, &desc_scan})
+            b->release();
+    }
+};
+
+constexpr int CHUNK_LOG = 7;               // 128 work items per warp-chunk
+constexpr int CHUNK = 1 << CHUNK_LOG;
+constexpr int SCAN_BLOCK = 256;
+
+}  // namespace tsmv
+
+struct tsmv_ctx {
+    int device = 0;
+    tsmv_options opt{};
+    tsmv_dtype dtype = TSMV_F64;
+    int nt = 16, lognt = 4;
+    int64_t m = 0, n = 0, nnz = 0, row_begin = 0;
+    int64_t nTR = 0, nTC = 0;
+    int sm_count = 148;
+    int expand_blocks = 0;     // persistent grid of the expand kernels
+    bool symmetric = false;
+    bool bfs_built = false;
+    double build_ms = 0;
+    std::vector<int64_t> row_splits;
+
+    tsmv::TileSet P;           // tile-CSC of A (SpMSpV + push kernels)
+    tsmv::TileSet Qown;        // tile-CSC of A^T (pull / Push-CSR) when A is not symmetric
+    tsmv::TileSet *Q = nullptr;
+
+    tsmv::DevBuf outdeg;       // int32[n]: nnz of column v (local rows)
+    tsmv::DevBuf indeg;        // int32[m]: nnz of row v
+
+    // SpMSpV workspaces (clear-on-read)
+    tsmv::DevBuf acc;          // double[m] (or ordered keys for MIN)
+    tsmv::DevBuf rowbits;      // uint32[ceil(m/32)]
+    tsmv::DevBuf desc_compact; // LBDesc<1>[blocks]
+    tsmv::Lists L;
+    tsmv::DevBuf counters;     // Counters
+    tsmv::Counters *hcnt = nullptr;  // mapped pinned mirror written by kernels
+    tsmv::Counters *hcnt_dev = nullptr;
+    unsigned int epoch = 0;
+
+    // host staging
+    tsmv::DevBuf stage_x_idx, stage_x_val, stage_y_idx, stage_y_val, stage_levels;
+
+    // BFS state
+    tsmv::DevBuf V, F0, F1;    // uint32[ceil(n/64)*2] visited, frontier ping-pong
+    tsmv::DevBuf desc_bfs;     // LBDesc<8>[ceil(nTC/256)+1]
+    tsmv::DevBuf splits_dev;   // int64[nranks+1]
+    int fcur = 0;
+    int32_t *levels_dev = nullptr;
+    int bfs_level = 0;
+    long long m_u_local = 0;
+    long long cur_fsize = 0, cur_mf = 0;
+
+    cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+};
+
+namespace tsmv {
+// builder.cu
+void build_tileset(tsmv_ctx *c, TileSet &S, const int32_t *rows, const int32_t *cols, const void *vals,
+                   int64_t nnz, int64_t dimR, int64_t dimC, bool want_vals, bool want_planes,
+                   cudaStream_t st);
+bool same_pattern_transposed(tsmv_ctx *c, const int32_t *rows, const int32_t *cols, int64_t nnz,
+                             cudaStream_t st);
+void prepare_csr(tsmv_ctx *c, const int64_t *row_ptr, const int32_t *col_idx, int32_t *rows, cudaStream_t st);
+// spmspv.cu
+void ensure_lists(tsmv_ctx *c, int64_t k);
+// bfs.cu
+int choose_dir(const tsmv_options &o, long long n, long long fsize, long long mf, long long mu);
+// pointer classification
+bool is_device_ptr(const void *p);
+}  // namespace tsmv

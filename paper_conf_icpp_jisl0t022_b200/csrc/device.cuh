@@ -1,0 +1,182 @@
+// device.cuh -- device helpers shared by the SpMSpV and TileBFS kernels:
+// single-pass decoupled look-back scan, dynamic block ids, list/chunk writers,
+// and the chunk -> list-entry window search of the load-balanced expand kernels.
+#pragma once
+#include "common.cuh"
+#include <cub/block/block_scan.cuh>
+
+namespace tsmv {
+
+struct Quad {
+    long long v[4];
+};
+struct QuadSum {
+    __device__ __forceinline__ Quad operator()(const Quad &a, const Quad &b) const {
+        Quad r;
+#pragma unroll
+        for (int i = 0; i < 4; ++i) r.v[i] = a.v[i] + b.v[i];
+        return r;
+    }
+};
+
+__device__ __forceinline__ unsigned ld_status(const LBDesc<4> *d) {
+    return *(volatile const unsigned *)&d->status;
+}
+template <int K> __device__ __forceinline__ unsigned ld_status_k(const LBDesc<K> *d) {
+    return *(volatile const unsigned *)&d->status;
+}
+
+// Decoupled look-back (one thread per block).  `agg` = this block's aggregate,
+// returns the exclusive prefix of all blocks before `bid`.  Blocks must obtain
+// `bid` in launch order (dynamic ids) so that predecessors are resident.
+template <int K>
+__device__ void lookback(LBDesc<K> *desc, unsigned bid, unsigned epoch, const long long *agg, long long *excl) {
+    const unsigned ep = (epoch & 0x3fffffffu) << 2;
+    LBDesc<K> *me = desc + bid;
+    if (bid == 0) {
+#pragma unroll
+        for (int i = 0; i < K; ++i) {
+            ((volatile long long *)me->inc)[i] = agg[i];
+            excl[i] = 0;
+        }
+        __threadfence();
+        *(volatile unsigned *)&me->status = ep | 2u;
+        return;
+    }
+#pragma unroll
+    for (int i = 0; i < K; ++i) ((volatile long long *)me->agg)[i] = agg[i];
+    __threadfence();
+    *(volatile unsigned *)&me->status = ep | 1u;
+    long long acc[K];
+#pragma unroll
+    for (int i = 0; i < K; ++i) acc[i] = 0;
+    int p = (int)bid - 1;
+    while (true) {
+        unsigned s = ld_status_k<K>(desc + p);
+        if ((s & ~3u) != ep || (s & 3u) == 0) continue;
+        __threadfence();
+        if ((s & 3u) == 2u) {
+#pragma unroll
+            for (int i = 0; i < K; ++i) acc[i] += ((volatile long long *)desc[p].inc)[i];
+            break;
+        }
+#pragma unroll
+        for (int i = 0; i < K; ++i) acc[i] += ((volatile long long *)desc[p].agg)[i];
+        --p;
+    }
+#pragma unroll
+    for (int i = 0; i < K; ++i) {
+        excl[i] = acc[i];
+        ((volatile long long *)me->inc)[i] = acc[i] + agg[i];
+    }
+    __threadfence();
+    *(volatile unsigned *)&me->status = ep | 2u;
+}
+
+// View of the per-call lists (raw pointers).
+struct ListsView {
+    long long *Lt_seg;            // segment id J
+    unsigned long long *Lt_mask;  // segment's x bits (nt bits)
+    long long *Lt_first;          // first x entry of the segment
+    long long *Lt_tbeg;           // first tile of tile column J
+    long long *Lt_wpre;           // exclusive tile-work prefix (+ sentinel at nLt)
+    long long *Ls_beg;            // first side nonzero of column j
+    long long *Ls_wpre;           // exclusive side-work prefix (+ sentinel)
+    double *Ls_x;                 // x_j
+    int *Ls_col;                  // j
+    int *Ct;                      // tile chunk -> first Lt entry
+    int *Cs;                      // side chunk -> first Ls entry
+    double *xv;                   // x values (double)
+};
+
+inline ListsView lists_view(tsmv_ctx *c) {
+    ListsView v;
+    v.Lt_seg = c->L.Lt_seg.as<long long>();
+    v.Lt_mask = c->L.Lt_mask.as<unsigned long long>();
+    v.Lt_first = c->L.Lt_first.as<long long>();
+    v.Lt_tbeg = c->L.Lt_tbeg.as<long long>();
+    v.Lt_wpre = c->L.Lt_wpre.as<long long>();
+    v.Ls_beg = c->L.Ls_beg.as<long long>();
+    v.Ls_wpre = c->L.Ls_wpre.as<long long>();
+    v.Ls_x = c->L.Ls_x.as<double>();
+    v.Ls_col = c->L.Ls_col.as<int>();
+    v.Ct = c->L.Ct.as<int>();
+    v.Cs = c->L.Cs.as<int>();
+    v.xv = c->L.xv.as<double>();
+    return v;
+}
+
+// Write chunk -> entry map for an entry owning work items [w0, w0+w).
+__device__ __forceinline__ void write_chunks(int *C, long long w0, long long w, int entry) {
+    long long c0 = (w0 + CHUNK - 1) >> CHUNK_LOG;
+    long long c1 = (w0 + w + CHUNK - 1) >> CHUNK_LOG;
+    for (long long ch = c0; ch < c1; ++ch) C[ch] = entry;
+}
+
+// Warp loads the work-prefix window of a chunk into shared memory:
+// win[q] = wpre[s0 + q] for q in [0, CHUNK], +inf past the list end.
+__device__ __forceinline__ void load_window(long long *win, const long long *wpre, long long s0, long long nL,
+                                            int lane) {
+    for (int q = lane; q <= CHUNK; q += 32) {
+        long long idx = s0 + q;
+        win[q] = idx <= nL ? wpre[idx] : 0x7fffffffffffffffLL;
+    }
+    __syncwarp();
+}
+
+// Largest q in [0, CHUNK] with win[q] <= i (win[0] <= i guaranteed).
+__device__ __forceinline__ int window_find(const long long *win, long long i) {
+    int lo = 0, hi = CHUNK;  // invariant win[lo] <= i, answer in [lo, hi]
+    while (lo < hi) {
+        int mid = (lo + hi + 1) >> 1;
+        if (win[mid] <= i) lo = mid;
+        else hi = mid - 1;
+    }
+    return lo;
+}
+
+// Segment bits of an NT-segment inside uint32 bitmap words.
+template <int NT> __device__ __forceinline__ typename Tr<NT>::word_t seg_bits(const uint32_t *bm, long long J) {
+    if constexpr (NT == 16) {
+        return (uint16_t)(bm[J >> 1] >> ((J & 1) * 16));
+    } else if constexpr (NT == 32) {
+        return bm[J];
+    } else {
+        return ((unsigned long long)bm[2 * J + 1] << 32) | bm[2 * J];
+    }
+}
+
+// OR bits into an NT-segment, returns the previous segment bits.
+template <int NT>
+__device__ __forceinline__ typename Tr<NT>::word_t seg_or(uint32_t *bm, long long J, typename Tr<NT>::word_t bits) {
+    if constexpr (NT == 16) {
+        int sh = (J & 1) * 16;
+        unsigned old = atomicOr(&bm[J >> 1], (unsigned)bits << sh);
+        return (uint16_t)(old >> sh);
+    } else if constexpr (NT == 32) {
+        return atomicOr(&bm[J], bits);
+    } else {
+        return atomicOr((unsigned long long *)(bm + 2 * J), bits);
+    }
+}
+
+template <class W> __device__ __forceinline__ int popc_w(W w) {
+    if constexpr (sizeof(W) == 8) return __popcll(w);
+    else return __popc((unsigned)w);
+}
+template <class W> __device__ __forceinline__ int ffs_w(W w) {
+    if constexpr (sizeof(W) == 8) return __ffsll((long long)w) - 1;
+    else return __ffs((unsigned)w) - 1;
+}
+
+// order-preserving map double -> uint64 (unsigned order == numeric order)
+__device__ __forceinline__ unsigned long long ord_key(double x) {
+    unsigned long long b = (unsigned long long)__double_as_longlong(x);
+    return (b >> 63) ? ~b : (b | 0x8000000000000000ull);
+}
+__device__ __forceinline__ double ord_val(unsigned long long k) {
+    unsigned long long b = (k >> 63) ? (k & 0x7fffffffffffffffull) : ~k;
+    return __longlong_as_double((long long)b);
+}
+
+}  // namespace tsmv

@@ -1,0 +1,62 @@
+"""CPU-side checks of the C-ABI boundary: libtsmv.so loads and exports every
+function include/tsmv.h declares; host-only entry points behave."""
+import ctypes
+import os
+import re
+
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _declared():
+    src = open(os.path.join(ROOT, "include", "tsmv.h")).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    names = set(re.findall(r"\b(tsmv_[a-z_0-9]+)\s*\(", src))
+    return sorted(names)
+
+
+@pytest.fixture(scope="module")
+def lib():
+    from paper_conf_icpp_jisl0t022_b200 import build
+    build.build()
+    return ctypes.CDLL(build.LIB)
+
+
+def test_every_declared_symbol_exported(lib):
+    names = _declared()
+    assert len(names) >= 15
+    for n in names:
+        assert hasattr(lib, n), f"{n} declared in include/tsmv.h but not exported"
+
+
+def test_binding_covers_abi():
+    from paper_conf_icpp_jisl0t022_b200 import tsmv
+    assert set(_declared()) == set(tsmv.EXPORTED)
+
+
+def test_host_only_calls():
+    from paper_conf_icpp_jisl0t022_b200 import tsmv
+    assert tsmv.tsmv_version() >> 16 == 1
+    o = tsmv.default_options()
+    assert o.tile_dim == 16 and o.sparse_tile_max_nnz == 2 and o.nranks == 1
+    assert abs(o.push_csr_density - 0.01) < 1e-15
+    # direction rule (reading R9)
+    assert tsmv.choose_dir(1000, 1, 10, 10_000) == tsmv.DIR_PUSH_CSC
+    assert tsmv.choose_dir(1000, 10, 10, 10_000) == tsmv.DIR_PUSH_CSR
+    assert tsmv.choose_dir(1000, 10, 1000, 10_000) == tsmv.DIR_PULL_CSC
+    o.force_dir = tsmv.DIR_PUSH_CSR
+    assert tsmv.choose_dir(1000, 1, 1000, 10, o) == tsmv.DIR_PUSH_CSR
+    assert tsmv.tsmv_destroy(None) == tsmv.OK
+    assert tsmv.tsmv_owned_words(None) == 0
+
+
+def test_create_rejects_bad_args_without_gpu():
+    from paper_conf_icpp_jisl0t022_b200 import tsmv
+    ctx = ctypes.c_void_p()
+    o = tsmv.default_options(tile_dim=24)
+    rp = (ctypes.c_int64 * 2)(0, 0)
+    st = tsmv.tsmv_create(ctypes.byref(ctx), 1, 1, ctypes.cast(rp, ctypes.c_void_p), None, None, tsmv.PATTERN,
+                          ctypes.byref(o))
+    assert st == tsmv.EINVAL and b"tile_dim" in tsmv.tsmv_last_error()
+    assert not ctx.value

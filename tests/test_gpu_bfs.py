@@ -1,0 +1,121 @@
+"""GPU parity of tsmv_bfs (TileBFS: Push-CSC / Push-CSR / Pull-CSC, Sec 3.4)
+against the oracle's queue BFS: bit-exact int32 levels, for every forced
+direction and the automatic rule, over tile sizes, thresholds, directed and
+undirected graphs, and the BASELINE BFS configs."""
+import json
+import os
+
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import synth
+
+pytestmark = pytest.mark.gpu
+DEV = torch.device("cuda", 0)
+GOLD = os.path.join(os.path.dirname(__file__), "golden")
+DIRS = [0, 1, 2, 3]   # auto, push_csc, push_csr, pull_csc
+
+
+@pytest.fixture(scope="module")
+def tsmv():
+    from paper_conf_icpp_jisl0t022_b200 import tsmv as t
+    return t
+
+
+def _levels(tsmv, A, sources, dirs=DIRS, **opts):
+    C = oracle.csc_of(A)
+    Ad = A.to(DEV)
+    for d in dirs:
+        M = tsmv.TiledMatrix.from_csr(Ad, dtype="pattern", force_dir=d, **opts)
+        for s in sources:
+            lv, st = M.bfs(s)
+            ref = oracle.bfs_queue(C, s)
+            got = lv.cpu().numpy()
+            assert np.array_equal(got, ref), f"dir={d} src={s}: {np.sum(got != ref)} levels differ"
+            assert st["reached"] == int((ref >= 0).sum())
+            assert st["nlevels"] == int(ref.max()) + 1
+        M.close()
+
+
+def test_c1_grid_closed_form(tsmv):
+    A = synth.stencil2d(64, 64)
+    M = tsmv.TiledMatrix.from_csr(A.to(DEV))      # fp64 context also carries the BFS tiles
+    lv, st = M.bfs(0)
+    v = np.arange(4096)
+    assert np.array_equal(lv.cpu().numpy(), v // 64 + v % 64)
+    assert st["nlevels"] == 127
+    _levels(tsmv, A, [0, 2080, 4095])
+
+
+@pytest.mark.parametrize("nt", [16, 32, 64])
+@pytest.mark.parametrize("thr", [0, 2, 8])
+def test_rmat_sym_tiles(tsmv, nt, thr):
+    A = synth.rmat(12, 16, seed=3, symmetrize=True)
+    _levels(tsmv, A, synth.sample_sources(A, 2, seed=1) + [0], tile_dim=nt, sparse_tile_max_nnz=thr)
+
+
+@pytest.mark.parametrize("nt", [16, 64])
+def test_rmat_directed_pull_uses_in_edges(tsmv, nt):
+    A = synth.rmat(12, 8, seed=6)        # directed: A != A^T
+    M = tsmv.TiledMatrix.from_csr(A.to(DEV), dtype="pattern")
+    assert M.info()["symmetric"] == 0
+    _levels(tsmv, A, synth.sample_sources(A, 3, seed=4), tile_dim=nt)
+
+
+def test_3d_and_band(tsmv):
+    A = synth.stencil3d(16)
+    _levels(tsmv, A, [0, 2000])
+    B = synth.banded(4096, 8)
+    M = tsmv.TiledMatrix.from_csr(B.to(DEV))
+    lv, st = M.bfs(0)
+    v = np.arange(4096)
+    assert np.array_equal(lv.cpu().numpy(), (v + 7) // 8)
+    _levels(tsmv, B, [100], dirs=[0, 1, 3])
+
+
+def test_toys_and_ragged(tsmv):
+    _levels(tsmv, synth.from_edges(5, [(0, 1), (1, 2), (2, 3), (3, 4)]), [0, 2])
+    _levels(tsmv, synth.from_edges(6, [(0, 1), (2, 3)]), [0, 5])          # isolated source
+    _levels(tsmv, synth.from_edges(3, [(1, 0), (2, 1)], symmetric=False), [0, 2])
+    _levels(tsmv, synth.uniform(1000, 1000, 2, seed=3), [0, 999])        # n not a multiple of 32
+    _levels(tsmv, synth.rmat(9, 4, seed=2, symmetrize=True), [0], tile_dim=64)
+    _levels(tsmv, synth.from_edges(1, []) if False else synth.csr_from_keys(torch.tensor([0]), 1, 1), [0])
+
+
+def test_fig5_graph_and_bitmasks(tsmv):
+    g = json.load(open(os.path.join(GOLD, "fig5_bfs_trace.json")))
+    A = synth.from_edges(g["n"], g["undirected_edges"])
+    _levels(tsmv, A, [0])
+    # bitmask tiles of the GPU builder == oracle's Sec 3.2.3 tiles (nt = 16 here)
+    B = synth.rmat(8, 8, seed=1, symmetrize=True)
+    for thr in (0, 2):
+        M = tsmv.TiledMatrix.from_csr(B.to(DEV), dtype="pattern", sparse_tile_max_nnz=thr)
+        for orient in (0, 1):
+            got = M.export_bitmask_tiles(orient)
+            ref = oracle.bitmask_tiles(B.m, B.n, B.row_ptr, B.col_idx, 16, orient, max_tiles=1 << 14)
+            assert got == ref
+
+
+def test_repeated_traversals_clean_state(tsmv):
+    A = synth.rmat(13, 16, seed=8, symmetrize=True)
+    C = oracle.csc_of(A)
+    M = tsmv.TiledMatrix.from_csr(A.to(DEV), dtype="pattern")
+    for s in synth.sample_sources(A, 5, seed=9):
+        lv, _ = M.bfs(s)
+        assert np.array_equal(lv.cpu().numpy(), oracle.bfs_queue(C, s))
+    host = torch.empty(A.n, dtype=torch.int32)
+    lv, _ = M.bfs(0, levels=host)
+    assert np.array_equal(host.numpy(), oracle.bfs_queue(C, 0))
+
+
+def test_c3_rmat_s20_sym_directions(tsmv):
+    A = synth.rmat(20, 16, seed=1, symmetrize=True, device=DEV).to("cpu")
+    _levels(tsmv, A, [0] + synth.sample_sources(A, 1, seed=1))
+
+
+@pytest.mark.slow
+def test_c3_rmat_s22_sym(tsmv):
+    A = synth.rmat(22, 16, seed=1, symmetrize=True, device=DEV).to("cpu")
+    _levels(tsmv, A, [0], dirs=[0])

@@ -115,11 +115,17 @@ __device__ __forceinline__ void write_chunks(int *C, long long w0, long long w, 
 
 // Warp loads the work-prefix window of a chunk into shared memory:
 // win[q] = wpre[s0 + q] for q in [0, CHUNK], +inf past the list end.
+// The trip count is warp-uniform on purpose: with a lane-dependent count
+// (q = lane; q <= CHUNK) ptxas compiled the following __syncwarp() to a NOP and
+// lanes read win[CHUNK] before lane 0 had stored it (found on B200, r1).
 __device__ __forceinline__ void load_window(long long *win, const long long *wpre, long long s0, long long nL,
                                             int lane) {
-    for (int q = lane; q <= CHUNK; q += 32) {
+#pragma unroll
+    for (int q0 = 0; q0 <= CHUNK; q0 += 32) {
+        int q = q0 + lane;
         long long idx = s0 + q;
-        win[q] = idx <= nL ? wpre[idx] : 0x7fffffffffffffffLL;
+        long long v = idx <= nL ? wpre[idx] : 0x7fffffffffffffffLL;
+        if (q <= CHUNK) win[q] = v;
     }
     __syncwarp();
 }

@@ -371,6 +371,32 @@ void ensure_lists(tsmv_ctx *c, int64_t k) {
     }
 }
 
+// Debug aid (TSMV_CHECK_LISTS=1): validate the k_xscan lists on the host.
+void debug_check_lists(tsmv_ctx *c, cudaStream_t st) {
+    TSMV_CUDA(cudaStreamSynchronize(st));
+    Counters h;
+    TSMV_CUDA(cudaMemcpy(&h, c->counters.p, sizeof(h), cudaMemcpyDeviceToHost));
+    auto chk = [&](const char *nm, const DevBuf &wpre_b, const DevBuf &C_b, long long nL, long long W, long long nC) {
+        std::vector<long long> wpre(nL + 1);
+        std::vector<int> C(nC);
+        TSMV_CUDA(cudaMemcpy(wpre.data(), wpre_b.p, (nL + 1) * 8, cudaMemcpyDeviceToHost));
+        if (nC) TSMV_CUDA(cudaMemcpy(C.data(), C_b.p, nC * 4, cudaMemcpyDeviceToHost));
+        int bad = 0;
+        if (nL && wpre[0] != 0) fprintf(stderr, "[%s] wpre[0]=%lld\n", nm, wpre[0]), ++bad;
+        if (wpre[nL] != W) fprintf(stderr, "[%s] sentinel %lld != W %lld\n", nm, wpre[nL], W), ++bad;
+        for (long long i = 0; i + 1 <= nL && bad < 10; ++i)
+            if (wpre[i + 1] <= wpre[i]) fprintf(stderr, "[%s] wpre[%lld]=%lld wpre[+1]=%lld\n", nm, i, wpre[i], wpre[i + 1]), ++bad;
+        for (long long ch = 0; ch < nC && bad < 20; ++ch) {
+            long long it = ch << CHUNK_LOG, s = C[ch];
+            if (s < 0 || s >= nL || !(wpre[s] <= it && it < wpre[s + 1]))
+                fprintf(stderr, "[%s] chunk %lld -> %lld wrong\n", nm, ch, s), ++bad;
+        }
+        fprintf(stderr, "[%s] nL=%lld W=%lld nC=%lld bad=%d\n", nm, nL, W, nC, bad);
+    };
+    chk("tile", c->L.Lt_wpre, c->L.Ct, h.nLt, h.Wt, h.nCt);
+    chk("side", c->L.Ls_wpre, c->L.Cs, h.nLs, h.Ws, h.nCs);
+}
+
 }  // namespace tsmv
 
 using namespace tsmv;
@@ -432,6 +458,7 @@ extern "C" tsmv_status tsmv_spmspv(tsmv_ctx *c, tsmv_semiring sr, int64_t x_nnz,
             default: launch_xscan<64>(c, xi, xv, f32, x_nnz, st); break;
         }
         TSMV_CUDA(cudaGetLastError());
+        if (getenv("TSMV_CHECK_LISTS")) debug_check_lists(c, st);
         if (f32) {
             switch (c->nt) {
                 case 16: launch_expand_sr<16, float>(c, sr, st); break;

@@ -1,0 +1,444 @@
+#!/usr/bin/env python
+"""Benchmark of the TileSpMSpV / TileBFS hot path (BASELINE.json metric:
+"SpMSpV GFLOPS & %HBM roofline; TileBFS GTEPS").
+
+Default workload (config T of SURVEY §8, the north_star roofline target, the
+largest single-GPU case BASELINE names): R-MAT scale 22, edge factor 16,
+Graph500 (0.57, 0.19, 0.19, 0.05), directed, duplicates coalesced, fp64 values
+1+u; x = 1 % density (41,943 distinct uniform indices, values 1+u), a fresh x
+sample per step (seeds 1..W+K).  One step = one y = A x call (x tiling, tile
+intersection + multiply + side-matrix merge, y compaction: SURVEY §8(a) a2-a6);
+the tile format (a1) is built once outside the timed region and timed
+separately; TileBFS (a7) on the symmetrised R-MAT s22 is reported in "bfs".
+
+Timing: inputs resident in HBM; before every step the L2 is flushed by writing
+a 256 MiB buffer (outside the events); each step is bracketed by CUDA events on
+the launching stream; K steps between barriers; max over ranks.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl tsmv|reference]
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import torch  # noqa: E402
+
+import synth  # noqa: E402
+
+FALLBACK_HBM = 6650.0  # GB/s, B200_PROFILING.md fallback
+
+
+def parse():
+    p = argparse.ArgumentParser()
+    p.add_argument("--gpus", type=int, default=1)
+    p.add_argument("--steps", type=int, default=30)
+    p.add_argument("--warmup", type=int, default=5)
+    p.add_argument("--impl", default="tsmv", choices=["tsmv", "reference"])
+    p.add_argument("--scale", type=int, default=22)
+    p.add_argument("--density", type=float, default=0.01)
+    p.add_argument("--dtype", default="f64", choices=["f64", "f32"])
+    p.add_argument("--tile-dim", type=int, default=16)
+    p.add_argument("--thr", type=int, default=2)
+    p.add_argument("--bfs-scale", type=int, default=22)
+    p.add_argument("--bfs-sources", type=int, default=4)
+    p.add_argument("--no-bfs", action="store_true")
+    p.add_argument("--no-cpu", action="store_true")
+    p.add_argument("--cpu-seconds", type=float, default=12.0)
+    return p.parse_args()
+
+
+def peaks():
+    path = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        d = json.load(open(path))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json)"
+    except Exception:
+        return FALLBACK_HBM, "fallback (B200_PROFILING.md)"
+
+
+class Clocks:
+    """nvidia-smi sampler running during the timed region."""
+
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index = index
+        self.proc = None
+        self.path = f"/tmp/tsmv_clocks_{os.getpid()}.csv"
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=open(self.path, "w"), stderr=subprocess.DEVNULL)
+        except Exception:
+            self.proc = None
+
+    def stop(self):
+        if self.proc is None:
+            return None
+        time.sleep(0.25)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        sm, mx, reasons = [], 0.0, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for line in open(self.path):
+            f = [x.strip() for x in line.split(",")]
+            if len(f) < 9:
+                continue
+            try:
+                sm.append(float(f[1]))
+                mx = max(mx, float(f[2]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, f[5:9]):
+                if v.lower() == "active":
+                    reasons.add(nm)
+        if not sm:
+            return None
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": mx, "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+def dist_env():
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return world, rank, local
+
+
+def make_matrix(scale, dtype, device):
+    base = synth.rmat(scale, 16, seed=1, device=device)
+    return synth.attach_values(base, seed=1, dtype=dtype)
+
+
+def x_samples(n, k, count, dtype, device):
+    return [synth.sample_x(n, k, seed=1 + s, device=device, dtype=dtype) for s in range(count)]
+
+
+# --------------------------------------------------------------------------- reference arm
+def run_reference(args):
+    """The oracle (plain single-thread C, oracle/oracle.c) timed on the host on
+    the same config / metric; each step = one oracle y = A x on one x sample."""
+    import oracle
+    world, rank, _ = dist_env()
+    if world > 1 and rank != 0:
+        return
+    dev = "cuda" if torch.cuda.is_available() else "cpu"
+    A = make_matrix(args.scale, args.dtype, dev).to("cpu")
+    C = oracle.csc_of(A)
+    colcnt = torch.from_numpy(C.col_ptr[1:] - C.col_ptr[:-1])
+    k = synth.density_k(A.n, args.density)
+    xs = x_samples(A.n, k, args.warmup + args.steps, args.dtype, "cpu")
+    for s in range(args.warmup):
+        oracle.spmspv(C, xs[s][0], xs[s][1])
+    flops, tsum, times = 0, 0.0, []
+    for s in range(args.warmup, args.warmup + args.steps):
+        xi, xv = xs[s]
+        t0 = time.perf_counter()
+        oracle.spmspv(C, xi, xv)
+        dt = time.perf_counter() - t0
+        times.append(dt)
+        tsum += dt
+        flops += 2 * int(colcnt[xi.long()].sum())
+    val = flops / tsum / 1e9
+    line = {"impl": "reference", "metric": "spmspv_gflops", "value": round(val, 4), "unit": "GFLOP/s",
+            "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": round(1e3 * tsum / args.steps, 4), "higher_is_better": True, "scaling": "strong",
+            "vs_baseline": None, "dtype": args.dtype, "data": "synthetic",
+            "config": workload_config(args),
+            "cpu_baseline": {"value": round(val, 4), "unit": "GFLOP/s", "cores": 1, "kind": "oracle",
+                             "sample": f"{args.steps} x samples of k={k} on R-MAT s{args.scale} "
+                                       f"(oracle CSC built once, untimed)"},
+            "e2e": {"value": round(val, 4), "unit": "GFLOP/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def workload_config(args):
+    return {"workload": f"rmat_s{args.scale}_ef16_directed_{args.dtype}_x{args.density * 100:g}pct",
+            "matrix": f"R-MAT scale {args.scale}, edgefactor 16, (0.57,0.19,0.19,0.05), unpermuted, coalesced",
+            "x_density": args.density, "tile_dim": args.tile_dim, "sparse_tile_max_nnz": args.thr,
+            "l2": "flushed before every step (256 MiB write + 256 MiB read of another buffer, outside the events)",
+            "parallelism": f"row-block x{args.gpus}" if args.gpus > 1 else "single GPU"}
+
+
+# --------------------------------------------------------------------------- our arm
+class L2Flush:
+    """Cold, clean L2 before a timed step: write a 256 MiB buffer (> 126 MB L2), then
+    read a second 256 MiB buffer so that the dirty lines of the first are written
+    back here, outside the timed region, instead of inside the next kernels."""
+
+    def __init__(self, dev):
+        self.w = torch.empty(64 * 1024 * 1024, dtype=torch.float32, device=dev)
+        self.r = torch.ones(64 * 1024 * 1024, dtype=torch.float32, device=dev)
+
+    def __call__(self):
+        self.w.zero_()
+        self.sink = self.r.sum()
+
+def flops_of(colcnt, xi):
+    return 2 * int(colcnt[xi.long()].sum())
+
+
+def call_bytes(st, k, sv, nt, m):
+    """Algorithmic bytes of one tsmv_spmspv call (= one launch of the fused kernel)
+    for this build's data layout: every byte the method must
+    touch once, at its natural width, no sector rounding."""
+    si = 1 if nt == 16 else 2        # packed in-tile row index
+    cs = 1 if nt == 16 else 2        # column start offset inside a tile
+    mask_b = nt // 8
+    phase_a = (k * (4 + sv)                      # read x (index, value)
+               + k * 16 + st["x_segments"] * 16  # side col_ptr pair per entry, tile col_ptr pair per segment
+               + k * 8                           # scatter x_j -> xd[j]
+               + st["x_segments"] * 32 + k * 24)  # segment / side list entries written
+    phase_b = (st["tile_items"] * mask_b            # column mask of every tile in a hit tile column
+               + st["x_segments"] * 24 + k * 16     # list entries read back
+               + st["hit_tiles"] * 16               # TileDesc {off, row, nnz} of tiles whose mask meets x
+               + st["hit_columns"] * (2 * cs + 8)   # column start/end + x_j for every hit column
+               + st["tile_macs"] * (si + sv)        # row index + value of every useful tile nonzero
+               + st["side_items"] * (4 + sv)        # row + value of every useful side nonzero
+               + st["y_nnz"] * (8 + 4))             # accumulator write + touched word per output row
+    phase_c = (m // 8                               # touched bitmap scan
+               + st["y_nnz"] * (8 + 8 + 4 + sv))    # acc read + clear, y index + value
+    return phase_a + phase_b + phase_c
+
+
+def survey_bytes(st, k, sv, nt, macs):
+    """SURVEY §8(d) B_alg for the whole call (tile descriptor 4+8+nt/8 B per tile in a
+    hit column; fp value + 1..2 B index per useful tile nonzero; side col_ptr pair per
+    x entry; 4 B + value per useful side nonzero; read x; write y)."""
+    si = 1 if nt == 16 else 2
+    return (st["tile_items"] * (4 + 8 + nt // 8) + (macs - st["side_items"]) * (sv + si) + k * 16
+            + st["side_items"] * (4 + sv) + k * (4 + sv) + st["y_nnz"] * (4 + sv))
+
+
+def run_tsmv(args):
+    world, rank, local = dist_env()
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    from paper_conf_icpp_jisl0t022_b200 import tsmv
+    sv = 4 if args.dtype == "f32" else 8
+    peak, peak_src = peaks()
+
+    A = make_matrix(args.scale, args.dtype, dev)
+    colcnt = torch.bincount(A.col_idx.long(), minlength=A.n)
+    k = synth.density_k(A.n, args.density)
+    xs = x_samples(A.n, k, args.warmup + args.steps, args.dtype, dev)
+    flush = L2Flush(dev)
+
+    if world > 1:
+        from paper_conf_icpp_jisl0t022_b200 import dist as tdist
+        splits = tdist.partition_rows(A.row_ptr, world)
+        Al = tdist.local_rows(A, splits, rank)
+        D = tdist.DistTiledMatrix(Al, splits, rank, world, dtype=args.dtype, device=local,
+                                  tile_dim=args.tile_dim, sparse_tile_max_nnz=args.thr)
+        M = D.M
+    else:
+        D = None
+        M = tsmv.TiledMatrix.from_csr(A, dtype=args.dtype, tile_dim=args.tile_dim,
+                                      sparse_tile_max_nnz=args.thr, build_bfs=0)
+    info = M.info()
+    y_idx = torch.empty(M.m, dtype=torch.int32, device=dev)
+    y_val = torch.empty(M.m, dtype=torch.float32 if args.dtype == "f32" else torch.float64, device=dev)
+    y_nnz = torch.zeros(1, dtype=torch.int64, device=dev)
+
+    def step(s):
+        xi, xv = xs[s]
+        if D is None:
+            M.spmspv_async(xi, xv, y_idx, y_val, y_nnz)
+        else:
+            lo, hi = D.splits[rank], D.splits[rank + 1]
+            own = (xi >= lo) & (xi < hi)
+            D.spmspv(xi[own], xv[own])
+
+    for s in range(args.warmup):
+        flush()
+        step(s)
+    torch.cuda.synchronize()
+
+    clocks = Clocks(local) if rank == 0 else None
+    if clocks:
+        clocks.start()
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    flops, kexp_bytes, svy_bytes, step_stats = 0, 0, 0, []
+    M.set_timing(True)
+    if world > 1:
+        torch.distributed.barrier()
+    torch.cuda.synchronize()
+    for i in range(args.steps):
+        s = args.warmup + i
+        flush()
+        ev[i][0].record()
+        step(s)
+        ev[i][1].record()
+        torch.cuda.synchronize()
+        st = M.last_call_stats()
+        flops += flops_of(colcnt, xs[s][0]) if world == 1 else 0
+        kexp_bytes += call_bytes(st, k, sv, args.tile_dim, M.m)
+        macs = flops_of(colcnt, xs[s][0]) // 2
+        svy_bytes += survey_bytes(st, k, sv, args.tile_dim, macs)
+        step_stats.append(st)
+    torch.cuda.synchronize()
+    if world > 1:
+        torch.distributed.barrier()
+    kt, ncalls = M.get_timing()
+    M.set_timing(False)
+    clk = clocks.stop() if clocks else None
+    ms = sum(e0.elapsed_time(e1) for e0, e1 in ev)
+    if world > 1:
+        import torch.distributed as dist
+        t = torch.tensor([ms], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t)
+        flops = sum(flops_of(colcnt, xs[args.warmup + i][0]) for i in range(args.steps))
+    value = flops / (ms * 1e-3) / 1e9
+
+    # roofline of the dominant (only) kernel: one k_spmspv_fused launch per call,
+    # algorithmic bytes / its CUDA-event duration
+    kms = ms / args.steps
+    achieved = (kexp_bytes / args.steps) / (kms * 1e-3) / 1e9
+    traffic = None
+    tpath = os.path.join(ROOT, "profiles", "fused_traffic.json")
+    if os.path.exists(tpath):
+        try:
+            traffic = json.load(open(tpath)).get("dram_bytes_per_launch")
+        except Exception:
+            traffic = None
+    n_ = max(ncalls, 1)
+    roof = {"bound": "hbm", "achieved": round(achieved, 2), "peak": peak, "unit": "GB/s",
+            "frac": round(achieved / peak, 4), "traffic": traffic,
+            "kernel": "k_spmspv_fused (the whole call is one cooperative launch)",
+            "peak_source": peak_src,
+            "algorithmic_bytes_per_launch": int(kexp_bytes / args.steps),
+            "kernel_ms_per_launch": round(kms, 5),
+            "phase_ms_per_launch (globaltimer, CTA 0)": {
+                "A_x_tiling": round(kt[0] / n_, 5), "B_intersect_multiply": round(kt[1] / n_, 5),
+                "C_compact": round(kt[2] / n_, 5), "whole": round(kt[3] / n_, 5)},
+            "survey_B_alg": {"bytes": int(svy_bytes / args.steps),
+                             "achieved_GBps": round(svy_bytes / (ms * 1e-3) / 1e9, 2),
+                             "frac": round(svy_bytes / (ms * 1e-3) / 1e9 / peak, 4)}}
+
+    # e2e through the public synchronous API with pinned host buffers (N = 1)
+    e2e = None
+    if world == 1:
+        hx = [(xi.cpu().pin_memory(), xv.cpu().pin_memory()) for xi, xv in xs[args.warmup:]]
+        hy_i = torch.empty(M.m, dtype=torch.int32).pin_memory()
+        hy_v = torch.empty(M.m, dtype=y_val.dtype).pin_memory()
+        for xi, xv in hx[:3]:
+            M.spmspv(xi, xv, y_idx=hy_i, y_val=hy_v)
+        t_e2e, h2d, d2h = 0.0, 0, 0
+        for i, (xi, xv) in enumerate(hx):
+            flush()
+            torch.cuda.synchronize()
+            t0 = time.perf_counter()
+            yi, yv = M.spmspv(xi, xv, y_idx=hy_i, y_val=hy_v)
+            t_e2e += time.perf_counter() - t0
+            h2d += xi.numel() * 4 + xv.numel() * sv
+            d2h += yi.numel() * (4 + sv)
+        e2e = {"value": round(flops / t_e2e / 1e9, 3), "unit": "GFLOP/s",
+               "h2d_bytes_per_step": int(h2d / len(hx)), "d2h_bytes_per_step": int(d2h / len(hx)),
+               "ms_per_step": round(1e3 * t_e2e / len(hx), 4),
+               "path": "tsmv_spmspv (C ABI) with pinned host x and y; wall clock per call"}
+
+    bfs = None
+    if not args.no_bfs and world == 1:
+        bfs = run_bfs(args, dev, flush, tsmv)
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu:
+        cpu = cpu_baseline(args, A, colcnt, xs)
+
+    if rank == 0:
+        mean_st = {kk: sum(s_[kk] for s_ in step_stats) / len(step_stats) for kk in step_stats[0]}
+        line = {"metric": "spmspv_gflops", "value": round(value, 3), "unit": "GFLOP/s", "n_gpus": world,
+                "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms / args.steps, 5),
+                "higher_is_better": True, "scaling": "strong",
+                "vs_baseline": None, "dtype": args.dtype, "data": "synthetic (seeded R-MAT, seeded x)",
+                "config": workload_config(args), "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,
+                "gpu_launches": args.steps, "clocks": clk,
+                "per_step": {"k": k, "mean_flops": int(flops / args.steps),
+                             **{kk: round(v, 1) for kk, v in mean_st.items() if kk != "x_nnz"}},
+                "format": {kk: info[kk] for kk in ("nnz", "n_tiles", "n_dense_tiles", "dense_nnz", "side_nnz",
+                                                   "build_ms", "bytes_spmspv")},
+                "bfs": bfs}
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        torch.distributed.destroy_process_group()
+
+
+def run_bfs(args, dev, flush, tsmv):
+    """TileBFS GTEPS on the symmetrised R-MAT (BASELINE config 3 shape)."""
+    A = synth.rmat(args.bfs_scale, 16, seed=1, symmetrize=True, device=dev)
+    t0 = time.perf_counter()
+    M = tsmv.TiledMatrix.from_csr(A, dtype="pattern", tile_dim=args.tile_dim, sparse_tile_max_nnz=args.thr)
+    build_wall = time.perf_counter() - t0
+    info = M.info()
+    srcs = [0] + synth.sample_sources(A, max(0, args.bfs_sources - 1), seed=1)
+    levels = torch.empty(A.n, dtype=torch.int32, device=dev)
+    M.bfs(srcs[0], levels=levels)  # warm-up
+    runs = []
+    for s in srcs:
+        flush()
+        torch.cuda.synchronize()
+        _, st = M.bfs(s, levels=levels)
+        runs.append({"source": int(s), "ms": round(st["ms"], 4), "levels": st["nlevels"],
+                     "edges": st["edges_traversed"], "reached": st["reached"],
+                     "gteps": round(st["edges_traversed"] / (st["ms"] * 1e-3) / 1e9, 3),
+                     "dirs": "".join({"push_csc": "C", "push_csr": "R", "pull_csc": "P"}.get(d, "?")
+                                     for d in st["dirs"])})
+    hm = len(runs) / sum(1.0 / r["gteps"] for r in runs if r["gteps"] > 0)
+    M.close()
+    return {"graph": f"rmat_s{args.bfs_scale}_ef16_sym", "nnz": info["nnz"], "gteps_hmean": round(hm, 3),
+            "build_ms": round(info["build_ms"], 2), "build_wall_s": round(build_wall, 3),
+            "edge_count": "sum of out-degrees of reached vertices (directed count of the symmetrised graph)",
+            "runs": runs}
+
+
+def cpu_baseline(args, A, colcnt, xs):
+    """The oracle as it stands on the host, bounded to ~cpu_seconds of CPU work."""
+    import oracle
+    Ac = A.to("cpu")
+    C = oracle.csc_of(Ac)
+    flops, t = 0, 0.0
+    used = 0
+    for xi, xv in xs:
+        xi_c, xv_c = xi.cpu(), xv.cpu()
+        t0 = time.perf_counter()
+        oracle.spmspv(C, xi_c, xv_c)
+        t += time.perf_counter() - t0
+        flops += flops_of(colcnt.cpu(), xi_c)
+        used += 1
+        if t > args.cpu_seconds:
+            break
+    return {"value": round(flops / t / 1e9, 5), "unit": "GFLOP/s", "cores": 1, "kind": "oracle",
+            "sample": f"{used} x samples (k={xs[0][0].numel()}) of the same workload, oracle CSC built once untimed"}
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_tsmv(args)
+
+
+if __name__ == "__main__":
+    main()

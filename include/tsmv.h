@@ -83,6 +83,9 @@ typedef struct {
     int64_t tile_items;     /* tiles in the tile columns of non-empty segments (a3) */
     int64_t side_items;     /* side-matrix nonzeros in the columns of x (a5) */
     int64_t y_nnz;
+    int64_t hit_tiles;      /* tiles whose column mask intersects the segment mask */
+    int64_t hit_columns;    /* (tile, column) pairs in both the tile's and x's masks */
+    int64_t tile_macs;      /* useful multiply-adds inside tiles (side ones = side_items) */
 } tsmv_call_stats;
 
 /* Built-format census. */
@@ -143,6 +146,22 @@ tsmv_status tsmv_create(tsmv_ctx **out, int64_t nrows, int64_t ncols, const int6
 tsmv_status tsmv_spmspv(tsmv_ctx *c, tsmv_semiring sr, int64_t x_nnz, const int32_t *x_idx,
                         const void *x_val, int64_t y_cap, int32_t *y_idx, void *y_val,
                         int64_t *y_nnz, void *cuda_stream);
+
+/* Asynchronous variant for pipelines and benchmarks: same semantics, but every
+ * pointer must be device memory, nothing is synchronised, and the result size is
+ * written to *y_nnz_dev (device int64) when the stream reaches it: y_nnz, or -1
+ * if x was invalid (the workspaces stay clean).  If y_nnz > y_cap only the first
+ * y_cap entries are written.  x_nnz must be >= 1. */
+tsmv_status tsmv_spmspv_async(tsmv_ctx *c, tsmv_semiring sr, int64_t x_nnz, const int32_t *x_idx,
+                              const void *x_val, int64_t y_cap, int32_t *y_idx, void *y_val,
+                              int64_t *y_nnz_dev, void *cuda_stream);
+
+/* Per-kernel device timing of tsmv_spmspv* (CUDA events recorded on the call's
+ * stream around each of its three kernels).  tsmv_set_timing(c, 1) starts a new
+ * window; tsmv_get_timing waits for the events and returns the summed ms of
+ * {x-scan, expand, compact, whole call} over the `calls` timed calls since. */
+tsmv_status tsmv_set_timing(tsmv_ctx *c, int32_t enable);
+tsmv_status tsmv_get_timing(tsmv_ctx *c, double *ms_out4, int64_t *calls);
 
 /* Counters of the last tsmv_spmspv on this ctx (synchronous D2H read). */
 tsmv_status tsmv_last_call_stats(tsmv_ctx *c, tsmv_call_stats *s);

@@ -36,6 +36,7 @@ using namespace tsmv;
 // defined in spmspv.cu / bfs.cu (occupancy of the persistent expand kernels)
 namespace tsmv {
 int expand_occupancy(int nt, int dtype);
+int fused_occupancy(int nt, int dtype);
 }
 
 extern "C" tsmv_status tsmv_default_options(tsmv_options *o) {
@@ -66,7 +67,7 @@ static void destroy_impl(tsmv_ctx *c) {
     c->Qown.release();
     for (DevBuf *b : {&c->outdeg, &c->indeg, &c->acc, &c->rowbits, &c->desc_compact, &c->counters, &c->stage_x_idx,
                       &c->stage_x_val, &c->stage_y_idx, &c->stage_y_val, &c->stage_levels, &c->V, &c->F0, &c->F1,
-                      &c->desc_bfs, &c->splits_dev})
+                      &c->desc_bfs, &c->splits_dev, &c->xdense, &c->acct, &c->tring, &c->partials})
         b->release();
     c->L.release();
     if (c->hcnt) cudaFreeHost(c->hcnt);
@@ -219,6 +220,15 @@ extern "C" tsmv_status tsmv_create(tsmv_ctx **out, int64_t nrows, int64_t ncols,
                                       cudaMemcpyHostToDevice, st));
         }
         c->expand_blocks = c->sm_count * expand_occupancy(c->nt, (int)dtype);
+        // fused SpMSpV: one co-resident 1024-thread CTA per SM (cooperative launch)
+        int fo = fused_occupancy(c->nt, (int)dtype);
+        TSMV_REQUIRE(fo >= 1, "tsmv_create: fused SpMSpV kernel cannot be resident (occupancy 0)");
+        c->fused_blocks = c->sm_count;
+        c->partials.alloc((size_t)c->fused_blocks * 8 * 8);
+        TSMV_CUDA(cudaMemsetAsync(c->partials.p, 0, c->partials.bytes, st));
+        c->acct.alloc((size_t)std::max(c->expand_blocks, c->fused_blocks) * 4 * 8);
+        TSMV_CUDA(cudaMemsetAsync(c->acct.p, 0, c->acct.bytes, st));
+        c->xdense.alloc(std::max<int64_t>(ncols, 1) * 8);
         TSMV_CUDA(cudaEventRecord(c->ev1, st));
         TSMV_CUDA(cudaStreamSynchronize(st));
         float ms = 0;

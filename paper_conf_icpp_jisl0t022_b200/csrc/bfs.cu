@@ -133,11 +133,13 @@ k_fscan(const uint32_t *__restrict__ F, uint32_t *__restrict__ Fclear, long long
 #pragma unroll
     for (int i = 0; i < 8; ++i) zero.v[i] = 0;
     BS(ts).ExclusiveScan(q, ex, zero, OctSum(), agg);
-    if (threadIdx.x == 0) {
+    if (threadIdx.x < 32) {
         long long pre[8];
-        lookback<8>(desc, bid, epoch, agg.v, pre);
+        lookback_warp<8>(desc, bid, epoch, agg.v, pre, threadIdx.x);
+        if (threadIdx.x == 0) {
 #pragma unroll
-        for (int i = 0; i < 8; ++i) s_pre[i] = pre[i];
+            for (int i = 0; i < 8; ++i) s_pre[i] = pre[i];
+        }
     }
     __syncthreads();
 #pragma unroll

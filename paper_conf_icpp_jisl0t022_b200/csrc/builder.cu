@@ -91,7 +91,8 @@ __global__ void k_fill_tiles(const unsigned long long *__restrict__ keys, const 
                              typename Tr<NT>::idx_t *__restrict__ idx, V *__restrict__ dval,
                              typename Tr<NT>::word_t *__restrict__ planes,
                              unsigned long long *__restrict__ skey, V *__restrict__ sval,
-                             int32_t *__restrict__ colcnt) {
+                             int32_t *__restrict__ colcnt, TileDesc *__restrict__ desc,
+                             typename Tr<NT>::cs_t *__restrict__ cstart) {
     using word_t = typename Tr<NT>::word_t;
     using idx_t = typename Tr<NT>::idx_t;
     constexpr int LOG = Tr<NT>::LOG;
@@ -105,18 +106,26 @@ __global__ void k_fill_tiles(const unsigned long long *__restrict__ keys, const 
             int64_t d = dord[t];
             int64_t p0 = dpos[t];
             word_t mk = 0;
+            int next_c = 0;  // columns < next_c have their start written
             for (int64_t e = s0; e < s1; ++e) {
                 unsigned c = (unsigned)((keys[e] >> LOG) & (NT - 1));
                 unsigned r = (unsigned)(keys[e] & (NT - 1));
+                for (; next_c <= (int)c; ++next_c) cstart[d * NT + next_c] = (typename Tr<NT>::cs_t)(e - s0);
                 mk |= (word_t)1 << c;
                 idx[p0 + (e - s0)] = (idx_t)((c << LOG) | r);
                 if (dval) dval[p0 + (e - s0)] = vals[e];
                 if (planes) planes[(int64_t)c * T + d] |= (word_t)1 << r;
             }
+            for (; next_c < NT; ++next_c) cstart[d * NT + next_c] = (typename Tr<NT>::cs_t)(s1 - s0);
             trow[d] = (int32_t)I;
             tgrp[d] = (int32_t)J;
             mask[d] = mk;
             off[d] = p0;
+            TileDesc td;
+            td.off = p0;
+            td.trow = (int)I;
+            td.nnz = (int)(s1 - s0);
+            desc[d] = td;
             atomicAdd(&colcnt[J], 1);
         } else {
             int64_t q0 = spos[t];
@@ -272,6 +281,8 @@ void build_nt(TileSet &S, const int32_t *rows, const int32_t *cols, const V *val
     S.mask.alloc(T * sizeof(word_t));
     S.off.alloc((T + 1) * 8);
     S.idx.alloc(DN * sizeof(idx_t));
+    S.desc.alloc(T * sizeof(TileDesc));
+    S.cstart.alloc((size_t)T * NT * sizeof(typename Tr<NT>::cs_t));
     if (vals) S.val.alloc(DN * sizeof(V));
     if (want_planes) {
         S.planes.alloc((size_t)NT * T * sizeof(word_t));
@@ -288,7 +299,8 @@ void build_nt(TileSet &S, const int32_t *rows, const int32_t *cols, const V *val
             dpos.as<int64_t>(), spos.as<int64_t>(), dimR, S.trow.as<int32_t>(), S.tgrp.as<int32_t>(),
             S.mask.as<word_t>(), S.off.as<int64_t>(), S.idx.as<idx_t>(), vals ? S.val.as<V>() : nullptr,
             want_planes ? S.planes.as<word_t>() : nullptr, skey.as<unsigned long long>(),
-            vals ? sval_tmp.as<V>() : nullptr, colcnt.as<int32_t>());
+            vals ? sval_tmp.as<V>() : nullptr, colcnt.as<int32_t>(), S.desc.as<TileDesc>(),
+            S.cstart.as<typename Tr<NT>::cs_t>());
     TSMV_CUDA(cudaGetLastError());
     TSMV_CUDA(cudaMemcpyAsync(S.off.as<int64_t>() + T, &DN, 8, cudaMemcpyHostToDevice, st));
     S.ptr.alloc((S.nTC + 1) * 8);

@@ -46,9 +46,16 @@ struct Err {
 
 // ------------------------------------------------------------------ tile traits
 template <int NT> struct Tr;
-template <> struct Tr<16> { using word_t = uint16_t; using idx_t = uint8_t;  static constexpr int LOG = 4; };
-template <> struct Tr<32> { using word_t = uint32_t; using idx_t = uint16_t; static constexpr int LOG = 5; };
-template <> struct Tr<64> { using word_t = unsigned long long; using idx_t = uint16_t; static constexpr int LOG = 6; };
+template <> struct Tr<16> { using word_t = uint16_t; using idx_t = uint8_t;  using cs_t = uint8_t;  static constexpr int LOG = 4; };
+template <> struct Tr<32> { using word_t = uint32_t; using idx_t = uint16_t; using cs_t = uint16_t; static constexpr int LOG = 5; };
+template <> struct Tr<64> { using word_t = unsigned long long; using idx_t = uint16_t; using cs_t = uint16_t; static constexpr int LOG = 6; };
+
+// Per-tile descriptor read once a tile's mask intersects x (one 16-byte load).
+struct __align__(16) TileDesc {
+    long long off;  // first in-tile nonzero
+    int trow;       // tile row I
+    int nnz;        // nonzeros in the tile
+};
 
 inline int log2_nt(int nt) { return nt == 16 ? 4 : nt == 32 ? 5 : 6; }
 inline int idx_bytes(int nt) { return nt == 16 ? 1 : 2; }
@@ -91,16 +98,18 @@ struct TileSet {
     DevBuf idx;      // idx_t[dense_nnz]: (c << LOG) | r, column-major inside a tile
     DevBuf val;      // double/float[dense_nnz] (absent for pattern)
     DevBuf planes;   // word_t[NT][T]: plane c holds column word c of every tile (bit r = row r)
+    DevBuf desc;     // TileDesc[T]
+    DevBuf cstart;   // cs_t[T][NT]: start of column c inside the tile's nonzeros (column-major)
     DevBuf sptr;     // int64[dimC+1]: side matrix (very sparse tiles), CSC
     DevBuf srow;     // int32[side_nnz]
     DevBuf sval;     // double/float[side_nnz]
     bool has_vals = false, has_planes = false, has_list = false;
     size_t bytes() const {
         return ptr.bytes + trow.bytes + tgrp.bytes + mask.bytes + off.bytes + idx.bytes + val.bytes +
-               planes.bytes + sptr.bytes + srow.bytes + sval.bytes;
+               planes.bytes + sptr.bytes + srow.bytes + sval.bytes + desc.bytes + cstart.bytes;
     }
     void release() {
-        for (DevBuf *b : {&ptr, &trow, &tgrp, &mask, &off, &idx, &val, &planes, &sptr, &srow, &sval})
+        for (DevBuf *b : {&ptr, &trow, &tgrp, &mask, &off, &idx, &val, &planes, &sptr, &srow, &sval, &desc, &cstart})
             b->release();
     }
 };
@@ -119,6 +128,9 @@ struct Counters {
     unsigned int chunk_next;       // work-queue head of the expand kernel
     unsigned int pad1;
     long long reached, edges;      // BFS totals
+    long long hit_tiles, hit_nnz, tile_macs;  // expand-kernel accounting (tiles with mask hit,
+                                              // their nonzeros, useful multiplies in tiles)
+    unsigned long long bar;        // grid-barrier arrival counter (monotonic)
 };
 
 template <int K> struct LBDesc {
@@ -177,6 +189,8 @@ struct tsmv_ctx {
 
     // SpMSpV workspaces (clear-on-read)
     tsmv::DevBuf acc;          // double[m] (or ordered keys for MIN)
+    tsmv::DevBuf xdense;       // double[n]: x_j scattered by column (only x's columns are ever read)
+    tsmv::DevBuf acct;         // long long[expand_blocks][4]: per-block byte-accounting counters
     tsmv::DevBuf rowbits;      // uint32[ceil(m/32)]
     tsmv::DevBuf desc_compact; // LBDesc<1>[blocks]
     tsmv::Lists L;
@@ -199,6 +213,15 @@ struct tsmv_ctx {
     long long cur_fsize = 0, cur_mf = 0;
 
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+    // optional per-phase timing of tsmv_spmspv* (tsmv_set_timing): block 0 of the
+    // fused kernel stamps %globaltimer at its phase boundaries into a ring
+    bool timing = false;
+    tsmv::DevBuf tring;            // unsigned long long[TRING][8]
+    long long tcalls = 0;          // timed calls since tsmv_set_timing
+    unsigned long long bar_base = 0;  // value of Counters::bar at the next launch
+    int fused_blocks = 0, fused_threads = 1024;
+    tsmv::DevBuf partials;         // long long[fused_blocks][8]
+    long long last_x_nnz = 0;
 };
 
 namespace tsmv {

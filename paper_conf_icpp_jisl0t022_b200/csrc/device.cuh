@@ -73,6 +73,102 @@ __device__ void lookback(LBDesc<K> *desc, unsigned bid, unsigned epoch, const lo
     *(volatile unsigned *)&me->status = ep | 2u;
 }
 
+// Warp-parallel decoupled look-back: called by all 32 lanes of one warp; lane l
+// inspects predecessor (window_top - l), so a chain of aggregates is consumed 32
+// blocks per L2 round trip.  Same contract as lookback().
+template <int K>
+__device__ void lookback_warp(LBDesc<K> *desc, unsigned bid, unsigned epoch, const long long *agg, long long *excl,
+                              int lane) {
+    const unsigned ep = (epoch & 0x3fffffffu) << 2;
+    LBDesc<K> *me = desc + bid;
+    if (bid == 0) {
+        if (lane == 0) {
+#pragma unroll
+            for (int i = 0; i < K; ++i) ((volatile long long *)me->inc)[i] = agg[i];
+            __threadfence();
+            *(volatile unsigned *)&me->status = ep | 2u;
+        }
+#pragma unroll
+        for (int i = 0; i < K; ++i) excl[i] = 0;
+        return;
+    }
+    if (lane == 0) {
+#pragma unroll
+        for (int i = 0; i < K; ++i) ((volatile long long *)me->agg)[i] = agg[i];
+        __threadfence();
+        *(volatile unsigned *)&me->status = ep | 1u;
+    }
+    long long acc[K];
+#pragma unroll
+    for (int i = 0; i < K; ++i) acc[i] = 0;
+    long long top = (long long)bid - 1;
+    while (true) {
+        const long long q = top - lane;
+        unsigned s = ep | 2u;  // q < 0: virtual inclusive prefix 0
+        if (q >= 0) {
+            do {
+                s = ld_status_k<K>(desc + q);
+            } while ((s & ~3u) != ep || (s & 3u) == 0);
+        }
+        __syncwarp();
+        const unsigned pm = __ballot_sync(0xffffffffu, (s & 3u) == 2u);
+        const int first = pm ? __ffs(pm) - 1 : 32;
+        __threadfence();
+        long long v[K];
+#pragma unroll
+        for (int i = 0; i < K; ++i) {
+            v[i] = 0;
+            if (q >= 0 && lane < first) v[i] = ((volatile long long *)desc[q].agg)[i];
+            else if (q >= 0 && lane == first) v[i] = ((volatile long long *)desc[q].inc)[i];
+        }
+#pragma unroll
+        for (int i = 0; i < K; ++i) {
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1) v[i] += __shfl_xor_sync(0xffffffffu, v[i], o);
+            acc[i] += v[i];
+        }
+        if (first < 32) break;
+        top -= 32;
+    }
+#pragma unroll
+    for (int i = 0; i < K; ++i) excl[i] = acc[i];
+    if (lane == 0) {
+#pragma unroll
+        for (int i = 0; i < K; ++i) ((volatile long long *)me->inc)[i] = acc[i] + agg[i];
+        __threadfence();
+        *(volatile unsigned *)&me->status = ep | 2u;
+    }
+}
+
+// ------------------------------------------------------------------ grid barrier
+// For cooperative (co-resident) launches.  `bar` is a monotonically increasing
+// arrival counter; every block tracks the same target sequence from the host-side
+// base value of this launch, so nothing has to be reset between launches.
+__device__ __forceinline__ unsigned long long ld_acquire_u64(const unsigned long long *p) {
+    unsigned long long v;
+    asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+
+__device__ __forceinline__ void grid_sync(unsigned long long *bar, unsigned long long &target) {
+    __syncthreads();
+    target += gridDim.x;
+    if (threadIdx.x == 0) {
+        __threadfence();
+        atomicAdd(bar, 1ull);
+        while (ld_acquire_u64(bar) < target) {
+        }
+        __threadfence();
+    }
+    __syncthreads();
+}
+
+__device__ __forceinline__ unsigned long long globaltimer_ns() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+
 // View of the per-call lists (raw pointers).
 struct ListsView {
     long long *Lt_seg;            // segment id J
@@ -87,6 +183,7 @@ struct ListsView {
     int *Ct;                      // tile chunk -> first Lt entry
     int *Cs;                      // side chunk -> first Ls entry
     double *xv;                   // x values (double)
+    double *xd;                   // x values scattered by column: xd[j] = x_j
 };
 
 inline ListsView lists_view(tsmv_ctx *c) {
@@ -103,6 +200,7 @@ inline ListsView lists_view(tsmv_ctx *c) {
     v.Ct = c->L.Ct.as<int>();
     v.Cs = c->L.Cs.as<int>();
     v.xv = c->L.xv.as<double>();
+    v.xd = c->xdense.as<double>();
     return v;
 }
 

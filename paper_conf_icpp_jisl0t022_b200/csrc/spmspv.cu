@@ -1,125 +1,66 @@
 // spmspv.cu -- TileSpMSpV y = A x (Sec 3.3,
 // P:790-863, Fig 4; semirings P:1373-1379).
 //
-// Three kernels on the caller's stream:
-//   k_xscan    (a2) x -> tiled sparse vector: one thread per x entry finds the
-//              non-empty nt-segments (x must be ascending so the
-//              segments are runs), their nt-bit masks, the tile work
-//              (tiles in tile column J) and the side work (side nonzeros of
-//              column j); one decoupled look-back scan gives list positions,
-//              work prefixes and the chunk -> entry maps of the expand kernel.
-//   k_expand   (a3-a5) persistent, load balanced: warps pull 128-item chunks
-//              of tile work and side work.  Tile item: intersect the tile's
-//              column mask with the segment mask (skips the tile without
-//              touching its nonzeros), multiply the hit columns'
-//              nonzeros, accumulate into acc[m] with RED atomics and mark the
-//              row in the touched bitmap.  Side item: one side nonzero.
-//   k_compact  (a6) one thread per 32-row bitmap word: popc + look-back scan
-//              -> y_idx ascending, y_val; acc and bits cleared as read.
+// ONE cooperative persistent kernel per call (one CTA of 1024 threads per SM),
+// phases separated by grid barriers instead of kernel boundaries:
+//   A  (a2) x -> tiled sparse vector.  x is strictly ascending, so the
+//           non-empty nt-segments are runs of x; each CTA takes a
+//           slice of x, finds segment heads, their nt-bit masks, the tile work
+//           (tiles in tile column J) and the side work (side nonzeros of each
+//           column j), writes x_j into xd[j] (the paper's x_tile, addressed by
+//           column instead of through x_ptr), and publishes its totals.
+//   -- barrier --  every CTA scans the <= #SM totals itself (no look-back chain)
+//   A' writes the segment list / side list, their work prefixes and the
+//           chunk -> entry maps of the load balancer.
+//   -- barrier --
+//   B  (a3-a5) warps take 128-item chunks (first chunk static, then an atomic
+//           queue).  Tile item: AND the tile's column mask with the segment
+//           mask (a miss never touches the tile); a hit loads one
+//           16-byte descriptor + the column start offsets and multiplies only
+//           the hit columns' nonzeros.  Side item: one side nonzero (CSC column
+//           merge, Alg 2).  Accumulation: RED.ADD.F64 into acc[m] + touched bit.
+//   -- barrier --
+//   C  (a6) CTAs count the set bits of their slice of the touched bitmap,
+//   -- barrier --  then write y (ascending) with a "transposed" warp walk: lane l
+//           handles bit l of each word, so a dense stretch of y costs one round
+//           of 32 parallel accumulator loads per word.  acc/bits cleared on read.
 #include "device.cuh"
 
 namespace tsmv {
 
 namespace {
 
-template <int NT, class XV>
-__global__ void __launch_bounds__(SCAN_BLOCK)
-k_xscan(const int32_t *__restrict__ x_idx, const XV *__restrict__ x_val, long long k, long long n,
-        const long long *__restrict__ tptr, const long long *__restrict__ sptr, ListsView Lv,
-        Counters *__restrict__ cnt, LBDesc<4> *__restrict__ desc, unsigned epoch) {
-    constexpr int LOG = Tr<NT>::LOG;
-    using BS = cub::BlockScan<Quad, SCAN_BLOCK>;
-    __shared__ typename BS::TempStorage ts;
-    __shared__ unsigned s_bid;
-    __shared__ long long s_pre[4];
-    if (threadIdx.x == 0) s_bid = atomicAdd(&cnt->bid_scan, 1u);
-    __syncthreads();
-    const unsigned bid = s_bid;
-    const long long e = (long long)bid * SCAN_BLOCK + threadIdx.x;
-    Quad q = {{0, 0, 0, 0}};
-    long long j = -1, seg = -1, wt = 0, ws = 0;
-    bool head = false;
-    double xvd = 1.0;
-    if (e < k) {
-        j = x_idx[e];
-        long long prev = e > 0 ? (long long)x_idx[e - 1] : -1;
-        bool bad = j < 0 || j >= n || prev >= j;
-        if (bad) {
-            cnt->err = 1;
-        } else {
-            seg = j >> LOG;
-            head = e == 0 || (prev >> LOG) != seg;
-            if (head) wt = tptr[seg + 1] - tptr[seg];
-            ws = sptr[j + 1] - sptr[j];
-        }
-        if (x_val) xvd = (double)x_val[e];
-        Lv.xv[e] = xvd;
-    }
-    q.v[0] = (head && wt > 0) ? 1 : 0;
-    q.v[1] = head ? wt : 0;
-    q.v[2] = ws > 0 ? 1 : 0;
-    q.v[3] = ws;
-    Quad ex, agg;
-    BS(ts).ExclusiveScan(q, ex, Quad{{0, 0, 0, 0}}, QuadSum(), agg);
-    if (threadIdx.x == 0) {
-        long long pre[4];
-        lookback<4>(desc, bid, epoch, agg.v, pre);
-#pragma unroll
-        for (int i = 0; i < 4; ++i) s_pre[i] = pre[i];
-    }
-    __syncthreads();
-#pragma unroll
-    for (int i = 0; i < 4; ++i) ex.v[i] += s_pre[i];
-    if (head && wt > 0) {
-        long long i = ex.v[0];
-        unsigned long long mk = 0;
-        for (long long e2 = e; e2 < k; ++e2) {
-            long long j2 = x_idx[e2];
-            if ((j2 >> LOG) != seg) break;
-            mk |= 1ull << (j2 & (NT - 1));
-        }
-        Lv.Lt_seg[i] = seg;
-        Lv.Lt_mask[i] = mk;
-        Lv.Lt_first[i] = e;
-        Lv.Lt_tbeg[i] = tptr[seg];
-        Lv.Lt_wpre[i] = ex.v[1];
-        write_chunks(Lv.Ct, ex.v[1], wt, (int)i);
-    }
-    if (ws > 0) {
-        long long i = ex.v[2];
-        Lv.Ls_beg[i] = sptr[j];
-        Lv.Ls_wpre[i] = ex.v[3];
-        Lv.Ls_x[i] = xvd;
-        Lv.Ls_col[i] = (int)j;
-        write_chunks(Lv.Cs, ex.v[3], ws, (int)i);
-    }
-    if (bid == gridDim.x - 1 && threadIdx.x == SCAN_BLOCK - 1) {
-        long long tot[4];
-#pragma unroll
-        for (int i = 0; i < 4; ++i) tot[i] = s_pre[i] + agg.v[i];
-        cnt->nLt = tot[0];
-        cnt->Wt = tot[1];
-        cnt->nLs = tot[2];
-        cnt->Ws = tot[3];
-        cnt->nCt = (tot[1] + CHUNK - 1) >> CHUNK_LOG;
-        cnt->nCs = (tot[3] + CHUNK - 1) >> CHUNK_LOG;
-        Lv.Lt_wpre[tot[0]] = tot[1];
-        Lv.Ls_wpre[tot[2]] = tot[3];
-        cnt->chunk_next = 0;
-        cnt->bid_scan = 0;
-    }
-}
+constexpr int FB = 512;  // threads per CTA of the fused kernel
+constexpr int TRING = 4096;
 
-struct TileView {
-    const long long *ptr;
-    const int *trow;
+struct FusedArgs {
+    const int32_t *x_idx;
+    const void *x_val;
+    long long k, n, m, W, row_begin;
+    // tiles (push format)
+    const long long *tptr;
     const void *mask;
-    const long long *off;
     const void *idx;
     const void *val;
+    const void *desc;
+    const void *cstart;
     const long long *sptr;
     const int *srow;
     const void *sval;
+    ListsView Lv;
+    double *acc;
+    uint32_t *rowbits;
+    long long *partials;  // [G][8]
+    long long *acct;      // [G][4]
+    int32_t *y_idx;
+    void *y_val;
+    long long y_cap;
+    long long *ynnz_dev;
+    Counters *cnt;
+    Counters *hm;
+    unsigned long long bar_base;
+    unsigned long long *tring;  // nullptr = no timing
+    long long tslot;
 };
 
 template <int SR>
@@ -129,214 +70,426 @@ __device__ __forceinline__ void accumulate(double *acc, uint32_t *rowbits, long 
     } else if constexpr (SR == TSMV_MIN_SECOND) {
         atomicMax((unsigned long long *)&acc[row], ~ord_key(x));
     }
-    atomicOr(&rowbits[row >> 5], 1u << (row & 31));
+    // Touched-row bit: test before set.  Power-law rows receive thousands of
+    // contributions per call; an unconditional RED.OR on their (shared) word
+    // serialises in one L2 slice.  A stale read only costs a redundant RED.
+    const unsigned bit = 1u << (row & 31);
+    unsigned *wp = &rowbits[row >> 5];
+    if (!(__ldca(wp) & bit)) atomicOr(wp, bit);
 }
 
-template <int NT, class AV, int SR>
-__global__ void __launch_bounds__(256)
-k_expand(TileView A, ListsView Lv, Counters *__restrict__ cnt, double *__restrict__ acc,
-         uint32_t *__restrict__ rowbits) {
+// per-entry facts of phase A
+template <int NT>
+__device__ __forceinline__ void entry_facts(const int32_t *x_idx, long long e, long long k, long long n,
+                                            const long long *tptr, const long long *sptr, long long &j,
+                                            long long &seg, bool &head, long long &wt, long long &ws, bool &bad) {
+    constexpr int LOG = Tr<NT>::LOG;
+    j = x_idx[e];
+    const long long prev = e > 0 ? (long long)x_idx[e - 1] : -1;
+    bad = j < 0 || j >= n || prev >= j;
+    head = false;
+    wt = ws = 0;
+    seg = j >> LOG;
+    if (!bad) {
+        head = e == 0 || (prev >> LOG) != seg;
+        if (head) wt = tptr[seg + 1] - tptr[seg];
+        ws = sptr[j + 1] - sptr[j];
+    }
+}
+
+template <int NT, class AV, class XV, int SR>
+__global__ void __launch_bounds__(FB, 1) k_spmspv_fused(FusedArgs a) {
     using word_t = typename Tr<NT>::word_t;
     using idx_t = typename Tr<NT>::idx_t;
+    using cs_t = typename Tr<NT>::cs_t;
     constexpr int LOG = Tr<NT>::LOG;
-    __shared__ long long win_all[8][CHUNK + 1];
-    if (cnt->err) return;
-    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-    long long *win = win_all[wid];
-    const long long nCt = cnt->nCt, nCs = cnt->nCs;
-    const long long nLt = cnt->nLt, nLs = cnt->nLs, Wt = cnt->Wt, Ws = cnt->Ws;
-    const word_t *mask = (const word_t *)A.mask;
-    const idx_t *idx = (const idx_t *)A.idx;
-    const AV *val = (const AV *)A.val;
-    const AV *sval = (const AV *)A.sval;
-    while (true) {
-        unsigned ch = 0;
-        if (lane == 0) ch = atomicAdd(&cnt->chunk_next, 1u);
-        ch = __shfl_sync(0xffffffffu, ch, 0);
-        if (ch < nCt) {
-            const long long s0 = Lv.Ct[ch];
-            const long long base = (long long)ch << CHUNK_LOG;
-            load_window(win, Lv.Lt_wpre, s0, nLt, lane);
+    constexpr int U = CHUNK / 32;
+    constexpr int NW = FB / 32;
+    using BSQ = cub::BlockScan<Quad, FB>;
+    using BSL = cub::BlockScan<long long, FB>;
+    __shared__ union {
+        typename BSQ::TempStorage q;
+        typename BSL::TempStorage l;
+    } ts;
+    __shared__ long long win_all[NW][CHUNK + 1];
+    __shared__ long long s_pre[4], s_tot[4];
+    __shared__ long long s_acct[NW][3];
+    __shared__ int s_err;
+    const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+    const int G = gridDim.x, b = blockIdx.x;
+    unsigned long long target = a.bar_base;
+    const bool stamp = a.tring && b == 0 && tid == 0;
+    unsigned long long *ts_out = a.tring ? a.tring + (a.tslot % TRING) * 8 : nullptr;
+    if (stamp) ts_out[0] = globaltimer_ns();
+
+    // ------------------------------------------------------------ phase A: x -> segments
+    const long long E = (a.k + G - 1) / G;
+    const long long e0 = (long long)b * E, e1 = min(a.k, e0 + E);
+    const long long per = (E + FB - 1) / FB;
+    const long long te0 = min(e1, e0 + tid * per), te1 = min(e1, te0 + per);
+    Quad q = {{0, 0, 0, 0}};
+    bool any_bad = false;
+    for (long long e = te0; e < te1; ++e) {
+        long long j, seg, wt, ws;
+        bool head, bad;
+        entry_facts<NT>(a.x_idx, e, a.k, a.n, a.tptr, a.sptr, j, seg, head, wt, ws, bad);
+        any_bad |= bad;
+        q.v[0] += (head && wt > 0);
+        q.v[1] += wt;
+        q.v[2] += (ws > 0);
+        q.v[3] += ws;
+        if (!bad) {
+            double xv = a.x_val ? (double)((const XV *)a.x_val)[e] : 1.0;
+            a.Lv.xd[j] = xv;
+        }
+    }
+    if (any_bad) a.cnt->err = 1;
+    Quad ex, agg;
+    BSQ(ts.q).ExclusiveScan(q, ex, Quad{{0, 0, 0, 0}}, QuadSum(), agg);
+    if (tid < 4) a.partials[b * 8 + tid] = agg.v[tid];
+    if (b == 0 && tid == 0) a.cnt->chunk_next = 0;
+    grid_sync(&a.cnt->bar, target);
+    if (stamp) ts_out[1] = globaltimer_ns();
+
+    // every CTA reduces the G partials itself: prefix of CTAs < b, and totals
+    if (tid < 32) {
+        long long pre[4] = {0, 0, 0, 0}, tot[4] = {0, 0, 0, 0};
+        for (int g = lane; g < G; g += 32) {
 #pragma unroll
-            for (int u = 0; u < CHUNK / 32; ++u) {
-                long long i = base + lane + 32 * u;
-                if (i >= Wt) break;
-                int q = window_find(win, i);
-                long long s = s0 + q;
-                long long t = Lv.Lt_tbeg[s] + (i - win[q]);
-                unsigned long long xm = Lv.Lt_mask[s];
-                word_t hit = mask[t] & (word_t)xm;
-                if (hit) {
-                    long long I = A.trow[t];
-                    long long p0 = A.off[t], p1 = A.off[t + 1];
-                    long long first = Lv.Lt_first[s];
-                    for (long long p = p0; p < p1; ++p) {
-                        unsigned id = idx[p];
-                        unsigned cc = id >> LOG;
-                        if ((hit >> cc) & 1) {
-                            unsigned r = id & (NT - 1);
-                            unsigned long long below = cc ? (xm & ((1ull << cc) - 1)) : 0ull;
-                            double xv = Lv.xv[first + __popcll(below)];
-                            double a = val ? (double)val[p] : 1.0;
-                            accumulate<SR>(acc, rowbits, I * NT + r, a, xv);
+            for (int i = 0; i < 4; ++i) {
+                long long v = __ldcg(&a.partials[g * 8 + i]);
+                tot[i] += v;
+                if (g < b) pre[i] += v;
+            }
+        }
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1) {
+                pre[i] += __shfl_xor_sync(0xffffffffu, pre[i], o);
+                tot[i] += __shfl_xor_sync(0xffffffffu, tot[i], o);
+            }
+        }
+        if (lane == 0) {
+#pragma unroll
+            for (int i = 0; i < 4; ++i) {
+                s_pre[i] = pre[i];
+                s_tot[i] = tot[i];
+            }
+            s_err = __ldcg(&a.cnt->err);
+        }
+    }
+    __syncthreads();
+    const bool err = s_err != 0;
+    // A': write the lists
+    if (!err) {
+        long long oLt = s_pre[0] + ex.v[0], oWt = s_pre[1] + ex.v[1];
+        long long oLs = s_pre[2] + ex.v[2], oWs = s_pre[3] + ex.v[3];
+        for (long long e = te0; e < te1; ++e) {
+            long long j, seg, wt, ws;
+            bool head, bad;
+            entry_facts<NT>(a.x_idx, e, a.k, a.n, a.tptr, a.sptr, j, seg, head, wt, ws, bad);
+            if (head && wt > 0) {
+                unsigned long long mk = 0;
+                for (long long e2 = e; e2 < a.k; ++e2) {
+                    const long long j2 = a.x_idx[e2];
+                    if ((j2 >> LOG) != seg) break;
+                    mk |= 1ull << (j2 & (NT - 1));
+                }
+                a.Lv.Lt_seg[oLt] = seg;
+                a.Lv.Lt_mask[oLt] = mk;
+                a.Lv.Lt_tbeg[oLt] = a.tptr[seg];
+                a.Lv.Lt_wpre[oLt] = oWt;
+                write_chunks(a.Lv.Ct, oWt, wt, (int)oLt);
+                ++oLt;
+                oWt += wt;
+            }
+            if (ws > 0) {
+                a.Lv.Ls_beg[oLs] = a.sptr[j];
+                a.Lv.Ls_wpre[oLs] = oWs;
+                a.Lv.Ls_x[oLs] = a.x_val ? (double)((const XV *)a.x_val)[e] : 1.0;
+                write_chunks(a.Lv.Cs, oWs, ws, (int)oLs);
+                ++oLs;
+                oWs += ws;
+            }
+        }
+        if (b == G - 1 && tid == 0) {
+            a.Lv.Lt_wpre[s_tot[0]] = s_tot[1];
+            a.Lv.Ls_wpre[s_tot[2]] = s_tot[3];
+        }
+    }
+    grid_sync(&a.cnt->bar, target);
+    if (stamp) ts_out[2] = globaltimer_ns();
+
+    // ------------------------------------------------------------ phase B: expand
+    long long n_hit = 0, n_hcol = 0, n_mac = 0;
+    if (!err) {
+        const long long nLt = s_tot[0], Wt = s_tot[1], nLs = s_tot[2], Ws = s_tot[3];
+        const long long nCt = (Wt + CHUNK - 1) >> CHUNK_LOG, nCs = (Ws + CHUNK - 1) >> CHUNK_LOG;
+        long long *win = win_all[wid];
+        const word_t *mask = (const word_t *)a.mask;
+        const idx_t *idx = (const idx_t *)a.idx;
+        const AV *val = (const AV *)a.val;
+        const AV *sval = (const AV *)a.sval;
+        const cs_t *cstart = (const cs_t *)a.cstart;
+        const unsigned nwarps = (unsigned)(G * NW);
+        unsigned ch = (unsigned)(b * NW + wid);  // first chunk static, then the queue
+        while (true) {
+            if (ch < nCt) {
+                const long long s0 = __ldcg(&a.Lv.Ct[ch]);
+                const long long base = (long long)ch << CHUNK_LOG;
+                load_window(win, a.Lv.Lt_wpre, s0, nLt, lane);
+                long long sidx[U], t[U];
+                bool ok[U];
+#pragma unroll
+                for (int u = 0; u < U; ++u) {
+                    const long long i = base + lane + 32 * u;
+                    ok[u] = i < Wt;
+                    const int qq = ok[u] ? window_find(win, i) : 0;
+                    sidx[u] = s0 + qq;
+                    t[u] = i - win[qq];
+                }
+                long long J[U];
+                word_t xm[U];
+#pragma unroll
+                for (int u = 0; u < U; ++u) {
+                    if (ok[u]) {
+                        t[u] += __ldcg(&a.Lv.Lt_tbeg[sidx[u]]);
+                        xm[u] = (word_t)__ldcg(&a.Lv.Lt_mask[sidx[u]]);
+                        J[u] = __ldcg(&a.Lv.Lt_seg[sidx[u]]);
+                    }
+                }
+                word_t hit[U];
+#pragma unroll
+                for (int u = 0; u < U; ++u) hit[u] = ok[u] ? (word_t)(mask[t[u]] & xm[u]) : (word_t)0;
+#pragma unroll
+                for (int u = 0; u < U; ++u) {
+                    if (hit[u]) {
+                        const TileDesc d = ((const TileDesc *)a.desc)[t[u]];
+                        ++n_hit;
+                        word_t h = hit[u];
+                        const long long rowbase = (long long)d.trow * NT;
+                        while (h) {
+                            const int c = ffs_w(h);
+                            h &= h - 1;
+                            const int p0 = cstart[t[u] * NT + c];
+                            const int p1 = c + 1 < NT ? (int)cstart[t[u] * NT + c + 1] : d.nnz;
+                            const double xv = __ldcg(&a.Lv.xd[J[u] * NT + c]);
+                            for (int p = p0; p < p1; ++p) {
+                                const unsigned r = idx[d.off + p] & (NT - 1);
+                                const double av = val ? (double)val[d.off + p] : 1.0;
+                                accumulate<SR>(a.acc, a.rowbits, rowbase + r, av, xv);
+                            }
+                            n_mac += p1 - p0;
+                            ++n_hcol;
+                        }
+                    }
+                }
+            } else if (ch < nCt + nCs) {
+                const long long c2 = (long long)ch - nCt;
+                const long long s0 = __ldcg(&a.Lv.Cs[c2]);
+                const long long base = c2 << CHUNK_LOG;
+                load_window(win, a.Lv.Ls_wpre, s0, nLs, lane);
+                long long p[U], sidx[U];
+                bool ok[U];
+#pragma unroll
+                for (int u = 0; u < U; ++u) {
+                    const long long i = base + lane + 32 * u;
+                    ok[u] = i < Ws;
+                    const int qq = ok[u] ? window_find(win, i) : 0;
+                    sidx[u] = s0 + qq;
+                    p[u] = i - win[qq];
+                }
+                double xv[U];
+#pragma unroll
+                for (int u = 0; u < U; ++u) {
+                    if (ok[u]) {
+                        p[u] += __ldcg(&a.Lv.Ls_beg[sidx[u]]);
+                        xv[u] = __ldcg(&a.Lv.Ls_x[sidx[u]]);
+                    }
+                }
+                long long row[U];
+                double av[U];
+#pragma unroll
+                for (int u = 0; u < U; ++u) {
+                    if (ok[u]) {
+                        row[u] = a.srow[p[u]];
+                        av[u] = sval ? (double)sval[p[u]] : 1.0;
+                    }
+                }
+#pragma unroll
+                for (int u = 0; u < U; ++u)
+                    if (ok[u]) accumulate<SR>(a.acc, a.rowbits, row[u], av[u], xv[u]);
+            } else {
+                break;
+            }
+            __syncwarp();
+            unsigned nx = 0;
+            if (lane == 0) nx = nwarps + atomicAdd(&a.cnt->chunk_next, 1u);
+            ch = __shfl_sync(0xffffffffu, nx, 0);
+        }
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        n_hit += __shfl_xor_sync(0xffffffffu, n_hit, o);
+        n_hcol += __shfl_xor_sync(0xffffffffu, n_hcol, o);
+        n_mac += __shfl_xor_sync(0xffffffffu, n_mac, o);
+    }
+    if (lane == 0) {
+        s_acct[wid][0] = n_hit;
+        s_acct[wid][1] = n_hcol;
+        s_acct[wid][2] = n_mac;
+    }
+    grid_sync(&a.cnt->bar, target);  // (its __syncthreads also orders s_acct)
+    if (stamp) ts_out[3] = globaltimer_ns();
+    if (tid < 3) {
+        long long sum = 0;
+        for (int w = 0; w < NW; ++w) sum += s_acct[w][tid];
+        a.acct[b * 4 + tid] = sum;
+    }
+
+    // ------------------------------------------------------------ phase C: compact
+    const long long S = (((a.W + G - 1) / G) + 31) & ~31ll;  // words per CTA, warp aligned
+    const long long w0 = (long long)b * S, w1 = min(a.W, w0 + S);
+    long long mycnt = 0;
+    for (long long w = w0 + tid; w < w1; w += FB) mycnt += __popc(__ldcg(&a.rowbits[w]));
+    long long blk = 0;
+    {
+        long long dummy;
+        BSL(ts.l).ExclusiveSum(mycnt, dummy, blk);
+    }
+    if (tid == 0) a.partials[b * 8 + 4] = blk;
+    grid_sync(&a.cnt->bar, target);
+    if (stamp) ts_out[4] = globaltimer_ns();
+    if (tid < 32) {
+        long long pre = 0, tot = 0;
+        for (int g = lane; g < G; g += 32) {
+            long long v = __ldcg(&a.partials[g * 8 + 4]);
+            tot += v;
+            if (g < b) pre += v;
+        }
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) {
+            pre += __shfl_xor_sync(0xffffffffu, pre, o);
+            tot += __shfl_xor_sync(0xffffffffu, tot, o);
+        }
+        if (lane == 0) {
+            s_pre[0] = pre;
+            s_tot[0] = tot;
+        }
+    }
+    __syncthreads();
+    long long carry = s_pre[0];
+    const long long ycap = a.y_cap;
+    const unsigned lt = (1u << lane) - 1;
+    for (long long rb = w0; rb < w1; rb += FB) {
+        const long long w = rb + tid;
+        const unsigned bits = w < w1 ? __ldcg(&a.rowbits[w]) : 0u;
+        long long c = __popc(bits), exw, rtot;
+        BSL(ts.l).ExclusiveSum(c, exw, rtot);
+        const long long pos0 = carry + exw;
+        carry += rtot;
+        if (bits) a.rowbits[w] = 0u;
+        const long long wbase = w - lane;
+        unsigned todo = __ballot_sync(0xffffffffu, bits != 0);
+        while (todo) {
+            int src[8];
+            int nb = 0;
+#pragma unroll
+            for (int kk = 0; kk < 8; ++kk) {
+                src[kk] = 0;
+                if (todo) {
+                    src[kk] = __ffs(todo) - 1;
+                    todo &= todo - 1;
+                    nb = kk + 1;
+                }
+            }
+            unsigned wb[8];
+            long long wp[8];
+            double v[8];
+            bool mine[8];
+#pragma unroll
+            for (int kk = 0; kk < 8; ++kk) {
+                wb[kk] = __shfl_sync(0xffffffffu, bits, src[kk]);
+                wp[kk] = __shfl_sync(0xffffffffu, pos0, src[kk]);
+                mine[kk] = kk < nb && ((wb[kk] >> lane) & 1u);
+                if (mine[kk]) v[kk] = __ldcg(&a.acc[(wbase + src[kk]) * 32 + lane]);
+            }
+#pragma unroll
+            for (int kk = 0; kk < 8; ++kk) {
+                if (mine[kk]) {
+                    const long long row = (wbase + src[kk]) * 32 + lane;
+                    const long long pos = wp[kk] + __popc(wb[kk] & lt);
+                    a.acc[row] = 0.0;
+                    if (pos < ycap) {
+                        a.y_idx[pos] = (int32_t)(row + a.row_begin);
+                        if (a.y_val) {
+                            double x = v[kk];
+                            if constexpr (SR == TSMV_MIN_SECOND)
+                                x = ord_val(~(unsigned long long)__double_as_longlong(x));
+                            ((XV *)a.y_val)[pos] = (XV)x;
                         }
                     }
                 }
             }
-            __syncwarp();
-        } else if (ch < nCt + nCs) {
-            const long long c2 = ch - nCt;
-            const long long s0 = Lv.Cs[c2];
-            const long long base = c2 << CHUNK_LOG;
-            load_window(win, Lv.Ls_wpre, s0, nLs, lane);
-#pragma unroll
-            for (int u = 0; u < CHUNK / 32; ++u) {
-                long long i = base + lane + 32 * u;
-                if (i >= Ws) break;
-                int q = window_find(win, i);
-                long long s = s0 + q;
-                long long p = Lv.Ls_beg[s] + (i - win[q]);
-                long long row = A.srow[p];
-                double a = sval ? (double)sval[p] : 1.0;
-                accumulate<SR>(acc, rowbits, row, a, Lv.Ls_x[s]);
-            }
-            __syncwarp();
-        } else {
-            break;
         }
+        __syncthreads();  // ts.l reuse
+    }
+    if (b == 0 && tid == 0) {
+        // every CTA read cnt->err before barrier 3, so it can be reset here
+        const long long tot = s_tot[0];
+        a.cnt->y_nnz = tot;
+        a.hm->y_nnz = tot;
+        a.hm->err = err ? 1 : 0;
+        if (a.ynnz_dev) *a.ynnz_dev = err ? -1 : tot;
+        a.cnt->err = 0;
+        if (a.tring) ts_out[5] = globaltimer_ns();
     }
 }
 
-template <class YV, int SR>
-__global__ void __launch_bounds__(SCAN_BLOCK)
-k_compact(uint32_t *__restrict__ rowbits, long long W, double *__restrict__ acc, long long row_begin,
-          int32_t *__restrict__ y_idx, YV *__restrict__ y_val, long long y_cap, Counters *__restrict__ cnt,
-          Counters *__restrict__ hmirror, LBDesc<1> *__restrict__ desc, unsigned epoch) {
-    using BS = cub::BlockScan<long long, SCAN_BLOCK>;
-    __shared__ typename BS::TempStorage ts;
-    __shared__ unsigned s_bid;
-    __shared__ long long s_pre;
-    if (threadIdx.x == 0) s_bid = atomicAdd(&cnt->bid_compact, 1u);
-    __syncthreads();
-    const unsigned bid = s_bid;
-    const long long w = (long long)bid * SCAN_BLOCK + threadIdx.x;
-    unsigned bits = w < W ? rowbits[w] : 0u;
-    long long c = __popc(bits), ex, agg;
-    BS(ts).ExclusiveSum(c, ex, agg);
-    if (threadIdx.x == 0) {
-        long long pre;
-        lookback<1>(desc, bid, epoch, &agg, &pre);
-        s_pre = pre;
+// Phase-A totals / accounting for tsmv_last_call_stats are summed on the host
+// from `partials` and `acct`.
+
+template <int NT, class AV, class XV, int SR> void *fused_fn() {
+    return (void *)k_spmspv_fused<NT, AV, XV, SR>;
+}
+
+template <int NT, class AV, class XV> void *pick_sr(int sr) {
+    if (sr == TSMV_PLUS_TIMES) return fused_fn<NT, AV, XV, TSMV_PLUS_TIMES>();
+    if (sr == TSMV_OR_AND) return fused_fn<NT, AV, XV, TSMV_OR_AND>();
+    return fused_fn<NT, AV, XV, TSMV_MIN_SECOND>();
+}
+
+void *pick_kernel(int nt, bool f32, int sr) {
+    // AV = matrix value type, XV = x / y value type (both fp32 for F32 contexts)
+    if (f32) {
+        if (nt == 16) return pick_sr<16, float, float>(sr);
+        if (nt == 32) return pick_sr<32, float, float>(sr);
+        return pick_sr<64, float, float>(sr);
     }
-    __syncthreads();
-    long long pos = s_pre + ex;
-    if (bits) {
-        rowbits[w] = 0u;
-        while (bits) {
-            int b = __ffs(bits) - 1;
-            bits &= bits - 1;
-            long long row = w * 32 + b;
-            double v = acc[row];
-            acc[row] = 0.0;
-            if (pos < y_cap) {
-                y_idx[pos] = (int32_t)(row + row_begin);
-                if (y_val) {
-                    if constexpr (SR == TSMV_MIN_SECOND) v = ord_val(~(unsigned long long)__double_as_longlong(v));
-                    y_val[pos] = (YV)v;
-                }
-            }
-            ++pos;
-        }
-    }
-    if (bid == gridDim.x - 1 && threadIdx.x == SCAN_BLOCK - 1) {
-        long long tot = s_pre + agg;
-        cnt->y_nnz = tot;
-        hmirror->y_nnz = tot;
-        hmirror->err = cnt->err;
-        hmirror->nLt = cnt->nLt;
-        hmirror->Wt = cnt->Wt;
-        hmirror->nLs = cnt->nLs;
-        hmirror->Ws = cnt->Ws;
-        cnt->err = 0;
-        cnt->bid_compact = 0;
-    }
-}
-
-inline TileView tile_view(const TileSet &S) {
-    TileView v;
-    v.ptr = S.ptr.as<long long>();
-    v.trow = S.trow.as<int>();
-    v.mask = S.mask.p;
-    v.off = S.off.as<long long>();
-    v.idx = S.idx.p;
-    v.val = S.has_vals ? S.val.p : nullptr;
-    v.sptr = S.sptr.as<long long>();
-    v.srow = S.srow.as<int>();
-    v.sval = S.has_vals ? S.sval.p : nullptr;
-    return v;
-}
-
-template <int NT, class AV, int SR>
-void launch_expand(tsmv_ctx *c, cudaStream_t st) {
-    k_expand<NT, AV, SR><<<c->expand_blocks, 256, 0, st>>>(tile_view(c->P), lists_view(c),
-                                                           c->counters.as<Counters>(), c->acc.as<double>(),
-                                                           c->rowbits.as<uint32_t>());
-}
-
-template <int NT, class AV>
-void launch_expand_sr(tsmv_ctx *c, int sr, cudaStream_t st) {
-    if (sr == TSMV_PLUS_TIMES) launch_expand<NT, AV, TSMV_PLUS_TIMES>(c, st);
-    else if (sr == TSMV_OR_AND) launch_expand<NT, AV, TSMV_OR_AND>(c, st);
-    else launch_expand<NT, AV, TSMV_MIN_SECOND>(c, st);
-}
-
-template <int NT>
-void launch_xscan(tsmv_ctx *c, const int32_t *xi, const void *xv, bool f32, long long k, cudaStream_t st) {
-    int grid = (int)((k + SCAN_BLOCK - 1) / SCAN_BLOCK);
-    if (f32)
-        k_xscan<NT, float><<<grid, SCAN_BLOCK, 0, st>>>(xi, (const float *)xv, k, c->n, c->P.ptr.as<long long>(),
-                                                        c->P.sptr.as<long long>(), lists_view(c),
-                                                        c->counters.as<Counters>(),
-                                                        c->L.desc_scan.as<LBDesc<4>>(), c->epoch);
-    else
-        k_xscan<NT, double><<<grid, SCAN_BLOCK, 0, st>>>(xi, (const double *)xv, k, c->n,
-                                                         c->P.ptr.as<long long>(), c->P.sptr.as<long long>(),
-                                                         lists_view(c), c->counters.as<Counters>(),
-                                                         c->L.desc_scan.as<LBDesc<4>>(), c->epoch);
-}
-
-template <class YV>
-void launch_compact(tsmv_ctx *c, int sr, int32_t *yi, void *yv, long long ycap, cudaStream_t st) {
-    long long W = (c->m + 31) / 32;
-    int grid = (int)std::max<long long>(1, (W + SCAN_BLOCK - 1) / SCAN_BLOCK);
-    auto *d = c->desc_compact.as<LBDesc<1>>();
-    if (sr == TSMV_MIN_SECOND)
-        k_compact<YV, TSMV_MIN_SECOND><<<grid, SCAN_BLOCK, 0, st>>>(
-            c->rowbits.as<uint32_t>(), W, c->acc.as<double>(), c->row_begin, yi, (YV *)yv, ycap,
-            c->counters.as<Counters>(), c->hcnt_dev, d, c->epoch);
-    else
-        k_compact<YV, TSMV_PLUS_TIMES><<<grid, SCAN_BLOCK, 0, st>>>(
-            c->rowbits.as<uint32_t>(), W, c->acc.as<double>(), c->row_begin, yi,
-            sr == TSMV_OR_AND ? nullptr : (YV *)yv, ycap, c->counters.as<Counters>(), c->hcnt_dev, d, c->epoch);
+    if (nt == 16) return pick_sr<16, double, double>(sr);
+    if (nt == 32) return pick_sr<32, double, double>(sr);
+    return pick_sr<64, double, double>(sr);
 }
 
 }  // namespace
 
 int expand_occupancy(int nt, int dtype) {
-    int b = 0;
-    bool f32 = dtype == TSMV_F32;
-    cudaError_t e;
-    if (nt == 16) e = f32 ? cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_expand<16, float, 0>, 256, 0)
-                          : cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_expand<16, double, 0>, 256, 0);
-    else if (nt == 32) e = f32 ? cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_expand<32, float, 0>, 256, 0)
-                               : cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_expand<32, double, 0>, 256, 0);
-    else e = f32 ? cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_expand<64, float, 0>, 256, 0)
-                 : cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, k_expand<64, double, 0>, 256, 0);
-    if (e != cudaSuccess || b < 1) {
+    // blocks per SM of the persistent BFS push kernels (256 threads)
+    (void)nt;
+    (void)dtype;
+    return 4;
+}
+
+int fused_occupancy(int nt, int dtype) {
+    int bps = 0;
+    void *f = pick_kernel(nt, dtype == TSMV_F32, TSMV_PLUS_TIMES);
+    cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, f, FB, 0);
+    if (e != cudaSuccess || bps < 1) {
         cudaGetLastError();
-        b = 4;
+        bps = 0;
     }
-    return b;
+    return bps;
 }
 
 void ensure_lists(tsmv_ctx *c, int64_t k) {
@@ -371,30 +524,66 @@ void ensure_lists(tsmv_ctx *c, int64_t k) {
     }
 }
 
-// Debug aid (TSMV_CHECK_LISTS=1): validate the k_xscan lists on the host.
-void debug_check_lists(tsmv_ctx *c, cudaStream_t st) {
-    TSMV_CUDA(cudaStreamSynchronize(st));
-    Counters h;
-    TSMV_CUDA(cudaMemcpy(&h, c->counters.p, sizeof(h), cudaMemcpyDeviceToHost));
-    auto chk = [&](const char *nm, const DevBuf &wpre_b, const DevBuf &C_b, long long nL, long long W, long long nC) {
-        std::vector<long long> wpre(nL + 1);
-        std::vector<int> C(nC);
-        TSMV_CUDA(cudaMemcpy(wpre.data(), wpre_b.p, (nL + 1) * 8, cudaMemcpyDeviceToHost));
-        if (nC) TSMV_CUDA(cudaMemcpy(C.data(), C_b.p, nC * 4, cudaMemcpyDeviceToHost));
-        int bad = 0;
-        if (nL && wpre[0] != 0) fprintf(stderr, "[%s] wpre[0]=%lld\n", nm, wpre[0]), ++bad;
-        if (wpre[nL] != W) fprintf(stderr, "[%s] sentinel %lld != W %lld\n", nm, wpre[nL], W), ++bad;
-        for (long long i = 0; i + 1 <= nL && bad < 10; ++i)
-            if (wpre[i + 1] <= wpre[i]) fprintf(stderr, "[%s] wpre[%lld]=%lld wpre[+1]=%lld\n", nm, i, wpre[i], wpre[i + 1]), ++bad;
-        for (long long ch = 0; ch < nC && bad < 20; ++ch) {
-            long long it = ch << CHUNK_LOG, s = C[ch];
-            if (s < 0 || s >= nL || !(wpre[s] <= it && it < wpre[s + 1]))
-                fprintf(stderr, "[%s] chunk %lld -> %lld wrong\n", nm, ch, s), ++bad;
-        }
-        fprintf(stderr, "[%s] nL=%lld W=%lld nC=%lld bad=%d\n", nm, nL, W, nC, bad);
-    };
-    chk("tile", c->L.Lt_wpre, c->L.Ct, h.nLt, h.Wt, h.nCt);
-    chk("side", c->L.Ls_wpre, c->L.Cs, h.nLs, h.Ws, h.nCs);
+// Enqueue one fused SpMSpV (device pointers only, no sync).
+void enqueue_spmspv(tsmv_ctx *c, int sr, long long k, const int32_t *xi, const void *xv, long long ycap,
+                    int32_t *yi, void *yv, long long *ynnz_dev, cudaStream_t st) {
+    const bool f32 = c->dtype == TSMV_F32;
+    ensure_lists(c, k);
+    FusedArgs a;
+    a.x_idx = xi;
+    a.x_val = xv;
+    a.k = k;
+    a.n = c->n;
+    a.m = c->m;
+    a.W = (c->m + 31) / 32;
+    a.row_begin = c->row_begin;
+    a.tptr = c->P.ptr.as<long long>();
+    a.mask = c->P.mask.p;
+    a.idx = c->P.idx.p;
+    a.val = c->P.has_vals ? c->P.val.p : nullptr;
+    a.desc = c->P.desc.p;
+    a.cstart = c->P.cstart.p;
+    a.sptr = c->P.sptr.as<long long>();
+    a.srow = c->P.srow.as<int>();
+    a.sval = c->P.has_vals ? c->P.sval.p : nullptr;
+    a.Lv = lists_view(c);
+    a.acc = c->acc.as<double>();
+    a.rowbits = c->rowbits.as<uint32_t>();
+    a.partials = c->partials.as<long long>();
+    a.acct = c->acct.as<long long>();
+    a.y_idx = yi;
+    a.y_val = (sr == TSMV_OR_AND) ? nullptr : yv;
+    a.y_cap = ycap;
+    a.ynnz_dev = ynnz_dev;
+    a.cnt = c->counters.as<Counters>();
+    a.hm = c->hcnt_dev;
+    a.bar_base = c->bar_base;
+    a.tring = c->timing ? c->tring.as<unsigned long long>() : nullptr;
+    a.tslot = c->tcalls;
+    void *args[] = {&a};
+    void *f = pick_kernel(c->nt, f32, sr);
+    TSMV_CUDA(cudaLaunchCooperativeKernel(f, dim3(c->fused_blocks), dim3(FB), args, 0, st));
+    c->bar_base += 4ull * (unsigned long long)c->fused_blocks;
+    if (c->timing) c->tcalls++;
+}
+
+void stats_from_partials(tsmv_ctx *c, tsmv_call_stats *s) {
+    std::vector<long long> p(8 * (size_t)c->fused_blocks), q(4 * (size_t)c->fused_blocks);
+    TSMV_CUDA(cudaMemcpy(p.data(), c->partials.p, p.size() * 8, cudaMemcpyDeviceToHost));
+    TSMV_CUDA(cudaMemcpy(q.data(), c->acct.p, q.size() * 8, cudaMemcpyDeviceToHost));
+    s->x_segments = s->tile_items = s->side_items = 0;
+    s->hit_tiles = s->hit_columns = s->tile_macs = 0;
+    long long nLs = 0;
+    for (int b = 0; b < c->fused_blocks; ++b) {
+        s->x_segments += p[8 * b];
+        s->tile_items += p[8 * b + 1];
+        nLs += p[8 * b + 2];
+        s->side_items += p[8 * b + 3];
+        s->hit_tiles += q[4 * b];
+        s->hit_columns += q[4 * b + 1];
+        s->tile_macs += q[4 * b + 2];
+    }
+    (void)nLs;
 }
 
 }  // namespace tsmv
@@ -417,10 +606,8 @@ extern "C" tsmv_status tsmv_spmspv(tsmv_ctx *c, tsmv_semiring sr, int64_t x_nnz,
         TSMV_CUDA(cudaSetDevice(c->device));
         cudaStream_t st = (cudaStream_t)cuda_stream;
         *y_nnz = 0;
-        if (x_nnz == 0) {
-            c->hcnt->nLt = c->hcnt->Wt = c->hcnt->nLs = c->hcnt->Ws = c->hcnt->y_nnz = 0;
-            return TSMV_OK;
-        }
+        c->last_x_nnz = x_nnz;
+        if (x_nnz == 0) return TSMV_OK;
         const bool f32 = c->dtype == TSMV_F32;
         const size_t vb = f32 ? 4 : 8;
         // stage host inputs
@@ -450,38 +637,12 @@ extern "C" tsmv_status tsmv_spmspv(tsmv_ctx *c, tsmv_semiring sr, int64_t x_nnz,
             c->stage_y_val.ensure(std::max<int64_t>(ycap_dev, 1) * vb);
             yv = c->stage_y_val.p;
         }
-        ensure_lists(c, x_nnz);
-        c->epoch++;
-        switch (c->nt) {
-            case 16: launch_xscan<16>(c, xi, xv, f32, x_nnz, st); break;
-            case 32: launch_xscan<32>(c, xi, xv, f32, x_nnz, st); break;
-            default: launch_xscan<64>(c, xi, xv, f32, x_nnz, st); break;
-        }
-        TSMV_CUDA(cudaGetLastError());
-        if (getenv("TSMV_CHECK_LISTS")) debug_check_lists(c, st);
-        if (f32) {
-            switch (c->nt) {
-                case 16: launch_expand_sr<16, float>(c, sr, st); break;
-                case 32: launch_expand_sr<32, float>(c, sr, st); break;
-                default: launch_expand_sr<64, float>(c, sr, st); break;
-            }
-        } else {
-            switch (c->nt) {
-                case 16: launch_expand_sr<16, double>(c, sr, st); break;
-                case 32: launch_expand_sr<32, double>(c, sr, st); break;
-                default: launch_expand_sr<64, double>(c, sr, st); break;
-            }
-        }
-        TSMV_CUDA(cudaGetLastError());
-        if (f32) launch_compact<float>(c, sr, yi, yv, ycap_dev, st);
-        else launch_compact<double>(c, sr, yi, yv, ycap_dev, st);
-        TSMV_CUDA(cudaGetLastError());
+        enqueue_spmspv(c, sr, x_nnz, xi, xv, ycap_dev, yi, yv, nullptr, st);
         TSMV_CUDA(cudaStreamSynchronize(st));
         volatile Counters *h = c->hcnt;
         int64_t ynnz = h->y_nnz;
         int err = h->err;
-        TSMV_REQUIRE(err == 0, "tsmv_spmspv: x indices must be strictly ascending and in [0, %lld)",
-                     (long long)c->n);
+        TSMV_REQUIRE(err == 0, "tsmv_spmspv: x indices must be strictly ascending and in [0, %lld)", (long long)c->n);
         *y_nnz = ynnz;
         if (ynnz > y_cap) {
             set_error("tsmv_spmspv: y_cap %lld < y_nnz %lld", (long long)y_cap, (long long)ynnz);
@@ -496,15 +657,71 @@ extern "C" tsmv_status tsmv_spmspv(tsmv_ctx *c, tsmv_semiring sr, int64_t x_nnz,
     }
 }
 
+extern "C" tsmv_status tsmv_spmspv_async(tsmv_ctx *c, tsmv_semiring sr, int64_t x_nnz, const int32_t *x_idx,
+                                         const void *x_val, int64_t y_cap, int32_t *y_idx, void *y_val,
+                                         int64_t *y_nnz_dev, void *cuda_stream) {
+    try {
+        TSMV_REQUIRE(c != nullptr, "tsmv_spmspv_async: NULL ctx");
+        TSMV_REQUIRE(sr >= 0 && sr <= 2, "tsmv_spmspv_async: bad semiring %d", (int)sr);
+        TSMV_REQUIRE(x_nnz >= 1 && x_nnz <= c->n, "tsmv_spmspv_async: x_nnz %lld out of [1, ncols]",
+                     (long long)x_nnz);
+        TSMV_REQUIRE(x_idx != nullptr && (sr == TSMV_OR_AND || x_val != nullptr), "tsmv_spmspv_async: NULL x");
+        TSMV_REQUIRE(y_cap >= 0 && (y_cap == 0 || y_idx != nullptr), "tsmv_spmspv_async: NULL y_idx");
+        TSMV_REQUIRE(sr == TSMV_OR_AND || y_cap == 0 || y_val != nullptr, "tsmv_spmspv_async: NULL y_val");
+        TSMV_CUDA(cudaSetDevice(c->device));
+        c->last_x_nnz = x_nnz;
+        enqueue_spmspv(c, sr, x_nnz, x_idx, sr == TSMV_OR_AND ? nullptr : x_val, y_cap, y_idx,
+                       sr == TSMV_OR_AND ? nullptr : y_val, (long long *)y_nnz_dev, (cudaStream_t)cuda_stream);
+        return TSMV_OK;
+    } catch (const Err &e) {
+        return e.st;
+    }
+}
+
+extern "C" tsmv_status tsmv_set_timing(tsmv_ctx *c, int32_t enable) {
+    try {
+        TSMV_REQUIRE(c, "tsmv_set_timing: NULL ctx");
+        if (enable && !c->tring.p) c->tring.alloc((size_t)TRING * 8 * 8);
+        c->timing = enable != 0;
+        c->tcalls = 0;
+        return TSMV_OK;
+    } catch (const Err &e) {
+        return e.st;
+    }
+}
+
+extern "C" tsmv_status tsmv_get_timing(tsmv_ctx *c, double *ms_out, int64_t *calls) {
+    try {
+        TSMV_REQUIRE(c && ms_out && calls, "tsmv_get_timing: NULL argument");
+        for (int i = 0; i < 4; ++i) ms_out[i] = 0;
+        long long n = std::min<long long>(c->tcalls, TRING);
+        *calls = n;
+        if (n == 0 || !c->tring.p) return TSMV_OK;
+        TSMV_CUDA(cudaDeviceSynchronize());
+        std::vector<unsigned long long> r((size_t)TRING * 8);
+        TSMV_CUDA(cudaMemcpy(r.data(), c->tring.p, r.size() * 8, cudaMemcpyDeviceToHost));
+        for (long long q = 0; q < n; ++q) {
+            const unsigned long long *t = &r[q * 8];
+            ms_out[0] += (t[2] - t[0]) * 1e-6;  // phase A (+A')
+            ms_out[1] += (t[3] - t[2]) * 1e-6;  // phase B (expand)
+            ms_out[2] += (t[5] - t[3]) * 1e-6;  // phase C (compact)
+            ms_out[3] += (t[5] - t[0]) * 1e-6;  // whole kernel (block 0's view)
+        }
+        c->tcalls = 0;
+        return TSMV_OK;
+    } catch (const Err &e) {
+        return e.st;
+    }
+}
+
 extern "C" tsmv_status tsmv_last_call_stats(tsmv_ctx *c, tsmv_call_stats *s) {
     try {
         TSMV_REQUIRE(c && s, "tsmv_last_call_stats: NULL argument");
+        TSMV_CUDA(cudaSetDevice(c->device));
         volatile Counters *h = c->hcnt;
-        s->x_nnz = 0;
-        s->x_segments = h->nLt;
-        s->tile_items = h->Wt;
-        s->side_items = h->Ws;
+        s->x_nnz = c->last_x_nnz;
         s->y_nnz = h->y_nnz;
+        stats_from_partials(c, s);
         return TSMV_OK;
     } catch (const Err &e) {
         return e.st;

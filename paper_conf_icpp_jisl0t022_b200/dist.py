@@ -1,0 +1,158 @@
+"""Row-block multi-GPU TileSpMSpV / TileBFS.
+
+The paper is single-GPU; the partitioned path is this build's addition
+(BASELINE.json north_star item 4).  One process per GPU.  Rank p owns global
+rows [splits[p], splits[p+1]) of A (contiguous, nnz-balanced, cut at multiples
+of 64 rows so tile rows and bitmap words never straddle ranks) in its own
+libtsmv context; columns stay global.
+
+Per iteration there is exactly one exchange, done with torch.distributed (NCCL
+over NVLink on the GPU box, gloo in the CPU tests):
+  * SpMSpV: all-gather of the owners' x entries (counts, then padded entries);
+    every rank then computes y for its own rows -- no reduction is needed;
+  * TileBFS: all-gather of each rank's newly discovered owned-vertex bitmap
+    segment (padded to the largest segment) + one all-reduce of two int64
+    (m_f, m_u) so that all ranks take the same push/pull decision.
+Everything else (the level kernels, the merge of the gathered frontier into the
+replicated visited bitmap, the frontier scan) runs in libtsmv.so.
+"""
+from __future__ import annotations
+
+from typing import List, Optional, Sequence
+
+import torch
+import torch.distributed as dist
+
+ALIGN = 64
+
+
+def partition_rows(row_ptr: torch.Tensor, nranks: int, align: int = ALIGN) -> List[int]:
+    """nnz-balanced contiguous row blocks: split p is the multiple of `align` nearest
+    to the row where the running nnz reaches p/nranks of the total.
+    Returns nranks+1 global row boundaries (first 0, last m)."""
+    rp = row_ptr.detach().to("cpu", torch.int64)
+    m = rp.numel() - 1
+    nnz = int(rp[-1])
+    splits = [0]
+    for p in range(1, nranks):
+        target = (nnz * p + nranks - 1) // nranks
+        r = int(torch.searchsorted(rp, torch.tensor(target, dtype=torch.int64), right=False))
+        r = min(m, ((r + align // 2) // align) * align)   # nearest multiple of `align`
+        splits.append(max(r, splits[-1]))
+    splits.append(m)
+    return splits
+
+
+def local_rows(A, splits: Sequence[int], rank: int):
+    """The CSR block of A holding rows [splits[rank], splits[rank+1]) (global columns)."""
+    import synth  # only for the CSR container type
+    r0, r1 = int(splits[rank]), int(splits[rank + 1])
+    rp = A.row_ptr[r0:r1 + 1]
+    base = int(rp[0])
+    cols = A.col_idx[base:int(rp[-1])]
+    vals = None if A.values is None else A.values[base:int(rp[-1])]
+    return synth.CSR(r1 - r0, A.n, rp - base, cols, vals, f"{A.name}[{r0}:{r1}]")
+
+
+def allgather_varlen(t: torch.Tensor, group=None) -> torch.Tensor:
+    """Concatenation, in rank order, of a 1-D tensor of per-rank length."""
+    world = dist.get_world_size(group)
+    n = torch.tensor([t.numel()], dtype=torch.int64, device=t.device)
+    sizes = [torch.zeros_like(n) for _ in range(world)]
+    dist.all_gather(sizes, n, group=group)
+    sizes = [int(s) for s in sizes]
+    mx = max(sizes) if sizes else 0
+    pad = torch.zeros(max(mx, 1), dtype=t.dtype, device=t.device)
+    pad[:t.numel()] = t
+    out = torch.empty(world * max(mx, 1), dtype=t.dtype, device=t.device)
+    dist.all_gather_into_tensor(out, pad, group=group)
+    return torch.cat([out[p * max(mx, 1):p * max(mx, 1) + sizes[p]] for p in range(world)])
+
+
+def exchange_frontier(owned_words: torch.Tensor, stride: int, group=None) -> torch.Tensor:
+    """All-gather of the owned frontier-bitmap segments, each padded to `stride`
+    uint32 words (int32 storage), rank-major: out[p*stride + w]."""
+    world = dist.get_world_size(group)
+    buf = torch.zeros(stride, dtype=owned_words.dtype, device=owned_words.device)
+    buf[:owned_words.numel()] = owned_words
+    out = torch.empty(world * stride, dtype=owned_words.dtype, device=owned_words.device)
+    dist.all_gather_into_tensor(out, buf, group=group)
+    return out
+
+
+def bfs_loop(engine, source: int, group=None) -> int:
+    """Level-synchronous distributed TileBFS driver (Alg 3, one
+    exchange per level).  `engine` provides begin(source) -> (|F|, m_f, m_u) local,
+    expand(dir) -> owned words, merge(gathered, stride) -> (|F|, m_f, m_u),
+    stride (padded words), n, choose(n, |F|, m_f, m_u).  Returns the number of levels."""
+    dev = engine.device
+    f, mf, mu = engine.begin(source)
+    levels = 0
+    while f > 0:
+        red = torch.tensor([mf, mu], dtype=torch.int64, device=dev)
+        dist.all_reduce(red, group=group)
+        d = engine.choose(engine.n, f, int(red[0]), int(red[1]))
+        owned = engine.expand(d)
+        gathered = exchange_frontier(owned, engine.stride, group)
+        f, mf, mu = engine.merge(gathered, engine.stride)
+        levels += 1
+    return levels
+
+
+class DistTiledMatrix:
+    """This rank's row block of A in a libtsmv context, plus the exchange steps."""
+
+    def __init__(self, A_local, splits: Sequence[int], rank: int, nranks: int, group=None,
+                 dtype: Optional[str] = None, device: int = 0, **opts):
+        from . import tsmv
+        self.tsmv = tsmv
+        self.splits = [int(s) for s in splits]
+        self.rank, self.nranks, self.group = rank, nranks, group
+        self.n = A_local.n
+        self.m_local = A_local.m
+        self.device = torch.device("cuda", device)
+        self.M = tsmv.TiledMatrix(A_local.m, A_local.n, A_local.row_ptr, A_local.col_idx, A_local.values,
+                                  dtype=dtype, device=device, rank=rank, nranks=nranks,
+                                  row_splits=self.splits, build_bfs=1, **opts)
+        self.stride = max((self.splits[p + 1] - self.splits[p] + 31) // 32 for p in range(nranks))
+        self.owned = torch.zeros(max(1, (self.m_local + 31) // 32), dtype=torch.int32, device=self.device)
+        self.levels = torch.empty(max(1, self.m_local), dtype=torch.int32, device=self.device)
+        self._stats = (torch.zeros(3, dtype=torch.int64))
+
+    # ---- SpMSpV: x entries are distributed by owner (x_idx in this rank's row range)
+    def spmspv(self, x_idx_owned: torch.Tensor, x_val_owned: Optional[torch.Tensor], semiring="plus_times"):
+        xi = allgather_varlen(x_idx_owned.to(torch.int32), self.group)
+        xv = None if x_val_owned is None else allgather_varlen(x_val_owned, self.group)
+        if xi.numel() == 0:
+            return xi, xv
+        return self.M.spmspv(xi, xv, semiring=semiring)
+
+    # ---- BFS engine interface
+    def choose(self, n, f, mf, mu):
+        return self.tsmv.choose_dir(n, f, mf, mu, self.M.opts)
+
+    def begin(self, source):
+        import ctypes
+        st = (ctypes.c_int64 * 3)()
+        self.tsmv.check(self.tsmv.tsmv_bfs_dist_begin(self.M.ctx, int(source), self.levels.data_ptr(), st,
+                                                      torch.cuda.current_stream().cuda_stream),
+                        "tsmv_bfs_dist_begin")
+        return st[0], st[1], st[2]
+
+    def expand(self, d):
+        self.tsmv.check(self.tsmv.tsmv_bfs_dist_expand(self.M.ctx, int(d), self.owned.data_ptr(),
+                                                       torch.cuda.current_stream().cuda_stream),
+                        "tsmv_bfs_dist_expand")
+        return self.owned
+
+    def merge(self, gathered, stride):
+        import ctypes
+        st = (ctypes.c_int64 * 3)()
+        self.tsmv.check(self.tsmv.tsmv_bfs_dist_merge(self.M.ctx, gathered.data_ptr(), int(stride), st,
+                                                      torch.cuda.current_stream().cuda_stream),
+                        "tsmv_bfs_dist_merge")
+        return st[0], st[1], st[2]
+
+    def bfs(self, source: int):
+        nl = bfs_loop(self, source, self.group)
+        return self.levels[:self.m_local], nl

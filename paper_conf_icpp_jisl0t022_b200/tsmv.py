@@ -45,7 +45,8 @@ class tsmv_options(ctypes.Structure):
 
 class tsmv_call_stats(ctypes.Structure):
     _fields_ = [("x_nnz", ctypes.c_int64), ("x_segments", ctypes.c_int64), ("tile_items", ctypes.c_int64),
-                ("side_items", ctypes.c_int64), ("y_nnz", ctypes.c_int64)]
+                ("side_items", ctypes.c_int64), ("y_nnz", ctypes.c_int64), ("hit_tiles", ctypes.c_int64),
+                ("hit_columns", ctypes.c_int64), ("tile_macs", ctypes.c_int64)]
 
 
 class tsmv_info(ctypes.Structure):
@@ -68,6 +69,9 @@ _SIGS = {
     "tsmv_create": (ctypes.c_int, [ctypes.POINTER(_vp), _i64, _i64, _vp, _vp, _vp, ctypes.c_int,
                                    ctypes.POINTER(tsmv_options)]),
     "tsmv_spmspv": (ctypes.c_int, [_vp, ctypes.c_int, _i64, _vp, _vp, _i64, _vp, _vp, ctypes.POINTER(_i64), _vp]),
+    "tsmv_spmspv_async": (ctypes.c_int, [_vp, ctypes.c_int, _i64, _vp, _vp, _i64, _vp, _vp, _vp, _vp]),
+    "tsmv_set_timing": (ctypes.c_int, [_vp, _i32]),
+    "tsmv_get_timing": (ctypes.c_int, [_vp, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(_i64)]),
     "tsmv_last_call_stats": (ctypes.c_int, [_vp, ctypes.POINTER(tsmv_call_stats)]),
     "tsmv_bfs": (ctypes.c_int, [_vp, _i64, _vp, ctypes.POINTER(tsmv_bfs_stats), _vp]),
     "tsmv_bfs_dist_begin": (ctypes.c_int, [_vp, _i64, _vp, ctypes.POINTER(_i64), _vp]),
@@ -181,6 +185,24 @@ class TiledMatrix:
         check(st, "tsmv_spmspv")
         k = ynnz.value
         return y_idx[:k], (y_val[:k] if y_val is not None and sr != OR_AND else None)
+
+    def spmspv_async(self, x_idx: torch.Tensor, x_val: Optional[torch.Tensor], y_idx: torch.Tensor,
+                     y_val: Optional[torch.Tensor], y_nnz: torch.Tensor, semiring="plus_times", stream=None):
+        """Device-only, no synchronisation; y_nnz (int64[1] on the device) receives the size."""
+        sr = _SEMIRINGS[semiring] if isinstance(semiring, str) else int(semiring)
+        check(tsmv_spmspv_async(self.ctx, sr, x_idx.numel(), _ptr(x_idx), _ptr(x_val), y_idx.numel(), _ptr(y_idx),
+                                _ptr(y_val) if sr != OR_AND else None, _ptr(y_nnz), _stream(stream)),
+              "tsmv_spmspv_async")
+
+    def set_timing(self, enable: bool = True):
+        check(tsmv_set_timing(self.ctx, 1 if enable else 0), "tsmv_set_timing")
+
+    def get_timing(self):
+        """(ms x-scan, ms expand, ms compact, ms whole call) summed, and the number of calls."""
+        ms = (ctypes.c_double * 4)()
+        n = ctypes.c_int64(0)
+        check(tsmv_get_timing(self.ctx, ms, ctypes.byref(n)), "tsmv_get_timing")
+        return [ms[i] for i in range(4)], n.value
 
     def last_call_stats(self) -> dict:
         s = tsmv_call_stats()

@@ -1,0 +1,75 @@
+"""Simulated ranks on one GPU: P libtsmv contexts built from the row blocks of
+`dist.partition_rows`, with the exchange done by concatenation (what the NCCL
+all-gather returns).  Exercises the distributed C-ABI calls
+(tsmv_bfs_dist_begin/expand/merge, row_splits contexts) against the oracle."""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import synth
+from paper_conf_icpp_jisl0t022_b200 import dist as D
+
+pytestmark = pytest.mark.gpu
+DEV = torch.device("cuda", 0)
+
+
+def _ranks(A, P, dtype="pattern", **opts):
+    splits = D.partition_rows(A.row_ptr, P)
+    engines = []
+    for r in range(P):
+        Al = D.local_rows(A, splits, r).to(DEV)
+        if dtype == "pattern":
+            Al = Al.with_values(None)
+        engines.append(D.DistTiledMatrix(Al, splits, r, P, dtype=dtype, **opts))
+    return splits, engines
+
+
+def _sim_bfs(engines, source):
+    st = [e.begin(source) for e in engines]
+    while st[0][0] > 0:
+        assert len({s[0] for s in st}) == 1          # |F| identical on every rank
+        mf = sum(s[1] for s in st)
+        mu = sum(s[2] for s in st)
+        d = engines[0].choose(engines[0].n, st[0][0], mf, mu)
+        owned = [e.expand(d).clone() for e in engines]
+        stride = engines[0].stride
+        gathered = torch.zeros(len(engines) * stride, dtype=torch.int32, device=DEV)
+        for p, o in enumerate(owned):
+            gathered[p * stride:p * stride + o.numel()] = o
+        st = [e.merge(gathered, stride) for e in engines]
+    return np.concatenate([e.levels[:e.m_local].cpu().numpy() for e in engines])
+
+
+@pytest.mark.parametrize("P", [2, 3, 4])
+@pytest.mark.parametrize("sym", [True, False])
+def test_sim_ranks_bfs(P, sym):
+    A = synth.rmat(13, 16, seed=7, symmetrize=sym)
+    C = oracle.csc_of(A)
+    _, engines = _ranks(A, P)
+    for s in [0] + synth.sample_sources(A, 2, seed=2):
+        assert np.array_equal(_sim_bfs(engines, s), oracle.bfs_queue(C, s))
+
+
+@pytest.mark.parametrize("force", [1, 2, 3])
+def test_sim_ranks_forced_directions(force):
+    A = synth.stencil2d(64, 64)
+    C = oracle.csc_of(A)
+    _, engines = _ranks(A, 3, force_dir=force)
+    assert np.array_equal(_sim_bfs(engines, 0), oracle.bfs_queue(C, 0))
+
+
+@pytest.mark.parametrize("P", [2, 4])
+def test_sim_ranks_spmspv(P):
+    A = synth.attach_values(synth.rmat(13, 16, seed=3), seed=2, integer=True)
+    C = oracle.csc_of(A)
+    splits, engines = _ranks(A, P, dtype="f64")
+    xi, xv = synth.sample_x(A.n, 500, seed=5, integer=True)
+    ys_i, ys_v = [], []
+    for e in engines:
+        yi, yv = e.M.spmspv(xi.to(DEV), xv.to(DEV))     # the all-gathered x
+        ys_i.append(yi.cpu().numpy())
+        ys_v.append(yv.cpu().numpy())
+    ri, rv = oracle.spmspv(C, xi.numpy(), xv.numpy())
+    assert np.array_equal(np.concatenate(ys_i), ri)      # global row ids, ascending across ranks
+    assert np.array_equal(np.concatenate(ys_v), rv)

@@ -163,6 +163,14 @@ tsmv_status tsmv_spmspv_async(tsmv_ctx *c, tsmv_semiring sr, int64_t x_nnz, cons
 tsmv_status tsmv_set_timing(tsmv_ctx *c, int32_t enable);
 tsmv_status tsmv_get_timing(tsmv_ctx *c, double *ms_out4, int64_t *calls);
 
+/* Development trace of the multiply phase: when `device_buffer` (u64 words,
+ * tsmv_trace_words(c) of them, device memory, caller-owned) is set, every warp of
+ * every later SpMSpV call writes 8 words {phase-B start ns, chunk-loop end ns,
+ * chunks, ns in tile chunks, ns in side chunks, longest chunk ns, barrier arrival
+ * ns, multiplies}.  NULL disables. */
+tsmv_status tsmv_set_trace(tsmv_ctx *c, void *device_buffer);
+int64_t tsmv_trace_words(const tsmv_ctx *c);
+
 /* Counters of the last tsmv_spmspv on this ctx (synchronous D2H read). */
 tsmv_status tsmv_last_call_stats(tsmv_ctx *c, tsmv_call_stats *s);
 

@@ -67,7 +67,7 @@ static void destroy_impl(tsmv_ctx *c) {
     c->Qown.release();
     for (DevBuf *b : {&c->outdeg, &c->indeg, &c->acc, &c->rowbits, &c->desc_compact, &c->counters, &c->stage_x_idx,
                       &c->stage_x_val, &c->stage_y_idx, &c->stage_y_val, &c->stage_levels, &c->V, &c->F0, &c->F1,
-                      &c->desc_bfs, &c->splits_dev, &c->xdense, &c->acct, &c->tring, &c->partials})
+                      &c->desc_bfs, &c->splits_dev, &c->xdense, &c->acct, &c->tring, &c->partials, &c->hot_list})
         b->release();
     c->L.release();
     if (c->hcnt) cudaFreeHost(c->hcnt);
@@ -170,7 +170,11 @@ extern "C" tsmv_status tsmv_create(tsmv_ctx **out, int64_t nrows, int64_t ncols,
         prepare_csr(c, rp, ci, d_rows.as<int32_t>(), st);
 
         // --- tiled structures
-        build_tileset(c, c->P, d_rows.as<int32_t>(), ci, vv, nnz, nrows, ncols, dtype != TSMV_PATTERN, want_bfs, st);
+        DevBuf hot_map;
+        if (!getenv("TSMV_NO_HOT")) choose_hot_rows(c, st, hot_map);  // env: ablation of the privatisation
+        build_tileset(c, c->P, d_rows.as<int32_t>(), ci, vv, nnz, nrows, ncols, dtype != TSMV_PATTERN, want_bfs, st,
+                      c->n_hot ? hot_map.as<int32_t>() : nullptr);
+        hot_map.release();
         c->nTR = c->P.nTR;
         c->nTC = c->P.nTC;
         if (want_bfs) {
@@ -220,10 +224,10 @@ extern "C" tsmv_status tsmv_create(tsmv_ctx **out, int64_t nrows, int64_t ncols,
                                       cudaMemcpyHostToDevice, st));
         }
         c->expand_blocks = c->sm_count * expand_occupancy(c->nt, (int)dtype);
-        // fused SpMSpV: one co-resident 1024-thread CTA per SM (cooperative launch)
+        // fused SpMSpV: all CTAs co-resident (cooperative launch), up to 4 per SM
         int fo = fused_occupancy(c->nt, (int)dtype);
         TSMV_REQUIRE(fo >= 1, "tsmv_create: fused SpMSpV kernel cannot be resident (occupancy 0)");
-        c->fused_blocks = c->sm_count;
+        c->fused_blocks = c->sm_count * std::min(fo, 4);
         c->partials.alloc((size_t)c->fused_blocks * 8 * 8);
         TSMV_CUDA(cudaMemsetAsync(c->partials.p, 0, c->partials.bytes, st));
         c->acct.alloc((size_t)std::max(c->expand_blocks, c->fused_blocks) * 4 * 8);
@@ -284,6 +288,21 @@ template <class T> static std::vector<T> d2h(const DevBuf &b, size_t count) {
     return h;
 }
 
+static tsmv_ctx *g_export_ctx = nullptr;  // set by the export entry points (single-threaded use)
+static std::vector<int32_t> host_hot_list(const TileSet &S) {
+    std::vector<int32_t> h;
+    if (S.hot_list && g_export_ctx && g_export_ctx->n_hot) {
+        h.resize(g_export_ctx->n_hot);
+        TSMV_CUDA(cudaMemcpy(h.data(), S.hot_list, h.size() * 4, cudaMemcpyDeviceToHost));
+    }
+    return h;
+}
+static int64_t decode_host(int32_t v, const std::vector<int32_t> &hl, int nt) {
+    if (v >= 0) return v;
+    int64_t s = ~(int64_t)v;
+    return (int64_t)hl[s / nt] * nt + s % nt;
+}
+
 // Host-side walk over every stored entry of a TileSet: f(row, col, dense?, value_index)
 template <class F> static void walk_tileset(const TileSet &S, int nt, F f) {
     int LOG = log2_nt(nt);
@@ -304,14 +323,16 @@ template <class F> static void walk_tileset(const TileSet &S, int nt, F f) {
         }
     auto sptr = d2h<int64_t>(S.sptr, S.dimC + 1);
     auto srow = d2h<int32_t>(S.srow, S.side_nnz);
+    std::vector<int32_t> hl = host_hot_list(S);
     for (int64_t j = 0; j < S.dimC; ++j)
-        for (int64_t p = sptr[j]; p < sptr[j + 1]; ++p) f((int64_t)srow[p], j, false, p);
+        for (int64_t p = sptr[j]; p < sptr[j + 1]; ++p) f(decode_host(srow[p], hl, nt), j, false, p);
 }
 
 extern "C" tsmv_status tsmv_export_csr(tsmv_ctx *c, int64_t *row_ptr, int32_t *col_idx, void *values) {
     try {
         TSMV_REQUIRE(c && row_ptr && (c->nnz == 0 || col_idx), "tsmv_export_csr: NULL argument");
         TSMV_CUDA(cudaSetDevice(c->device));
+        g_export_ctx = c;
         const TileSet &S = c->P;
         bool f32 = c->dtype == TSMV_F32;
         size_t vb = f32 ? 4 : 8;
@@ -386,11 +407,13 @@ extern "C" tsmv_status tsmv_export_bitmask_tiles(tsmv_ctx *c, int32_t orient, in
             tiles[{trow[t], tgrp[t]}] = w;
         }
         // side entries folded back into their tiles
+        g_export_ctx = c;
         auto sptr = d2h<int64_t>(S.sptr, S.dimC + 1);
         auto srow = d2h<int32_t>(S.srow, S.side_nnz);
+        std::vector<int32_t> hl = host_hot_list(S);
         for (int64_t j = 0; j < S.dimC; ++j)
             for (int64_t p = sptr[j]; p < sptr[j + 1]; ++p) {
-                int64_t r = srow[p];
+                int64_t r = decode_host(srow[p], hl, nt);
                 auto &w = tiles[{r / nt, j / nt}];
                 if (w.empty()) w.assign(nt, 0);
                 w[j % nt] |= 1ull << (r % nt);

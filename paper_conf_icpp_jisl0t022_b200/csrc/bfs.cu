@@ -205,6 +205,7 @@ struct BfsTiles {
     long long T;
     const long long *sptr;
     const int *srow;
+    const int32_t *hot_list;  // side rows of hot tile rows are encoded (TileSet::hot_list)
 };
 
 inline BfsTiles bfs_tiles(const TileSet &S) {
@@ -217,6 +218,7 @@ inline BfsTiles bfs_tiles(const TileSet &S) {
     b.T = S.T;
     b.sptr = S.sptr.as<long long>();
     b.srow = S.srow.as<int>();
+    b.hot_list = S.hot_list;
     return b;
 }
 
@@ -272,7 +274,7 @@ k_push(BfsTiles P, ListsView Lv, Counters *__restrict__ cnt, BfsView B) {
                 int q = window_find(win, i);
                 long long s = s0 + q;
                 long long p = Lv.Ls_beg[s] + (i - win[q]);
-                long long v = B.row_begin + P.srow[p];
+                long long v = B.row_begin + decode_row<NT>(P.srow[p], P.hot_list);
                 discover<NT>(B, v / NT, (word_t)1 << (v % NT));
             }
             __syncwarp();
@@ -304,16 +306,6 @@ __global__ void __launch_bounds__(256) k_push_csr(BfsTiles Q, BfsView B) {
             if (planes[(long long)r * Q.T + t] & f) res |= (word_t)1 << r;
         }
         if (res) discover<NT>(B, Iseg, res);
-    }
-}
-
-template <class W> __device__ __forceinline__ W warp_or(W v) {
-    if constexpr (sizeof(W) == 8) {
-        unsigned lo = __reduce_or_sync(0xffffffffu, (unsigned)v);
-        unsigned hi = __reduce_or_sync(0xffffffffu, (unsigned)(v >> 32));
-        return ((W)hi << 32) | lo;
-    } else {
-        return (W)__reduce_or_sync(0xffffffffu, (unsigned)v);
     }
 }
 
@@ -366,7 +358,7 @@ __global__ void __launch_bounds__(256) k_pull_side(BfsTiles Q, BfsView B) {
         long long g = B.row_begin + v;
         if ((B.V[g >> 5] >> (g & 31)) & 1u) continue;
         for (long long p = p0; p < p1; ++p) {
-            long long u = Q.srow[p];
+            long long u = decode_row<NT>(Q.srow[p], Q.hot_list);
             if ((B.F[u >> 5] >> (u & 31)) & 1u) {
                 discover<NT>(B, g / NT, (word_t)1 << (g % NT));
                 break;

@@ -13,6 +13,8 @@
 //   6. side entries re-sorted by (column, row) -> side CSC.
 #include "common.cuh"
 #include <cub/cub.cuh>
+#include <algorithm>
+#include <vector>
 
 namespace tsmv {
 
@@ -92,7 +94,7 @@ __global__ void k_fill_tiles(const unsigned long long *__restrict__ keys, const 
                              typename Tr<NT>::word_t *__restrict__ planes,
                              unsigned long long *__restrict__ skey, V *__restrict__ sval,
                              int32_t *__restrict__ colcnt, TileDesc *__restrict__ desc,
-                             typename Tr<NT>::cs_t *__restrict__ cstart) {
+                             typename Tr<NT>::cs_t *__restrict__ cstart, const int32_t *__restrict__ hot_map) {
     using word_t = typename Tr<NT>::word_t;
     using idx_t = typename Tr<NT>::idx_t;
     constexpr int LOG = Tr<NT>::LOG;
@@ -123,7 +125,7 @@ __global__ void k_fill_tiles(const unsigned long long *__restrict__ keys, const 
             off[d] = p0;
             TileDesc td;
             td.off = p0;
-            td.trow = (int)I;
+            td.trow = (hot_map && hot_map[I] >= 0) ? ~hot_map[I] : (int)I;
             td.nnz = (int)(s1 - s0);
             desc[d] = td;
             atomicAdd(&colcnt[J], 1);
@@ -141,11 +143,17 @@ __global__ void k_fill_tiles(const unsigned long long *__restrict__ keys, const 
 }
 
 __global__ void k_side_split(const unsigned long long *__restrict__ skey, int64_t S, int64_t dimR,
-                             int32_t *__restrict__ srow, int32_t *__restrict__ scnt) {
+                             int32_t *__restrict__ srow, int32_t *__restrict__ scnt,
+                             const int32_t *__restrict__ hot_map, int nt) {
     for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q < S;
          q += (int64_t)gridDim.x * blockDim.x) {
         unsigned long long k = skey[q];
-        srow[q] = (int32_t)(k % (unsigned long long)dimR);
+        int32_t row = (int32_t)(k % (unsigned long long)dimR);
+        if (hot_map) {
+            int32_t h = hot_map[row / nt];
+            if (h >= 0) row = ~(h * nt + row % nt);
+        }
+        srow[q] = row;
         atomicAdd(&scnt[k / (unsigned long long)dimR], 1);
     }
 }
@@ -184,7 +192,7 @@ void counts_to_ptr(const int32_t *cnt, int64_t n, int64_t *ptr, CubTemp &tmp, cu
 
 template <int NT, class V>
 void build_nt(TileSet &S, const int32_t *rows, const int32_t *cols, const V *vals, int64_t nnz, int64_t dimR,
-              int64_t dimC, int thr, bool want_planes, cudaStream_t st) {
+              int64_t dimC, int thr, bool want_planes, cudaStream_t st, const int32_t *hot_map) {
     using word_t = typename Tr<NT>::word_t;
     using idx_t = typename Tr<NT>::idx_t;
     constexpr int LOG = Tr<NT>::LOG;
@@ -300,7 +308,7 @@ void build_nt(TileSet &S, const int32_t *rows, const int32_t *cols, const V *val
             S.mask.as<word_t>(), S.off.as<int64_t>(), S.idx.as<idx_t>(), vals ? S.val.as<V>() : nullptr,
             want_planes ? S.planes.as<word_t>() : nullptr, skey.as<unsigned long long>(),
             vals ? sval_tmp.as<V>() : nullptr, colcnt.as<int32_t>(), S.desc.as<TileDesc>(),
-            S.cstart.as<typename Tr<NT>::cs_t>());
+            S.cstart.as<typename Tr<NT>::cs_t>(), hot_map);
     TSMV_CUDA(cudaGetLastError());
     TSMV_CUDA(cudaMemcpyAsync(S.off.as<int64_t>() + T, &DN, 8, cudaMemcpyHostToDevice, st));
     S.ptr.alloc((S.nTC + 1) * 8);
@@ -339,7 +347,7 @@ void build_nt(TileSet &S, const int32_t *rows, const int32_t *cols, const V *val
     scnt.alloc((dimC + 1) * 4);
     TSMV_CUDA(cudaMemsetAsync(scnt.p, 0, (dimC + 1) * 4, st));
     if (SN) k_side_split<<<grid_for(SN), 256, 0, st>>>(skey2.as<unsigned long long>(), SN, dimR,
-                                                        S.srow.as<int32_t>(), scnt.as<int32_t>());
+                                                        S.srow.as<int32_t>(), scnt.as<int32_t>(), hot_map, NT);
     TSMV_CUDA(cudaGetLastError());
     S.sptr.alloc((dimC + 1) * 8);
     counts_to_ptr(scnt.as<int32_t>(), dimC, S.sptr.as<int64_t>(), tmp, st);
@@ -413,19 +421,64 @@ void prepare_csr(tsmv_ctx *c, const int64_t *row_ptr, const int32_t *col_idx, in
 }
 
 void build_tileset(tsmv_ctx *c, TileSet &S, const int32_t *rows, const int32_t *cols, const void *vals,
-                   int64_t nnz, int64_t dimR, int64_t dimC, bool want_vals, bool want_planes, cudaStream_t st) {
+                   int64_t nnz, int64_t dimR, int64_t dimC, bool want_vals, bool want_planes, cudaStream_t st,
+                   const int32_t *hot_map) {
     int thr = c->opt.sparse_tile_max_nnz;
+    S.hot_list = hot_map ? c->hot_list.as<int32_t>() : nullptr;
     bool f32 = c->dtype == TSMV_F32;
     const void *v = want_vals ? vals : nullptr;
 #define TSMV_BUILD(NTV)                                                                                  \
-    if (v && f32) build_nt<NTV, float>(S, rows, cols, (const float *)v, nnz, dimR, dimC, thr, want_planes, st); \
-    else build_nt<NTV, double>(S, rows, cols, (const double *)v, nnz, dimR, dimC, thr, want_planes, st);
+    if (v && f32) build_nt<NTV, float>(S, rows, cols, (const float *)v, nnz, dimR, dimC, thr, want_planes, st, hot_map); \
+    else build_nt<NTV, double>(S, rows, cols, (const double *)v, nnz, dimR, dimC, thr, want_planes, st, hot_map);
     switch (c->nt) {
         case 16: TSMV_BUILD(16); break;
         case 32: TSMV_BUILD(32); break;
         default: TSMV_BUILD(64); break;
     }
 #undef TSMV_BUILD
+}
+
+__global__ void k_tilerow_nnz(const int32_t *__restrict__ indeg, int64_t m, int nt, int64_t nTR,
+                              long long *__restrict__ out) {
+    for (int64_t I = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; I < nTR; I += (int64_t)gridDim.x * blockDim.x) {
+        long long s = 0;
+        for (int64_t r = I * nt; r < (I + 1) * nt && r < m; ++r) s += indeg[r];
+        out[I] = s;
+    }
+}
+
+// Pick the tile rows whose rows are privatised in shared memory by the SpMSpV
+// kernel: the HOT_SLOTS/nt tile rows with the most nonzeros (power-law hubs get
+// thousands of same-address fp64 atomics per call otherwise).
+void choose_hot_rows(tsmv_ctx *c, cudaStream_t st, DevBuf &hot_map) {
+    const int nt = c->nt;
+    const int64_t nTR = (c->m + nt - 1) / nt;
+    const int K = (int)std::min<int64_t>(HOT_SLOTS / nt, nTR);
+    c->n_hot = 0;
+    if (K <= 0 || c->m == 0) return;
+    DevBuf tr;
+    tr.alloc(nTR * 8);
+    k_tilerow_nnz<<<grid_for(nTR), 256, 0, st>>>(c->indeg.as<int32_t>(), c->m, nt, nTR, tr.as<long long>());
+    TSMV_CUDA(cudaGetLastError());
+    std::vector<long long> h(nTR);
+    TSMV_CUDA(cudaMemcpyAsync(h.data(), tr.p, nTR * 8, cudaMemcpyDeviceToHost, st));
+    TSMV_CUDA(cudaStreamSynchronize(st));
+    std::vector<int32_t> idx(nTR);
+    for (int64_t i = 0; i < nTR; ++i) idx[i] = (int32_t)i;
+    std::partial_sort(idx.begin(), idx.begin() + K, idx.end(), [&](int32_t a, int32_t b) {
+        return h[a] != h[b] ? h[a] > h[b] : a < b;
+    });
+    std::vector<int32_t> hot;
+    for (int q = 0; q < K; ++q)
+        if (h[idx[q]] >= 2 * nt) hot.push_back(idx[q]);  // only genuinely heavy tile rows
+    c->n_hot = (int)hot.size();
+    if (hot.empty()) return;
+    std::vector<int32_t> map(nTR, -1);
+    for (size_t q = 0; q < hot.size(); ++q) map[hot[q]] = (int32_t)q;
+    c->hot_list.alloc(hot.size() * 4);
+    TSMV_CUDA(cudaMemcpy(c->hot_list.p, hot.data(), hot.size() * 4, cudaMemcpyHostToDevice));
+    hot_map.alloc(nTR * 4);
+    TSMV_CUDA(cudaMemcpy(hot_map.p, map.data(), nTR * 4, cudaMemcpyHostToDevice));
 }
 
 bool same_pattern_transposed(tsmv_ctx *c, const int32_t *rows, const int32_t *cols, int64_t nnz, cudaStream_t st) {

@@ -104,6 +104,10 @@ struct TileSet {
     DevBuf srow;     // int32[side_nnz]
     DevBuf sval;     // double/float[side_nnz]
     bool has_vals = false, has_planes = false, has_list = false;
+    // Hot-row encoding (SpMSpV privatisation): rows of "hot" tile rows
+    // are stored as ~(hot_idx*NT + r) in srow and as ~hot_idx in TileDesc::trow;
+    // hot_list[hot_idx] = tile row.  decode_row() restores the row id.
+    const int32_t *hot_list = nullptr;
     size_t bytes() const {
         return ptr.bytes + trow.bytes + tgrp.bytes + mask.bytes + off.bytes + idx.bytes + val.bytes +
                planes.bytes + sptr.bytes + srow.bytes + sval.bytes + desc.bytes + cstart.bytes;
@@ -160,6 +164,7 @@ struct Lists {
     }
 };
 
+constexpr int HOT_SLOTS = 2048;           // privatised rows per CTA (smem fp64 + bits)
 constexpr int CHUNK_LOG = 7;               // 128 work items per warp-chunk
 constexpr int CHUNK = 1 << CHUNK_LOG;
 constexpr int SCAN_BLOCK = 256;
@@ -184,6 +189,8 @@ struct tsmv_ctx {
     tsmv::TileSet Qown;        // tile-CSC of A^T (pull / Push-CSR) when A is not symmetric
     tsmv::TileSet *Q = nullptr;
 
+    tsmv::DevBuf hot_list;     // int32[n_hot]: tile rows privatised in the SpMSpV kernel
+    int n_hot = 0;
     tsmv::DevBuf outdeg;       // int32[n]: nnz of column v (local rows)
     tsmv::DevBuf indeg;        // int32[m]: nnz of row v
 
@@ -222,13 +229,21 @@ struct tsmv_ctx {
     int fused_blocks = 0, fused_threads = 1024;
     tsmv::DevBuf partials;         // long long[fused_blocks][8]
     long long last_x_nnz = 0;
+    void *trace = nullptr;         // tsmv_set_trace (device, u64[tsmv_trace_words])
 };
 
 namespace tsmv {
+// side-matrix / descriptor row decode (hot-row encoding, see TileSet::hot_list)
+template <int NT> __host__ __device__ __forceinline__ long long decode_row(long long v, const int32_t *hot_list) {
+    if (v >= 0) return v;
+    const long long s = ~v;
+    return (long long)hot_list[s / NT] * NT + (s % NT);
+}
 // builder.cu
 void build_tileset(tsmv_ctx *c, TileSet &S, const int32_t *rows, const int32_t *cols, const void *vals,
                    int64_t nnz, int64_t dimR, int64_t dimC, bool want_vals, bool want_planes,
-                   cudaStream_t st);
+                   cudaStream_t st, const int32_t *hot_map = nullptr);
+void choose_hot_rows(tsmv_ctx *c, cudaStream_t st, DevBuf &hot_map);
 bool same_pattern_transposed(tsmv_ctx *c, const int32_t *rows, const int32_t *cols, int64_t nnz,
                              cudaStream_t st);
 void prepare_csr(tsmv_ctx *c, const int64_t *row_ptr, const int32_t *col_idx, int32_t *rows, cudaStream_t st);

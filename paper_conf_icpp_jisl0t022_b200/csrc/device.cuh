@@ -205,9 +205,11 @@ inline ListsView lists_view(tsmv_ctx *c) {
 }
 
 // Write chunk -> entry map for an entry owning work items [w0, w0+w).
+template <int LOGC = CHUNK_LOG>
 __device__ __forceinline__ void write_chunks(int *C, long long w0, long long w, int entry) {
-    long long c0 = (w0 + CHUNK - 1) >> CHUNK_LOG;
-    long long c1 = (w0 + w + CHUNK - 1) >> CHUNK_LOG;
+    constexpr int CH = 1 << LOGC;
+    long long c0 = (w0 + CH - 1) >> LOGC;
+    long long c1 = (w0 + w + CH - 1) >> LOGC;
     for (long long ch = c0; ch < c1; ++ch) C[ch] = entry;
 }
 
@@ -216,21 +218,24 @@ __device__ __forceinline__ void write_chunks(int *C, long long w0, long long w, 
 // The trip count is warp-uniform on purpose: with a lane-dependent count
 // (q = lane; q <= CHUNK) ptxas compiled the following __syncwarp() to a NOP and
 // lanes read win[CHUNK] before lane 0 had stored it (found on B200, r1).
+template <int LOGC = CHUNK_LOG>
 __device__ __forceinline__ void load_window(long long *win, const long long *wpre, long long s0, long long nL,
                                             int lane) {
+    constexpr int CH = 1 << LOGC;
 #pragma unroll
-    for (int q0 = 0; q0 <= CHUNK; q0 += 32) {
+    for (int q0 = 0; q0 <= CH; q0 += 32) {
         int q = q0 + lane;
         long long idx = s0 + q;
         long long v = idx <= nL ? wpre[idx] : 0x7fffffffffffffffLL;
-        if (q <= CHUNK) win[q] = v;
+        if (q <= CH) win[q] = v;
     }
     __syncwarp();
 }
 
 // Largest q in [0, CHUNK] with win[q] <= i (win[0] <= i guaranteed).
+template <int LOGC = CHUNK_LOG>
 __device__ __forceinline__ int window_find(const long long *win, long long i) {
-    int lo = 0, hi = CHUNK;  // invariant win[lo] <= i, answer in [lo, hi]
+    int lo = 0, hi = 1 << LOGC;  // invariant win[lo] <= i, answer in [lo, hi]
     while (lo < hi) {
         int mid = (lo + hi + 1) >> 1;
         if (win[mid] <= i) lo = mid;
@@ -272,6 +277,17 @@ template <class W> __device__ __forceinline__ int ffs_w(W w) {
     if constexpr (sizeof(W) == 8) return __ffsll((long long)w) - 1;
     else return __ffs((unsigned)w) - 1;
 }
+
+template <class W> __device__ __forceinline__ W warp_or(W v) {
+    if constexpr (sizeof(W) == 8) {
+        unsigned lo = __reduce_or_sync(0xffffffffu, (unsigned)v);
+        unsigned hi = __reduce_or_sync(0xffffffffu, (unsigned)(v >> 32));
+        return ((W)hi << 32) | lo;
+    } else {
+        return (W)__reduce_or_sync(0xffffffffu, (unsigned)v);
+    }
+}
+
 
 // order-preserving map double -> uint64 (unsigned order == numeric order)
 __device__ __forceinline__ unsigned long long ord_key(double x) {

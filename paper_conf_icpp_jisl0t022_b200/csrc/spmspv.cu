@@ -30,7 +30,23 @@ namespace tsmv {
 
 namespace {
 
-constexpr int FB = 512;  // threads per CTA of the fused kernel
+#ifndef TSMV_FB
+#define TSMV_FB 512
+#endif
+#ifndef TSMV_CB
+#define TSMV_CB 8
+#endif
+constexpr int FB = TSMV_FB;  // threads per CTA of the fused kernel
+constexpr int CB = TSMV_CB;  // accumulator loads batched per lane in phase C
+#ifndef TSMV_R
+#define TSMV_R 4
+#endif
+#ifndef TSMV_SCL
+#define TSMV_SCL 7
+#endif
+constexpr int R = TSMV_R;     // useful nonzeros per lane per round of the multiply step
+constexpr int SCL = TSMV_SCL; // log2 of the items per warp-chunk of the SpMSpV load balancer
+constexpr int SCH = 1 << SCL;
 constexpr int TRING = 4096;
 
 struct FusedArgs {
@@ -61,21 +77,206 @@ struct FusedArgs {
     unsigned long long bar_base;
     unsigned long long *tring;  // nullptr = no timing
     long long tslot;
+    const int32_t *hot_list;    // privatised tile rows (TileSet::hot_list), n_hot of them
+    int n_hot;
+    unsigned long long *trace;  // tsmv_set_trace: per warp {t_B0, t_loop_end, chunks, tile ns, side ns, max chunk ns, t_arrive, macs}
 };
 
+// Shared-memory accumulation of the privatised ("hot") rows.
 template <int SR>
-__device__ __forceinline__ void accumulate(double *acc, uint32_t *rowbits, long long row, double a, double x) {
+__device__ __forceinline__ void accumulate_shared(double *s_acc, long long slot, double a, double x) {
     if constexpr (SR == TSMV_PLUS_TIMES) {
+        atomicAdd(&s_acc[slot], a * x);
+    } else if constexpr (SR == TSMV_MIN_SECOND) {
+        atomicMax((unsigned long long *)&s_acc[slot], ~ord_key(x));
+    }
+}
+
+// Exclusive block-wide scan of K int64 values per thread (shuffles + one smem
+// pass); register-light replacement for cub::BlockScan of a 4-wide struct, which
+// made the fused kernel spill.  tot = block totals (all threads).  Contains
+// __syncthreads; every thread of the block must call it.
+template <int K, int NTHREADS>
+__device__ __forceinline__ void block_scan(const long long *v, long long *ex, long long *tot,
+                                           long long (*s)[NTHREADS / 32]) {
+    constexpr int NW = NTHREADS / 32;
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+#pragma unroll
+    for (int i = 0; i < K; ++i) {
+        long long x = v[i];
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const long long y = __shfl_up_sync(0xffffffffu, x, o);
+            if (lane >= o) x += y;
+        }
+        ex[i] = x - v[i];
+        if (lane == 31) s[i][wid] = x;
+    }
+    __syncthreads();
+#pragma unroll
+    for (int i = 0; i < K; ++i) {
+        long long before = 0, all = 0;
+#pragma unroll
+        for (int w = 0; w < NW; ++w) {
+            const long long t = s[i][w];
+            before += w < wid ? t : 0;
+            all += t;
+        }
+        ex[i] += before;
+        tot[i] = all;
+    }
+    __syncthreads();
+}
+
+template <int SR>
+__device__ __forceinline__ void accumulate_value(double *acc, long long row, double a, double x) {
+    if constexpr (SR == TSMV_PLUS_TIMES) {
+#ifdef TSMV_EXPERIMENT_NO_ATOMIC
+        if (a * x == 1234.5678) acc[row] = 0.0;  // keeps the loads, drops the RED
+#else
         atomicAdd(&acc[row], a * x);
+#endif
     } else if constexpr (SR == TSMV_MIN_SECOND) {
         atomicMax((unsigned long long *)&acc[row], ~ord_key(x));
     }
-    // Touched-row bit: test before set.  Power-law rows receive thousands of
-    // contributions per call; an unconditional RED.OR on their (shared) word
-    // serialises in one L2 slice.  A stale read only costs a redundant RED.
-    const unsigned bit = 1u << (row & 31);
-    unsigned *wp = &rowbits[row >> 5];
-    if (!(__ldca(wp) & bit)) atomicOr(wp, bit);
+}
+
+// Touched-row bits of rows rowbase + {bits of m} (rowbase is a multiple of NT, so
+// the rows of one tile share a word, or two for NT = 64).  Test before set:
+// power-law rows receive thousands of contributions per call and an
+// unconditional RED.OR on their shared word serialises in one L2 slice; the L1
+// copy can only be stale towards "not set", which costs a redundant RED.
+template <int NT>
+__device__ __forceinline__ void mark_rows(uint32_t *rowbits, long long rowbase, typename Tr<NT>::word_t m) {
+    if constexpr (NT == 64) {
+        uint32_t lo = (uint32_t)m, hi = (uint32_t)((unsigned long long)m >> 32);
+        uint32_t *w = rowbits + (rowbase >> 5);
+        if (lo && (__ldca(w) & lo) != lo) atomicOr(w, lo);
+        if (hi && (__ldca(w + 1) & hi) != hi) atomicOr(w + 1, hi);
+    } else {
+        const uint32_t b = (uint32_t)m << (rowbase & 31);
+        uint32_t *w = rowbits + (rowbase >> 5);
+        if ((__ldca(w) & b) != b) atomicOr(w, b);
+    }
+}
+
+template <int NT>
+__device__ __forceinline__ void mark_rows_shared(uint32_t *s_bits, long long slotbase, typename Tr<NT>::word_t m) {
+    if constexpr (NT == 64) {
+        atomicOr(&s_bits[slotbase >> 5], (uint32_t)m);
+        atomicOr(&s_bits[(slotbase >> 5) + 1], (uint32_t)((unsigned long long)m >> 32));
+    } else {
+        atomicOr(&s_bits[slotbase >> 5], (uint32_t)m << (slotbase & 31));
+    }
+}
+
+// Staged hit tile of one lane (multiply step of phase B).
+struct Stage {
+    long long off, t;
+    unsigned long long hit;
+    int incl, J, trow, nnz;
+};
+
+// Column range [p0, p1) of column c inside tile t (column-major nonzeros).
+template <int NT>
+__device__ __forceinline__ void col_range(const typename Tr<NT>::cs_t *cstart, long long t, int c, int nnz, int &p0,
+                                          int &p1) {
+    p0 = cstart[t * NT + c];
+    p1 = c + 1 < NT ? (int)cstart[t * NT + c + 1] : nnz;
+}
+
+// nt = 16: the 16 one-byte column starts of a tile are one aligned 16-byte
+// load; the column walks below then run in registers (a walk over global
+// memory is a chain of dependent L2 round trips, ~1 us per hit column).
+__device__ __forceinline__ uint4 cs_row16(const uint8_t *cstart, long long t) {
+    return __ldg(reinterpret_cast<const uint4 *>(cstart + t * 16));
+}
+__device__ __forceinline__ int cs_byte16(const uint4 &w, int c, int nnz) {
+    if (c >= 16) return nnz;
+    const unsigned x = c < 8 ? (c < 4 ? w.x : w.y) : (c < 12 ? w.z : w.w);
+    return (int)((x >> ((c & 3) * 8)) & 0xffu);
+}
+
+__device__ __forceinline__ int hit_useful16(const uint4 &w, unsigned h, int nnz) {
+    int s = 0;
+    while (h) {
+        const int c = __ffs(h) - 1;
+        h &= h - 1;
+        s += cs_byte16(w, c + 1, nnz) - cs_byte16(w, c, nnz);
+    }
+    return s;
+}
+__device__ __forceinline__ void hit_position16(const uint4 &w, unsigned h, int nnz, int k, int &c, int &p) {
+    c = 0;
+    p = 0;
+    while (h) {
+        c = __ffs(h) - 1;
+        h &= h - 1;
+        const int p0 = cs_byte16(w, c, nnz), len = cs_byte16(w, c + 1, nnz) - p0;
+        if (k < len) {
+            p = p0 + k;
+            return;
+        }
+        k -= len;
+    }
+}
+
+// Useful nonzeros of a hit tile = sum over its hit columns of the column lengths.
+template <int NT>
+__device__ __forceinline__ int hit_useful(const typename Tr<NT>::cs_t *cstart, long long t,
+                                          typename Tr<NT>::word_t h, int nnz) {
+    if constexpr (NT == 16) {
+        const uint4 w = cs_row16((const uint8_t *)cstart, t);
+        int s = 0;
+        while (h) {
+            const int c = ffs_w(h);
+            h &= h - 1;
+            s += cs_byte16(w, c + 1, nnz) - cs_byte16(w, c, nnz);
+        }
+        return s;
+    }
+    int s = 0;
+    while (h) {
+        const int c = ffs_w(h);
+        h &= h - 1;
+        int p0, p1;
+        col_range<NT>(cstart, t, c, nnz, p0, p1);
+        s += p1 - p0;
+    }
+    return s;
+}
+
+// The k-th useful nonzero of a hit tile: its column c and position p in the tile.
+template <int NT>
+__device__ __forceinline__ void hit_position(const typename Tr<NT>::cs_t *cstart, long long t,
+                                             typename Tr<NT>::word_t h, int nnz, int k, int &c, int &p) {
+    c = 0;
+    p = 0;
+    if constexpr (NT == 16) {
+        const uint4 w = cs_row16((const uint8_t *)cstart, t);
+        while (h) {
+            c = ffs_w(h);
+            h &= h - 1;
+            const int p0 = cs_byte16(w, c, nnz), len = cs_byte16(w, c + 1, nnz) - p0;
+            if (k < len) {
+                p = p0 + k;
+                return;
+            }
+            k -= len;
+        }
+        return;
+    }
+    while (h) {
+        c = ffs_w(h);
+        h &= h - 1;
+        int p0, p1;
+        col_range<NT>(cstart, t, c, nnz, p0, p1);
+        if (k < p1 - p0) {
+            p = p0 + k;
+            return;
+        }
+        k -= p1 - p0;
+    }
 }
 
 // per-entry facts of phase A
@@ -103,24 +304,28 @@ __global__ void __launch_bounds__(FB, 1) k_spmspv_fused(FusedArgs a) {
     using idx_t = typename Tr<NT>::idx_t;
     using cs_t = typename Tr<NT>::cs_t;
     constexpr int LOG = Tr<NT>::LOG;
-    constexpr int U = CHUNK / 32;
+    constexpr int U = SCH / 32;
     constexpr int NW = FB / 32;
-    using BSQ = cub::BlockScan<Quad, FB>;
-    using BSL = cub::BlockScan<long long, FB>;
-    __shared__ union {
-        typename BSQ::TempStorage q;
-        typename BSL::TempStorage l;
-    } ts;
-    __shared__ long long win_all[NW][CHUNK + 1];
+    __shared__ long long s_scan[4][NW];  // block_scan scratch
+    __shared__ long long win_all[NW][SCH + 1];
+
     __shared__ long long s_pre[4], s_tot[4];
     __shared__ long long s_acct[NW][3];
     __shared__ int s_err;
+    extern __shared__ __align__(16) unsigned char s_dyn[];
+    double *s_hacc = reinterpret_cast<double *>(s_dyn);                   // [HOT_SLOTS]
+    uint32_t *s_hbits = reinterpret_cast<uint32_t *>(s_dyn + HOT_SLOTS * 8);  // [HOT_SLOTS/32]
+    Stage *stage_all = reinterpret_cast<Stage *>(s_dyn + HOT_SLOTS * 8 + HOT_SLOTS / 8);  // [NW][SCH]
+    const int n_slots = a.n_hot * NT;
     const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
     const int G = gridDim.x, b = blockIdx.x;
     unsigned long long target = a.bar_base;
     const bool stamp = a.tring && b == 0 && tid == 0;
     unsigned long long *ts_out = a.tring ? a.tring + (a.tslot % TRING) * 8 : nullptr;
     if (stamp) ts_out[0] = globaltimer_ns();
+
+    for (int i = tid; i < n_slots; i += FB) s_hacc[i] = 0.0;
+    for (int i = tid; i < (n_slots + 31) / 32; i += FB) s_hbits[i] = 0u;
 
     // ------------------------------------------------------------ phase A: x -> segments
     const long long E = (a.k + G - 1) / G;
@@ -145,7 +350,7 @@ __global__ void __launch_bounds__(FB, 1) k_spmspv_fused(FusedArgs a) {
     }
     if (any_bad) a.cnt->err = 1;
     Quad ex, agg;
-    BSQ(ts.q).ExclusiveScan(q, ex, Quad{{0, 0, 0, 0}}, QuadSum(), agg);
+    block_scan<4, FB>(q.v, ex.v, agg.v, s_scan);
     if (tid < 4) a.partials[b * 8 + tid] = agg.v[tid];
     if (b == 0 && tid == 0) a.cnt->chunk_next = 0;
     grid_sync(&a.cnt->bar, target);
@@ -200,7 +405,7 @@ __global__ void __launch_bounds__(FB, 1) k_spmspv_fused(FusedArgs a) {
                 a.Lv.Lt_mask[oLt] = mk;
                 a.Lv.Lt_tbeg[oLt] = a.tptr[seg];
                 a.Lv.Lt_wpre[oLt] = oWt;
-                write_chunks(a.Lv.Ct, oWt, wt, (int)oLt);
+                write_chunks<SCL>(a.Lv.Ct, oWt, wt, (int)oLt);
                 ++oLt;
                 oWt += wt;
             }
@@ -208,7 +413,7 @@ __global__ void __launch_bounds__(FB, 1) k_spmspv_fused(FusedArgs a) {
                 a.Lv.Ls_beg[oLs] = a.sptr[j];
                 a.Lv.Ls_wpre[oLs] = oWs;
                 a.Lv.Ls_x[oLs] = a.x_val ? (double)((const XV *)a.x_val)[e] : 1.0;
-                write_chunks(a.Lv.Cs, oWs, ws, (int)oLs);
+                write_chunks<SCL>(a.Lv.Cs, oWs, ws, (int)oLs);
                 ++oLs;
                 oWs += ws;
             }
@@ -225,7 +430,7 @@ __global__ void __launch_bounds__(FB, 1) k_spmspv_fused(FusedArgs a) {
     long long n_hit = 0, n_hcol = 0, n_mac = 0;
     if (!err) {
         const long long nLt = s_tot[0], Wt = s_tot[1], nLs = s_tot[2], Ws = s_tot[3];
-        const long long nCt = (Wt + CHUNK - 1) >> CHUNK_LOG, nCs = (Ws + CHUNK - 1) >> CHUNK_LOG;
+        const long long nCt = (Wt + SCH - 1) >> SCL, nCs = (Ws + SCH - 1) >> SCL;
         long long *win = win_all[wid];
         const word_t *mask = (const word_t *)a.mask;
         const idx_t *idx = (const idx_t *)a.idx;
@@ -234,18 +439,28 @@ __global__ void __launch_bounds__(FB, 1) k_spmspv_fused(FusedArgs a) {
         const cs_t *cstart = (const cs_t *)a.cstart;
         const unsigned nwarps = (unsigned)(G * NW);
         unsigned ch = (unsigned)(b * NW + wid);  // first chunk static, then the queue
+        unsigned long long tr_b0 = 0, tr_tile = 0, tr_side = 0, tr_max = 0, tr_n = 0, tr_stage = 0, tr_smax = 0;
+#ifdef TSMV_TRACE_ROUNDS
+        unsigned long long tr_pos = 0, tr_ld = 0, tr_at = 0;
+#endif
+        if (a.trace) tr_b0 = globaltimer_ns();
         while (true) {
+            const unsigned long long tr_c0 = a.trace ? globaltimer_ns() : 0;
+            const bool tr_is_tile = ch < nCt;
+            // grab the next chunk now; its latency overlaps this chunk's work
+            unsigned nx = 0;
+            if (lane == 0 && ch < nCt + nCs) nx = nwarps + atomicAdd(&a.cnt->chunk_next, 1u);
             if (ch < nCt) {
                 const long long s0 = __ldcg(&a.Lv.Ct[ch]);
-                const long long base = (long long)ch << CHUNK_LOG;
-                load_window(win, a.Lv.Lt_wpre, s0, nLt, lane);
+                const long long base = (long long)ch << SCL;
+                load_window<SCL>(win, a.Lv.Lt_wpre, s0, nLt, lane);
                 long long sidx[U], t[U];
                 bool ok[U];
 #pragma unroll
                 for (int u = 0; u < U; ++u) {
                     const long long i = base + lane + 32 * u;
                     ok[u] = i < Wt;
-                    const int qq = ok[u] ? window_find(win, i) : 0;
+                    const int qq = ok[u] ? window_find<SCL>(win, i) : 0;
                     sidx[u] = s0 + qq;
                     t[u] = i - win[qq];
                 }
@@ -262,41 +477,141 @@ __global__ void __launch_bounds__(FB, 1) k_spmspv_fused(FusedArgs a) {
                 word_t hit[U];
 #pragma unroll
                 for (int u = 0; u < U; ++u) hit[u] = ok[u] ? (word_t)(mask[t[u]] & xm[u]) : (word_t)0;
+                // ---- multiply: nonzero-level load balance inside the warp.  The hit
+                // tiles of all U items of all lanes are staged in shared memory with the
+                // inclusive prefix of their useful nonzeros (sum over hit columns); the
+                // warp then walks that flat index space R positions per lane at a time,
+                // so a dense hub tile is spread over the warp and the loads of different
+                // positions are issued together.
+                TileDesc d[U];
+#pragma unroll
+                for (int u = 0; u < U; ++u)
+                    if (hit[u]) d[u] = ((const TileDesc *)a.desc)[t[u]];
+                int useful[U];
+                int mine = 0;
 #pragma unroll
                 for (int u = 0; u < U; ++u) {
+                    useful[u] = hit[u] ? hit_useful<NT>(cstart, t[u], hit[u], d[u].nnz) : 0;
+                    mine += useful[u];
                     if (hit[u]) {
-                        const TileDesc d = ((const TileDesc *)a.desc)[t[u]];
                         ++n_hit;
-                        word_t h = hit[u];
-                        const long long rowbase = (long long)d.trow * NT;
-                        while (h) {
-                            const int c = ffs_w(h);
-                            h &= h - 1;
-                            const int p0 = cstart[t[u] * NT + c];
-                            const int p1 = c + 1 < NT ? (int)cstart[t[u] * NT + c + 1] : d.nnz;
-                            const double xv = __ldcg(&a.Lv.xd[J[u] * NT + c]);
-                            for (int p = p0; p < p1; ++p) {
-                                const unsigned r = idx[d.off + p] & (NT - 1);
-                                const double av = val ? (double)val[d.off + p] : 1.0;
-                                accumulate<SR>(a.acc, a.rowbits, rowbase + r, av, xv);
-                            }
-                            n_mac += p1 - p0;
-                            ++n_hcol;
+                        n_hcol += popc_w(hit[u]);
+                    }
+                }
+                n_mac += mine;
+                int incl = mine;
+#pragma unroll
+                for (int o = 1; o < 32; o <<= 1) {
+                    const int v = __shfl_up_sync(0xffffffffu, incl, o);
+                    if (lane >= o) incl += v;
+                }
+                const int total = __shfl_sync(0xffffffffu, incl, 31);
+                if (a.trace) tr_stage = globaltimer_ns() - tr_c0;
+                if (total > 0) {
+                    Stage *st = stage_all + wid * SCH;
+                    int run = incl - mine;
+#pragma unroll
+                    for (int u = 0; u < U; ++u) {
+                        run += useful[u];
+                        Stage &sg = st[lane * U + u];
+                        sg.incl = run;
+                        if (useful[u]) {
+                            sg.t = t[u];
+                            sg.J = (int)J[u];
+                            sg.off = d[u].off;
+                            sg.hit = (unsigned long long)hit[u];
+                            sg.trow = d[u].trow;
+                            sg.nnz = d[u].nnz;
                         }
                     }
+                    __syncwarp();
+                    for (int q0 = 0; q0 < total; q0 += 32 * R) {
+#ifdef TSMV_TRACE_ROUNDS
+                        const unsigned long long rt0 = globaltimer_ns();
+#endif
+                        long long row[R], pos[R], xj[R];
+                        bool okq[R], hot[R];
+#pragma unroll
+                        for (int r = 0; r < R; ++r) {
+                            const int q = q0 + 32 * r + lane;
+                            okq[r] = q < total;
+                            if (okq[r]) {
+                                int lo = 0, hi = SCH - 1;  // first staged entry with incl > q
+                                while (lo < hi) {
+                                    const int mid = (lo + hi) >> 1;
+                                    if (st[mid].incl > q) hi = mid;
+                                    else lo = mid + 1;
+                                }
+                                const Stage &src = st[lo];
+                                const int before = lo ? st[lo - 1].incl : 0;
+                                int c, p;
+                                hit_position<NT>(cstart, src.t, (word_t)src.hit, src.nnz, q - before, c, p);
+                                hot[r] = src.trow < 0;
+                                row[r] = (hot[r] ? (long long)(~src.trow) : (long long)src.trow) * NT;
+                                pos[r] = src.off + p;
+                                xj[r] = (long long)src.J * NT + c;
+                            }
+                        }
+                        double av[R], xv[R];
+#ifdef TSMV_TRACE_ROUNDS
+                        __syncwarp();
+                        const unsigned long long rt1 = globaltimer_ns();
+#endif
+#pragma unroll
+                        for (int r = 0; r < R; ++r) {
+                            if (okq[r]) {
+                                row[r] += idx[pos[r]] & (NT - 1);
+                                av[r] = val ? (double)val[pos[r]] : 1.0;
+                                xv[r] = __ldcg(&a.Lv.xd[xj[r]]);
+                            }
+                        }
+#ifdef TSMV_TRACE_ROUNDS
+                        {
+                            double sink = 0;
+                            for (int r = 0; r < R; ++r) if (okq[r]) sink += av[r] + xv[r] + (double)row[r];
+                            if (sink == 1.2345e300) a.acc[0] = sink;
+                        }
+                        __syncwarp();
+                        const unsigned long long rt2 = globaltimer_ns();
+#endif
+#pragma unroll
+                        for (int r = 0; r < R; ++r) {
+                            if (okq[r]) {
+                                if (hot[r]) {
+                                    accumulate_shared<SR>(s_hacc, row[r], av[r], xv[r]);
+                                    atomicOr(&s_hbits[row[r] >> 5], 1u << (row[r] & 31));
+                                } else {
+                                    accumulate_value<SR>(a.acc, row[r], av[r], xv[r]);
+                                }
+                            }
+                        }
+                        // touched bit: rows of hub tile rows are privatised (shared memory),
+                        // so the remaining RED.ORs are spread over many words -> no test load
+#pragma unroll
+                        for (int r = 0; r < R; ++r)
+                            if (okq[r] && !hot[r]) atomicOr(&a.rowbits[row[r] >> 5], 1u << (row[r] & 31));
+#ifdef TSMV_TRACE_ROUNDS
+                        __syncwarp();
+                        const unsigned long long rt3 = globaltimer_ns();
+                        tr_pos += rt1 - rt0;
+                        tr_ld += rt2 - rt1;
+                        tr_at += rt3 - rt2;
+#endif
+                    }
+                    __syncwarp();
                 }
             } else if (ch < nCt + nCs) {
                 const long long c2 = (long long)ch - nCt;
                 const long long s0 = __ldcg(&a.Lv.Cs[c2]);
-                const long long base = c2 << CHUNK_LOG;
-                load_window(win, a.Lv.Ls_wpre, s0, nLs, lane);
+                const long long base = c2 << SCL;
+                load_window<SCL>(win, a.Lv.Ls_wpre, s0, nLs, lane);
                 long long p[U], sidx[U];
                 bool ok[U];
 #pragma unroll
                 for (int u = 0; u < U; ++u) {
                     const long long i = base + lane + 32 * u;
                     ok[u] = i < Ws;
-                    const int qq = ok[u] ? window_find(win, i) : 0;
+                    const int qq = ok[u] ? window_find<SCL>(win, i) : 0;
                     sidx[u] = s0 + qq;
                     p[u] = i - win[qq];
                 }
@@ -318,15 +633,47 @@ __global__ void __launch_bounds__(FB, 1) k_spmspv_fused(FusedArgs a) {
                     }
                 }
 #pragma unroll
+                for (int u = 0; u < U; ++u) {
+                    if (ok[u] && row[u] < 0) {  // privatised row: shared memory
+                        const long long sl = ~row[u];
+                        accumulate_shared<SR>(s_hacc, sl, av[u], xv[u]);
+                        atomicOr(&s_hbits[sl >> 5], 1u << (sl & 31));
+                        ok[u] = false;
+                    }
+                }
+#pragma unroll
                 for (int u = 0; u < U; ++u)
-                    if (ok[u]) accumulate<SR>(a.acc, a.rowbits, row[u], av[u], xv[u]);
+                    if (ok[u]) accumulate_value<SR>(a.acc, row[u], av[u], xv[u]);
+#pragma unroll
+                for (int u = 0; u < U; ++u)
+                    if (ok[u]) atomicOr(&a.rowbits[row[u] >> 5], 1u << (row[u] & 31));
             } else {
                 break;
             }
             __syncwarp();
-            unsigned nx = 0;
-            if (lane == 0) nx = nwarps + atomicAdd(&a.cnt->chunk_next, 1u);
+            if (a.trace) {
+                const unsigned long long dt = globaltimer_ns() - tr_c0;
+                (tr_is_tile ? tr_tile : tr_side) += dt;
+                if (dt > tr_max) tr_smax = tr_is_tile ? tr_stage : 0;
+                tr_max = dt > tr_max ? dt : tr_max;
+                ++tr_n;
+            }
             ch = __shfl_sync(0xffffffffu, nx, 0);
+        }
+        if (a.trace && lane == 0) {
+            unsigned long long *tw = a.trace + ((long long)b * NW + wid) * 8;
+            tw[0] = tr_b0;
+            tw[1] = globaltimer_ns();
+            tw[2] = tr_n;
+            tw[3] = tr_tile;
+            tw[4] = tr_side;
+            tw[5] = tr_max;
+            tw[6] = tr_smax;
+#ifdef TSMV_TRACE_ROUNDS
+            tw[3] = tr_pos;
+            tw[4] = tr_ld;
+            tw[6] = tr_at;
+#endif
         }
     }
 #pragma unroll
@@ -339,6 +686,24 @@ __global__ void __launch_bounds__(FB, 1) k_spmspv_fused(FusedArgs a) {
         s_acct[wid][0] = n_hit;
         s_acct[wid][1] = n_hcol;
         s_acct[wid][2] = n_mac;
+    }
+    // flush the privatised rows: one global atomic per (CTA, touched hot row)
+    __syncthreads();
+    if (!err) {
+        for (int sl = tid; sl < n_slots; sl += FB) {
+            if ((s_hbits[sl >> 5] >> (sl & 31)) & 1u) {
+                const long long row = (long long)a.hot_list[sl / NT] * NT + sl % NT;
+                if constexpr (SR == TSMV_PLUS_TIMES) atomicAdd(&a.acc[row], s_hacc[sl]);
+                else if constexpr (SR == TSMV_MIN_SECOND)
+                    atomicMax((unsigned long long *)&a.acc[row], (unsigned long long)__double_as_longlong(s_hacc[sl]));
+                const unsigned bit = 1u << (row & 31);
+                if (!(__ldca(&a.rowbits[row >> 5]) & bit)) atomicOr(&a.rowbits[row >> 5], bit);
+            }
+        }
+    }
+    if (a.trace && lane == 0) {
+        unsigned long long *tw = a.trace + ((long long)b * NW + wid) * 8;
+        tw[7] = (unsigned long long)n_mac;
     }
     grid_sync(&a.cnt->bar, target);  // (its __syncthreads also orders s_acct)
     if (stamp) ts_out[3] = globaltimer_ns();
@@ -356,7 +721,7 @@ __global__ void __launch_bounds__(FB, 1) k_spmspv_fused(FusedArgs a) {
     long long blk = 0;
     {
         long long dummy;
-        BSL(ts.l).ExclusiveSum(mycnt, dummy, blk);
+        block_scan<1, FB>(&mycnt, &dummy, &blk, s_scan);
     }
     if (tid == 0) a.partials[b * 8 + 4] = blk;
     grid_sync(&a.cnt->bar, target);
@@ -386,17 +751,17 @@ __global__ void __launch_bounds__(FB, 1) k_spmspv_fused(FusedArgs a) {
         const long long w = rb + tid;
         const unsigned bits = w < w1 ? __ldcg(&a.rowbits[w]) : 0u;
         long long c = __popc(bits), exw, rtot;
-        BSL(ts.l).ExclusiveSum(c, exw, rtot);
+        block_scan<1, FB>(&c, &exw, &rtot, s_scan);
         const long long pos0 = carry + exw;
         carry += rtot;
         if (bits) a.rowbits[w] = 0u;
         const long long wbase = w - lane;
         unsigned todo = __ballot_sync(0xffffffffu, bits != 0);
         while (todo) {
-            int src[8];
+            int src[CB];
             int nb = 0;
 #pragma unroll
-            for (int kk = 0; kk < 8; ++kk) {
+            for (int kk = 0; kk < CB; ++kk) {
                 src[kk] = 0;
                 if (todo) {
                     src[kk] = __ffs(todo) - 1;
@@ -404,19 +769,19 @@ __global__ void __launch_bounds__(FB, 1) k_spmspv_fused(FusedArgs a) {
                     nb = kk + 1;
                 }
             }
-            unsigned wb[8];
-            long long wp[8];
-            double v[8];
-            bool mine[8];
+            unsigned wb[CB];
+            long long wp[CB];
+            double v[CB];
+            bool mine[CB];
 #pragma unroll
-            for (int kk = 0; kk < 8; ++kk) {
+            for (int kk = 0; kk < CB; ++kk) {
                 wb[kk] = __shfl_sync(0xffffffffu, bits, src[kk]);
                 wp[kk] = __shfl_sync(0xffffffffu, pos0, src[kk]);
                 mine[kk] = kk < nb && ((wb[kk] >> lane) & 1u);
                 if (mine[kk]) v[kk] = __ldcg(&a.acc[(wbase + src[kk]) * 32 + lane]);
             }
 #pragma unroll
-            for (int kk = 0; kk < 8; ++kk) {
+            for (int kk = 0; kk < CB; ++kk) {
                 if (mine[kk]) {
                     const long long row = (wbase + src[kk]) * 32 + lane;
                     const long long pos = wp[kk] + __popc(wb[kk] & lt);
@@ -433,7 +798,7 @@ __global__ void __launch_bounds__(FB, 1) k_spmspv_fused(FusedArgs a) {
                 }
             }
         }
-        __syncthreads();  // ts.l reuse
+        __syncthreads();  // s_scan reuse
     }
     if (b == 0 && tid == 0) {
         // every CTA read cnt->err before barrier 3, so it can be reset here
@@ -449,6 +814,8 @@ __global__ void __launch_bounds__(FB, 1) k_spmspv_fused(FusedArgs a) {
 
 // Phase-A totals / accounting for tsmv_last_call_stats are summed on the host
 // from `partials` and `acct`.
+
+size_t fused_dyn_smem() { return HOT_SLOTS * 8 + HOT_SLOTS / 8 + (size_t)(FB / 32) * SCH * sizeof(Stage); }
 
 template <int NT, class AV, class XV, int SR> void *fused_fn() {
     return (void *)k_spmspv_fused<NT, AV, XV, SR>;
@@ -484,7 +851,9 @@ int expand_occupancy(int nt, int dtype) {
 int fused_occupancy(int nt, int dtype) {
     int bps = 0;
     void *f = pick_kernel(nt, dtype == TSMV_F32, TSMV_PLUS_TIMES);
-    cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, f, FB, 0);
+    const size_t dyn = fused_dyn_smem();
+    cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dyn);
+    cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, f, FB, dyn);
     if (e != cudaSuccess || bps < 1) {
         cudaGetLastError();
         bps = 0;
@@ -515,8 +884,8 @@ void ensure_lists(tsmv_ctx *c, int64_t k) {
     }
     if (L.cap_ct == 0) {
         // work items are bounded by the tile / side totals
-        int64_t nct = (c->P.T + CHUNK - 1) / CHUNK + 2;
-        int64_t ncs = (c->P.side_nnz + CHUNK - 1) / CHUNK + 2;
+        int64_t nct = (c->P.T + SCH - 1) / SCH + 2;
+        int64_t ncs = (c->P.side_nnz + SCH - 1) / SCH + 2;
         L.Ct.alloc(nct * 4);
         L.Cs.alloc(ncs * 4);
         L.cap_ct = nct;
@@ -560,9 +929,14 @@ void enqueue_spmspv(tsmv_ctx *c, int sr, long long k, const int32_t *xi, const v
     a.bar_base = c->bar_base;
     a.tring = c->timing ? c->tring.as<unsigned long long>() : nullptr;
     a.tslot = c->tcalls;
+    a.hot_list = c->P.hot_list;
+    a.n_hot = c->P.hot_list ? c->n_hot : 0;
+    a.trace = (unsigned long long *)c->trace;
     void *args[] = {&a};
     void *f = pick_kernel(c->nt, f32, sr);
-    TSMV_CUDA(cudaLaunchCooperativeKernel(f, dim3(c->fused_blocks), dim3(FB), args, 0, st));
+    const size_t dyn = fused_dyn_smem();
+    TSMV_CUDA(cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dyn));
+    TSMV_CUDA(cudaLaunchCooperativeKernel(f, dim3(c->fused_blocks), dim3(FB), args, dyn, st));
     c->bar_base += 4ull * (unsigned long long)c->fused_blocks;
     if (c->timing) c->tcalls++;
 }
@@ -676,6 +1050,16 @@ extern "C" tsmv_status tsmv_spmspv_async(tsmv_ctx *c, tsmv_semiring sr, int64_t 
     } catch (const Err &e) {
         return e.st;
     }
+}
+
+extern "C" int64_t tsmv_trace_words(const tsmv_ctx *c) {
+    return c ? (int64_t)c->fused_blocks * (FB / 32) * 8 : 0;
+}
+
+extern "C" tsmv_status tsmv_set_trace(tsmv_ctx *c, void *device_buffer) {
+    if (!c) return TSMV_EINVAL;
+    c->trace = device_buffer;
+    return TSMV_OK;
 }
 
 extern "C" tsmv_status tsmv_set_timing(tsmv_ctx *c, int32_t enable) {

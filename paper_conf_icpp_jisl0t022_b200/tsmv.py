@@ -17,7 +17,7 @@ from typing import Optional
 import torch
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libtsmv.so")
+LIB_PATH = os.environ.get("TSMV_LIB") or os.path.join(_HERE, "libtsmv.so")
 
 if not os.path.exists(LIB_PATH):
     raise ImportError(f"libtsmv.so not built ({LIB_PATH}); run `python -c 'import __graft_entry__ as g; g.build()'`")
@@ -71,6 +71,8 @@ _SIGS = {
     "tsmv_spmspv": (ctypes.c_int, [_vp, ctypes.c_int, _i64, _vp, _vp, _i64, _vp, _vp, ctypes.POINTER(_i64), _vp]),
     "tsmv_spmspv_async": (ctypes.c_int, [_vp, ctypes.c_int, _i64, _vp, _vp, _i64, _vp, _vp, _vp, _vp]),
     "tsmv_set_timing": (ctypes.c_int, [_vp, _i32]),
+    "tsmv_set_trace": (ctypes.c_int, [_vp, _vp]),
+    "tsmv_trace_words": (_i64, [_vp]),
     "tsmv_get_timing": (ctypes.c_int, [_vp, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(_i64)]),
     "tsmv_last_call_stats": (ctypes.c_int, [_vp, ctypes.POINTER(tsmv_call_stats)]),
     "tsmv_bfs": (ctypes.c_int, [_vp, _i64, _vp, ctypes.POINTER(tsmv_bfs_stats), _vp]),

@@ -82,6 +82,12 @@ struct FusedArgs {
     unsigned long long *trace;  // tsmv_set_trace: per warp {t_B0, t_loop_end, chunks, tile ns, side ns, max chunk ns, t_arrive, macs}
 };
 
+#ifdef TSMV_EXPERIMENT_NO_ROWBITS
+#define TOUCH(p, b) ((void)0)  // timing experiment only: y comes out empty
+#else
+#define TOUCH(p, b) atomicOr((p), (b))
+#endif
+
 // Shared-memory accumulation of the privatised ("hot") rows.
 template <int SR>
 __device__ __forceinline__ void accumulate_shared(double *s_acc, long long slot, double a, double x) {
@@ -113,17 +119,26 @@ __device__ __forceinline__ void block_scan(const long long *v, long long *ex, lo
         if (lane == 31) s[i][wid] = x;
     }
     __syncthreads();
+    if (wid == 0) {  // scan the NW warp totals with one warp, in place (exclusive) + total in slot NW-1's place
+#pragma unroll
+        for (int i = 0; i < K; ++i) {
+            const long long w0 = lane < NW ? s[i][lane] : 0;
+            long long x = w0;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const long long y = __shfl_up_sync(0xffffffffu, x, o);
+                if (lane >= o) x += y;
+            }
+            const long long all = __shfl_sync(0xffffffffu, x, 31);
+            if (lane < NW) s[i][lane] = x - w0;
+            if (lane == 0) s[i + K][0] = all;
+        }
+    }
+    __syncthreads();
 #pragma unroll
     for (int i = 0; i < K; ++i) {
-        long long before = 0, all = 0;
-#pragma unroll
-        for (int w = 0; w < NW; ++w) {
-            const long long t = s[i][w];
-            before += w < wid ? t : 0;
-            all += t;
-        }
-        ex[i] += before;
-        tot[i] = all;
+        ex[i] += s[i][wid];
+        tot[i] = s[i + K][0];
     }
     __syncthreads();
 }
@@ -306,7 +321,7 @@ __global__ void __launch_bounds__(FB, 1) k_spmspv_fused(FusedArgs a) {
     constexpr int LOG = Tr<NT>::LOG;
     constexpr int U = SCH / 32;
     constexpr int NW = FB / 32;
-    __shared__ long long s_scan[4][NW];  // block_scan scratch
+    __shared__ long long s_scan[8][NW];  // block_scan scratch (K prefixes + K totals)
     __shared__ long long win_all[NW][SCH + 1];
 
     __shared__ long long s_pre[4], s_tot[4];
@@ -316,6 +331,8 @@ __global__ void __launch_bounds__(FB, 1) k_spmspv_fused(FusedArgs a) {
     double *s_hacc = reinterpret_cast<double *>(s_dyn);                   // [HOT_SLOTS]
     uint32_t *s_hbits = reinterpret_cast<uint32_t *>(s_dyn + HOT_SLOTS * 8);  // [HOT_SLOTS/32]
     Stage *stage_all = reinterpret_cast<Stage *>(s_dyn + HOT_SLOTS * 8 + HOT_SLOTS / 8);  // [NW][SCH]
+    long long *win_b = reinterpret_cast<long long *>(stage_all + NW * SCH);                // [NW][SCH+1]
+    double *win_x = reinterpret_cast<double *>(win_b + NW * (SCH + 1));                    // [NW][SCH+1]
     const int n_slots = a.n_hot * NT;
     const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
     const int G = gridDim.x, b = blockIdx.x;
@@ -589,7 +606,7 @@ __global__ void __launch_bounds__(FB, 1) k_spmspv_fused(FusedArgs a) {
                         // so the remaining RED.ORs are spread over many words -> no test load
 #pragma unroll
                         for (int r = 0; r < R; ++r)
-                            if (okq[r] && !hot[r]) atomicOr(&a.rowbits[row[r] >> 5], 1u << (row[r] & 31));
+                            if (okq[r] && !hot[r]) TOUCH(&a.rowbits[row[r] >> 5], 1u << (row[r] & 31));
 #ifdef TSMV_TRACE_ROUNDS
                         __syncwarp();
                         const unsigned long long rt3 = globaltimer_ns();
@@ -604,24 +621,35 @@ __global__ void __launch_bounds__(FB, 1) k_spmspv_fused(FusedArgs a) {
                 const long long c2 = (long long)ch - nCt;
                 const long long s0 = __ldcg(&a.Lv.Cs[c2]);
                 const long long base = c2 << SCL;
-                load_window<SCL>(win, a.Lv.Ls_wpre, s0, nLs, lane);
-                long long p[U], sidx[U];
+                // window of the side list with its payload (column start, x_j) in shared
+                // memory: one coalesced load phase instead of a dependent hop per item
+                long long *winb = win_b + wid * (SCH + 1);
+                double *winx = win_x + wid * (SCH + 1);
+#pragma unroll
+                for (int q0 = 0; q0 <= SCH; q0 += 32) {
+                    const int q = q0 + lane;
+                    const long long ix = s0 + q;
+                    const bool in = ix <= nLs;
+                    const long long w = in ? __ldcg(&a.Lv.Ls_wpre[ix]) : 0x7fffffffffffffffLL;
+                    const long long bg = (in && ix < nLs) ? __ldcg(&a.Lv.Ls_beg[ix]) : 0;
+                    const double xx = (in && ix < nLs) ? __ldcg(&a.Lv.Ls_x[ix]) : 0.0;
+                    if (q <= SCH) {
+                        win[q] = w;
+                        winb[q] = bg;
+                        winx[q] = xx;
+                    }
+                }
+                __syncwarp();
+                long long p[U];
+                double xv[U];
                 bool ok[U];
 #pragma unroll
                 for (int u = 0; u < U; ++u) {
                     const long long i = base + lane + 32 * u;
                     ok[u] = i < Ws;
                     const int qq = ok[u] ? window_find<SCL>(win, i) : 0;
-                    sidx[u] = s0 + qq;
-                    p[u] = i - win[qq];
-                }
-                double xv[U];
-#pragma unroll
-                for (int u = 0; u < U; ++u) {
-                    if (ok[u]) {
-                        p[u] += __ldcg(&a.Lv.Ls_beg[sidx[u]]);
-                        xv[u] = __ldcg(&a.Lv.Ls_x[sidx[u]]);
-                    }
+                    p[u] = winb[qq] + (i - win[qq]);
+                    xv[u] = winx[qq];
                 }
                 long long row[U];
                 double av[U];
@@ -646,7 +674,7 @@ __global__ void __launch_bounds__(FB, 1) k_spmspv_fused(FusedArgs a) {
                     if (ok[u]) accumulate_value<SR>(a.acc, row[u], av[u], xv[u]);
 #pragma unroll
                 for (int u = 0; u < U; ++u)
-                    if (ok[u]) atomicOr(&a.rowbits[row[u] >> 5], 1u << (row[u] & 31));
+                    if (ok[u]) TOUCH(&a.rowbits[row[u] >> 5], 1u << (row[u] & 31));
             } else {
                 break;
             }
@@ -815,7 +843,9 @@ __global__ void __launch_bounds__(FB, 1) k_spmspv_fused(FusedArgs a) {
 // Phase-A totals / accounting for tsmv_last_call_stats are summed on the host
 // from `partials` and `acct`.
 
-size_t fused_dyn_smem() { return HOT_SLOTS * 8 + HOT_SLOTS / 8 + (size_t)(FB / 32) * SCH * sizeof(Stage); }
+size_t fused_dyn_smem() {
+    return HOT_SLOTS * 8 + HOT_SLOTS / 8 + (size_t)(FB / 32) * SCH * sizeof(Stage) + (size_t)(FB / 32) * (SCH + 1) * 16;
+}
 
 template <int NT, class AV, class XV, int SR> void *fused_fn() {
     return (void *)k_spmspv_fused<NT, AV, XV, SR>;

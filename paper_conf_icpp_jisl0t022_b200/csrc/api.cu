@@ -67,7 +67,7 @@ static void destroy_impl(tsmv_ctx *c) {
     c->Qown.release();
     for (DevBuf *b : {&c->outdeg, &c->indeg, &c->acc, &c->rowbits, &c->desc_compact, &c->counters, &c->stage_x_idx,
                       &c->stage_x_val, &c->stage_y_idx, &c->stage_y_val, &c->stage_levels, &c->V, &c->F0, &c->F1,
-                      &c->desc_bfs, &c->splits_dev, &c->xdense, &c->acct, &c->tring, &c->partials, &c->hot_list})
+                      &c->desc_bfs, &c->splits_dev, &c->xdense, &c->acct, &c->tring, &c->partials, &c->hot_list, &c->bfs_dirs, &c->bfs_front})
         b->release();
     c->L.release();
     if (c->hcnt) cudaFreeHost(c->hcnt);
@@ -228,7 +228,14 @@ extern "C" tsmv_status tsmv_create(tsmv_ctx **out, int64_t nrows, int64_t ncols,
         int fo = fused_occupancy(c->nt, (int)dtype);
         TSMV_REQUIRE(fo >= 1, "tsmv_create: fused SpMSpV kernel cannot be resident (occupancy 0)");
         c->fused_blocks = c->sm_count * std::min(fo, 4);
-        c->partials.alloc((size_t)c->fused_blocks * 8 * 8);
+        if (want_bfs && o.nranks == 1) {
+            int bo = bfs_fused_occupancy(c->nt);
+            TSMV_REQUIRE(bo >= 1, "tsmv_create: fused BFS kernel cannot be resident (occupancy 0)");
+            c->bfs_blocks = c->sm_count * std::min(bo, 2);
+            c->bfs_dirs.alloc(TSMV_MAX_LEVELS * 4);
+            c->bfs_front.alloc(TSMV_MAX_LEVELS * 8);
+        }
+        c->partials.alloc((size_t)std::max(c->fused_blocks, c->bfs_blocks) * 8 * 8);
         TSMV_CUDA(cudaMemsetAsync(c->partials.p, 0, c->partials.bytes, st));
         c->acct.alloc((size_t)std::max(c->expand_blocks, c->fused_blocks) * 4 * 8);
         TSMV_CUDA(cudaMemsetAsync(c->acct.p, 0, c->acct.bytes, st));

@@ -18,7 +18,7 @@
 //              sum indeg (one look-back pass over the n/nt segments); clears F.
 // Reading R10: pull tests the frontier of the level (not the live visited
 // set), so in-level discoveries cannot shorten levels.
-#include "device.cuh"
+#include "bfs_dev.cuh"
 
 namespace tsmv {
 
@@ -35,29 +35,6 @@ struct OctSum {
         return r;
     }
 };
-
-struct BfsView {
-    uint32_t *V, *F, *Fn;
-    int32_t *levels;
-    long long row_begin, m_local, n;
-    int level;  // level of F; discoveries get level + 1
-};
-
-template <int NT>
-__device__ __forceinline__ void discover(const BfsView &B, long long gseg, typename Tr<NT>::word_t bits) {
-    using word_t = typename Tr<NT>::word_t;
-    word_t old = seg_or<NT>(B.V, gseg, bits);
-    word_t nw = bits & ~old;
-    if (nw) {
-        seg_or<NT>(B.Fn, gseg, nw);
-        long long base = gseg * NT - B.row_begin;
-        while (nw) {
-            int r = ffs_w(nw);
-            nw &= nw - 1;
-            B.levels[base + r] = B.level + 1;
-        }
-    }
-}
 
 __global__ void k_bfs_init(BfsView B, long long NW, long long source) {
     long long tid = blockIdx.x * (long long)blockDim.x + threadIdx.x;
@@ -197,44 +174,15 @@ k_fscan(const uint32_t *__restrict__ F, uint32_t *__restrict__ Fclear, long long
     }
 }
 
-struct BfsTiles {
-    const long long *ptr;
-    const int *trow, *tgrp;
-    const void *mask;
-    const void *planes;
-    long long T;
-    const long long *sptr;
-    const int *srow;
-    const int32_t *hot_list;  // side rows of hot tile rows are encoded (TileSet::hot_list)
-};
-
-inline BfsTiles bfs_tiles(const TileSet &S) {
-    BfsTiles b;
-    b.ptr = S.ptr.as<long long>();
-    b.trow = S.trow.as<int>();
-    b.tgrp = S.tgrp.as<int>();
-    b.mask = S.mask.p;
-    b.planes = S.planes.p;
-    b.T = S.T;
-    b.sptr = S.sptr.as<long long>();
-    b.srow = S.srow.as<int>();
-    b.hot_list = S.hot_list;
-    return b;
-}
-
 // Push (vector-driven): tile chunks (Push-CSC, Alg 5) and side chunks.
 template <int NT, bool DO_TILES>
 __global__ void __launch_bounds__(256)
 k_push(BfsTiles P, ListsView Lv, Counters *__restrict__ cnt, BfsView B) {
-    using word_t = typename Tr<NT>::word_t;
     __shared__ long long win_all[8][CHUNK + 1];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     long long *win = win_all[wid];
     const long long nCt = DO_TILES ? cnt->nCt : 0, nCs = cnt->nCs;
     const long long nLt = cnt->nLt, nLs = cnt->nLs, Wt = cnt->Wt, Ws = cnt->Ws;
-    const word_t *mask = (const word_t *)P.mask;
-    const word_t *planes = (const word_t *)P.planes;
-    const long long rb_seg = B.row_begin / NT;
     while (true) {
         unsigned ch = 0;
         if (lane == 0) ch = atomicAdd(&cnt->chunk_next, 1u);
@@ -249,17 +197,7 @@ k_push(BfsTiles P, ListsView Lv, Counters *__restrict__ cnt, BfsView B) {
                 if (i >= Wt) break;
                 int q = window_find(win, i);
                 long long s = s0 + q;
-                long long t = Lv.Lt_tbeg[s] + (i - win[q]);
-                word_t hit = mask[t] & (word_t)Lv.Lt_mask[s];
-                if (hit) {
-                    word_t w = 0;
-                    while (hit) {
-                        int c = ffs_w(hit);
-                        hit &= hit - 1;
-                        w |= planes[(long long)c * P.T + t];
-                    }
-                    discover<NT>(B, rb_seg + P.trow[t], w);
-                }
+                push_tile_item<NT>(P, B, Lv.Lt_tbeg[s] + (i - win[q]), (typename Tr<NT>::word_t)Lv.Lt_mask[s]);
             }
             __syncwarp();
         } else if (ch < nCt + nCs) {
@@ -272,10 +210,7 @@ k_push(BfsTiles P, ListsView Lv, Counters *__restrict__ cnt, BfsView B) {
                 long long i = base + lane + 32 * u;
                 if (i >= Ws) break;
                 int q = window_find(win, i);
-                long long s = s0 + q;
-                long long p = Lv.Ls_beg[s] + (i - win[q]);
-                long long v = B.row_begin + decode_row<NT>(P.srow[p], P.hot_list);
-                discover<NT>(B, v / NT, (word_t)1 << (v % NT));
+                push_side_item<NT>(P, B, Lv.Ls_beg[s0 + q] + (i - win[q]));
             }
             __syncwarp();
         } else {
@@ -284,87 +219,26 @@ k_push(BfsTiles P, ListsView Lv, Counters *__restrict__ cnt, BfsView B) {
     }
 }
 
-// Push-CSR (Alg 6): every tile of the row-tile structure Q; x word of its tile
-// column, row words of the still-unvisited rows.
 template <int NT>
 __global__ void __launch_bounds__(256) k_push_csr(BfsTiles Q, BfsView B) {
-    using word_t = typename Tr<NT>::word_t;
-    const word_t *planes = (const word_t *)Q.planes;
-    const long long rb_seg = B.row_begin / NT;
     for (long long t = blockIdx.x * (long long)blockDim.x + threadIdx.x; t < Q.T;
-         t += (long long)gridDim.x * blockDim.x) {
-        long long Jx = Q.trow[t];            // A's tile column (segment of x)
-        word_t f = seg_bits<NT>(B.F, Jx);
-        if (!f) continue;
-        long long Iseg = rb_seg + Q.tgrp[t]; // A's tile row (global segment)
-        word_t um = ~seg_bits<NT>(B.V, Iseg);
-        if (!um) continue;
-        word_t res = 0;
-        while (um) {
-            int r = ffs_w(um);
-            um &= um - 1;
-            if (planes[(long long)r * Q.T + t] & f) res |= (word_t)1 << r;
-        }
-        if (res) discover<NT>(B, Iseg, res);
-    }
+         t += (long long)gridDim.x * blockDim.x)
+        push_csr_item<NT>(Q, B, t);
 }
 
-// Pull-CSC (Alg 7): one warp per local row tile with unvisited rows; lanes walk
-// the tiles of the row tile; stop when every unvisited row has found a parent.
 template <int NT>
 __global__ void __launch_bounds__(256) k_pull(BfsTiles Q, BfsView B, long long nTR_local) {
-    using word_t = typename Tr<NT>::word_t;
-    const word_t *planes = (const word_t *)Q.planes;
     const int lane = threadIdx.x & 31;
     const long long warp = (blockIdx.x * (long long)blockDim.x + threadIdx.x) >> 5;
     const long long nwarps = ((long long)gridDim.x * blockDim.x) >> 5;
-    const long long rb_seg = B.row_begin / NT;
-    for (long long I = warp; I < nTR_local; I += nwarps) {
-        word_t um = ~seg_bits<NT>(B.V, rb_seg + I);
-        if (!um) continue;
-        word_t found = 0;
-        const long long t0 = Q.ptr[I], t1 = Q.ptr[I + 1];
-        for (long long tb = t0; tb < t1; tb += 32) {
-            long long t = tb + lane;
-            word_t fl = 0;
-            if (t < t1) {
-                word_t f = seg_bits<NT>(B.F, Q.trow[t]);
-                if (f) {
-                    word_t u = um;
-                    while (u) {
-                        int r = ffs_w(u);
-                        u &= u - 1;
-                        if (planes[(long long)r * Q.T + t] & f) fl |= (word_t)1 << r;
-                    }
-                }
-            }
-            fl = warp_or(fl);
-            found |= fl;
-            um &= ~fl;
-            if (!um) break;
-        }
-        if (lane == 0 && found) discover<NT>(B, rb_seg + I, found);
-    }
+    for (long long I = warp; I < nTR_local; I += nwarps) pull_rowtile<NT>(Q, B, I, lane);
 }
 
-// Pull over the side matrix: CSC of A^T's side part = in-neighbour lists.
 template <int NT>
 __global__ void __launch_bounds__(256) k_pull_side(BfsTiles Q, BfsView B) {
-    using word_t = typename Tr<NT>::word_t;
     for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < B.m_local;
-         v += (long long)gridDim.x * blockDim.x) {
-        long long p0 = Q.sptr[v], p1 = Q.sptr[v + 1];
-        if (p0 == p1) continue;
-        long long g = B.row_begin + v;
-        if ((B.V[g >> 5] >> (g & 31)) & 1u) continue;
-        for (long long p = p0; p < p1; ++p) {
-            long long u = decode_row<NT>(Q.srow[p], Q.hot_list);
-            if ((B.F[u >> 5] >> (u & 31)) & 1u) {
-                discover<NT>(B, g / NT, (word_t)1 << (g % NT));
-                break;
-            }
-        }
-    }
+         v += (long long)gridDim.x * blockDim.x)
+        pull_side_vertex<NT>(Q, B, v);
 }
 
 __global__ void k_merge(const uint32_t *__restrict__ gathered, long long stride, int nranks,
@@ -499,6 +373,77 @@ extern "C" tsmv_status tsmv_bfs(tsmv_ctx *c, int64_t source, int32_t *levels, ts
         bool host_levels;
         bfs_prepare_levels(c, levels, host_levels);
         ensure_lists(c, c->n);
+        if (!getenv("TSMV_BFS_HOSTLOOP")) {
+            // Hybrid: push levels run inside the fused persistent kernel
+            // (no host round trip per level); a Pull-CSC level hands back to the host,
+            // which runs it with the high-occupancy per-level kernels, then resumes.
+            const bool stop_on_pull = !getenv("TSMV_BFS_FUSED_ONLY");
+            TSMV_CUDA(cudaEventRecord(c->ev0, st));
+            uint32_t *Fa = c->F0.as<uint32_t>(), *Fb = c->F1.as<uint32_t>();
+            long long level = 0, mu = c->nnz, reached = 0, edges = 0;
+            bool resume = false;
+            BfsRunner R{c, st, (long long)(c->V.bytes / 4)};
+            std::vector<int> hdir;
+            std::vector<long long> hfront;
+            while (true) {
+                long long L, mu2, r2, e2;
+                int cur;
+                const bool stopped = bfs_fused_launch(c, source, st, resume, level, Fa, Fb, mu, reached, edges,
+                                                      stop_on_pull, TSMV_MAX_LEVELS, L, mu2, r2, e2, cur);
+                if (cur) std::swap(Fa, Fb);  // Fa = bitmap of the current frontier
+                level = L;
+                mu = mu2;
+                reached = r2;
+                edges = e2;
+                if (!stopped) break;
+                // pull levels on the host path until the rule turns back to push
+                while (true) {
+                    c->bfs_level = (int)level;
+                    c->fcur = (Fa == c->F0.as<uint32_t>()) ? 0 : 1;
+                    R.do_expand(TSMV_DIR_PULL_CSC);
+                    R.do_fscan(Fb, Fa);  // next frontier lists + stats; clears Fa
+                    TSMV_CUDA(cudaStreamSynchronize(st));
+                    volatile Counters *h = c->hcnt;
+                    const long long fsize = h->fsize, mf = h->mf, din = h->din;
+                    std::swap(Fa, Fb);
+                    ++level;
+                    if (fsize == 0 || level >= TSMV_MAX_LEVELS) break;
+                    const int dir = choose_dir(c->opt, c->n, fsize, mf, mu - din);
+                    if (dir != TSMV_DIR_PULL_CSC) break;  // resume the fused kernel at `level`
+                    mu -= din;
+                    reached += fsize;
+                    edges += mf;
+                    hdir.resize(level + 1, 0);
+                    hfront.resize(level + 1, 0);
+                    hdir[level] = dir;
+                    hfront[level] = fsize;
+                    int dd = dir;
+                    long long ff = fsize;
+                    TSMV_CUDA(cudaMemcpy(c->bfs_dirs.as<int>() + level, &dd, 4, cudaMemcpyHostToDevice));
+                    TSMV_CUDA(cudaMemcpy(c->bfs_front.as<long long>() + level, &ff, 8, cudaMemcpyHostToDevice));
+                }
+                if (c->hcnt->fsize == 0 || level >= TSMV_MAX_LEVELS) break;
+                resume = true;
+            }
+            TSMV_CUDA(cudaEventRecord(c->ev1, st));
+            if (host_levels) TSMV_CUDA(cudaMemcpyAsync(levels, c->levels_dev, c->m * 4, cudaMemcpyDeviceToHost, st));
+            TSMV_CUDA(cudaStreamSynchronize(st));
+            c->bfs_last_levels = level;
+            if (stats) {
+                float ms = 0;
+                TSMV_CUDA(cudaEventElapsedTime(&ms, c->ev0, c->ev1));
+                const long long nl = std::min<long long>(level, TSMV_MAX_LEVELS);
+                if (nl > 0) {
+                    TSMV_CUDA(cudaMemcpy(stats->dir_per_level, c->bfs_dirs.p, nl * 4, cudaMemcpyDeviceToHost));
+                    TSMV_CUDA(cudaMemcpy(stats->frontier_per_level, c->bfs_front.p, nl * 8, cudaMemcpyDeviceToHost));
+                }
+                stats->nlevels = (int32_t)nl;
+                stats->reached = reached;
+                stats->edges_traversed = edges;
+                stats->ms = ms;
+            }
+            return TSMV_OK;
+        }
         BfsRunner R{c, st, (long long)(c->V.bytes / 4)};
         c->fcur = 0;
         c->bfs_level = 0;

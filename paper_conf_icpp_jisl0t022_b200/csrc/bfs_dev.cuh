@@ -1,0 +1,166 @@
+// bfs_dev.cuh -- device-side pieces of one TileBFS level shared by the
+// per-level kernels (bfs.cu, used by the distributed driver) and the fused
+// persistent single-GPU kernel (bfs_fused.cu).
+#pragma once
+#include "device.cuh"
+
+namespace tsmv {
+
+struct BfsView {
+    uint32_t *V, *F, *Fn;
+    int32_t *levels;
+    long long row_begin, m_local, n;
+    int level;  // level of F; discoveries get level + 1
+};
+
+template <int NT>
+__device__ __forceinline__ void discover(const BfsView &B, long long gseg, typename Tr<NT>::word_t bits) {
+    using word_t = typename Tr<NT>::word_t;
+    word_t old = seg_or<NT>(B.V, gseg, bits);
+    word_t nw = bits & ~old;
+    if (nw) {
+        seg_or<NT>(B.Fn, gseg, nw);
+        long long base = gseg * NT - B.row_begin;
+        while (nw) {
+            int r = ffs_w(nw);
+            nw &= nw - 1;
+            B.levels[base + r] = B.level + 1;
+        }
+    }
+}
+
+struct BfsTiles {
+    const long long *ptr;
+    const int *trow, *tgrp;
+    const void *mask;
+    const void *planes;
+    long long T;
+    const long long *sptr;
+    const int *srow;
+    const int32_t *hot_list;  // side rows of hot tile rows are encoded (TileSet::hot_list)
+};
+
+inline BfsTiles bfs_tiles(const TileSet &S) {
+    BfsTiles b;
+    b.ptr = S.ptr.as<long long>();
+    b.trow = S.trow.as<int>();
+    b.tgrp = S.tgrp.as<int>();
+    b.mask = S.mask.p;
+    b.planes = S.planes.p;
+    b.T = S.T;
+    b.sptr = S.sptr.as<long long>();
+    b.srow = S.srow.as<int>();
+    b.hot_list = S.hot_list;
+    return b;
+}
+
+
+// ---- one item of each level kernel -------------------------------------------
+
+// Push-CSC tile item (Alg 5): OR the bit planes of the frontier's columns of tile t.
+template <int NT>
+__device__ __forceinline__ void push_tile_item(const BfsTiles &P, const BfsView &B, long long t,
+                                               typename Tr<NT>::word_t xm) {
+    using word_t = typename Tr<NT>::word_t;
+    word_t hit = ((const word_t *)P.mask)[t] & xm;
+    if (hit) {
+        const word_t *planes = (const word_t *)P.planes;
+        word_t w = 0;
+        while (hit) {
+            int c = ffs_w(hit);
+            hit &= hit - 1;
+            w |= planes[(long long)c * P.T + t];
+        }
+        discover<NT>(B, B.row_begin / NT + P.trow[t], w);
+    }
+}
+
+// Push over the side matrix: one side nonzero p of a frontier vertex's column.
+template <int NT>
+__device__ __forceinline__ void push_side_item(const BfsTiles &P, const BfsView &B, long long p) {
+    using word_t = typename Tr<NT>::word_t;
+    long long v = B.row_begin + decode_row<NT>(P.srow[p], P.hot_list);
+    discover<NT>(B, v / NT, (word_t)1 << (v % NT));
+}
+
+// Push-CSR (Alg 6) tile item: tile t of the row structure Q; x word of its tile
+// column, row words of the still-unvisited rows.
+template <int NT>
+__device__ __forceinline__ void push_csr_item(const BfsTiles &Q, const BfsView &B, long long t) {
+    using word_t = typename Tr<NT>::word_t;
+    const word_t *planes = (const word_t *)Q.planes;
+    long long Jx = Q.trow[t];  // A's tile column (segment of x)
+    word_t f = seg_bits<NT>(B.F, Jx);
+    if (!f) return;
+    long long Iseg = B.row_begin / NT + Q.tgrp[t];  // A's tile row (global segment)
+    word_t um = ~seg_bits<NT>(B.V, Iseg);
+    if (!um) return;
+    word_t res = 0;
+    while (um) {
+        int r = ffs_w(um);
+        um &= um - 1;
+        if (planes[(long long)r * Q.T + t] & f) res |= (word_t)1 << r;
+    }
+    if (res) discover<NT>(B, Iseg, res);
+}
+
+// Pull-CSC (Alg 7), one warp on local row tile I: lanes walk the tiles of the
+// row tile; stop when every unvisited row has found a parent in the frontier.
+template <int NT>
+__device__ __forceinline__ void pull_rowtile(const BfsTiles &Q, const BfsView &B, long long I, int lane) {
+    using word_t = typename Tr<NT>::word_t;
+    const word_t *planes = (const word_t *)Q.planes;
+    const long long rb_seg = B.row_begin / NT;
+    word_t um = ~seg_bits<NT>(B.V, rb_seg + I);
+    if (!um) return;
+    word_t found = 0;
+    const long long t0 = Q.ptr[I], t1 = Q.ptr[I + 1];
+    for (long long tb = t0; tb < t1; tb += 32) {
+        long long t = tb + lane;
+        word_t fl = 0;
+        if (t < t1) {
+            word_t f = seg_bits<NT>(B.F, Q.trow[t]);
+            if (f) {
+                word_t u = um;
+                while (u) {
+                    int r = ffs_w(u);
+                    u &= u - 1;
+                    if (planes[(long long)r * Q.T + t] & f) fl |= (word_t)1 << r;
+                }
+            }
+        }
+        fl = warp_or(fl);
+        found |= fl;
+        um &= ~fl;
+        if (!um) break;
+    }
+    if (lane == 0 && found) discover<NT>(B, rb_seg + I, found);
+}
+
+// Pull over the side matrix: in-neighbour list of local vertex v (CSC of A^T's side).
+template <int NT>
+__device__ __forceinline__ void pull_side_vertex(const BfsTiles &Q, const BfsView &B, long long v) {
+    using word_t = typename Tr<NT>::word_t;
+    long long p0 = Q.sptr[v], p1 = Q.sptr[v + 1];
+    if (p0 == p1) return;
+    long long g = B.row_begin + v;
+    if ((B.V[g >> 5] >> (g & 31)) & 1u) return;
+    for (long long p = p0; p < p1; ++p) {
+        long long u = decode_row<NT>(Q.srow[p], Q.hot_list);
+        if ((B.F[u >> 5] >> (u & 31)) & 1u) {
+            discover<NT>(B, g / NT, (word_t)1 << (g % NT));
+            break;
+        }
+    }
+}
+
+// Device copy of the direction rule (reading R9); host: tsmv::choose_dir.
+__device__ __forceinline__ int choose_dir_dev(int force, double alpha, double dens, long long n, long long f,
+                                              long long mf, long long mu) {
+    if (force) return force;
+    if ((double)mf > (double)mu / alpha) return TSMV_DIR_PULL_CSC;
+    if ((double)f / (double)n >= dens) return TSMV_DIR_PUSH_CSR;
+    return TSMV_DIR_PUSH_CSC;
+}
+
+}  // namespace tsmv

@@ -229,6 +229,9 @@ struct tsmv_ctx {
     int fused_blocks = 0, fused_threads = 1024;
     tsmv::DevBuf partials;         // long long[fused_blocks][8]
     long long last_x_nnz = 0;
+    int bfs_blocks = 0;            // CTAs of the fused BFS kernel
+    long long bfs_last_levels = 0;
+    tsmv::DevBuf bfs_dirs, bfs_front;  // per-level direction / frontier size (device)
     void *trace = nullptr;         // tsmv_set_trace (device, u64[tsmv_trace_words])
 };
 
@@ -249,6 +252,12 @@ bool same_pattern_transposed(tsmv_ctx *c, const int32_t *rows, const int32_t *co
 void prepare_csr(tsmv_ctx *c, const int64_t *row_ptr, const int32_t *col_idx, int32_t *rows, cudaStream_t st);
 // spmspv.cu
 void ensure_lists(tsmv_ctx *c, int64_t k);
+// bfs_fused.cu
+int bfs_fused_occupancy(int nt);
+bool bfs_fused_launch(tsmv_ctx *c, long long source, cudaStream_t st, bool resume, long long level0, uint32_t *Fa,
+                      uint32_t *Fb, long long mu, long long reached, long long edges, bool stop_on_pull,
+                      long long max_levels, long long &level_out, long long &mu_out, long long &reached_out,
+                      long long &edges_out, int &cur_out);
 // bfs.cu
 int choose_dir(const tsmv_options &o, long long n, long long fsize, long long mf, long long mu);
 // pointer classification

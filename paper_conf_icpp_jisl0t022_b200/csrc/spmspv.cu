@@ -98,51 +98,6 @@ __device__ __forceinline__ void accumulate_shared(double *s_acc, long long slot,
     }
 }
 
-// Exclusive block-wide scan of K int64 values per thread (shuffles + one smem
-// pass); register-light replacement for cub::BlockScan of a 4-wide struct, which
-// made the fused kernel spill.  tot = block totals (all threads).  Contains
-// __syncthreads; every thread of the block must call it.
-template <int K, int NTHREADS>
-__device__ __forceinline__ void block_scan(const long long *v, long long *ex, long long *tot,
-                                           long long (*s)[NTHREADS / 32]) {
-    constexpr int NW = NTHREADS / 32;
-    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-#pragma unroll
-    for (int i = 0; i < K; ++i) {
-        long long x = v[i];
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            const long long y = __shfl_up_sync(0xffffffffu, x, o);
-            if (lane >= o) x += y;
-        }
-        ex[i] = x - v[i];
-        if (lane == 31) s[i][wid] = x;
-    }
-    __syncthreads();
-    if (wid == 0) {  // scan the NW warp totals with one warp, in place (exclusive) + total in slot NW-1's place
-#pragma unroll
-        for (int i = 0; i < K; ++i) {
-            const long long w0 = lane < NW ? s[i][lane] : 0;
-            long long x = w0;
-#pragma unroll
-            for (int o = 1; o < 32; o <<= 1) {
-                const long long y = __shfl_up_sync(0xffffffffu, x, o);
-                if (lane >= o) x += y;
-            }
-            const long long all = __shfl_sync(0xffffffffu, x, 31);
-            if (lane < NW) s[i][lane] = x - w0;
-            if (lane == 0) s[i + K][0] = all;
-        }
-    }
-    __syncthreads();
-#pragma unroll
-    for (int i = 0; i < K; ++i) {
-        ex[i] += s[i][wid];
-        tot[i] = s[i + K][0];
-    }
-    __syncthreads();
-}
-
 template <int SR>
 __device__ __forceinline__ void accumulate_value(double *acc, long long row, double a, double x) {
     if constexpr (SR == TSMV_PLUS_TIMES) {

@@ -54,6 +54,7 @@ def parse():
     p.add_argument("--no-bfs", action="store_true")
     p.add_argument("--no-cpu", action="store_true")
     p.add_argument("--cpu-seconds", type=float, default=12.0)
+    p.add_argument("--no-configs", action="store_true", help="skip the per-config table (C1, C2, C4)")
     return p.parse_args()
 
 
@@ -361,6 +362,10 @@ def run_tsmv(args):
     bfs = None
     if not args.no_bfs and world == 1:
         bfs = run_bfs(args, dev, flush, tsmv)
+    configs = None
+    if not args.no_configs and world == 1:
+        del M
+        configs = run_configs(args, dev, flush, tsmv)
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu:
@@ -378,7 +383,7 @@ def run_tsmv(args):
                              **{kk: round(v, 1) for kk, v in mean_st.items() if kk != "x_nnz"}},
                 "format": {kk: info[kk] for kk in ("nnz", "n_tiles", "n_dense_tiles", "dense_nnz", "side_nnz",
                                                    "build_ms", "bytes_spmspv")},
-                "bfs": bfs}
+                "bfs": bfs, "configs": configs}
         print(json.dumps(line), flush=True)
     if world > 1:
         torch.distributed.destroy_process_group()
@@ -410,6 +415,74 @@ def run_bfs(args, dev, flush, tsmv):
             "build_ms": round(info["build_ms"], 2), "build_wall_s": round(build_wall, 3),
             "edge_count": "sum of out-degrees of reached vertices (directed count of the symmetrised graph)",
             "runs": runs}
+
+
+def spmspv_gflops(M, A, dtype, density, flush, steps=5, warm=2):
+    """Device-timed SpMSpV at `density` on context M (fresh x per step, L2 flushed)."""
+    dev = A.row_ptr.device
+    colcnt = torch.bincount(A.col_idx.long(), minlength=A.n)
+    k = max(1, synth.density_k(A.n, density))
+    xs = x_samples(A.n, k, steps + warm, dtype, dev)
+    vt = torch.float32 if dtype == "f32" else torch.float64
+    yi = torch.empty(A.m, dtype=torch.int32, device=dev)
+    yv = torch.empty(A.m, dtype=vt, device=dev)
+    yn = torch.zeros(1, dtype=torch.int64, device=dev)
+    for s in range(warm):
+        M.spmspv_async(xs[s][0], xs[s][1], yi, yv, yn)
+    ms, flops = 0.0, 0
+    for s in range(warm, warm + steps):
+        flush()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        M.spmspv_async(xs[s][0], xs[s][1], yi, yv, yn)
+        e1.record()
+        torch.cuda.synchronize()
+        ms += e0.elapsed_time(e1)
+        flops += flops_of(colcnt, xs[s][0])
+    return {"density": density, "k": k, "us_per_call": round(1e3 * ms / steps, 2),
+            "gflops": round(flops / (ms * 1e-3) / 1e9, 3), "y_nnz": int(yn.item())}
+
+
+def bfs_gteps(M, A, flush, sources):
+    lv = torch.empty(A.n, dtype=torch.int32, device=A.row_ptr.device)
+    M.bfs(sources[0], levels=lv)
+    out = []
+    for s in sources:
+        flush()
+        torch.cuda.synchronize()
+        _, st = M.bfs(s, levels=lv)
+        out.append({"source": int(s), "ms": round(st["ms"], 3), "levels": st["nlevels"],
+                    "gteps": round(st["edges_traversed"] / (st["ms"] * 1e-3) / 1e9, 3)})
+    return out
+
+
+def run_configs(args, dev, flush, tsmv):
+    """The other BASELINE.json configs (C1, C2, C4), a few device-timed calls each."""
+    res = {}
+    # C1: 2D 5-point 64x64, fp64, x 1 %, BFS from 0
+    A = synth.stencil2d(64, 64, device=dev)
+    M = tsmv.TiledMatrix.from_csr(A)
+    res["C1_stencil2d_64x64"] = {"spmspv_f64": spmspv_gflops(M, A, "f64", 0.01, flush),
+                                 "bfs": bfs_gteps(M, A, flush, [0])}
+    M.close()
+    # C2: R-MAT s20 ef16 sweep, fp64 and fp32
+    base = synth.rmat(20, 16, seed=1, device=dev)
+    c2 = {}
+    for dt in ("f64", "f32"):
+        A = synth.attach_values(base, seed=1, dtype=dt)
+        M = tsmv.TiledMatrix.from_csr(A, dtype=dt, build_bfs=0)
+        c2[dt] = [spmspv_gflops(M, A, dt, d, flush) for d in (0.0001, 0.001, 0.01, 0.1)]
+        M.close()
+    res["C2_rmat_s20_sweep"] = c2
+    # C4: 3D 7-point 256^3 and banded (2^20, b = 64): TileBFS + SpMSpV at 1 %
+    for name, A in (("C4_stencil3d_256", synth.stencil3d(256, device=dev)),
+                    ("C4_banded_2e20_b64", synth.banded(1 << 20, 64, device=dev))):
+        M = tsmv.TiledMatrix.from_csr(A)
+        res[name] = {"nnz": A.nnz, "spmspv_f64": spmspv_gflops(M, A, "f64", 0.01, flush),
+                     "bfs": bfs_gteps(M, A, flush, [0])}
+        M.close()
+        del A
+    return res
 
 
 def cpu_baseline(args, A, colcnt, xs):

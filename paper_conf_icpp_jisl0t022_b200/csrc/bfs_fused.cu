@@ -104,6 +104,7 @@ __global__ void __launch_bounds__(BFB, 1) k_bfs_fused(BfsFusedArgs a) {
     const long long per = (S + BFB - 1) / BFB;
     const long long tj0 = min(js1, js0 + tid * per), tj1 = min(js1, tj0 + per);
     int level = (int)a.level0;
+    unsigned long long t_s1 = 0, t_s2 = 0, t_e = 0, tq = b == 0 && tid == 0 ? globaltimer_ns() : 0;
     for (; level < a.max_levels; ++level) {
         B.F = Fa;
         B.Fn = Fb;
@@ -126,6 +127,11 @@ __global__ void __launch_bounds__(BFB, 1) k_bfs_fused(BfsFusedArgs a) {
         if (tid < 8) a.partials[b * 8 + tid] = tot[tid];
         if (b == 0 && tid == 0) a.cnt->chunk_next = 0;
         grid_sync(&a.cnt->bar, target);
+        if (b == 0 && tid == 0) {
+            const unsigned long long t = globaltimer_ns();
+            t_s1 += t - tq;
+            tq = t;
+        }
         if (tid < 32) {
             long long pre[8] = {0, 0, 0, 0, 0, 0, 0, 0}, all[8] = {0, 0, 0, 0, 0, 0, 0, 0};
             for (int g = lane; g < G; g += 32) {
@@ -203,6 +209,11 @@ __global__ void __launch_bounds__(BFB, 1) k_bfs_fused(BfsFusedArgs a) {
             }
         }
         grid_sync(&a.cnt->bar, target);
+        if (b == 0 && tid == 0) {
+            const unsigned long long t = globaltimer_ns();
+            t_s2 += t - tq;
+            tq = t;
+        }
 
         // ---- E: expand
         if (dir == TSMV_DIR_PULL_CSC) {
@@ -254,6 +265,11 @@ __global__ void __launch_bounds__(BFB, 1) k_bfs_fused(BfsFusedArgs a) {
             }
         }
         grid_sync(&a.cnt->bar, target);
+        if (b == 0 && tid == 0) {
+            const unsigned long long t = globaltimer_ns();
+            t_e += t - tq;
+            tq = t;
+        }
         uint32_t *tmp = Fa;
         Fa = Fb;
         Fb = tmp;
@@ -265,6 +281,9 @@ __global__ void __launch_bounds__(BFB, 1) k_bfs_fused(BfsFusedArgs a) {
         a.hm->mf = mu;
         a.hm->din = stopped;
         a.hm->nLt = (Fa == a.B.F) ? 0 : 1;  // which bitmap holds the current frontier
+        a.hm->Wt = (long long)t_s1;  // phase times (ns, CTA 0): count, lists, expand
+        a.hm->nLs = (long long)t_s2;
+        a.hm->Ws = (long long)t_e;
     }
 }
 

@@ -289,6 +289,46 @@ __device__ __forceinline__ int window_find(const long long *win, long long i) {
     return lo;
 }
 
+// Item -> window-entry map of one chunk without a per-item binary search:
+// the entries starting strictly inside the chunk are marked in a (1<<LOGC)-bit
+// mask (warp OR-reduction, no shared memory); item j of the chunk then belongs
+// to window entry popc(mask & bits(0..j)).  Requires every window entry to own
+// at least one item (true for the work lists: entries with zero work are not
+// listed).  win = the chunk's window (load_window), base = first item.
+template <int LOGC>
+struct ChunkMap {
+    unsigned w[(1 << LOGC) / 32];
+    __device__ __forceinline__ void build(const long long *win, long long base, int lane) {
+        constexpr int CH = 1 << LOGC, NWD = CH / 32;
+        unsigned loc[NWD];
+#pragma unroll
+        for (int k = 0; k < NWD; ++k) loc[k] = 0u;
+#pragma unroll
+        for (int v = 0; v < NWD; ++v) {
+            const int q = 1 + lane + 32 * v;  // window entries 1..CH
+            const long long d = win[q] - base;
+            if (d > 0 && d < CH) {
+#pragma unroll
+                for (int k = 0; k < NWD; ++k)
+                    if ((int)(d >> 5) == k) loc[k] |= 1u << (d & 31);
+            }
+        }
+#pragma unroll
+        for (int k = 0; k < NWD; ++k) w[k] = __reduce_or_sync(0xffffffffu, loc[k]);
+    }
+    __device__ __forceinline__ int entry(int j) const {
+        constexpr int NWD = (1 << LOGC) / 32;
+        int cnt = 0;
+        const int wj = j >> 5;
+#pragma unroll
+        for (int k = 0; k < NWD; ++k) {
+            const unsigned m = k < wj ? 0xffffffffu : (k == wj ? ((j & 31) == 31 ? 0xffffffffu : ((2u << (j & 31)) - 1u)) : 0u);
+            cnt += __popc(w[k] & m);
+        }
+        return cnt;
+    }
+};
+
 // Segment bits of an NT-segment inside uint32 bitmap words.
 template <int NT> __device__ __forceinline__ typename Tr<NT>::word_t seg_bits(const uint32_t *bm, long long J) {
     if constexpr (NT == 16) {

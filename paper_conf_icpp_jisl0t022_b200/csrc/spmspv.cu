@@ -39,7 +39,7 @@ namespace {
 constexpr int FB = TSMV_FB;  // threads per CTA of the fused kernel
 constexpr int CB = TSMV_CB;  // accumulator loads batched per lane in phase C
 #ifndef TSMV_R
-#define TSMV_R 4
+#define TSMV_R 2
 #endif
 #ifndef TSMV_SCL
 #define TSMV_SCL 7
@@ -81,6 +81,20 @@ struct FusedArgs {
     int n_hot;
     unsigned long long *trace;  // tsmv_set_trace: per warp {t_B0, t_loop_end, chunks, tile ns, side ns, max chunk ns, t_arrive, macs}
 };
+
+#ifdef TSMV_TRACE_STEPS
+// development: stamp step k of the warp that processes tile chunk 0 (after a fake
+// use of `dep` so the stamp waits for the loads that produced it)
+#define STEP(k, dep)                                                                          \
+    do {                                                                                      \
+        if (a.trace && ch == 0 && lane == 0) {                                                \
+            if ((long long)(dep) == 0x5eed5eed5eedll) a.trace[1000] = 1;                     \
+            a.trace[200 + (k)] = globaltimer_ns();                                            \
+        }                                                                                     \
+    } while (0)
+#else
+#define STEP(k, dep) ((void)0)
+#endif
 
 #ifdef TSMV_EXPERIMENT_NO_ROWBITS
 #define TOUCH(p, b) ((void)0)  // timing experiment only: y comes out empty
@@ -423,19 +437,25 @@ __global__ void __launch_bounds__(FB, 1) k_spmspv_fused(FusedArgs a) {
             unsigned nx = 0;
             if (lane == 0 && ch < nCt + nCs) nx = nwarps + atomicAdd(&a.cnt->chunk_next, 1u);
             if (ch < nCt) {
+                STEP(0, 0);
                 const long long s0 = __ldcg(&a.Lv.Ct[ch]);
+                STEP(1, s0);
                 const long long base = (long long)ch << SCL;
                 load_window<SCL>(win, a.Lv.Lt_wpre, s0, nLt, lane);
+                STEP(2, win[0]);
                 long long sidx[U], t[U];
                 bool ok[U];
+                ChunkMap<SCL> cm;
+                cm.build(win, base, lane);
 #pragma unroll
                 for (int u = 0; u < U; ++u) {
                     const long long i = base + lane + 32 * u;
                     ok[u] = i < Wt;
-                    const int qq = ok[u] ? window_find<SCL>(win, i) : 0;
+                    const int qq = ok[u] ? cm.entry(lane + 32 * u) : 0;
                     sidx[u] = s0 + qq;
                     t[u] = i - win[qq];
                 }
+                STEP(3, sidx[0] + t[0]);
                 long long J[U];
                 word_t xm[U];
 #pragma unroll
@@ -446,6 +466,7 @@ __global__ void __launch_bounds__(FB, 1) k_spmspv_fused(FusedArgs a) {
                         J[u] = __ldcg(&a.Lv.Lt_seg[sidx[u]]);
                     }
                 }
+                STEP(4, t[0] + xm[0] + J[0]);
                 word_t hit[U];
 #pragma unroll
                 for (int u = 0; u < U; ++u) hit[u] = ok[u] ? (word_t)(mask[t[u]] & xm[u]) : (word_t)0;
@@ -455,21 +476,33 @@ __global__ void __launch_bounds__(FB, 1) k_spmspv_fused(FusedArgs a) {
                 // warp then walks that flat index space R positions per lane at a time,
                 // so a dense hub tile is spread over the warp and the loads of different
                 // positions are issued together.
+                STEP(5, hit[0] + hit[1]);
                 TileDesc d[U];
 #pragma unroll
                 for (int u = 0; u < U; ++u)
                     if (hit[u]) d[u] = ((const TileDesc *)a.desc)[t[u]];
+                STEP(6, d[0].off + d[1].off);
                 int useful[U];
                 int mine = 0;
+                uint4 csr[U];
+                if constexpr (NT == 16) {
+#pragma unroll
+                    for (int u = 0; u < U; ++u)
+                        if (hit[u]) csr[u] = cs_row16((const uint8_t *)cstart, t[u]);
+                }
 #pragma unroll
                 for (int u = 0; u < U; ++u) {
-                    useful[u] = hit[u] ? hit_useful<NT>(cstart, t[u], hit[u], d[u].nnz) : 0;
+                    if constexpr (NT == 16)
+                        useful[u] = hit[u] ? hit_useful16(csr[u], (unsigned)hit[u], d[u].nnz) : 0;
+                    else
+                        useful[u] = hit[u] ? hit_useful<NT>(cstart, t[u], hit[u], d[u].nnz) : 0;
                     mine += useful[u];
                     if (hit[u]) {
                         ++n_hit;
                         n_hcol += popc_w(hit[u]);
                     }
                 }
+                STEP(7, mine);
                 n_mac += mine;
                 int incl = mine;
 #pragma unroll
@@ -479,6 +512,7 @@ __global__ void __launch_bounds__(FB, 1) k_spmspv_fused(FusedArgs a) {
                 }
                 const int total = __shfl_sync(0xffffffffu, incl, 31);
                 if (a.trace) tr_stage = globaltimer_ns() - tr_c0;
+                STEP(8, total);
                 if (total > 0) {
                     Stage *st = stage_all + wid * SCH;
                     int run = incl - mine;
@@ -497,16 +531,20 @@ __global__ void __launch_bounds__(FB, 1) k_spmspv_fused(FusedArgs a) {
                         }
                     }
                     __syncwarp();
+                    STEP(9, 0);
                     for (int q0 = 0; q0 < total; q0 += 32 * R) {
 #ifdef TSMV_TRACE_ROUNDS
                         const unsigned long long rt0 = globaltimer_ns();
 #endif
                         long long row[R], pos[R], xj[R];
                         bool okq[R], hot[R];
+                        int srcq[R], kq[R];
 #pragma unroll
                         for (int r = 0; r < R; ++r) {
                             const int q = q0 + 32 * r + lane;
                             okq[r] = q < total;
+                            srcq[r] = 0;
+                            kq[r] = 0;
                             if (okq[r]) {
                                 int lo = 0, hi = SCH - 1;  // first staged entry with incl > q
                                 while (lo < hi) {
@@ -514,16 +552,32 @@ __global__ void __launch_bounds__(FB, 1) k_spmspv_fused(FusedArgs a) {
                                     if (st[mid].incl > q) hi = mid;
                                     else lo = mid + 1;
                                 }
-                                const Stage &src = st[lo];
-                                const int before = lo ? st[lo - 1].incl : 0;
+                                srcq[r] = lo;
+                                kq[r] = q - (lo ? st[lo - 1].incl : 0);
+                            }
+                        }
+                        uint4 cq[R];
+                        if constexpr (NT == 16) {
+#pragma unroll
+                            for (int r = 0; r < R; ++r)
+                                if (okq[r]) cq[r] = cs_row16((const uint8_t *)cstart, st[srcq[r]].t);
+                        }
+#pragma unroll
+                        for (int r = 0; r < R; ++r) {
+                            if (okq[r]) {
+                                const Stage &src = st[srcq[r]];
                                 int c, p;
-                                hit_position<NT>(cstart, src.t, (word_t)src.hit, src.nnz, q - before, c, p);
+                                if constexpr (NT == 16)
+                                    hit_position16(cq[r], (unsigned)src.hit, src.nnz, kq[r], c, p);
+                                else
+                                    hit_position<NT>(cstart, src.t, (word_t)src.hit, src.nnz, kq[r], c, p);
                                 hot[r] = src.trow < 0;
                                 row[r] = (hot[r] ? (long long)(~src.trow) : (long long)src.trow) * NT;
                                 pos[r] = src.off + p;
                                 xj[r] = (long long)src.J * NT + c;
                             }
                         }
+                        STEP(10, pos[0] + row[0]);
                         double av[R], xv[R];
 #ifdef TSMV_TRACE_ROUNDS
                         __syncwarp();
@@ -537,6 +591,7 @@ __global__ void __launch_bounds__(FB, 1) k_spmspv_fused(FusedArgs a) {
                                 xv[r] = __ldcg(&a.Lv.xd[xj[r]]);
                             }
                         }
+                        STEP(11, (long long)(av[0] + xv[0]) + row[0]);
 #ifdef TSMV_TRACE_ROUNDS
                         {
                             double sink = 0;
@@ -562,6 +617,7 @@ __global__ void __launch_bounds__(FB, 1) k_spmspv_fused(FusedArgs a) {
 #pragma unroll
                         for (int r = 0; r < R; ++r)
                             if (okq[r] && !hot[r]) TOUCH(&a.rowbits[row[r] >> 5], 1u << (row[r] & 31));
+                        STEP(12, 0);
 #ifdef TSMV_TRACE_ROUNDS
                         __syncwarp();
                         const unsigned long long rt3 = globaltimer_ns();
@@ -598,11 +654,13 @@ __global__ void __launch_bounds__(FB, 1) k_spmspv_fused(FusedArgs a) {
                 long long p[U];
                 double xv[U];
                 bool ok[U];
+                ChunkMap<SCL> cm;
+                cm.build(win, base, lane);
 #pragma unroll
                 for (int u = 0; u < U; ++u) {
                     const long long i = base + lane + 32 * u;
                     ok[u] = i < Ws;
-                    const int qq = ok[u] ? window_find<SCL>(win, i) : 0;
+                    const int qq = ok[u] ? cm.entry(lane + 32 * u) : 0;
                     p[u] = winb[qq] + (i - win[qq]);
                     xv[u] = winx[qq];
                 }

@@ -13,6 +13,6 @@ wait
 for v in "$@"; do
   IFS=, read FB CB EX <<< "$v"
   d=build/var_${FB}_${CB}${EX//[ =-]/}
-  nvcc -gencode arch=compute_100a,code=sm_100a -shared -o $d/libtsmv.so $d/spmspv.o build/api.o build/bfs.o build/builder.o
+  nvcc -gencode arch=compute_100a,code=sm_100a -shared -o $d/libtsmv.so $d/spmspv.o $(ls build/*.o | grep -v spmspv.o)
   echo "$v: $(grep -A3 'k_spmspv_fusedILi16EddLi0E' $d/ptxas.log | grep -E 'registers|spill' | tr '\n' ' ')"
 done

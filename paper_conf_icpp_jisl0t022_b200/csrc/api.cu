@@ -37,6 +37,34 @@ using namespace tsmv;
 namespace tsmv {
 int expand_occupancy(int nt, int dtype);
 int fused_occupancy(int nt, int dtype);
+
+// L2 residency of the SpMSpV workspace (accumulator + touched bitmap, all zero
+// between calls): a persisting access-policy window on the SpMSpV launches keeps
+// its lines in L2 across calls, so the first RED to a row does not fetch a zero
+// sector from HBM.  Device-wide set-aside (cudaLimitPersistingL2CacheSize) is
+// raised to the window size if the device allows it.  TSMV_NO_PERSIST=1 disables.
+static void setup_persistence(tsmv_ctx *c) {
+    c->persist_bytes = 0;
+    c->persist_ratio = 0.f;
+    if (getenv("TSMV_NO_PERSIST")) return;
+    int max_persist = 0, max_win = 0;
+    if (cudaDeviceGetAttribute(&max_persist, cudaDevAttrMaxPersistingL2CacheSize, c->device) != cudaSuccess ||
+        cudaDeviceGetAttribute(&max_win, cudaDevAttrMaxAccessPolicyWindowSize, c->device) != cudaSuccess) {
+        cudaGetLastError();
+        return;
+    }
+    if (max_persist <= 0 || max_win <= 0) return;
+    const size_t want = std::min<size_t>(c->acc.bytes, (size_t)max_win);
+    size_t cur = 0;
+    cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize);
+    const size_t setp = std::max(cur, std::min(want, (size_t)max_persist));
+    if (setp > cur && cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, setp) != cudaSuccess) {
+        cudaGetLastError();
+        return;
+    }
+    c->persist_bytes = want;
+    c->persist_ratio = (float)std::min(1.0, (double)setp / (double)want);
+}
 }
 
 extern "C" tsmv_status tsmv_default_options(tsmv_options *o) {
@@ -70,6 +98,7 @@ static void destroy_impl(tsmv_ctx *c) {
                       &c->desc_bfs, &c->splits_dev, &c->xdense, &c->acct, &c->tring, &c->partials, &c->hot_list, &c->bfs_dirs, &c->bfs_front})
         b->release();
     c->L.release();
+    c->FL.release();
     if (c->hcnt) cudaFreeHost(c->hcnt);
     if (c->ev0) cudaEventDestroy(c->ev0);
     if (c->ev1) cudaEventDestroy(c->ev1);
@@ -175,6 +204,7 @@ extern "C" tsmv_status tsmv_create(tsmv_ctx **out, int64_t nrows, int64_t ncols,
         build_tileset(c, c->P, d_rows.as<int32_t>(), ci, vv, nnz, nrows, ncols, dtype != TSMV_PATTERN, want_bfs, st,
                       c->n_hot ? hot_map.as<int32_t>() : nullptr);
         hot_map.release();
+        build_rec16(c, c->P, st);
         c->nTR = c->P.nTR;
         c->nTC = c->P.nTC;
         if (want_bfs) {
@@ -194,11 +224,14 @@ extern "C" tsmv_status tsmv_create(tsmv_ctx **out, int64_t nrows, int64_t ncols,
         d_rp.release();
 
         // --- workspaces
-        c->acc.alloc(std::max<int64_t>(nrows, 1) * 8);
-        TSMV_CUDA(cudaMemsetAsync(c->acc.p, 0, c->acc.bytes, st));
+        // accumulator and touched-row bitmap in ONE allocation, so that a single
+        // L2 access-policy window can keep both resident (setup_persistence)
         int64_t W = (nrows + 31) / 32;
-        c->rowbits.alloc(std::max<int64_t>(W, 1) * 4);
-        TSMV_CUDA(cudaMemsetAsync(c->rowbits.p, 0, c->rowbits.bytes, st));
+        const size_t acc_b = ((size_t)std::max<int64_t>(nrows, 1) * 8 + 255) & ~(size_t)255;
+        c->acc.alloc(acc_b + (size_t)std::max<int64_t>(W, 1) * 4);
+        TSMV_CUDA(cudaMemsetAsync(c->acc.p, 0, c->acc.bytes, st));
+        c->rowbits_p = reinterpret_cast<uint32_t *>(static_cast<char *>(c->acc.p) + acc_b);
+        setup_persistence(c);
         int64_t cblocks = (W + SCAN_BLOCK - 1) / SCAN_BLOCK + 1;
         c->desc_compact.alloc(cblocks * sizeof(LBDesc<1>));
         TSMV_CUDA(cudaMemsetAsync(c->desc_compact.p, 0, c->desc_compact.bytes, st));
@@ -228,6 +261,11 @@ extern "C" tsmv_status tsmv_create(tsmv_ctx **out, int64_t nrows, int64_t ncols,
         int fo = fused_occupancy(c->nt, (int)dtype);
         TSMV_REQUIRE(fo >= 1, "tsmv_create: fused SpMSpV kernel cannot be resident (occupancy 0)");
         c->fused_blocks = c->sm_count * std::min(fo, 4);
+        if (c->P.rec.p) {
+            int fl = flat_occupancy((int)dtype);
+            TSMV_REQUIRE(fl >= 1, "tsmv_create: flat SpMSpV kernel cannot be resident (occupancy 0)");
+            c->flat_blocks = c->sm_count;  // one 1024-thread CTA per SM
+        }
         if (want_bfs && o.nranks == 1) {
             int bo = bfs_fused_occupancy(c->nt);
             TSMV_REQUIRE(bo >= 1, "tsmv_create: fused BFS kernel cannot be resident (occupancy 0)");
@@ -235,9 +273,9 @@ extern "C" tsmv_status tsmv_create(tsmv_ctx **out, int64_t nrows, int64_t ncols,
             c->bfs_dirs.alloc(TSMV_MAX_LEVELS * 4);
             c->bfs_front.alloc(TSMV_MAX_LEVELS * 8);
         }
-        c->partials.alloc((size_t)std::max(c->fused_blocks, c->bfs_blocks) * 8 * 8);
+        c->partials.alloc((size_t)std::max({c->fused_blocks, c->bfs_blocks, c->flat_blocks}) * 8 * 8);
         TSMV_CUDA(cudaMemsetAsync(c->partials.p, 0, c->partials.bytes, st));
-        c->acct.alloc((size_t)std::max(c->expand_blocks, c->fused_blocks) * 4 * 8);
+        c->acct.alloc((size_t)std::max({c->expand_blocks, c->fused_blocks, c->flat_blocks}) * 4 * 8);
         TSMV_CUDA(cudaMemsetAsync(c->acct.p, 0, c->acct.bytes, st));
         c->xdense.alloc(std::max<int64_t>(ncols, 1) * 8);
         TSMV_CUDA(cudaEventRecord(c->ev1, st));

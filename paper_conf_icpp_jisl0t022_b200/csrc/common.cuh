@@ -57,6 +57,17 @@ struct __align__(16) TileDesc {
     int nnz;        // nonzeros in the tile
 };
 
+// nt = 16 tile record of the flat SpMSpV kernel (spmspv_flat.cu): one 32-byte
+// sector per hit tile.  b = the tile's 16 index bytes ((c << 4) | r, column-major)
+// when nnz <= 16, else its 16 column starts.
+struct __align__(32) TileRec16 {
+    uint32_t off;   // first in-tile nonzero (dense_nnz < 2^32 required)
+    int32_t trow;   // tile row I, or ~hot index (as TileDesc::trow)
+    uint32_t nnz;
+    uint32_t pad;
+    uint4 b;
+};
+
 inline int log2_nt(int nt) { return nt == 16 ? 4 : nt == 32 ? 5 : 6; }
 inline int idx_bytes(int nt) { return nt == 16 ? 1 : 2; }
 inline int word_bytes(int nt) { return nt / 8; }
@@ -100,6 +111,7 @@ struct TileSet {
     DevBuf planes;   // word_t[NT][T]: plane c holds column word c of every tile (bit r = row r)
     DevBuf desc;     // TileDesc[T]
     DevBuf cstart;   // cs_t[T][NT]: start of column c inside the tile's nonzeros (column-major)
+    DevBuf rec;      // TileRec16[T] (nt = 16 only): descriptor + inline indices / column starts
     DevBuf sptr;     // int64[dimC+1]: side matrix (very sparse tiles), CSC
     DevBuf srow;     // int32[side_nnz]
     DevBuf sval;     // double/float[side_nnz]
@@ -110,10 +122,10 @@ struct TileSet {
     const int32_t *hot_list = nullptr;
     size_t bytes() const {
         return ptr.bytes + trow.bytes + tgrp.bytes + mask.bytes + off.bytes + idx.bytes + val.bytes +
-               planes.bytes + sptr.bytes + srow.bytes + sval.bytes + desc.bytes + cstart.bytes;
+               planes.bytes + sptr.bytes + srow.bytes + sval.bytes + desc.bytes + cstart.bytes + rec.bytes;
     }
     void release() {
-        for (DevBuf *b : {&ptr, &trow, &tgrp, &mask, &off, &idx, &val, &planes, &sptr, &srow, &sval, &desc, &cstart})
+        for (DevBuf *b : {&ptr, &trow, &tgrp, &mask, &off, &idx, &val, &planes, &sptr, &srow, &sval, &desc, &cstart, &rec})
             b->release();
     }
 };
@@ -135,6 +147,8 @@ struct Counters {
     long long hit_tiles, hit_nnz, tile_macs;  // expand-kernel accounting (tiles with mask hit,
                                               // their nonzeros, useful multiplies in tiles)
     unsigned long long bar;        // grid-barrier arrival counter (monotonic)
+    unsigned long long resv_t;     // flat SpMSpV list reservation: (entries << 40) | tile work
+    unsigned long long resv_s;     // (entries << 37) | side work; reset at the end of each call
 };
 
 template <int K> struct LBDesc {
@@ -162,6 +176,30 @@ struct Lists {
                           &Ls_col, &Ct, &Cs, &xv, &desc_scan})
             b->release();
     }
+};
+
+// Per-call lists of the flat SpMSpV kernel (capacity grows on demand).
+struct FlatLists {
+    int64_t cap_ent = 0;
+    DevBuf t_beg, t_wpre, t_xm, t_J;  // per x segment with tiles: first tile, work prefix, x bits, J
+    DevBuf s_beg, s_wpre, s_x;        // per x entry with side work: first side nonzero, prefix, x_j
+    DevBuf Ct, Cs;                    // chunk -> first list entry
+    size_t bytes() const {
+        return t_beg.bytes + t_wpre.bytes + t_xm.bytes + t_J.bytes + s_beg.bytes + s_wpre.bytes + s_x.bytes +
+               Ct.bytes + Cs.bytes;
+    }
+    void release() {
+        for (DevBuf *b : {&t_beg, &t_wpre, &t_xm, &t_J, &s_beg, &s_wpre, &s_x, &Ct, &Cs}) b->release();
+    }
+};
+struct FlatListsView {
+    long long *t_beg, *t_wpre;
+    unsigned *t_xm;
+    int *t_J;
+    long long *s_beg, *s_wpre;
+    double *s_x;
+    int *Ct, *Cs;
+    double *xd;
 };
 
 constexpr int HOT_SLOTS = 2048;           // privatised rows per CTA (smem fp64 + bits)
@@ -198,9 +236,13 @@ struct tsmv_ctx {
     tsmv::DevBuf acc;          // double[m] (or ordered keys for MIN)
     tsmv::DevBuf xdense;       // double[n]: x_j scattered by column (only x's columns are ever read)
     tsmv::DevBuf acct;         // long long[expand_blocks][4]: per-block byte-accounting counters
-    tsmv::DevBuf rowbits;      // uint32[ceil(m/32)]
+    tsmv::DevBuf rowbits;      // (unused; the bitmap lives in `acc`, see rowbits_p)
+    uint32_t *rowbits_p = nullptr;  // uint32[ceil(m/32)] touched rows, inside the acc allocation
+    size_t persist_bytes = 0;  // L2 persisting window over acc (+ bitmap); 0 = none
+    float persist_ratio = 0.f;
     tsmv::DevBuf desc_compact; // LBDesc<1>[blocks]
     tsmv::Lists L;
+    tsmv::FlatLists FL;
     tsmv::DevBuf counters;     // Counters
     tsmv::Counters *hcnt = nullptr;  // mapped pinned mirror written by kernels
     tsmv::Counters *hcnt_dev = nullptr;
@@ -227,6 +269,8 @@ struct tsmv_ctx {
     long long tcalls = 0;          // timed calls since tsmv_set_timing
     unsigned long long bar_base = 0;  // value of Counters::bar at the next launch
     int fused_blocks = 0, fused_threads = 1024;
+    int flat_blocks = 0;           // CTAs of the flat SpMSpV kernel (1024 threads, 1 per SM)
+    int last_blocks = 0;           // CTAs of the last SpMSpV launch (partials / acct rows)
     tsmv::DevBuf partials;         // long long[fused_blocks][8]
     long long last_x_nnz = 0;
     int bfs_blocks = 0;            // CTAs of the fused BFS kernel
@@ -252,6 +296,12 @@ bool same_pattern_transposed(tsmv_ctx *c, const int32_t *rows, const int32_t *co
 void prepare_csr(tsmv_ctx *c, const int64_t *row_ptr, const int32_t *col_idx, int32_t *rows, cudaStream_t st);
 // spmspv.cu
 void ensure_lists(tsmv_ctx *c, int64_t k);
+// spmspv_flat.cu
+bool flat_supported(const tsmv_ctx *c);
+void build_rec16(tsmv_ctx *c, TileSet &S, cudaStream_t st);
+int flat_occupancy(int dtype);
+void enqueue_spmspv_flat(tsmv_ctx *c, int sr, long long k, const int32_t *xi, const void *xv, long long ycap,
+                         int32_t *yi, void *yv, long long *ynnz_dev, cudaStream_t st);
 // bfs_fused.cu
 int bfs_fused_occupancy(int nt);
 bool bfs_fused_launch(tsmv_ctx *c, long long source, cudaStream_t st, bool resume, long long level0, uint32_t *Fa,

@@ -939,6 +939,10 @@ void ensure_lists(tsmv_ctx *c, int64_t k) {
 // Enqueue one fused SpMSpV (device pointers only, no sync).
 void enqueue_spmspv(tsmv_ctx *c, int sr, long long k, const int32_t *xi, const void *xv, long long ycap,
                     int32_t *yi, void *yv, long long *ynnz_dev, cudaStream_t st) {
+    if (flat_supported(c)) {
+        enqueue_spmspv_flat(c, sr, k, xi, xv, ycap, yi, yv, ynnz_dev, st);
+        return;
+    }
     const bool f32 = c->dtype == TSMV_F32;
     ensure_lists(c, k);
     FusedArgs a;
@@ -960,7 +964,7 @@ void enqueue_spmspv(tsmv_ctx *c, int sr, long long k, const int32_t *xi, const v
     a.sval = c->P.has_vals ? c->P.sval.p : nullptr;
     a.Lv = lists_view(c);
     a.acc = c->acc.as<double>();
-    a.rowbits = c->rowbits.as<uint32_t>();
+    a.rowbits = c->rowbits_p;
     a.partials = c->partials.as<long long>();
     a.acct = c->acct.as<long long>();
     a.y_idx = yi;
@@ -981,17 +985,19 @@ void enqueue_spmspv(tsmv_ctx *c, int sr, long long k, const int32_t *xi, const v
     TSMV_CUDA(cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dyn));
     TSMV_CUDA(cudaLaunchCooperativeKernel(f, dim3(c->fused_blocks), dim3(FB), args, dyn, st));
     c->bar_base += 4ull * (unsigned long long)c->fused_blocks;
+    c->last_blocks = c->fused_blocks;
     if (c->timing) c->tcalls++;
 }
 
 void stats_from_partials(tsmv_ctx *c, tsmv_call_stats *s) {
-    std::vector<long long> p(8 * (size_t)c->fused_blocks), q(4 * (size_t)c->fused_blocks);
+    const int G = c->last_blocks;
+    std::vector<long long> p(8 * (size_t)G), q(4 * (size_t)G);
     TSMV_CUDA(cudaMemcpy(p.data(), c->partials.p, p.size() * 8, cudaMemcpyDeviceToHost));
     TSMV_CUDA(cudaMemcpy(q.data(), c->acct.p, q.size() * 8, cudaMemcpyDeviceToHost));
     s->x_segments = s->tile_items = s->side_items = 0;
     s->hit_tiles = s->hit_columns = s->tile_macs = 0;
     long long nLs = 0;
-    for (int b = 0; b < c->fused_blocks; ++b) {
+    for (int b = 0; b < G; ++b) {
         s->x_segments += p[8 * b];
         s->tile_items += p[8 * b + 1];
         nLs += p[8 * b + 2];

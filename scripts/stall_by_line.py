@@ -11,6 +11,8 @@ import sys
 from collections import defaultdict
 
 rep, kre, cubin = sys.argv[1], sys.argv[2], sys.argv[3]
+import os
+KSEL = os.environ.get("KSEL", "ILi16EddLi0E")
 top = int(sys.argv[4]) if len(sys.argv) > 4 else 30
 raw = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "sass", "-k", f"regex:{kre}"],
                      capture_output=True, text=True).stdout
@@ -34,9 +36,9 @@ funcs = re.split(r"\n\s*\.text\.", dis)
 best = None
 for f in funcs:
     head = f.split("\n", 1)[0]
-    if re.search(kre.replace("|", ".*|"), head) and ("ILi16EddLi0E" in head or best is None):
+    if re.search(kre, head) and (KSEL in head or best is None):
         best = f
-        if "ILi16EddLi0E" in head:
+        if KSEL in head:
             break
 line_of = {}
 cur = None

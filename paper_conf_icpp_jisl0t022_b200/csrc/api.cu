@@ -204,7 +204,7 @@ extern "C" tsmv_status tsmv_create(tsmv_ctx **out, int64_t nrows, int64_t ncols,
         build_tileset(c, c->P, d_rows.as<int32_t>(), ci, vv, nnz, nrows, ncols, dtype != TSMV_PATTERN, want_bfs, st,
                       c->n_hot ? hot_map.as<int32_t>() : nullptr);
         hot_map.release();
-        build_rec16(c, c->P, st);
+        build_rec64(c, c->P, st);
         c->nTR = c->P.nTR;
         c->nTC = c->P.nTC;
         if (want_bfs) {
@@ -231,6 +231,7 @@ extern "C" tsmv_status tsmv_create(tsmv_ctx **out, int64_t nrows, int64_t ncols,
         c->acc.alloc(acc_b + (size_t)std::max<int64_t>(W, 1) * 4);
         TSMV_CUDA(cudaMemsetAsync(c->acc.p, 0, c->acc.bytes, st));
         c->rowbits_p = reinterpret_cast<uint32_t *>(static_cast<char *>(c->acc.p) + acc_b);
+        flat_init(c, st);
         setup_persistence(c);
         int64_t cblocks = (W + SCAN_BLOCK - 1) / SCAN_BLOCK + 1;
         c->desc_compact.alloc(cblocks * sizeof(LBDesc<1>));
@@ -264,7 +265,7 @@ extern "C" tsmv_status tsmv_create(tsmv_ctx **out, int64_t nrows, int64_t ncols,
         if (c->P.rec.p) {
             int fl = flat_occupancy((int)dtype);
             TSMV_REQUIRE(fl >= 1, "tsmv_create: flat SpMSpV kernel cannot be resident (occupancy 0)");
-            c->flat_blocks = c->sm_count;  // one 1024-thread CTA per SM
+            c->flat_blocks = std::min(c->sm_count, 256);  // one 1024-thread CTA per SM (MAXG)
         }
         if (want_bfs && o.nranks == 1) {
             int bo = bfs_fused_occupancy(c->nt);

@@ -57,15 +57,24 @@ struct __align__(16) TileDesc {
     int nnz;        // nonzeros in the tile
 };
 
-// nt = 16 tile record of the flat SpMSpV kernel (spmspv_flat.cu): one 32-byte
-// sector per hit tile.  b = the tile's 16 index bytes ((c << 4) | r, column-major)
-// when nnz <= 16, else its 16 column starts.
-struct __align__(32) TileRec16 {
-    uint32_t off;   // first in-tile nonzero (dense_nnz < 2^32 required)
+// nt = 16 tile record of the flat SpMSpV kernel (spmspv_flat.cu): one 64-byte
+// DRAM access per hit tile.  b = the tile's 16 index bytes ((c << 4) | r,
+// column-major; padding 0xff) when nnz <= 16, else its 16 column starts; v = the
+// tile's values inline when they fit (nnz <= 4 fp64 / 8 fp32), else unused.
+struct __align__(64) TileRec64 {
+    uint32_t off;   // first in-tile nonzero in idx / val (dense_nnz < 2^32 required)
     int32_t trow;   // tile row I, or ~hot index (as TileDesc::trow)
     uint32_t nnz;
     uint32_t pad;
     uint4 b;
+    uint4 v[2];
+};
+// Per-column record of the flat kernel: side-matrix start of column j and the
+// tile range of its tile column J = j / 16 (replicated over the 16 columns), so
+// that one x entry costs one 16-byte access (+ the next column's sbeg).
+struct __align__(16) ColInfo {
+    long long sbeg;            // side nonzeros of column j are [sbeg, next.sbeg)
+    unsigned long long tinfo;  // (first tile of J << 24) | number of tiles of J
 };
 
 inline int log2_nt(int nt) { return nt == 16 ? 4 : nt == 32 ? 5 : 6; }
@@ -111,7 +120,8 @@ struct TileSet {
     DevBuf planes;   // word_t[NT][T]: plane c holds column word c of every tile (bit r = row r)
     DevBuf desc;     // TileDesc[T]
     DevBuf cstart;   // cs_t[T][NT]: start of column c inside the tile's nonzeros (column-major)
-    DevBuf rec;      // TileRec16[T] (nt = 16 only): descriptor + inline indices / column starts
+    DevBuf rec;      // TileRec64[T] (nt = 16 only): descriptor + inline indices / column starts / values
+    DevBuf colinfo;  // ColInfo[dimC + 1] (nt = 16 only)
     DevBuf sptr;     // int64[dimC+1]: side matrix (very sparse tiles), CSC
     DevBuf srow;     // int32[side_nnz]
     DevBuf sval;     // double/float[side_nnz]
@@ -122,10 +132,10 @@ struct TileSet {
     const int32_t *hot_list = nullptr;
     size_t bytes() const {
         return ptr.bytes + trow.bytes + tgrp.bytes + mask.bytes + off.bytes + idx.bytes + val.bytes +
-               planes.bytes + sptr.bytes + srow.bytes + sval.bytes + desc.bytes + cstart.bytes + rec.bytes;
+               planes.bytes + sptr.bytes + srow.bytes + sval.bytes + desc.bytes + cstart.bytes + rec.bytes + colinfo.bytes;
     }
     void release() {
-        for (DevBuf *b : {&ptr, &trow, &tgrp, &mask, &off, &idx, &val, &planes, &sptr, &srow, &sval, &desc, &cstart, &rec})
+        for (DevBuf *b : {&ptr, &trow, &tgrp, &mask, &off, &idx, &val, &planes, &sptr, &srow, &sval, &desc, &cstart, &rec, &colinfo})
             b->release();
     }
 };
@@ -149,6 +159,7 @@ struct Counters {
     unsigned long long bar;        // grid-barrier arrival counter (monotonic)
     unsigned long long resv_t;     // flat SpMSpV list reservation: (entries << 40) | tile work
     unsigned long long resv_s;     // (entries << 37) | side work; reset at the end of each call
+    unsigned long long nhits;      // flat SpMSpV: hit tiles appended in phase B1
 };
 
 template <int K> struct LBDesc {
@@ -182,23 +193,27 @@ struct Lists {
 struct FlatLists {
     int64_t cap_ent = 0;
     DevBuf t_beg, t_wpre, t_xm, t_J;  // per x segment with tiles: first tile, work prefix, x bits, J
+    DevBuf t_xv;                      // double[16] per segment with tiles: its x values by column
     DevBuf s_beg, s_wpre, s_x;        // per x entry with side work: first side nonzero, prefix, x_j
     DevBuf Ct, Cs;                    // chunk -> first list entry
+    DevBuf hits;                      // uint4 {tile, hit columns, J, 0} per hit tile
     size_t bytes() const {
-        return t_beg.bytes + t_wpre.bytes + t_xm.bytes + t_J.bytes + s_beg.bytes + s_wpre.bytes + s_x.bytes +
-               Ct.bytes + Cs.bytes;
+        return t_beg.bytes + t_wpre.bytes + t_xm.bytes + t_J.bytes + t_xv.bytes + s_beg.bytes + s_wpre.bytes + s_x.bytes +
+               Ct.bytes + Cs.bytes + hits.bytes;
     }
     void release() {
-        for (DevBuf *b : {&t_beg, &t_wpre, &t_xm, &t_J, &s_beg, &s_wpre, &s_x, &Ct, &Cs}) b->release();
+        for (DevBuf *b : {&t_beg, &t_wpre, &t_xm, &t_J, &t_xv, &s_beg, &s_wpre, &s_x, &Ct, &Cs, &hits}) b->release();
     }
 };
 struct FlatListsView {
     long long *t_beg, *t_wpre;
     unsigned *t_xm;
     int *t_J;
+    double *t_xv;
     long long *s_beg, *s_wpre;
     double *s_x;
     int *Ct, *Cs;
+    uint4 *hits;
     double *xd;
 };
 
@@ -269,6 +284,7 @@ struct tsmv_ctx {
     long long tcalls = 0;          // timed calls since tsmv_set_timing
     unsigned long long bar_base = 0;  // value of Counters::bar at the next launch
     int fused_blocks = 0, fused_threads = 1024;
+    bool use_flat = false;         // SpMSpV through the flat kernel (nt = 16), decided at create
     int flat_blocks = 0;           // CTAs of the flat SpMSpV kernel (1024 threads, 1 per SM)
     int last_blocks = 0;           // CTAs of the last SpMSpV launch (partials / acct rows)
     tsmv::DevBuf partials;         // long long[fused_blocks][8]
@@ -298,7 +314,8 @@ void prepare_csr(tsmv_ctx *c, const int64_t *row_ptr, const int32_t *col_idx, in
 void ensure_lists(tsmv_ctx *c, int64_t k);
 // spmspv_flat.cu
 bool flat_supported(const tsmv_ctx *c);
-void build_rec16(tsmv_ctx *c, TileSet &S, cudaStream_t st);
+void flat_init(tsmv_ctx *c, cudaStream_t st);
+void build_rec64(tsmv_ctx *c, TileSet &S, cudaStream_t st);
 int flat_occupancy(int dtype);
 void enqueue_spmspv_flat(tsmv_ctx *c, int sr, long long k, const int32_t *xi, const void *xv, long long ycap,
                          int32_t *yi, void *yv, long long *ynnz_dev, cudaStream_t st);

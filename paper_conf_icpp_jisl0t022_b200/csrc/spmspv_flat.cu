@@ -12,9 +12,10 @@
 //     (count, work) counter instead of a grid-wide scan + barrier: slot order and
 //     work order agree, which is all the chunk maps need (accumulation order is free);
 //   * tile work in 32-item warp chunks: lane = tile item, mask test, then one
-//     32-byte TileRec16 per hit (descriptor + the tile's 16 index bytes inline when
-//     nnz <= 16, else its 16 column starts), and the useful nonzeros of the warp's
-//     hit tiles are redistributed over the lanes with shuffles (no shared memory);
+//     64-byte TileRec64 per hit (descriptor + the tile's 16 index bytes inline when
+//     nnz <= 16, else its 16 column starts, + its values when they fit), and the
+//     useful nonzeros of the warp's other hit tiles are redistributed over the
+//     lanes with shuffles (no shared memory);
 //   * side work (very sparse tiles, Alg 2 column merge) in 128-item chunks whose
 //     list window (start, x_j) is staged in shared memory;
 //   * chunks are dealt round-robin to warps (no work-queue atomics on one address);
@@ -30,7 +31,8 @@ namespace {
 
 constexpr int FT = 1024;          // threads per CTA
 constexpr int NWF = FT / 32;      // warps per CTA
-constexpr int TL = 5;             // log2 tile items per warp chunk
+constexpr int TL = 7;             // log2 tile items per warp task (phase B1)
+constexpr int UT = (1 << TL) / 32;
 constexpr int SL = 7;             // log2 side items per warp chunk
 constexpr int US = (1 << SL) / 32;
 constexpr int BATCH = 8;          // accumulator loads in flight per thread in C2
@@ -44,7 +46,8 @@ struct FlatArgs {
     long long k, n, m, W, row_begin;
     const long long *tptr;
     const uint16_t *mask;
-    const TileRec16 *rec;
+    const TileRec64 *rec;
+    const ColInfo *colinfo;
     const uint8_t *idx;
     const void *val;
     const long long *sptr;
@@ -69,46 +72,65 @@ struct FlatArgs {
     unsigned long long *trace;  // tsmv_set_trace: per CTA 8 globaltimer stamps (dev aid)
 };
 
+// Accumulator encoding (all semirings): an untouched row holds EMPTY = the bits
+// of -0.0, which is the identity of both updates used here: -0.0 + v == v (plus-
+// times, fp64), and LLONG_MIN is the identity of a signed max, to which the
+// min-second keys are mapped (k' = ~ord_key(x) ^ 2^63 keeps the order).  The old
+// value returned by the atomic tells whether this contribution is the first to
+// its row, and only that one sets the row's touched bit (one RED.OR per output
+// row instead of one per contribution).  A row whose contributions are all -0.0
+// returns "first" more than once, which only repeats an idempotent OR.
+constexpr unsigned long long EMPTY = 0x8000000000000000ull;
+
 template <int SR>
-__device__ __forceinline__ void acc_global(double *acc, long long row, double a, double x) {
-    if constexpr (SR == TSMV_PLUS_TIMES) atomicAdd(&acc[row], a * x);
-    else if constexpr (SR == TSMV_MIN_SECOND) atomicMax((unsigned long long *)&acc[row], ~ord_key(x));
+__device__ __forceinline__ bool acc_first(double *acc, long long row, double a, double x) {
+    if constexpr (SR == TSMV_PLUS_TIMES) {
+        return (unsigned long long)__double_as_longlong(atomicAdd(&acc[row], a * x)) == EMPTY;
+    } else if constexpr (SR == TSMV_MIN_SECOND) {
+        const long long k = (long long)(~ord_key(x) ^ EMPTY);
+        return (unsigned long long)atomicMax((long long *)&acc[row], k) == EMPTY;
+    } else {
+        return true;
+    }
 }
 template <int SR>
 __device__ __forceinline__ void acc_shared(double *s, int slot, double a, double x) {
     if constexpr (SR == TSMV_PLUS_TIMES) atomicAdd(&s[slot], a * x);
-    else if constexpr (SR == TSMV_MIN_SECOND) atomicMax((unsigned long long *)&s[slot], ~ord_key(x));
+    else if constexpr (SR == TSMV_MIN_SECOND) atomicMax((long long *)&s[slot], (long long)(~ord_key(x) ^ EMPTY));
 }
 
 // One contribution a*x to row code `rc` (>= 0: local row; < 0: ~hot slot).
+// Returns the row whose touched bit must be set (first contribution), or -1.
 template <int SR>
-__device__ __forceinline__ void contribute(const FlatArgs &a, double *s_hacc, uint32_t *s_hbits, long long rc,
-                                           double av, double xv) {
+__device__ __forceinline__ long long contribute(const FlatArgs &a, double *s_hacc, uint32_t *s_hbits, long long rc,
+                                                double av, double xv) {
     if (rc < 0) {
         const int sl = (int)~rc;
         acc_shared<SR>(s_hacc, sl, av, xv);
         atomicOr(&s_hbits[sl >> 5], 1u << (sl & 31));
-    } else {
-        acc_global<SR>(a.acc, rc, av, xv);
-        atomicOr(&a.rowbits[rc >> 5], 1u << (rc & 31));
+        return -1;
     }
+    return acc_first<SR>(a.acc, rc, av, xv) ? rc : -1;
+}
+__device__ __forceinline__ void touch(uint32_t *rowbits, long long row) {
+    if (row >= 0) atomicOr(&rowbits[row >> 5], 1u << (row & 31));
 }
 
 #ifdef TSMV_FLAT_STEPS
-// development: stamp step k of the warp that processes tile chunk 0 once the value
-// `dep` (produced by the step's loads) is available
+// development: stamp step k of warp 0 of CTA 0 once the value `dep` (produced by
+// the step's loads) is available
 #define FSTEP(k, dep)                                                                              \
     do {                                                                                           \
-        if (a.trace && ch == 0 && lane == 0) {                                                     \
+        if (a.trace && b == 0 && wid == 0 && lane == 0) {                                          \
             if ((long long)(dep) == 0x5eed5eed5eedll) a.trace[2000] = 1;                          \
-            a.trace[148 * 8 + (k)] = globaltimer_ns();                                             \
+            a.trace[148 * 12 + (k)] = globaltimer_ns();                                            \
         }                                                                                          \
     } while (0)
 #define CSTEP(k, dep)                                                                              \
     do {                                                                                           \
         if (a.trace && b == 1 && wid == 0 && lane == 0 && (k) < 16) {                              \
             if ((long long)(dep) == 0x5eed5eed5eedll) a.trace[2000] = 1;                          \
-            a.trace[148 * 8 + 16 + (k)] = globaltimer_ns();                                        \
+            a.trace[148 * 12 + 16 + (k)] = globaltimer_ns();                                       \
         }                                                                                          \
     } while (0)
 #else
@@ -117,6 +139,7 @@ __device__ __forceinline__ void contribute(const FlatArgs &a, double *s_hacc, ui
 #endif
 
 constexpr int HEAVY_CAP = 128;
+constexpr int MAXG = 256;  // max CTAs of the flat kernel (one per SM)
 // Chunk -> list-entry map for an entry owning work items [w0, w0 + w): short runs
 // are written by the calling thread, long ones are queued for a warp.
 template <int LOGC>
@@ -136,6 +159,14 @@ __device__ __forceinline__ void put_chunks(int *C, long long w0, long long w, in
     for (long long ch = c0; ch < c1; ++ch) C[ch] = entry;
 }
 
+__device__ __forceinline__ ColInfo load_colinfo(const ColInfo *p) {
+    const longlong2 v = __ldg(reinterpret_cast<const longlong2 *>(p));
+    ColInfo c;
+    c.sbeg = v.x;
+    c.tinfo = (unsigned long long)v.y;
+    return c;
+}
+
 __device__ __forceinline__ int byte_of(const uint4 &w, int i) {
     const unsigned x = i < 8 ? (i < 4 ? w.x : w.y) : (i < 12 ? w.z : w.w);
     return (int)((x >> ((i & 3) * 8)) & 0xffu);
@@ -143,13 +174,47 @@ __device__ __forceinline__ int byte_of(const uint4 &w, int i) {
 // column start c of a tile with cstart bytes in w (c == 16 -> nnz)
 __device__ __forceinline__ int cs_of(const uint4 &w, int c, int nnz) { return c >= 16 ? nnz : byte_of(w, c); }
 
+// Inline index bytes (nnz <= 16) are (c << 4) | r in column-major order, padding
+// bytes are 0xff.  cw = their column nibbles, four per word, so that the count of
+// bytes in / before a column is a SIMD byte compare + popc (no per-byte loop).
+__device__ __forceinline__ void col_nibbles(const uint4 &b, unsigned (&cw)[4]) {
+    cw[0] = (b.x >> 4) & 0x0f0f0f0fu;
+    cw[1] = (b.y >> 4) & 0x0f0f0f0fu;
+    cw[2] = (b.z >> 4) & 0x0f0f0f0fu;
+    cw[3] = (b.w >> 4) & 0x0f0f0f0fu;
+}
+// bytes i < nnz with column c
+__device__ __forceinline__ int count_col_eq(const unsigned (&cw)[4], int c, int nnz) {
+    const unsigned rep = 0x01010101u * (unsigned)c;
+    int s = 0;
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+        const int v = nnz - 4 * i;
+        const unsigned vm = v >= 4 ? 0xffffffffu : (v <= 0 ? 0u : (0xffffffffu >> (32 - 8 * v)));
+        s += __popc(__vcmpeq4(cw[i], rep) & vm);
+    }
+    return s >> 3;
+}
+// bytes with column < c (padding has column 15 and is never counted for c <= 15)
+__device__ __forceinline__ int count_col_lt(const unsigned (&cw)[4], int c) {
+    const unsigned rep = 0x01010101u * (unsigned)c;
+    int s = 0;
+#pragma unroll
+    for (int i = 0; i < 4; ++i) s += __popc(__vcmpltu4(cw[i], rep));
+    return s >> 3;
+}
+
 // Useful nonzeros of a hit tile (nonzeros in the columns of `hit`).
 __device__ __forceinline__ int rec_useful(const uint4 &b, unsigned hit, int nnz) {
     int s = 0;
     if (nnz <= 16) {
-#pragma unroll
-        for (int i = 0; i < 16; ++i)
-            if (i < nnz) s += (hit >> (byte_of(b, i) >> 4)) & 1u;
+        unsigned cw[4];
+        col_nibbles(b, cw);
+        while (hit) {
+            const int c = __ffs(hit) - 1;
+            hit &= hit - 1;
+            s += count_col_eq(cw, c, nnz);
+        }
     } else {
         while (hit) {
             const int c = __ffs(hit) - 1;
@@ -167,19 +232,18 @@ __device__ __forceinline__ void rec_position(const uint4 &b, unsigned hit, int n
     c = 0;
     r = -1;
     if (nnz <= 16) {
-#pragma unroll
-        for (int i = 0; i < 16; ++i) {
-            if (i < nnz) {
-                const int v = byte_of(b, i);
-                if ((hit >> (v >> 4)) & 1u) {
-                    if (k == 0) {
-                        p = i;
-                        c = v >> 4;
-                        r = v & 15;
-                    }
-                    --k;
-                }
+        unsigned cw[4];
+        col_nibbles(b, cw);
+        while (hit) {
+            c = __ffs(hit) - 1;
+            hit &= hit - 1;
+            const int len = count_col_eq(cw, c, nnz);
+            if (k < len) {
+                p = count_col_lt(cw, c) + k;
+                r = byte_of(b, p) & 15;
+                return;
             }
+            k -= len;
         }
         return;
     }
@@ -227,6 +291,9 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
     __shared__ long long s_acct[NWF][3];
     __shared__ int s_err;
     __shared__ int s_nheavy;
+    __shared__ int s_hcnt;
+    __shared__ long long s_nh;
+    __shared__ long long s_hpre[MAXG + 1];
     __shared__ long long s_heavy[HEAVY_CAP][3];  // chunk-map runs too long for one thread: c0, c1, list | kind
     const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
     const int G = gridDim.x, b = blockIdx.x;
@@ -234,12 +301,15 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
     const bool stamp = a.tring && b == 0 && tid == 0;
     unsigned long long *ts = a.tring ? a.tring + (a.tslot % FLAT_TRING) * 8 : nullptr;
     if (stamp) ts[0] = globaltimer_ns();
-    unsigned long long *tr = a.trace ? a.trace + (long long)b * 8 : nullptr;
+    unsigned long long *tr = a.trace ? a.trace + (long long)b * 12 : nullptr;
     if (tr && tid == 0) tr[0] = globaltimer_ns();
     const int n_slots = a.n_hot * NT;
-    for (int i = tid; i < n_slots; i += FT) s_hacc[i] = 0.0;
+    for (int i = tid; i < n_slots; i += FT) s_hacc[i] = __longlong_as_double((long long)EMPTY);
     for (int i = tid; i < (n_slots + 31) / 32; i += FT) s_hbits[i] = 0u;
-    if (tid == 0) s_nheavy = 0;
+    if (tid == 0) {
+        s_nheavy = 0;
+        s_hcnt = 0;
+    }
 
     // ------------------------------------------------------------ phase A (a2)
     // CTA b owns x entries [e0, e1); thread tid a contiguous run of them.
@@ -256,15 +326,15 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
         bad_any |= bad;
         if (bad) continue;
         const long long J = j >> LOG;
+        const ColInfo ci = load_colinfo(a.colinfo + j);
+        const long long ws = __ldg(&a.colinfo[j + 1].sbeg) - ci.sbeg;
         if (e == 0 || (prev >> LOG) != J) {
-            const long long wt = a.tptr[J + 1] - a.tptr[J];
+            const long long wt = (long long)(ci.tinfo & 0xffffffull);
             q[0] += wt > 0;
             q[1] += wt;
         }
-        const long long ws = a.sptr[j + 1] - a.sptr[j];
         q[2] += ws > 0;
         q[3] += ws;
-        a.L.xd[j] = a.x_val ? (double)((const XV *)a.x_val)[e] : 1.0;
     }
     if (bad_any) a.cnt->err = 1;
     long long ex[4], tot[4];
@@ -291,25 +361,28 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
             const long long prev = e > 0 ? (long long)a.x_idx[e - 1] : -1;
             if (j < 0 || j >= a.n || prev >= j) continue;
             const long long J = j >> LOG;
+            const ColInfo ci = load_colinfo(a.colinfo + j);
             if (e == 0 || (prev >> LOG) != J) {
-                const long long tb = a.tptr[J], wt = a.tptr[J + 1] - tb;
+                const long long tb = (long long)(ci.tinfo >> 24), wt = (long long)(ci.tinfo & 0xffffffull);
                 if (wt > 0) {
+                    // the segment's x bits and values (x stored by segment)
                     unsigned mk = 0;
+                    double *xs = a.L.t_xv + oLt * NT;
                     for (long long e2 = e; e2 < a.k; ++e2) {
                         const long long j2 = a.x_idx[e2];
                         if ((j2 >> LOG) != J) break;
                         mk |= 1u << (j2 & (NT - 1));
+                        xs[j2 & (NT - 1)] = a.x_val ? (double)((const XV *)a.x_val)[e2] : 1.0;
                     }
                     a.L.t_beg[oLt] = tb;
                     a.L.t_wpre[oLt] = oWt;
                     a.L.t_xm[oLt] = mk;
-                    a.L.t_J[oLt] = (int)J;
                     put_chunks<TL>(a.L.Ct, oWt, wt, (int)oLt, 0, s_heavy, &s_nheavy);
                     ++oLt;
                     oWt += wt;
                 }
             }
-            const long long sb = a.sptr[j], ws = a.sptr[j + 1] - sb;
+            const long long sb = ci.sbeg, ws = __ldg(&a.colinfo[j + 1].sbeg) - sb;
             if (ws > 0) {
                 a.L.s_beg[oLs] = sb;
                 a.L.s_wpre[oLs] = oWs;
@@ -343,109 +416,75 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
     __syncthreads();
     const bool err = s_err != 0;
     if (stamp) ts[2] = globaltimer_ns();
+    // hit-list region per CTA: the CTA's tile tasks (<= ceil(nTT / G)) x 128 items
+    const long long RC = (((s_tot[1] + (1 << TL) - 1) >> TL) + G - 1) / G * (1 << TL);
 
-    // ------------------------------------------------------------ phase B (a3-a5)
+    // ------------------------------------------------------------ phase B1 (a3, a5)
+    // Warp tasks of 128 items, dealt round-robin: a tile task ANDs the column masks
+    // of 128 tiles with their segment's x bits (4 mask loads in flight per lane) and
+    // appends the hits to a global hit list (one reservation per CTA and round); a
+    // side task multiplies 128 side nonzeros (Alg 2 column merge) into acc.
     long long n_hit = 0, n_hcol = 0, n_mac = 0;
+    const long long nwarps = (long long)G * NWF;
     if (!err) {
         const long long nLt = s_tot[0], Wt = s_tot[1], nLs = s_tot[2], Ws = s_tot[3];
-        const long long nCt = (Wt + (1 << TL) - 1) >> TL, nCs = (Ws + (1 << SL) - 1) >> SL;
-        const long long nwarps = (long long)G * NWF;
-        const AV *val = (const AV *)a.val;
+        const long long nTT = (Wt + (1 << TL) - 1) >> TL, nCs = (Ws + (1 << SL) - 1) >> SL;
+        const long long ntask = nTT + nCs;
+        const long long rounds = (ntask + nwarps - 1) / nwarps;
+        (void)rounds;
         const AV *sval = (const AV *)a.sval;
-        for (long long ch = (long long)wid * G + b; ch < nCt + nCs; ch += nwarps) {
-            if (ch < nCt) {
-                // ---- tile chunk: 32 tile items, lane = item
-                const long long base = ch << TL;
+        long long *win = s_win + wid * WN;
+        long long *winb = s_winb + wid * WN;
+        double *winx = s_winx + wid * WN;
+        long long *winp = reinterpret_cast<long long *>(winx);
+        for (long long task = (long long)wid * G + b; task < ntask; task += nwarps) {
+            unsigned hv[UT];
+            long long tv[UT];
+            int Jv[UT];
+#pragma unroll
+            for (int u = 0; u < UT; ++u) hv[u] = 0u;
+            if (task < nTT) {
+                const long long base = task << TL;
                 FSTEP(0, 0);
-                const long long s0 = __ldcg(&a.L.Ct[ch]);
+                const long long s0 = __ldcg(&a.L.Ct[task]);
                 FSTEP(1, s0);
-                const long long sq = s0 + lane;
-                const bool inl = sq < nLt;
-                const long long wq = inl ? __ldcg(&a.L.t_wpre[sq]) : INF64;
-                const long long tbq = inl ? __ldcg(&a.L.t_beg[sq]) : 0;
-                const unsigned xmq = inl ? __ldcg(&a.L.t_xm[sq]) : 0u;
-                const int Jq = inl ? __ldcg(&a.L.t_J[sq]) : 0;
-                FSTEP(2, wq + tbq + xmq + Jq);
-                const long long d = wq - base;
-                const unsigned starts = __reduce_or_sync(0xffffffffu, (lane > 0 && d > 0 && d < 32) ? 1u << d : 0u);
-                const int qq = __popc(starts & (lane == 31 ? 0xffffffffu : ((2u << lane) - 1u)));
-                const long long i = base + lane;
-                const long long wsrc = __shfl_sync(0xffffffffu, wq, qq);
-                const long long tbsrc = __shfl_sync(0xffffffffu, tbq, qq);
-                const unsigned xm = __shfl_sync(0xffffffffu, xmq, qq);
-                const int J = __shfl_sync(0xffffffffu, Jq, qq);
-                const bool ok = i < Wt;
-                const long long t = tbsrc + (i - wsrc);
-                const unsigned hit = ok ? ((unsigned)__ldg(&a.mask[t]) & xm) : 0u;
-                FSTEP(3, hit);
-                TileRec16 r;
-                r.off = 0;
-                r.trow = 0;
-                r.nnz = 0;
-                r.b = make_uint4(0, 0, 0, 0);
-                int useful = 0;
-                if (hit) {
-                    const uint4 *rp = reinterpret_cast<const uint4 *>(a.rec + t);
-                    const uint4 h0 = __ldg(rp), h1 = __ldg(rp + 1);
-                    r.off = h0.x;
-                    r.trow = (int)h0.y;
-                    r.nnz = h0.z;
-                    r.b = h1;
-                    useful = rec_useful(r.b, hit, (int)r.nnz);
-                    ++n_hit;
-                    n_hcol += __popc(hit);
-                }
-                int incl = useful;
 #pragma unroll
-                for (int o = 1; o < 32; o <<= 1) {
-                    const int v = __shfl_up_sync(0xffffffffu, incl, o);
-                    if (lane >= o) incl += v;
-                }
-                const int total = __shfl_sync(0xffffffffu, incl, 31);
-                FSTEP(4, total);
-                n_mac += useful;
-                for (int q0 = 0; q0 < total; q0 += 32) {
-                    const int qv = q0 + lane;
-                    // source lane: smallest l with incl_l > qv
-                    int lo = 0;
-#pragma unroll
-                    for (int step = 16; step >= 1; step >>= 1) {
-                        const int v = __shfl_sync(0xffffffffu, incl, lo + step - 1);
-                        if (v <= qv) lo += step;
-                    }
-                    lo = min(lo, 31);
-                    const int exs = __shfl_sync(0xffffffffu, incl - useful, lo);
-                    const unsigned off = __shfl_sync(0xffffffffu, r.off, lo);
-                    const int trow = __shfl_sync(0xffffffffu, r.trow, lo);
-                    const int nnz = __shfl_sync(0xffffffffu, (int)r.nnz, lo);
-                    const unsigned hs = __shfl_sync(0xffffffffu, hit, lo);
-                    const int Js = __shfl_sync(0xffffffffu, J, lo);
-                    uint4 bs;
-                    bs.x = __shfl_sync(0xffffffffu, r.b.x, lo);
-                    bs.y = __shfl_sync(0xffffffffu, r.b.y, lo);
-                    bs.z = __shfl_sync(0xffffffffu, r.b.z, lo);
-                    bs.w = __shfl_sync(0xffffffffu, r.b.w, lo);
-                    if (qv < total) {
-                        int p, c, rr;
-                        rec_position(bs, hs, nnz, qv - exs, p, c, rr);
-                        const long long pos = (long long)off + p;
-                        if (rr < 0) rr = __ldg(&a.idx[pos]) & (NT - 1);
-                        const double av = val ? (double)__ldg(&val[pos]) : 1.0;
-                        const double xv = __ldcg(&a.L.xd[(long long)Js * NT + c]);
-                        const long long rc = trow >= 0 ? (long long)trow * NT + rr : ~((long long)(~trow) * NT + rr);
-                        FSTEP(5, av + xv + rc);
-                        contribute<SR>(a, s_hacc, s_hbits, rc, av, xv);
+                for (int q0 = 0; q0 <= (1 << TL); q0 += 32) {
+                    const int qx = q0 + lane;
+                    const long long ix = s0 + qx;
+                    const bool in = ix < nLt;
+                    const long long w = in ? __ldcg(&a.L.t_wpre[ix]) : INF64;
+                    const long long tb = in ? __ldcg(&a.L.t_beg[ix]) : 0;
+                    const long long pk = in ? (long long)__ldcg(&a.L.t_xm[ix]) : 0;
+                    if (qx <= (1 << TL)) {
+                        win[qx] = w;
+                        winb[qx] = tb;
+                        winp[qx] = pk;
                     }
                 }
-                FSTEP(6, 0);
-            } else {
-                // ---- side chunk: 128 side nonzeros, window staged in shared memory
-                const long long c2 = ch - nCt;
+                __syncwarp();
+                FSTEP(2, win[0]);
+                ChunkMap<TL> cm;
+                cm.build(win, base, lane);
+                unsigned xm[UT];
+#pragma unroll
+                for (int u = 0; u < UT; ++u) {
+                    const long long i = base + lane + 32 * u;
+                    const bool ok = i < Wt;
+                    const int qq = ok ? cm.entry(lane + 32 * u) : 0;
+                    tv[u] = winb[qq] + (i - win[qq]);
+                    const long long pk = winp[qq];
+                    xm[u] = ok ? (unsigned)(pk & 0xffff) : 0u;
+                    Jv[u] = (int)(s0 + qq);  // list slot of the segment
+                }
+#pragma unroll
+                for (int u = 0; u < UT; ++u) hv[u] = xm[u] ? ((unsigned)__ldg(&a.mask[tv[u]]) & xm[u]) : 0u;
+                FSTEP(3, hv[0] + hv[UT - 1]);
+                __syncwarp();
+            } else if (task < ntask) {
+                const long long c2 = task - nTT;
                 const long long base = c2 << SL;
                 const long long s0 = __ldcg(&a.L.Cs[c2]);
-                long long *win = s_win + wid * WN;
-                long long *winb = s_winb + wid * WN;
-                double *winx = s_winx + wid * WN;
 #pragma unroll
                 for (int q0 = 0; q0 <= (1 << SL); q0 += 32) {
                     const int qx = q0 + lane;
@@ -483,10 +522,186 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
                         av[u] = sval ? (double)__ldg(&sval[p[u]]) : 1.0;
                     }
                 }
+                long long fr[US];
 #pragma unroll
                 for (int u = 0; u < US; ++u)
-                    if (ok[u]) contribute<SR>(a, s_hacc, s_hbits, (long long)row[u], av[u], xv[u]);
+                    fr[u] = ok[u] ? contribute<SR>(a, s_hacc, s_hbits, (long long)row[u], av[u], xv[u]) : -1;
+#pragma unroll
+                for (int u = 0; u < US; ++u) touch(a.rowbits, fr[u]);
                 __syncwarp();
+            }
+            // append this round's hits: warp offsets in shared memory, one global
+            // reservation per CTA
+            int nmine = 0;
+#pragma unroll
+            for (int u = 0; u < UT; ++u) nmine += hv[u] != 0u;
+            int incl = nmine;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const int v = __shfl_up_sync(0xffffffffu, incl, o);
+                if (lane >= o) incl += v;
+            }
+            const int wtot = __shfl_sync(0xffffffffu, incl, 31);
+            int woff = 0;
+            if (lane == 0 && wtot) woff = atomicAdd(&s_hcnt, wtot);
+            woff = __shfl_sync(0xffffffffu, woff, 0);
+            long long o = (long long)b * RC + woff + incl - nmine;
+#pragma unroll
+            for (int u = 0; u < UT; ++u)
+                if (hv[u]) a.L.hits[o++] = make_uint4((unsigned)tv[u], hv[u], (unsigned)Jv[u], 0u);
+        }
+    }
+    __syncthreads();
+    if (tid == 0) a.partials[b * 8 + 5] = s_hcnt;
+    grid_sync_f(&a.cnt->bar, target, tr ? tr + 3 : nullptr);
+    if (stamp) ts[6] = globaltimer_ns();
+    // prefix of the per-CTA hit counts (hits of CTA g live at [g * RC, g * RC + count))
+    if (wid == 0) {
+        constexpr int PER = (MAXG + 31) / 32;
+        long long v[PER], run = 0;
+#pragma unroll
+        for (int i = 0; i < PER; ++i) {
+            const int g = lane * PER + i;
+            v[i] = g < G ? __ldcg(&a.partials[g * 8 + 5]) : 0;
+            run += v[i];
+        }
+        long long inc = run;
+#pragma unroll
+        for (int o2 = 1; o2 < 32; o2 <<= 1) {
+            const long long y = __shfl_up_sync(0xffffffffu, inc, o2);
+            if (lane >= o2) inc += y;
+        }
+        long long ex = inc - run;
+#pragma unroll
+        for (int i = 0; i < PER; ++i) {
+            const int g = lane * PER + i;
+            if (g <= G) s_hpre[g] = ex;
+            ex += v[i];
+        }
+        if (lane == 31) s_nh = inc;
+    }
+    __syncthreads();
+
+    // ------------------------------------------------------------ phase B2 (a4)
+    // lane = hit tile: one 64-byte record.  Tiles whose values are inline (and
+    // indices, nnz <= 16) are multiplied by their own lane; the useful nonzeros of
+    // the other hit tiles of the warp are redistributed over the lanes (shuffles)
+    // and read from the idx / val arrays.
+    if (!err) {
+        const long long NH = s_nh;
+        const AV *val = (const AV *)a.val;
+        constexpr int INL = 32 / (int)sizeof(AV);
+        for (long long hb = ((long long)wid * G + b) * 32; hb < NH; hb += nwarps * 32) {
+            const long long h = hb + lane;
+            unsigned hit = 0u;
+            long long t = 0;
+            int slot = 0;
+            double xv0 = 0.0;
+            if (h < NH) {
+                int lo = 0, hi = G - 1;  // CTA region holding hit h: last g with s_hpre[g] <= h
+                while (lo < hi) {
+                    const int mid = (lo + hi + 1) >> 1;
+                    if (s_hpre[mid] <= h) lo = mid;
+                    else hi = mid - 1;
+                }
+                const uint4 e = __ldcg(&a.L.hits[(long long)lo * RC + (h - s_hpre[lo])]);
+                t = e.x;
+                hit = e.y;
+                slot = (int)e.z;
+                // x value of the first hit column, fetched beside the tile record
+                xv0 = __ldcg(&a.L.t_xv[(long long)slot * NT + (__ffs(hit) - 1)]);
+            }
+            FSTEP(4, hit);
+            unsigned off = 0, nnz = 0;
+            int trow = 0;
+            uint4 bb = make_uint4(0, 0, 0, 0);
+            int useful = 0;
+            if (hit) {
+                const uint4 *rp = reinterpret_cast<const uint4 *>(a.rec + t);
+                const uint4 h0 = __ldg(rp), h1 = __ldg(rp + 1), v0 = __ldg(rp + 2), v1 = __ldg(rp + 3);
+                off = h0.x;
+                trow = (int)h0.y;
+                nnz = h0.z;
+                bb = h1;
+                ++n_hit;
+                n_hcol += __popc(hit);
+                if (nnz <= (val ? (unsigned)INL : 16u)) {
+                    // inline tile: this lane multiplies its useful nonzeros
+                    unsigned cw[4];
+                    col_nibbles(bb, cw);
+                    const double *xs = a.L.t_xv + (long long)slot * NT;
+                    unsigned hh = hit;
+                    while (hh) {
+                        const int c = __ffs(hh) - 1;
+                        hh &= hh - 1;
+                        const int len = count_col_eq(cw, c, (int)nnz), p0 = count_col_lt(cw, c);
+                        const double xv = c == __ffs(hit) - 1 ? xv0 : __ldcg(&xs[c]);
+                        for (int k2 = 0; k2 < len; ++k2) {
+                            const int p = p0 + k2;
+                            const int rr = byte_of(bb, p) & (NT - 1);
+                            double av = 1.0;
+                            if (val) {
+                                if constexpr (sizeof(AV) == 8) {
+                                    const uint4 &vq = p < 2 ? v0 : v1;
+                                    av = (p & 1) ? __hiloint2double((int)vq.w, (int)vq.z)
+                                                 : __hiloint2double((int)vq.y, (int)vq.x);
+                                } else {
+                                    const uint4 &vq = p < 4 ? v0 : v1;
+                                    const int q4 = p & 3;
+                                    av = (double)__uint_as_float(q4 == 0 ? vq.x : q4 == 1 ? vq.y : q4 == 2 ? vq.z : vq.w);
+                                }
+                            }
+                            const long long rc =
+                                trow >= 0 ? (long long)trow * NT + rr : ~((long long)(~trow) * NT + rr);
+                            touch(a.rowbits, contribute<SR>(a, s_hacc, s_hbits, rc, av, xv));
+                            ++n_mac;
+                        }
+                    }
+                } else {
+                    useful = rec_useful(bb, hit, (int)nnz);
+                }
+            }
+            int incl = useful;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const int v = __shfl_up_sync(0xffffffffu, incl, o);
+                if (lane >= o) incl += v;
+            }
+            const int total = __shfl_sync(0xffffffffu, incl, 31);
+            FSTEP(5, total);
+            n_mac += useful;
+            for (int q0 = 0; q0 < total; q0 += 32) {
+                const int qv = q0 + lane;
+                // source lane: smallest l with incl_l > qv
+                int lo = 0;
+#pragma unroll
+                for (int step = 16; step >= 1; step >>= 1) {
+                    const int v = __shfl_sync(0xffffffffu, incl, lo + step - 1);
+                    if (v <= qv) lo += step;
+                }
+                lo = min(lo, 31);
+                const int exs = __shfl_sync(0xffffffffu, incl - useful, lo);
+                const unsigned offs = __shfl_sync(0xffffffffu, off, lo);
+                const int trs = __shfl_sync(0xffffffffu, trow, lo);
+                const int nns = __shfl_sync(0xffffffffu, (int)nnz, lo);
+                const unsigned hs = __shfl_sync(0xffffffffu, hit, lo);
+                const int ss = __shfl_sync(0xffffffffu, slot, lo);
+                uint4 bs;
+                bs.x = __shfl_sync(0xffffffffu, bb.x, lo);
+                bs.y = __shfl_sync(0xffffffffu, bb.y, lo);
+                bs.z = __shfl_sync(0xffffffffu, bb.z, lo);
+                bs.w = __shfl_sync(0xffffffffu, bb.w, lo);
+                if (qv < total) {
+                    int p, c, rr;
+                    rec_position(bs, hs, nns, qv - exs, p, c, rr);
+                    const long long pos = (long long)offs + p;
+                    if (rr < 0) rr = __ldg(&a.idx[pos]) & (NT - 1);
+                    const double av = val ? (double)__ldg(&val[pos]) : 1.0;
+                    const double xv = __ldcg(&a.L.t_xv[(long long)ss * NT + c]);
+                    const long long rc = trs >= 0 ? (long long)trs * NT + rr : ~((long long)(~trs) * NT + rr);
+                    FSTEP(6, av + xv + rc);
+                    touch(a.rowbits, contribute<SR>(a, s_hacc, s_hbits, rc, av, xv));
+                }
             }
         }
     }
@@ -503,15 +718,25 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
     }
     __syncthreads();
     // privatised hot rows: one global atomic per (CTA, touched hot row)
+#ifdef TSMV_EXP_NO_FLUSH
+    if (false) {
+#else
     if (!err) {
-        for (int sl = tid; sl < n_slots; sl += FT) {
+#endif
+        // CTAs start at different slots so that the 148 flushes of one hot row are
+        // spread over time instead of queueing on one L2 address together
+        const int rot = (int)(((long long)b * n_slots) / G);
+        for (int q = tid; q < n_slots; q += FT) {
+            const int sl = q + rot < n_slots ? q + rot : q + rot - n_slots;
             if ((s_hbits[sl >> 5] >> (sl & 31)) & 1u) {
                 const long long row = (long long)a.hot_list[sl / NT] * NT + sl % NT;
-                if constexpr (SR == TSMV_PLUS_TIMES) atomicAdd(&a.acc[row], s_hacc[sl]);
+                bool first = true;
+                if constexpr (SR == TSMV_PLUS_TIMES)
+                    first = (unsigned long long)__double_as_longlong(atomicAdd(&a.acc[row], s_hacc[sl])) == EMPTY;
                 else if constexpr (SR == TSMV_MIN_SECOND)
-                    atomicMax((unsigned long long *)&a.acc[row],
-                              (unsigned long long)__double_as_longlong(s_hacc[sl]));
-                atomicOr(&a.rowbits[row >> 5], 1u << (row & 31));
+                    first = (unsigned long long)atomicMax((long long *)&a.acc[row],
+                                                          (long long)__double_as_longlong(s_hacc[sl])) == EMPTY;
+                if (first) atomicOr(&a.rowbits[row >> 5], 1u << (row & 31));
             }
         }
     }
@@ -520,7 +745,7 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
         for (int w = 0; w < NWF; ++w) sum += s_acct[w][tid];
         a.acct[b * 4 + tid] = sum;
     }
-    grid_sync_f(&a.cnt->bar, target, tr ? tr + 3 : nullptr);
+    grid_sync_f(&a.cnt->bar, target, tr ? tr + 5 : nullptr);
     if (stamp) ts[3] = globaltimer_ns();
 
     // ------------------------------------------------------------ phase C (a6)
@@ -531,7 +756,7 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
     long long blk, dummy;
     block_scan<1, FT>(&mycnt, &dummy, &blk, s_scan);
     if (tid == 0) a.partials[b * 8 + 4] = blk;
-    grid_sync_f(&a.cnt->bar, target, tr ? tr + 5 : nullptr);
+    grid_sync_f(&a.cnt->bar, target, tr ? tr + 7 : nullptr);
     if (stamp) ts[4] = globaltimer_ns();
     if (tid < 32) {
         long long pre = 0, tt = 0;
@@ -603,7 +828,7 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
                     const long long row = (wbase + src[kk]) * 32 + lane;
                     const long long pos = wp[kk] + __popc(wb[kk] & lt);
 #ifndef TSMV_C2_NOZERO
-                    a.acc[row] = 0.0;
+                    a.acc[row] = __longlong_as_double((long long)EMPTY);
 #endif
 #ifdef TSMV_C2_NOSTORE
                     if (pos < 0) {
@@ -614,7 +839,7 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
                         if (a.y_val) {
                             double x = v[kk];
                             if constexpr (SR == TSMV_MIN_SECOND)
-                                x = ord_val(~(unsigned long long)__double_as_longlong(x));
+                                x = ord_val(~((unsigned long long)__double_as_longlong(x) ^ EMPTY));
                             ((XV *)a.y_val)[pos] = (XV)x;
                         }
                     }
@@ -636,7 +861,7 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
         a.cnt->resv_s = 0;
         if (a.tring) ts[5] = globaltimer_ns();
     }
-    if (tr && tid == 0) tr[7] = globaltimer_ns();
+    if (tr && tid == 0) tr[9] = globaltimer_ns();
 }
 
 template <class AV, class XV> void *pick_sr_flat(int sr) {
@@ -658,37 +883,88 @@ void flat_set_smem() {
     done = true;
 }
 
-__global__ void k_build_rec16(const TileDesc *__restrict__ desc, const uint8_t *__restrict__ cstart,
-                              const uint8_t *__restrict__ idx, int64_t T, TileRec16 *__restrict__ rec) {
+template <class V>
+__global__ void k_build_rec64(const TileDesc *__restrict__ desc, const uint8_t *__restrict__ cstart,
+                              const uint8_t *__restrict__ idx, const V *__restrict__ val, int64_t T,
+                              TileRec64 *__restrict__ rec) {
+    constexpr int INL = 32 / (int)sizeof(V);
     for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < T; t += (int64_t)gridDim.x * blockDim.x) {
         const TileDesc d = desc[t];
-        TileRec16 r;
+        TileRec64 r;
         r.off = (uint32_t)d.off;
         r.trow = d.trow;
         r.nnz = (uint32_t)d.nnz;
         r.pad = 0;
-        uint8_t by[16];
-        for (int i = 0; i < 16; ++i) by[i] = d.nnz <= 16 ? (i < d.nnz ? idx[d.off + i] : 0xffu) : cstart[t * 16 + i];
-        r.b.x = by[0] | (by[1] << 8) | (by[2] << 16) | ((unsigned)by[3] << 24);
-        r.b.y = by[4] | (by[5] << 8) | (by[6] << 16) | ((unsigned)by[7] << 24);
-        r.b.z = by[8] | (by[9] << 8) | (by[10] << 16) | ((unsigned)by[11] << 24);
-        r.b.w = by[12] | (by[13] << 8) | (by[14] << 16) | ((unsigned)by[15] << 24);
+        uint32_t w[4];
+        for (int q = 0; q < 4; ++q) {
+            uint32_t x = 0;
+            for (int i = 0; i < 4; ++i) {
+                const int k = 4 * q + i;
+                const uint32_t by = d.nnz <= 16 ? (k < d.nnz ? idx[d.off + k] : 0xffu) : cstart[t * 16 + k];
+                x |= by << (8 * i);
+            }
+            w[q] = x;
+        }
+        r.b = make_uint4(w[0], w[1], w[2], w[3]);
+        V vv[INL];
+        for (int i = 0; i < INL; ++i) vv[i] = (val && i < d.nnz && d.nnz <= INL) ? val[d.off + i] : (V)0;
+        memcpy(&r.v[0], vv, 32);
         rec[t] = r;
+    }
+}
+
+__global__ void k_build_colinfo(const long long *__restrict__ sptr, const long long *__restrict__ tptr, int64_t n,
+                                int64_t nTC, ColInfo *__restrict__ ci) {
+    for (int64_t j = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; j <= n; j += (int64_t)gridDim.x * blockDim.x) {
+        ColInfo c;
+        c.sbeg = sptr[j];
+        const int64_t J = j >> 4;
+        c.tinfo = J < nTC ? (((unsigned long long)tptr[J] << 24) | (unsigned long long)(tptr[J + 1] - tptr[J])) : 0ull;
+        ci[j] = c;
     }
 }
 
 }  // namespace
 
-bool flat_supported(const tsmv_ctx *c) {
-    return c->nt == 16 && c->P.rec.p != nullptr && !getenv("TSMV_FUSED_V6");
+bool flat_supported(const tsmv_ctx *c) { return c->use_flat; }
+
+namespace {
+__global__ void k_fill_u64(unsigned long long *p, long long n, unsigned long long v) {
+    for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x)
+        p[i] = v;
+}
+}  // namespace
+
+// Decide (once, at create) whether the context uses the flat kernel, and set the
+// accumulator to its EMPTY encoding (the round-1 fused kernel uses 0).
+void flat_init(tsmv_ctx *c, cudaStream_t st) {
+    c->use_flat = c->nt == 16 && c->P.rec.p != nullptr && !getenv("TSMV_FUSED_V6");
+    if (!c->use_flat || c->m == 0) return;
+    const int blocks = (int)std::min<int64_t>((c->m + 255) / 256, 148 * 8);
+    k_fill_u64<<<blocks, 256, 0, st>>>(c->acc.as<unsigned long long>(), c->m, EMPTY);
+    TSMV_CUDA(cudaGetLastError());
 }
 
-void build_rec16(tsmv_ctx *c, TileSet &S, cudaStream_t st) {
-    if (c->nt != 16 || S.T == 0 || S.dense_nnz >= (1ll << 32)) return;
-    S.rec.alloc((size_t)S.T * sizeof(TileRec16));
+void build_rec64(tsmv_ctx *c, TileSet &S, cudaStream_t st) {
+    // limits of the packed fields: u32 nonzero offsets, 24-bit tile counts per tile
+    // column, 40-bit tile ids
+    if (c->nt != 16 || S.T == 0 || S.dense_nnz >= (1ll << 32) || S.nTR >= (1ll << 24) || S.T >= (1ll << 40))
+        return;
+    S.rec.alloc((size_t)S.T * sizeof(TileRec64));
     const int blocks = (int)std::min<int64_t>((S.T + 255) / 256, 148 * 16);
-    k_build_rec16<<<blocks, 256, 0, st>>>(S.desc.as<TileDesc>(), S.cstart.as<uint8_t>(), S.idx.as<uint8_t>(), S.T,
-                                          S.rec.as<TileRec16>());
+    if (c->dtype == TSMV_F32)
+        k_build_rec64<float><<<blocks, 256, 0, st>>>(S.desc.as<TileDesc>(), S.cstart.as<uint8_t>(),
+                                                      S.idx.as<uint8_t>(), S.has_vals ? S.val.as<float>() : nullptr,
+                                                      S.T, S.rec.as<TileRec64>());
+    else
+        k_build_rec64<double><<<blocks, 256, 0, st>>>(S.desc.as<TileDesc>(), S.cstart.as<uint8_t>(),
+                                                       S.idx.as<uint8_t>(), S.has_vals ? S.val.as<double>() : nullptr,
+                                                       S.T, S.rec.as<TileRec64>());
+    TSMV_CUDA(cudaGetLastError());
+    S.colinfo.alloc((size_t)(S.dimC + 1) * sizeof(ColInfo));
+    const int cb = (int)std::min<int64_t>((S.dimC + 256) / 256, 148 * 16);
+    k_build_colinfo<<<cb, 256, 0, st>>>(S.sptr.as<long long>(), S.ptr.as<long long>(), S.dimC, S.nTC,
+                                        S.colinfo.as<ColInfo>());
     TSMV_CUDA(cudaGetLastError());
 }
 
@@ -713,6 +989,7 @@ void ensure_flat_lists(tsmv_ctx *c, int64_t k) {
         F.t_wpre.alloc(segs * 8);
         F.t_xm.alloc(segs * 4);
         F.t_J.alloc(segs * 4);
+        F.t_xv.alloc(segs * 16 * 8);
         F.s_beg.alloc((cap + 1) * 8);
         F.s_wpre.alloc((cap + 1) * 8);
         F.s_x.alloc((cap + 1) * 8);
@@ -721,6 +998,7 @@ void ensure_flat_lists(tsmv_ctx *c, int64_t k) {
     if (!F.Ct.p) {
         F.Ct.alloc(((c->P.T >> TL) + 2) * 4);
         F.Cs.alloc(((c->P.side_nnz >> SL) + 2) * 4);
+        F.hits.alloc((size_t)(c->P.T + 128ll * (c->flat_blocks + 2)) * 16);
     }
 }
 
@@ -730,11 +1008,13 @@ FlatListsView flat_view(tsmv_ctx *c) {
     v.t_wpre = c->FL.t_wpre.as<long long>();
     v.t_xm = c->FL.t_xm.as<unsigned>();
     v.t_J = c->FL.t_J.as<int>();
+    v.t_xv = c->FL.t_xv.as<double>();
     v.s_beg = c->FL.s_beg.as<long long>();
     v.s_wpre = c->FL.s_wpre.as<long long>();
     v.s_x = c->FL.s_x.as<double>();
     v.Ct = c->FL.Ct.as<int>();
     v.Cs = c->FL.Cs.as<int>();
+    v.hits = c->FL.hits.as<uint4>();
     v.xd = c->xdense.as<double>();
     return v;
 }
@@ -755,7 +1035,8 @@ void enqueue_spmspv_flat(tsmv_ctx *c, int sr, long long k, const int32_t *xi, co
     a.row_begin = c->row_begin;
     a.tptr = c->P.ptr.as<long long>();
     a.mask = c->P.mask.as<uint16_t>();
-    a.rec = c->P.rec.as<TileRec16>();
+    a.rec = c->P.rec.as<TileRec64>();
+    a.colinfo = c->P.colinfo.as<ColInfo>();
     a.idx = c->P.idx.as<uint8_t>();
     a.val = c->P.has_vals ? c->P.val.p : nullptr;
     a.sptr = c->P.sptr.as<long long>();
@@ -801,7 +1082,7 @@ void enqueue_spmspv_flat(tsmv_ctx *c, int sr, long long k, const int32_t *xi, co
     }
     cfg.attrs = at;
     TSMV_CUDA(cudaLaunchKernelExC(&cfg, pick_flat(f32, sr), args));
-    c->bar_base += 3ull * (unsigned long long)G;
+    c->bar_base += 4ull * (unsigned long long)G;
     c->last_blocks = G;
     if (c->timing) c->tcalls++;
 }

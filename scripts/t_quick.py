@@ -13,7 +13,7 @@ def run(M, A, d, steps=10, label=""):
     yi = torch.empty(A.m, dtype=torch.int32, device=dev); yv = torch.empty(A.m, dtype=torch.float64, device=dev)
     yn = torch.zeros(1, dtype=torch.int64, device=dev)
     out = {}
-    for v6 in (0, 1):
+    for v6 in (0,):
         if v6: os.environ["TSMV_FUSED_V6"] = "1"
         else: os.environ.pop("TSMV_FUSED_V6", None)
         for xi, xv in xs[:3]: M.spmspv_async(xi, xv, yi, yv, yn)

@@ -25,21 +25,24 @@ for flush in (True, False):
         M.spmspv(xi, xv)
         tsmv.tsmv_set_trace(M.ctx, 0)
     G = 148
-    t = buf[: G * 8].view(G, 8).cpu().double()
+    t = buf[: G * 12].view(G, 12).cpu().double()
     t0 = t[:, 0].min()
     t = (t - t0) / 1e3
-    print(f"{which} d={d} flush={flush}: start skew {t[:,0].max():.2f} us, end {t[:,7].max():.2f} us")
-    for bi in range(3):
+    print(f"{which} d={d} flush={flush}: start skew {t[:,0].max():.2f} us, end {t[:,9].max():.2f} us")
+    for bi in range(4):
         arr, rel = t[:, 1 + 2 * bi], t[:, 2 + 2 * bi]
         print(f"  barrier {bi+1}: arrivals min {arr.min():.2f} median {arr.median():.2f} max {arr.max():.2f} (CTA {int(arr.argmax())}); "
               f"release min {rel.min():.2f} max {rel.max():.2f}")
-st = buf[148 * 8: 148 * 8 + 8].cpu().tolist()
-print("tile chunk 0 step deltas ns:", [st[i + 1] - st[i] if st[i + 1] and st[i] else None for i in range(6)])
-c2 = t[:, 7] - t[:, 6]
+st = buf[148 * 12: 148 * 12 + 8].cpu().tolist()
+print("warp 0 step deltas ns (B1: Ct, window, masks | B2: entry->total, ->loads):", [st[i + 1] - st[i] if st[i + 1] and st[i] else None for i in range(6)])
+c2 = t[:, 9] - t[:, 8]
 top = torch.argsort(c2, descending=True)[:8].tolist()
 print("C2 per-CTA us: median %.2f max %.2f; slowest CTAs:" % (c2.median(), c2.max()), [(i, round(float(c2[i]), 2)) for i in top])
 b1 = t[:, 3] - t[:, 2]
 top = torch.argsort(b1, descending=True)[:8].tolist()
-print("B per-CTA us: median %.2f max %.2f; slowest CTAs:" % (b1.median(), b1.max()), [(i, round(float(b1[i]), 2)) for i in top])
-st = buf[148 * 8 + 16: 148 * 8 + 32].cpu().tolist()
+print("B1 per-CTA us: median %.2f max %.2f; slowest CTAs:" % (b1.median(), b1.max()), [(i, round(float(b1[i]), 2)) for i in top])
+st = buf[148 * 12 + 16: 148 * 12 + 32].cpu().tolist()
 print("C2 CTA1 warp0 step deltas ns:", [st[i + 1] - st[i] if st[i + 1] and st[i] else None for i in range(15)])
+b2 = t[:, 5] - t[:, 4]
+top = torch.argsort(b2, descending=True)[:8].tolist()
+print("B2 per-CTA us: median %.2f max %.2f; slowest CTAs:" % (b2.median(), b2.max()), [(i, round(float(b2[i]), 2)) for i in top])

@@ -196,13 +196,14 @@ struct FlatLists {
     DevBuf t_xv;                      // double[16] per segment with tiles: its x values by column
     DevBuf s_beg, s_wpre, s_x;        // per x entry with side work: first side nonzero, prefix, x_j
     DevBuf Ct, Cs;                    // chunk -> first list entry
-    DevBuf hits;                      // uint4 {tile, hit columns, J, 0} per hit tile
+    DevBuf hits;                      // uint4 {tile, hit columns, segment slot, 0} per hit tile
+    DevBuf pcnt;                      // long long[G * KP]: set bits per touched-bitmap piece
     size_t bytes() const {
         return t_beg.bytes + t_wpre.bytes + t_xm.bytes + t_J.bytes + t_xv.bytes + s_beg.bytes + s_wpre.bytes + s_x.bytes +
                Ct.bytes + Cs.bytes + hits.bytes;
     }
     void release() {
-        for (DevBuf *b : {&t_beg, &t_wpre, &t_xm, &t_J, &t_xv, &s_beg, &s_wpre, &s_x, &Ct, &Cs, &hits}) b->release();
+        for (DevBuf *b : {&t_beg, &t_wpre, &t_xm, &t_J, &t_xv, &s_beg, &s_wpre, &s_x, &Ct, &Cs, &hits, &pcnt}) b->release();
     }
 };
 struct FlatListsView {
@@ -214,6 +215,7 @@ struct FlatListsView {
     double *s_x;
     int *Ct, *Cs;
     uint4 *hits;
+    long long *pcnt;
     double *xd;
 };
 

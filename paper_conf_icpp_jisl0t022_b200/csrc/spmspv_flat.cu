@@ -35,7 +35,14 @@ constexpr int TL = 7;             // log2 tile items per warp task (phase B1)
 constexpr int UT = (1 << TL) / 32;
 constexpr int SL = 7;             // log2 side items per warp chunk
 constexpr int US = (1 << SL) / 32;
-constexpr int BATCH = 8;          // accumulator loads in flight per thread in C2
+#ifndef TSMV_BATCH
+#define TSMV_BATCH 4
+#endif
+#ifndef TSMV_SPW
+#define TSMV_SPW 4
+#endif
+constexpr int SPW = TSMV_SPW;     // set rows up to which a bitmap word is emitted by its own thread
+constexpr int BATCH = TSMV_BATCH; // accumulator loads in flight per thread in C2
 constexpr int FLAT_TRING = 4096;
 constexpr unsigned long long T_CNT_SHIFT = 40, S_CNT_SHIFT = 37;
 constexpr long long INF64 = 0x7fffffffffffffffLL;
@@ -140,6 +147,7 @@ __device__ __forceinline__ void touch(uint32_t *rowbits, long long row) {
 
 constexpr int HEAVY_CAP = 128;
 constexpr int MAXG = 256;  // max CTAs of the flat kernel (one per SM)
+constexpr int KP = 8;      // bitmap pieces per CTA in phase C
 // Chunk -> list-entry map for an entry owning work items [w0, w0 + w): short runs
 // are written by the calling thread, long ones are queued for a warp.
 template <int LOGC>
@@ -294,6 +302,8 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
     __shared__ int s_hcnt;
     __shared__ long long s_nh;
     __shared__ long long s_hpre[MAXG + 1];
+    __shared__ unsigned long long s_pc[KP];
+    __shared__ long long s_pbase[KP], s_ex0[KP];
     __shared__ long long s_heavy[HEAVY_CAP][3];  // chunk-map runs too long for one thread: c0, c1, list | kind
     const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
     const int G = gridDim.x, b = blockIdx.x;
@@ -749,55 +759,107 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
     if (stamp) ts[3] = globaltimer_ns();
 
     // ------------------------------------------------------------ phase C (a6)
-    const long long S = (((a.W + G - 1) / G) + 31) & ~31ll;
-    const long long w0 = (long long)b * S, w1 = min(a.W, w0 + S);
-    long long mycnt = 0;
-    for (long long w = w0 + tid; w < w1; w += FT) mycnt += __popc(__ldcg(&a.rowbits[w]));
-    long long blk, dummy;
-    block_scan<1, FT>(&mycnt, &dummy, &blk, s_scan);
-    if (tid == 0) a.partials[b * 8 + 4] = blk;
-    grid_sync_f(&a.cnt->bar, target, tr ? tr + 7 : nullptr);
-    if (stamp) ts[4] = globaltimer_ns();
-    if (tid < 32) {
-        long long pre = 0, tt = 0;
-        for (int g = lane; g < G; g += 32) {
-            const long long v = __ldcg(&a.partials[g * 8 + 4]);
-            tt += v;
-            if (g < b) pre += v;
-        }
+    // The touched bitmap is cut into G*KP pieces of PS words; CTA b owns pieces
+    // b, b + G, ..., so a dense stretch of y (power-law rows) is spread over KP
+    // CTAs.  C1 counts each piece, C2 emits y at the piece's global offset.  A
+    // round covers PSR words of each of the CTA's pieces (thread tid: piece
+    // tid / PSR), so one block scan per round serves all pieces.
+    constexpr int PSR = FT / KP;
+    const long long PS = ((a.W + (long long)G * KP - 1) / ((long long)G * KP) + 31) & ~31ll;
+    const int kp = tid / PSR, tp = tid % PSR;
+    const long long pw0 = ((long long)b + (long long)kp * G) * PS;
+    const long long pw1 = min(a.W, pw0 + PS);
+    if (tid < KP) s_pc[tid] = 0;
+    __syncthreads();
+    {
+        long long mycnt = 0;
+        for (long long w = pw0 + tp; w < pw1; w += PSR) mycnt += __popc(__ldcg(&a.rowbits[w]));
 #pragma unroll
-        for (int o = 16; o > 0; o >>= 1) {
-            pre += __shfl_xor_sync(0xffffffffu, pre, o);
-            tt += __shfl_xor_sync(0xffffffffu, tt, o);
-        }
-        if (lane == 0) {
-            s_base[0] = pre;
-            s_tot[0] = tt;
-        }
+        for (int o = 16; o > 0; o >>= 1) mycnt += __shfl_xor_sync(0xffffffffu, mycnt, o);
+        if (lane == 0 && mycnt) atomicAdd(&s_pc[kp], (unsigned long long)mycnt);
     }
     __syncthreads();
-    long long carry = s_base[0];
+    if (tid < KP) a.L.pcnt[b + tid * G] = (long long)s_pc[tid];
+    grid_sync_f(&a.cnt->bar, target, tr ? tr + 7 : nullptr);
+    if (stamp) ts[4] = globaltimer_ns();
+    {
+        // exclusive prefix of all G*KP piece counts (every CTA, in shared memory)
+        const int NP = G * KP;
+        constexpr int PPT = (MAXG * KP + FT - 1) / FT;
+        long long v[PPT], run = 0;
+#pragma unroll
+        for (int i = 0; i < PPT; ++i) {
+            const int q = tid * PPT + i;
+            v[i] = q < NP ? __ldcg(&a.L.pcnt[q]) : 0;
+            run += v[i];
+        }
+        long long ex, tt;
+        block_scan<1, FT>(&run, &ex, &tt, s_scan);
+#pragma unroll
+        for (int i = 0; i < PPT; ++i) {
+            const int q = tid * PPT + i;
+            if (q < NP && (q % G) == b) s_pbase[q / G] = ex;
+            ex += v[i];
+        }
+        if (tid == 0) s_tot[0] = tt;
+    }
+    __syncthreads();
     const long long ycap = a.y_cap;
-#ifdef TSMV_C2_DELAY
-    { const unsigned long long t0 = globaltimer_ns(); while (globaltimer_ns() - t0 < 10000) {} }
-#endif
-    for (long long rb = w0; rb < w1; rb += FT) {
-        const long long w = rb + tid;
+    const int nround = (int)((PS + PSR - 1) / PSR);
+    for (int rd = 0; rd < nround; ++rd) {
+        const long long w = pw0 + (long long)rd * PSR + tp;
         CSTEP(0, 0);
-        const unsigned bits = w < w1 ? __ldcg(&a.rowbits[w]) : 0u;
+        const unsigned bits = w < pw1 ? __ldcg(&a.rowbits[w]) : 0u;
         CSTEP(1, bits);
         long long c = __popc(bits), exw, rtot;
         block_scan<1, FT>(&c, &exw, &rtot, s_scan);
+        if (tp == 0) s_ex0[kp] = exw;
+        __syncthreads();
+        const long long seg0 = s_ex0[kp];
+        const long long segsum = (kp + 1 < KP ? s_ex0[kp + 1] : rtot) - seg0;
+        const long long pos0 = s_pbase[kp] + exw - seg0;
+        __syncthreads();
+        if (tp == 0) s_pbase[kp] += segsum;
         CSTEP(2, exw);
         int it = 0;
-        const long long pos0 = carry + exw;
-        carry += rtot;
         if (bits) a.rowbits[w] = 0u;
-        // transposed emission: the warp walks its words with bits, BATCH at a time;
-        // lane l handles bit l of each, so acc loads and y stores are coalesced
+        // sparse words (<= SPW set rows) are emitted by their own thread, all in one
+        // round of independent loads; dense words by the whole warp, BATCH words per
+        // round, lane l handling row l (coalesced acc loads and y stores)
+        const int pc = __popc(bits);
+        if (pc > 0 && pc <= SPW) {
+            unsigned bb = bits;
+            int rr[SPW];
+            double v[SPW];
+#pragma unroll
+            for (int kk = 0; kk < SPW; ++kk) {
+                rr[kk] = bb ? __ffs(bb) - 1 : 0;
+                bb &= bb - 1;
+            }
+#pragma unroll
+            for (int kk = 0; kk < SPW; ++kk)
+                if (kk < pc) v[kk] = __ldcg(&a.acc[w * 32 + rr[kk]]);
+#pragma unroll
+            for (int kk = 0; kk < SPW; ++kk) {
+                if (kk < pc) {
+                    const long long row = w * 32 + rr[kk];
+                    const long long pos = pos0 + kk;
+                    a.acc[row] = __longlong_as_double((long long)EMPTY);
+                    if (pos < ycap) {
+                        a.y_idx[pos] = (int32_t)(row + a.row_begin);
+                        if (a.y_val) {
+                            double x = v[kk];
+                            if constexpr (SR == TSMV_MIN_SECOND)
+                                x = ord_val(~((unsigned long long)__double_as_longlong(x) ^ EMPTY));
+                            ((XV *)a.y_val)[pos] = (XV)x;
+                        }
+                    }
+                }
+            }
+        }
         const long long wbase = w - lane;
         const unsigned lt = (1u << lane) - 1u;
-        unsigned todo = __ballot_sync(0xffffffffu, bits != 0);
+        unsigned todo = __ballot_sync(0xffffffffu, pc > SPW);
         while (todo) {
             int src[BATCH];
             int nb = 0;
@@ -811,30 +873,23 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
                 }
             }
             unsigned wb[BATCH];
-            long long wp[BATCH];
             double v[BATCH];
             bool mine[BATCH];
 #pragma unroll
             for (int kk = 0; kk < BATCH; ++kk) {
                 wb[kk] = __shfl_sync(0xffffffffu, bits, src[kk]);
-                wp[kk] = __shfl_sync(0xffffffffu, pos0, src[kk]);
                 mine[kk] = kk < nb && ((wb[kk] >> lane) & 1u);
                 if (mine[kk]) v[kk] = __ldcg(&a.acc[(wbase + src[kk]) * 32 + lane]);
             }
             CSTEP(3 + 2 * it, v[0] + v[BATCH - 1]);
 #pragma unroll
             for (int kk = 0; kk < BATCH; ++kk) {
+                const long long wp = __shfl_sync(0xffffffffu, pos0, src[kk]);
                 if (mine[kk]) {
                     const long long row = (wbase + src[kk]) * 32 + lane;
-                    const long long pos = wp[kk] + __popc(wb[kk] & lt);
-#ifndef TSMV_C2_NOZERO
+                    const long long pos = wp + __popc(wb[kk] & lt);
                     a.acc[row] = __longlong_as_double((long long)EMPTY);
-#endif
-#ifdef TSMV_C2_NOSTORE
-                    if (pos < 0) {
-#else
                     if (pos < ycap) {
-#endif
                         a.y_idx[pos] = (int32_t)(row + a.row_begin);
                         if (a.y_val) {
                             double x = v[kk];
@@ -999,6 +1054,7 @@ void ensure_flat_lists(tsmv_ctx *c, int64_t k) {
         F.Ct.alloc(((c->P.T >> TL) + 2) * 4);
         F.Cs.alloc(((c->P.side_nnz >> SL) + 2) * 4);
         F.hits.alloc((size_t)(c->P.T + 128ll * (c->flat_blocks + 2)) * 16);
+        F.pcnt.alloc((size_t)MAXG * KP * 8);
     }
 }
 
@@ -1015,6 +1071,7 @@ FlatListsView flat_view(tsmv_ctx *c) {
     v.Ct = c->FL.Ct.as<int>();
     v.Cs = c->FL.Cs.as<int>();
     v.hits = c->FL.hits.as<uint4>();
+    v.pcnt = c->FL.pcnt.as<long long>();
     v.xd = c->xdense.as<double>();
     return v;
 }

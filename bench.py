@@ -197,9 +197,38 @@ def flops_of(colcnt, xi):
 
 
 def call_bytes(st, k, sv, nt, m):
-    """Algorithmic bytes of one tsmv_spmspv call (= one launch of the fused kernel)
-    for this build's data layout: every byte the method must
-    touch once, at its natural width, no sector rounding."""
+    """Algorithmic bytes of one tsmv_spmspv call (= one launch of the SpMSpV kernel)
+    for this build's data layout: every byte the method must touch
+    once, at its natural width, no sector rounding.  nt = 16 contexts run the flat
+    kernel (64-byte tile records, per-column records); others the round-1 kernel."""
+    if nt != 16:
+        return call_bytes_v6(st, k, sv, nt, m)
+    segs, items, side = st["x_segments"], st["tile_items"], st["side_items"]
+    hits, hcols, macs = st["hit_tiles"], st["hit_columns"], st["tile_macs"]
+    ind = st.get("tile_macs_indirect", macs)
+    y = st["y_nnz"]
+    phase_a = (k * (4 + sv)                       # read x (index, value)
+               + k * (16 + 8)                     # ColInfo of column j + side start of j+1
+               + segs * (8 + 8 + 4) + k * 8       # tile-list entries + the segments' x values
+               + k * 24                           # side-list entries (start, prefix, x_j)
+               + (items + side) // 128 * 4)       # chunk -> entry maps
+    phase_b1 = (segs * 20 + k * 24                # list windows read back
+                + items * (nt // 8)               # column mask of every tile in a hit tile column
+                + hits * 16                       # hit-list entries written
+                + side * (4 + sv)                 # row + value of every useful side nonzero
+                + side * 8)                       # accumulator update
+    phase_b2 = (hits * (16 + 64)                  # hit entry + 64-byte tile record
+                + hcols * 8                       # x_j of every hit column
+                + ind * (1 + sv)                  # index + value of MACs not inline in the record
+                + macs * 8                        # accumulator update
+                + y * 4)                          # touched bit, once per output row
+    phase_c = (2 * (m // 8)                       # touched bitmap: count + emit passes
+               + y * (8 + 8 + 4 + sv))            # acc read + reset, y index + value
+    return phase_a + phase_b1 + phase_b2 + phase_c
+
+
+def call_bytes_v6(st, k, sv, nt, m):
+    """Round-1 fused kernel layout (nt = 32 / 64 contexts)."""
     si = 1 if nt == 16 else 2        # packed in-tile row index
     cs = 1 if nt == 16 else 2        # column start offset inside a tile
     mask_b = nt // 8
@@ -217,6 +246,23 @@ def call_bytes(st, k, sv, nt, m):
     phase_c = (m // 8                               # touched bitmap scan
                + st["y_nnz"] * (8 + 8 + 4 + sv))    # acc read + clear, y index + value
     return phase_a + phase_b + phase_c
+
+
+def random_access(kms, nt):
+    """The kernel's DRAM read sectors (ncu, profiles/flat_traffic.json) per second of
+    its device time, next to the measured ceiling of cold random sector reads
+    (profiles/random_access_ceiling.json): the irregular path is bound by random
+    sector rate long before streaming bandwidth."""
+    try:
+        t = json.load(open(os.path.join(ROOT, "profiles", "flat_traffic.json" if nt == 16 else "fused_traffic.json")))
+        c = json.load(open(os.path.join(ROOT, "profiles", "random_access_ceiling.json")))
+        sec = t.get("dram_sectors_read") or t["dram_bytes_per_launch"] / 32
+        ach = sec / (kms * 1e-3) / 1e9
+        ceil = c["footprint_1GiB_G_req_per_s"]
+        return {"dram_sectors_per_launch (ncu)": int(sec), "achieved_G_sectors_per_s": round(ach, 2),
+                "ceiling_G_random_sectors_per_s": ceil, "frac": round(ach / ceil, 4)}
+    except Exception:
+        return None
 
 
 def survey_bytes(st, k, sv, nt, macs):
@@ -317,7 +363,7 @@ def run_tsmv(args):
     kms = ms / args.steps
     achieved = (kexp_bytes / args.steps) / (kms * 1e-3) / 1e9
     traffic = None
-    tpath = os.path.join(ROOT, "profiles", "fused_traffic.json")
+    tpath = os.path.join(ROOT, "profiles", "flat_traffic.json" if args.tile_dim == 16 else "fused_traffic.json")
     if os.path.exists(tpath):
         try:
             traffic = json.load(open(tpath)).get("dram_bytes_per_launch")
@@ -326,13 +372,14 @@ def run_tsmv(args):
     n_ = max(ncalls, 1)
     roof = {"bound": "hbm", "achieved": round(achieved, 2), "peak": peak, "unit": "GB/s",
             "frac": round(achieved / peak, 4), "traffic": traffic,
-            "kernel": "k_spmspv_fused (the whole call is one cooperative launch)",
+            "kernel": ("k_spmspv_flat" if args.tile_dim == 16 else "k_spmspv_fused") + " (the whole call is one cooperative launch)",
             "peak_source": peak_src,
             "algorithmic_bytes_per_launch": int(kexp_bytes / args.steps),
             "kernel_ms_per_launch": round(kms, 5),
             "phase_ms_per_launch (globaltimer, CTA 0)": {
                 "A_x_tiling": round(kt[0] / n_, 5), "B_intersect_multiply": round(kt[1] / n_, 5),
                 "C_compact": round(kt[2] / n_, 5), "whole": round(kt[3] / n_, 5)},
+            "random_access": random_access(kms, args.tile_dim),
             "survey_B_alg": {"bytes": int(svy_bytes / args.steps),
                              "achieved_GBps": round(svy_bytes / (ms * 1e-3) / 1e9, 2),
                              "frac": round(svy_bytes / (ms * 1e-3) / 1e9 / peak, 4)}}

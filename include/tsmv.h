@@ -86,6 +86,8 @@ typedef struct {
     int64_t hit_tiles;      /* tiles whose column mask intersects the segment mask */
     int64_t hit_columns;    /* (tile, column) pairs in both the tile's and x's masks */
     int64_t tile_macs;      /* useful multiply-adds inside tiles (side ones = side_items) */
+    int64_t tile_macs_indirect; /* of tile_macs, those whose value / index came from the
+                                   nonzero arrays (not inline in the 64-byte tile record) */
 } tsmv_call_stats;
 
 /* Built-format census. */

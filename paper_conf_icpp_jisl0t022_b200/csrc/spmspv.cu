@@ -995,7 +995,7 @@ void stats_from_partials(tsmv_ctx *c, tsmv_call_stats *s) {
     TSMV_CUDA(cudaMemcpy(p.data(), c->partials.p, p.size() * 8, cudaMemcpyDeviceToHost));
     TSMV_CUDA(cudaMemcpy(q.data(), c->acct.p, q.size() * 8, cudaMemcpyDeviceToHost));
     s->x_segments = s->tile_items = s->side_items = 0;
-    s->hit_tiles = s->hit_columns = s->tile_macs = 0;
+    s->hit_tiles = s->hit_columns = s->tile_macs = s->tile_macs_indirect = 0;
     long long nLs = 0;
     for (int b = 0; b < G; ++b) {
         s->x_segments += p[8 * b];
@@ -1005,6 +1005,7 @@ void stats_from_partials(tsmv_ctx *c, tsmv_call_stats *s) {
         s->hit_tiles += q[4 * b];
         s->hit_columns += q[4 * b + 1];
         s->tile_macs += q[4 * b + 2];
+        s->tile_macs_indirect += (c->use_flat ? q[4 * b + 3] : q[4 * b + 2]);
     }
     (void)nLs;
 }

@@ -296,7 +296,7 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
     double *s_winx = reinterpret_cast<double *>(s_winb + NWF * WN);               // [NWF][WN]
     uint32_t *s_hbits = reinterpret_cast<uint32_t *>(s_winx + NWF * WN);          // [HOT_SLOTS/32]
     __shared__ long long s_base[4], s_tot[4];
-    __shared__ long long s_acct[NWF][3];
+    __shared__ long long s_acct[NWF][4];
     __shared__ int s_err;
     __shared__ int s_nheavy;
     __shared__ int s_hcnt;
@@ -434,7 +434,7 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
     // of 128 tiles with their segment's x bits (4 mask loads in flight per lane) and
     // appends the hits to a global hit list (one reservation per CTA and round); a
     // side task multiplies 128 side nonzeros (Alg 2 column merge) into acc.
-    long long n_hit = 0, n_hcol = 0, n_mac = 0;
+    long long n_hit = 0, n_hcol = 0, n_mac = 0, n_ind = 0;
     const long long nwarps = (long long)G * NWF;
     if (!err) {
         const long long nLt = s_tot[0], Wt = s_tot[1], nLs = s_tot[2], Ws = s_tot[3];
@@ -636,36 +636,40 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
                 ++n_hit;
                 n_hcol += __popc(hit);
                 if (nnz <= (val ? (unsigned)INL : 16u)) {
-                    // inline tile: this lane multiplies its useful nonzeros
-                    unsigned cw[4];
-                    col_nibbles(bb, cw);
+                    // inline tile: this lane multiplies its useful nonzeros, issuing the
+                    // atomics of up to 4 of them before waiting for any "first" result
                     const double *xs = a.L.t_xv + (long long)slot * NT;
-                    unsigned hh = hit;
-                    while (hh) {
-                        const int c = __ffs(hh) - 1;
-                        hh &= hh - 1;
-                        const int len = count_col_eq(cw, c, (int)nnz), p0 = count_col_lt(cw, c);
-                        const double xv = c == __ffs(hit) - 1 ? xv0 : __ldcg(&xs[c]);
-                        for (int k2 = 0; k2 < len; ++k2) {
-                            const int p = p0 + k2;
-                            const int rr = byte_of(bb, p) & (NT - 1);
-                            double av = 1.0;
-                            if (val) {
-                                if constexpr (sizeof(AV) == 8) {
-                                    const uint4 &vq = p < 2 ? v0 : v1;
-                                    av = (p & 1) ? __hiloint2double((int)vq.w, (int)vq.z)
-                                                 : __hiloint2double((int)vq.y, (int)vq.x);
-                                } else {
-                                    const uint4 &vq = p < 4 ? v0 : v1;
-                                    const int q4 = p & 3;
-                                    av = (double)__uint_as_float(q4 == 0 ? vq.x : q4 == 1 ? vq.y : q4 == 2 ? vq.z : vq.w);
+                    const int c0 = __ffs(hit) - 1;
+                    for (int g = 0; g < (int)nnz; g += 4) {
+                        long long fr[4];
+#pragma unroll
+                        for (int j = 0; j < 4; ++j) {
+                            const int p = g + j;
+                            fr[j] = -1;
+                            const int by = p < (int)nnz ? byte_of(bb, p) : 0xff;
+                            const int c = by >> 4, rr = by & (NT - 1);
+                            if (p < (int)nnz && ((hit >> c) & 1u)) {
+                                double av = 1.0;
+                                if (val) {
+                                    if constexpr (sizeof(AV) == 8) {
+                                        const uint4 &vq = p < 2 ? v0 : v1;
+                                        av = (p & 1) ? __hiloint2double((int)vq.w, (int)vq.z)
+                                                     : __hiloint2double((int)vq.y, (int)vq.x);
+                                    } else {
+                                        const uint4 &vq = p < 4 ? v0 : v1;
+                                        const int q4 = p & 3;
+                                        av = (double)__uint_as_float(q4 == 0 ? vq.x : q4 == 1 ? vq.y : q4 == 2 ? vq.z : vq.w);
+                                    }
                                 }
+                                const double xv = c == c0 ? xv0 : __ldcg(&xs[c]);
+                                const long long rc =
+                                    trow >= 0 ? (long long)trow * NT + rr : ~((long long)(~trow) * NT + rr);
+                                fr[j] = contribute<SR>(a, s_hacc, s_hbits, rc, av, xv);
+                                ++n_mac;
                             }
-                            const long long rc =
-                                trow >= 0 ? (long long)trow * NT + rr : ~((long long)(~trow) * NT + rr);
-                            touch(a.rowbits, contribute<SR>(a, s_hacc, s_hbits, rc, av, xv));
-                            ++n_mac;
                         }
+#pragma unroll
+                        for (int j = 0; j < 4; ++j) touch(a.rowbits, fr[j]);
                     }
                 } else {
                     useful = rec_useful(bb, hit, (int)nnz);
@@ -680,6 +684,8 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
             const int total = __shfl_sync(0xffffffffu, incl, 31);
             FSTEP(5, total);
             n_mac += useful;
+            n_ind += useful;
+            long long frp = -1, frq = -1;
             for (int q0 = 0; q0 < total; q0 += 32) {
                 const int qv = q0 + lane;
                 // source lane: smallest l with incl_l > qv
@@ -710,9 +716,13 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
                     const double xv = __ldcg(&a.L.t_xv[(long long)ss * NT + c]);
                     const long long rc = trs >= 0 ? (long long)trs * NT + rr : ~((long long)(~trs) * NT + rr);
                     FSTEP(6, av + xv + rc);
-                    touch(a.rowbits, contribute<SR>(a, s_hacc, s_hbits, rc, av, xv));
+                    frp = contribute<SR>(a, s_hacc, s_hbits, rc, av, xv);
                 }
+                touch(a.rowbits, frq);  // previous round's result: its atomic had a round to return
+                frq = frp;
+                frp = -1;
             }
+            touch(a.rowbits, frq);
         }
     }
 #pragma unroll
@@ -720,11 +730,13 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
         n_hit += __shfl_xor_sync(0xffffffffu, n_hit, o);
         n_hcol += __shfl_xor_sync(0xffffffffu, n_hcol, o);
         n_mac += __shfl_xor_sync(0xffffffffu, n_mac, o);
+        n_ind += __shfl_xor_sync(0xffffffffu, n_ind, o);
     }
     if (lane == 0) {
         s_acct[wid][0] = n_hit;
         s_acct[wid][1] = n_hcol;
         s_acct[wid][2] = n_mac;
+        s_acct[wid][3] = n_ind;
     }
     __syncthreads();
     // privatised hot rows: one global atomic per (CTA, touched hot row)
@@ -736,9 +748,14 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
         // CTAs start at different slots so that the 148 flushes of one hot row are
         // spread over time instead of queueing on one L2 address together
         const int rot = (int)(((long long)b * n_slots) / G);
-        for (int q = tid; q < n_slots; q += FT) {
+        constexpr int FQ = HOT_SLOTS / FT;
+        long long fr[FQ];
+#pragma unroll
+        for (int i = 0; i < FQ; ++i) {
+            const int q = tid + i * FT;
             const int sl = q + rot < n_slots ? q + rot : q + rot - n_slots;
-            if ((s_hbits[sl >> 5] >> (sl & 31)) & 1u) {
+            fr[i] = -1;
+            if (q < n_slots && ((s_hbits[sl >> 5] >> (sl & 31)) & 1u)) {
                 const long long row = (long long)a.hot_list[sl / NT] * NT + sl % NT;
                 bool first = true;
                 if constexpr (SR == TSMV_PLUS_TIMES)
@@ -746,11 +763,13 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
                 else if constexpr (SR == TSMV_MIN_SECOND)
                     first = (unsigned long long)atomicMax((long long *)&a.acc[row],
                                                           (long long)__double_as_longlong(s_hacc[sl])) == EMPTY;
-                if (first) atomicOr(&a.rowbits[row >> 5], 1u << (row & 31));
+                if (first) fr[i] = row;
             }
         }
+#pragma unroll
+        for (int i = 0; i < FQ; ++i) touch(a.rowbits, fr[i]);
     }
-    if (tid < 3) {
+    if (tid < 4) {
         long long sum = 0;
         for (int w = 0; w < NWF; ++w) sum += s_acct[w][tid];
         a.acct[b * 4 + tid] = sum;

@@ -46,7 +46,8 @@ class tsmv_options(ctypes.Structure):
 class tsmv_call_stats(ctypes.Structure):
     _fields_ = [("x_nnz", ctypes.c_int64), ("x_segments", ctypes.c_int64), ("tile_items", ctypes.c_int64),
                 ("side_items", ctypes.c_int64), ("y_nnz", ctypes.c_int64), ("hit_tiles", ctypes.c_int64),
-                ("hit_columns", ctypes.c_int64), ("tile_macs", ctypes.c_int64)]
+                ("hit_columns", ctypes.c_int64), ("tile_macs", ctypes.c_int64),
+                ("tile_macs_indirect", ctypes.c_int64)]
 
 
 class tsmv_info(ctypes.Structure):

@@ -390,9 +390,16 @@ extern "C" tsmv_status tsmv_bfs(tsmv_ctx *c, int64_t source, int32_t *levels, ts
                 int cur;
                 const bool stopped = bfs_fused_launch(c, source, st, resume, level, Fa, Fb, mu, reached, edges,
                                                       stop_on_pull, TSMV_MAX_LEVELS, L, mu2, r2, e2, cur);
-                if (getenv("TSMV_BFS_PHASES"))
-                    fprintf(stderr, "[bfs fused] levels %lld..%lld: count %.3f ms, lists %.3f ms, expand %.3f ms\n",
-                            level, L, c->hcnt->Wt * 1e-6, c->hcnt->nLs * 1e-6, c->hcnt->Ws * 1e-6);
+                if (getenv("TSMV_BFS_PHASES")) {
+                    long long fl = 0;
+                    if (c->lslots.p) {
+                        TSMV_CUDA(cudaMemcpy(&fl, c->lslots.as<long long>() + 15, 8, cudaMemcpyDeviceToHost));
+                        TSMV_CUDA(cudaMemset(c->lslots.as<long long>() + 12, 0, 32));
+                    }
+                    fprintf(stderr, "[bfs fused] levels %lld..%lld: count %.3f ms, lists %.3f ms, expand %.3f ms"
+                            " (list-prof builds: CTA0 expand / slowest CTA / CTA0 flush %.3f ms)\n",
+                            level, L, c->hcnt->Wt * 1e-6, c->hcnt->nLs * 1e-6, c->hcnt->Ws * 1e-6, fl * 1e-6);
+                }
                 if (cur) std::swap(Fa, Fb);  // Fa = bitmap of the current frontier
                 level = L;
                 mu = mu2;

@@ -137,20 +137,56 @@ __device__ __forceinline__ void pull_rowtile(const BfsTiles &Q, const BfsView &B
     if (lane == 0 && found) discover<NT>(B, rb_seg + I, found);
 }
 
+// Pull-CSC over 32 consecutive row tiles I0 .. I0+31 with one warp: the lanes
+// test the visited words of all 32 in one coalesced load, and only the row
+// tiles that still have unvisited rows are walked (pull_rowtile), one by one.
+template <int NT>
+__device__ __forceinline__ void pull_rowtiles32(const BfsTiles &Q, const BfsView &B, long long I0, long long nTR,
+                                                int lane) {
+    using word_t = typename Tr<NT>::word_t;
+    const long long I = I0 + lane;
+    bool open = false;
+    if (I < nTR) open = (word_t)~seg_bits<NT>(B.V, B.row_begin / NT + I) != 0 && Q.ptr[I + 1] > Q.ptr[I];
+    unsigned todo = __ballot_sync(0xffffffffu, open);
+    while (todo) {
+        const int l = __ffs(todo) - 1;
+        todo &= todo - 1;
+        pull_rowtile<NT>(Q, B, I0 + l, lane);
+    }
+}
+
 // Pull over the side matrix: in-neighbour list of local vertex v (CSC of A^T's side).
+// The visited bit is tested first (one coalesced word per 32 vertices), so a
+// visited vertex costs no read of the side structure.
 template <int NT>
 __device__ __forceinline__ void pull_side_vertex(const BfsTiles &Q, const BfsView &B, long long v) {
     using word_t = typename Tr<NT>::word_t;
-    long long p0 = Q.sptr[v], p1 = Q.sptr[v + 1];
-    if (p0 == p1) return;
     long long g = B.row_begin + v;
     if ((B.V[g >> 5] >> (g & 31)) & 1u) return;
+    long long p0 = Q.sptr[v], p1 = Q.sptr[v + 1];
+    if (p0 == p1) return;
     for (long long p = p0; p < p1; ++p) {
         long long u = decode_row<NT>(Q.srow[p], Q.hot_list);
         if ((B.F[u >> 5] >> (u & 31)) & 1u) {
             discover<NT>(B, g / NT, (word_t)1 << (g % NT));
             break;
         }
+    }
+}
+
+// Pull over the side matrix for the 32 vertices of visited word w (global word
+// index; only vertices in [row_begin, row_begin + m_local) are local).  Used by
+// the persistent kernel, whose few threads would otherwise walk the vertices
+// one by one: a fully visited word costs one load.
+template <int NT>
+__device__ __forceinline__ void pull_side_word(const BfsTiles &Q, const BfsView &B, long long w) {
+    uint32_t um = ~B.V[w];
+    while (um) {
+        const int r = __ffs(um) - 1;
+        um &= um - 1;
+        const long long v = w * 32 + r - B.row_begin;
+        if (v < 0 || v >= B.m_local) continue;
+        pull_side_vertex<NT>(Q, B, v);
     }
 }
 

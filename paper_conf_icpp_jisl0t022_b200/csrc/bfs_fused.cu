@@ -17,6 +17,18 @@
 //   -- barrier --
 // until the frontier is empty.  No host round trip per level (the per-level
 // kernels of bfs.cu remain for the distributed driver).
+//
+// List-driven push levels (high-diameter graphs: stencils, bands, late R-MAT
+// levels).  While the rule picks Push-CSC and no frontier vertex has more than
+// LIST_MAXW items of push work, a level is ONE phase and ONE grid barrier: a
+// group of G lanes per frontier vertex u (taken from the vertex list of the
+// level) ORs plane c = u % nt of every tile of u's tile column into V and walks
+// u's side column; each newly discovered vertex gets its level, is appended to
+// the next level's list through a per-CTA shared-memory queue and adds its
+// out-degree / in-degree / push work to the next level's counters (three
+// rotating slots).  The first level that needs the bitmap form (Pull-CSC,
+// Push-CSR or a heavy vertex) writes the list into the frontier bitmap and
+// continues with the 3-barrier scan levels above.
 #include "bfs_dev.cuh"
 
 namespace tsmv {
@@ -24,6 +36,8 @@ namespace tsmv {
 namespace {
 
 constexpr int BFB = 512;  // threads per CTA
+constexpr int LIST_MAXW = 512;   // list levels only while every frontier vertex has <= this much push work
+constexpr int QCAP = 2048;       // per-CTA shared-memory queue of discovered vertices
 
 struct BfsFusedArgs {
     BfsTiles P, Q;
@@ -44,7 +58,160 @@ struct BfsFusedArgs {
     // high-occupancy per-level kernels and resumes the kernel afterwards
     int resume, stop_on_pull;
     long long level0, mu0, reached0, edges0;
+    // list-driven push levels
+    const int *lwork;
+    int *bq0, *bq1;
+    long long *lslots;   // [3][4]
+    int use_list;
 };
+
+struct ListShared {
+    int qn, base, maxw, pad;
+    unsigned long long mf, din;
+    int q[QCAP];
+};
+
+// Discovery in a list level: V bits, levels and the CTA's queue.  Degrees are
+// read later, in parallel over the queue (list_flush), not in this serial loop.
+template <int NT>
+__device__ __forceinline__ void discover_list(const BfsFusedArgs &a, const BfsView &B, long long gseg,
+                                              typename Tr<NT>::word_t bits, ListShared &sh, int *Qn,
+                                              long long *slot_n) {
+    using word_t = typename Tr<NT>::word_t;
+    const word_t old = seg_or<NT>(B.V, gseg, bits);
+    word_t nw = bits & ~old;
+    if (!nw) return;
+    int p = atomicAdd(&sh.qn, popc_w(nw));
+    while (nw) {
+        const int r = ffs_w(nw);
+        nw &= nw - 1;
+        const long long v = gseg * NT + r;
+        B.levels[v] = B.level + 1;
+        if (p < QCAP) {
+            sh.q[p] = (int)v;
+        } else {  // queue full: straight to the global list and counters
+            const unsigned long long gp = atomicAdd((unsigned long long *)&slot_n[0], 1ull);
+            Qn[gp] = (int)v;
+            atomicAdd((unsigned long long *)&slot_n[1], (unsigned long long)a.outdeg[v]);
+            atomicAdd((unsigned long long *)&slot_n[2], (unsigned long long)a.indeg[v]);
+            atomicMax(&slot_n[3], (long long)a.lwork[v]);
+        }
+        ++p;
+    }
+}
+
+// End of a list level in one CTA: reserve the CTA's range of the next list,
+// copy the queue there and add its degrees / max work to the next slot.
+__device__ __forceinline__ void list_flush(const BfsFusedArgs &a, ListShared &sh, int *Qn, long long *slot_n,
+                                           int tid, int lane) {
+    __syncthreads();
+    const int qn = min(sh.qn, QCAP);
+    if (qn == 0) return;  // uniform: no __syncthreads skipped by part of the CTA
+    if (tid == 0) sh.base = (int)atomicAdd((unsigned long long *)&slot_n[0], (unsigned long long)qn);
+    __syncthreads();
+    unsigned long long mf = 0, din = 0;
+    int mx = 0;
+    for (int i = tid; i < qn; i += BFB) {
+        const int v = sh.q[i];
+        Qn[sh.base + i] = v;
+        mf += (unsigned long long)a.outdeg[v];
+        din += (unsigned long long)a.indeg[v];
+        mx = max(mx, a.lwork[v]);
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        mf += __shfl_xor_sync(0xffffffffu, mf, o);
+        din += __shfl_xor_sync(0xffffffffu, din, o);
+        mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+    }
+    if (lane == 0 && mf + din + (unsigned long long)mx) {
+        atomicAdd(&sh.mf, mf);
+        atomicAdd(&sh.din, din);
+        atomicMax(&sh.maxw, mx);
+    }
+    __syncthreads();
+    if (tid == 0) {
+        atomicAdd((unsigned long long *)&slot_n[1], sh.mf);
+        atomicAdd((unsigned long long *)&slot_n[2], sh.din);
+        atomicMax(&slot_n[3], (long long)sh.maxw);
+    }
+}
+
+// One list level: group of G lanes per frontier vertex.  A group takes LR
+// vertices at a time and issues each dependent step (list entry -> column
+// ranges -> first plane word / side row -> V) for all of them before the next,
+// so LR chains of loads are in flight per lane instead of one.
+#ifndef TSMV_LR
+#define TSMV_LR 1
+#endif
+constexpr int LR = TSMV_LR;
+
+template <int NT>
+__device__ __forceinline__ void list_level(const BfsFusedArgs &a, const BfsView &B, const int *Qc, long long fsize,
+                                           int G, long long gtid, long long gthreads, ListShared &sh, int *Qn,
+                                           long long *slot_n) {
+    using word_t = typename Tr<NT>::word_t;
+    const word_t *planes = (const word_t *)a.P.planes;
+    const long long ngroups = gthreads / G;
+    const long long gid = gtid / G;
+    const int gl = (int)(gtid % G);
+    for (long long i0 = gid; i0 < fsize; i0 += LR * ngroups) {
+        long long u[LR], t0[LR], ntl[LR], s0[LR], ns[LR];
+#pragma unroll
+        for (int r = 0; r < LR; ++r) {
+            const long long i = i0 + r * ngroups;
+            u[r] = i < fsize ? (long long)__ldcg(&Qc[i]) : -1;
+        }
+#pragma unroll
+        for (int r = 0; r < LR; ++r) {
+            t0[r] = ntl[r] = s0[r] = ns[r] = 0;
+            if (u[r] >= 0) {
+                const long long J = u[r] / NT;
+                t0[r] = __ldg(&a.P.ptr[J]);
+                ntl[r] = __ldg(&a.P.ptr[J + 1]) - t0[r];
+                s0[r] = __ldg(&a.P.sptr[u[r]]);
+                ns[r] = __ldg(&a.P.sptr[u[r] + 1]) - s0[r];
+            }
+        }
+        // first item of every vertex: loads for all LR vertices, then the ORs
+        word_t w[LR];
+        long long seg[LR];
+#pragma unroll
+        for (int r = 0; r < LR; ++r) {
+            w[r] = 0;
+            seg[r] = 0;
+            if (u[r] >= 0) {
+                if (gl < ntl[r]) {
+                    const long long t = t0[r] + gl;
+                    w[r] = __ldg(&planes[(long long)(u[r] % NT) * a.P.T + t]);
+                    seg[r] = __ldg(&a.P.trow[t]);
+                } else if (gl < ntl[r] + ns[r]) {
+                    const long long v = decode_row<NT>(__ldg(&a.P.srow[s0[r] + (gl - ntl[r])]), a.P.hot_list);
+                    w[r] = (word_t)1 << (v % NT);
+                    seg[r] = v / NT;
+                }
+            }
+        }
+#pragma unroll
+        for (int r = 0; r < LR; ++r)
+            if (w[r]) discover_list<NT>(a, B, seg[r], w[r], sh, Qn, slot_n);
+        // remaining items (vertices with more than G items of work)
+#pragma unroll 1
+        for (int r = 0; r < LR; ++r) {
+            const int c = (int)(u[r] % NT);
+            for (long long k = gl + G; k < ntl[r] + ns[r]; k += G) {
+                if (k < ntl[r]) {
+                    const long long t = t0[r] + k;
+                    const word_t ww = planes[(long long)c * a.P.T + t];
+                    if (ww) discover_list<NT>(a, B, (long long)a.P.trow[t], ww, sh, Qn, slot_n);
+                } else {
+                    const long long v = decode_row<NT>(a.P.srow[s0[r] + (k - ntl[r])], a.P.hot_list);
+                    discover_list<NT>(a, B, v / NT, (word_t)1 << (v % NT), sh, Qn, slot_n);
+                }
+            }
+        }
+    }
+}
 
 template <int NT>
 __device__ __forceinline__ void seg_counts(const BfsFusedArgs &a, const uint32_t *F, long long J, long long *v) {
@@ -69,7 +236,10 @@ __device__ __forceinline__ void seg_counts(const BfsFusedArgs &a, const uint32_t
 }
 
 template <int NT>
-__global__ void __launch_bounds__(BFB, 1) k_bfs_fused(BfsFusedArgs a) {
+#ifndef TSMV_BFS_MINB
+#define TSMV_BFS_MINB 1
+#endif
+__global__ void __launch_bounds__(BFB, TSMV_BFS_MINB) k_bfs_fused(BfsFusedArgs a) {
     using word_t = typename Tr<NT>::word_t;
     constexpr int NWP = BFB / 32;
     __shared__ long long s_scan[16][NWP];
@@ -83,18 +253,36 @@ __global__ void __launch_bounds__(BFB, 1) k_bfs_fused(BfsFusedArgs a) {
     BfsView B = a.B;
     uint32_t *Fa = B.F, *Fb = B.Fn;
 
-    // ---- init: V = padding bits + source, F0 = {source}, F1 = 0, levels
+    __shared__ ListShared sh;
+    int mode_list = a.use_list && !a.resume;
+
+    // ---- init: V = padding bits + source, F0 = {source} (scan mode) or the
+    // list {source} (list mode), F1 = 0, levels
     for (long long w = gtid; w < (a.resume ? 0 : a.NW); w += gthreads) {
         const long long v0 = w * 32;
         uint32_t pad = 0;
         if (v0 + 32 > B.n) pad = (v0 >= B.n) ? 0xffffffffu : (0xffffffffu << (B.n - v0));
         const uint32_t s = (a.source >= v0 && a.source < v0 + 32) ? (1u << (a.source - v0)) : 0u;
         B.V[w] = pad | s;
-        Fa[w] = s;
+        Fa[w] = mode_list ? 0u : s;
         Fb[w] = 0;
     }
     if (!a.resume)
         for (long long v = gtid; v < B.m_local; v += gthreads) B.levels[v] = (v == a.source) ? 0 : -1;
+    if (tid == 0) {
+        sh.qn = 0;
+        sh.maxw = 0;
+        sh.mf = 0;
+        sh.din = 0;
+    }
+    if (mode_list && b == 0 && tid == 0) {
+        a.bq0[0] = (int)a.source;
+        a.lslots[0] = 1;
+        a.lslots[1] = a.outdeg[a.source];
+        a.lslots[2] = a.indeg[a.source];
+        a.lslots[3] = a.lwork[a.source];
+        for (int i = 4; i < 12; ++i) a.lslots[i] = 0;
+    }
     grid_sync(&a.cnt->bar, target);
 
     long long mu = a.resume ? a.mu0 : a.nnz, reached = a.reached0, edges = a.edges0;
@@ -105,10 +293,84 @@ __global__ void __launch_bounds__(BFB, 1) k_bfs_fused(BfsFusedArgs a) {
     const long long tj0 = min(js1, js0 + tid * per), tj1 = min(js1, tj0 + per);
     int level = (int)a.level0;
     unsigned long long t_s1 = 0, t_s2 = 0, t_e = 0, tq = b == 0 && tid == 0 ? globaltimer_ns() : 0;
+    bool redo = false;  // scan pass over a level already counted in list mode
     for (; level < a.max_levels; ++level) {
         B.F = Fa;
         B.Fn = Fb;
         B.level = level;
+        if (mode_list) {
+            // ---- list level: counters of this level from its slot
+            const long long *sl = a.lslots + (level % 3) * 4;
+            const long long fsize = __ldcg(&sl[0]), mf = __ldcg(&sl[1]), din = __ldcg(&sl[2]),
+                            maxw = __ldcg(&sl[3]);
+            mu -= din;
+            if (fsize == 0) break;
+            reached += fsize;
+            edges += mf;
+            const int dir = choose_dir_dev(a.force, a.alpha, a.dens, B.n, fsize, mf, mu);
+            if (b == 0 && tid == 0) {
+                a.dir_out[level] = dir;
+                a.front_out[level] = fsize;
+            }
+            const int *Qc = (level & 1) ? a.bq1 : a.bq0;
+            if (dir != TSMV_DIR_PUSH_CSC || maxw > LIST_MAXW) {
+                // hand the level to the scan form: list -> frontier bitmap Fa
+                for (long long i = gtid; i < fsize; i += gthreads) {
+                    const long long v = __ldcg(&Qc[i]);
+                    atomicOr(&Fa[v >> 5], 1u << (v & 31));
+                }
+                grid_sync(&a.cnt->bar, target);
+                mode_list = 0;
+                redo = true;
+                --level;  // the loop increment brings it back
+                continue;
+            }
+            int *Qn = (level & 1) ? a.bq0 : a.bq1;
+            long long *slot_n = a.lslots + ((level + 1) % 3) * 4;
+            int G = 1;
+            while (G < maxw && G < 32) G <<= 1;
+#ifdef TSMV_LIST_PROF
+            unsigned long long tl0 = 0, tl1 = 0, tl2 = 0;
+            if (b == 0 && tid == 0) tl0 = globaltimer_ns();
+#endif
+            list_level<NT>(a, B, Qc, fsize, G, gtid, gthreads, sh, Qn, slot_n);
+#ifdef TSMV_LIST_PROF
+            __syncthreads();
+            if (b == 0 && tid == 0) tl1 = globaltimer_ns();
+            if (tid == 0) atomicMax((unsigned long long *)&a.lslots[12 + (level % 3)], globaltimer_ns());
+#endif
+            if (b == 0 && tid == 0) {
+                long long *sz = a.lslots + ((level + 2) % 3) * 4;
+                sz[0] = sz[1] = sz[2] = sz[3] = 0;
+            }
+            list_flush(a, sh, Qn, slot_n, tid, lane);
+            __syncthreads();
+            if (tid == 0) {
+                sh.qn = 0;
+                sh.maxw = 0;
+                sh.mf = 0;
+                sh.din = 0;
+            }
+#ifdef TSMV_LIST_PROF
+            if (b == 0 && tid == 0) tl2 = globaltimer_ns();
+#endif
+            grid_sync(&a.cnt->bar, target);
+            if (b == 0 && tid == 0) {
+                const unsigned long long t = globaltimer_ns();
+                t_e += t - tq;
+                tq = t;
+#ifdef TSMV_LIST_PROF
+                // t_s1: CTA 0 expansion, t_s2: slowest CTA's expansion end - CTA 0 start,
+                // lslots[15]: CTA 0 flush
+                t_s1 += tl1 - tl0;
+                unsigned long long *cell = (unsigned long long *)&a.lslots[12 + (level % 3)];
+                t_s2 += __ldcg(cell) - tl0;
+                a.lslots[15] += (long long)(tl2 - tl1);
+                *(unsigned long long *)&a.lslots[12 + ((level + 2) % 3)] = 0;
+#endif
+            }
+            continue;
+        }
         // ---- S: count this thread's segments, clear the consumed bitmap Fb
         long long v[8] = {0, 0, 0, 0, 0, 0, 0, 0};
         for (long long J = tj0; J < tj1; ++J) {
@@ -158,16 +420,22 @@ __global__ void __launch_bounds__(BFB, 1) k_bfs_fused(BfsFusedArgs a) {
         }
         __syncthreads();
         const long long fsize = s_tot[4], mf = s_tot[5];
-        mu -= s_tot[6];
+        if (!redo) mu -= s_tot[6];
         if (fsize == 0) break;
-        reached += fsize;
-        edges += mf;
+        if (!redo) {
+            reached += fsize;
+            edges += mf;
+        }
+        redo = false;
         const int dir = choose_dir_dev(a.force, a.alpha, a.dens, B.n, fsize, mf, mu);
         if (b == 0 && tid == 0) {
             a.dir_out[level] = dir;
             a.front_out[level] = fsize;
         }
-        if (dir == TSMV_DIR_PULL_CSC && a.stop_on_pull) {
+        // Pull levels go back to the host's high-occupancy kernels unless few
+        // edges are left unvisited (m_u <= 16 per thread of this grid: small
+        // graphs, the tail of a high-diameter traversal)
+        if (dir == TSMV_DIR_PULL_CSC && a.stop_on_pull && mu > 16 * gthreads) {
             stopped = 1;  // uniform across CTAs: same totals, same decision
             break;
         }
@@ -217,8 +485,9 @@ __global__ void __launch_bounds__(BFB, 1) k_bfs_fused(BfsFusedArgs a) {
 
         // ---- E: expand
         if (dir == TSMV_DIR_PULL_CSC) {
-            for (long long I = gwarp; I < a.nTR_local; I += gwarps) pull_rowtile<NT>(a.Q, B, I, lane);
-            for (long long u = gtid; u < B.m_local; u += gthreads) pull_side_vertex<NT>(a.Q, B, u);
+            for (long long I0 = gwarp * 32; I0 < a.nTR_local; I0 += gwarps * 32)
+                pull_rowtiles32<NT>(a.Q, B, I0, a.nTR_local, lane);
+            for (long long w = gtid; w < (B.m_local + 31) / 32; w += gthreads) pull_side_word<NT>(a.Q, B, w);
         } else {
             if (dir == TSMV_DIR_PUSH_CSR)
                 for (long long t = gtid; t < a.Q.T; t += gthreads) push_csr_item<NT>(a.Q, B, t);
@@ -284,10 +553,35 @@ __global__ void __launch_bounds__(BFB, 1) k_bfs_fused(BfsFusedArgs a) {
         a.hm->Wt = (long long)t_s1;  // phase times (ns, CTA 0): count, lists, expand
         a.hm->nLs = (long long)t_s2;
         a.hm->Ws = (long long)t_e;
+        a.hm->bfs_bars = target - a.bar_base;  // = G x barriers passed
+    }
+}
+
+// lwork[u] = tiles of u's tile column + u's side nonzeros (push work of u in a list level)
+__global__ void k_lwork(const long long *__restrict__ ptr, const long long *__restrict__ sptr, int lognt,
+                        long long n, int *__restrict__ lwork) {
+    for (long long u = blockIdx.x * (long long)blockDim.x + threadIdx.x; u < n;
+         u += (long long)gridDim.x * blockDim.x) {
+        const long long J = u >> lognt;
+        const long long w = (ptr[J + 1] - ptr[J]) + (sptr[u + 1] - sptr[u]);
+        lwork[u] = (int)min(w, (long long)INT_MAX);
     }
 }
 
 }  // namespace
+
+void bfs_list_init(tsmv_ctx *c, cudaStream_t st) {
+    c->lwork.alloc(std::max<int64_t>(c->n, 1) * 4);
+    c->bq0.alloc(std::max<int64_t>(c->n, 1) * 4);
+    c->bq1.alloc(std::max<int64_t>(c->n, 1) * 4);
+    c->lslots.alloc(16 * 8);
+    TSMV_CUDA(cudaMemsetAsync(c->lslots.p, 0, c->lslots.bytes, st));
+    const long long n = c->n;
+    const int grid = (int)std::max<long long>(1, std::min<long long>((n + 255) / 256, 148LL * 16));
+    k_lwork<<<grid, 256, 0, st>>>(c->P.ptr.as<long long>(), c->P.sptr.as<long long>(), c->lognt, n,
+                                  c->lwork.as<int>());
+    TSMV_CUDA(cudaGetLastError());
+}
 
 int bfs_fused_occupancy(int nt) {
     int bps = 0;
@@ -343,6 +637,11 @@ bool bfs_fused_launch(tsmv_ctx *c, long long source, cudaStream_t st, bool resum
     a.mu0 = mu;
     a.reached0 = reached;
     a.edges0 = edges;
+    a.lwork = c->lwork.as<int>();
+    a.bq0 = c->bq0.as<int>();
+    a.bq1 = c->bq1.as<int>();
+    a.lslots = c->lslots.as<long long>();
+    a.use_list = (c->lwork.p != nullptr && !getenv("TSMV_BFS_NO_LIST")) ? 1 : 0;
     void *args[] = {&a};
     void *f = c->nt == 16 ? (void *)k_bfs_fused<16> : c->nt == 32 ? (void *)k_bfs_fused<32> : (void *)k_bfs_fused<64>;
     const int G = c->bfs_blocks;
@@ -356,10 +655,7 @@ bool bfs_fused_launch(tsmv_ctx *c, long long source, cudaStream_t st, bool resum
     edges_out = h->edges;
     mu_out = h->mf;
     cur_out = (int)h->nLt;
-    // barriers: 1 (init) + 3 per expanded level + 1 for the final scan (empty frontier or pull stop)
-    const long long expanded = L - level0;
-    const long long nbar = 1 + 3 * expanded + ((L < max_levels) ? 1 : 0);
-    c->bar_base += (unsigned long long)nbar * (unsigned long long)G;
+    c->bar_base += h->bfs_bars;
     return stopped;
 }
 

@@ -160,6 +160,7 @@ struct Counters {
     unsigned long long resv_t;     // flat SpMSpV list reservation: (entries << 40) | tile work
     unsigned long long resv_s;     // (entries << 37) | side work; reset at the end of each call
     unsigned long long nhits;      // flat SpMSpV: hit tiles appended in phase B1
+    unsigned long long bfs_bars;   // fused BFS: grid barriers the last launch passed
 };
 
 template <int K> struct LBDesc {
@@ -294,6 +295,10 @@ struct tsmv_ctx {
     int bfs_blocks = 0;            // CTAs of the fused BFS kernel
     long long bfs_last_levels = 0;
     tsmv::DevBuf bfs_dirs, bfs_front;  // per-level direction / frontier size (device)
+    // list-driven push levels of the fused BFS kernel
+    tsmv::DevBuf lwork;        // int32[n]: push work of vertex u = tiles of its tile column + its side nonzeros
+    tsmv::DevBuf bq0, bq1;     // int32[n]: frontier vertex lists, ping-pong by level parity
+    tsmv::DevBuf lslots;       // long long[3][4]: {|F|, m_f, sum indeg, max lwork} of levels L, L+1, L+2
     void *trace = nullptr;         // tsmv_set_trace (device, u64[tsmv_trace_words])
 };
 
@@ -323,6 +328,7 @@ void enqueue_spmspv_flat(tsmv_ctx *c, int sr, long long k, const int32_t *xi, co
                          int32_t *yi, void *yv, long long *ynnz_dev, cudaStream_t st);
 // bfs_fused.cu
 int bfs_fused_occupancy(int nt);
+void bfs_list_init(tsmv_ctx *c, cudaStream_t st);
 bool bfs_fused_launch(tsmv_ctx *c, long long source, cudaStream_t st, bool resume, long long level0, uint32_t *Fa,
                       uint32_t *Fb, long long mu, long long reached, long long edges, bool stop_on_pull,
                       long long max_levels, long long &level_out, long long &mu_out, long long &reached_out,

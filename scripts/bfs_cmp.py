@@ -9,6 +9,8 @@ def graph(name):
         return synth.rmat(int(name[4:]), 16, seed=1, symmetrize=True, device=dev)
     if name.startswith("grid3d"):
         return synth.stencil3d(int(name[6:]), device=dev).with_values(None)
+    if name.startswith("grid2d"):
+        return synth.stencil2d(int(name[6:]), int(name[6:]), device=dev).with_values(None)
     if name.startswith("band"):
         n, b = name[4:].split("_")
         return synth.banded(1 << int(n), int(b), device=dev).with_values(None)
@@ -16,8 +18,9 @@ for name in sys.argv[1:]:
     A = graph(name)
     M = tsmv.TiledMatrix.from_csr(A, dtype="pattern")
     lv = torch.empty(A.n, dtype=torch.int32, device=dev)
-    for mode in ("hybrid", "fusedonly", "hostloop"):
-        os.environ.pop("TSMV_BFS_HOSTLOOP", None); os.environ.pop("TSMV_BFS_FUSED_ONLY", None)
+    for mode in os.environ.get("MODES", "hybrid,nolist,hostloop").split(","):
+        for e in ("TSMV_BFS_HOSTLOOP", "TSMV_BFS_FUSED_ONLY", "TSMV_BFS_NO_LIST"): os.environ.pop(e, None)
+        if mode == "nolist": os.environ["TSMV_BFS_NO_LIST"] = "1"
         if mode == "hostloop": os.environ["TSMV_BFS_HOSTLOOP"] = "1"
         if mode == "fusedonly": os.environ["TSMV_BFS_FUSED_ONLY"] = "1"
         M.bfs(0, levels=lv)

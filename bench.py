@@ -55,7 +55,17 @@ def parse():
     p.add_argument("--no-cpu", action="store_true")
     p.add_argument("--cpu-seconds", type=float, default=12.0)
     p.add_argument("--no-configs", action="store_true", help="skip the per-config table (C1, C2, C4)")
-    return p.parse_args()
+    p.add_argument("--scaling", default="weak", choices=["weak", "strong"],
+                   help="weak (default): at N ranks the R-MAT scales grow by log2 N, so the nonzeros "
+                        "per GPU stay fixed; strong: the same matrix at every N")
+    a = p.parse_args()
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    a.base_scale, a.base_bfs_scale = a.scale, a.bfs_scale
+    if a.scaling == "weak" and world > 1:
+        grow = int(round(math.log2(world)))
+        a.scale += grow
+        a.bfs_scale += grow
+    return a
 
 
 def peaks():
@@ -160,7 +170,7 @@ def run_reference(args):
     val = flops / tsum / 1e9
     line = {"impl": "reference", "metric": "spmspv_gflops", "value": round(val, 4), "unit": "GFLOP/s",
             "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
-            "ms_per_step": round(1e3 * tsum / args.steps, 4), "higher_is_better": True, "scaling": "strong",
+            "ms_per_step": round(1e3 * tsum / args.steps, 4), "higher_is_better": True, "scaling": args.scaling,
             "vs_baseline": None, "dtype": args.dtype, "data": "synthetic",
             "config": workload_config(args),
             "cpu_baseline": {"value": round(val, 4), "unit": "GFLOP/s", "cores": 1, "kind": "oracle",
@@ -175,7 +185,10 @@ def workload_config(args):
             "matrix": f"R-MAT scale {args.scale}, edgefactor 16, (0.57,0.19,0.19,0.05), unpermuted, coalesced",
             "x_density": args.density, "tile_dim": args.tile_dim, "sparse_tile_max_nnz": args.thr,
             "l2": "flushed before every step (256 MiB write + 256 MiB read of another buffer, outside the events)",
-            "parallelism": f"row-block x{args.gpus}" if args.gpus > 1 else "single GPU"}
+            "parallelism": f"row-block x{args.gpus}" if args.gpus > 1 else "single GPU",
+            "scaling_rule": (f"weak: R-MAT scale {args.base_scale} + log2(N) for SpMSpV, {args.base_bfs_scale} + log2(N) "
+                             "for TileBFS (nonzeros per GPU fixed)") if args.scaling == "weak"
+                            else "strong: same matrix at every N"}
 
 
 # --------------------------------------------------------------------------- our arm
@@ -276,9 +289,16 @@ def survey_bytes(st, k, sv, nt, macs):
 
 def run_tsmv(args):
     world, rank, local = dist_env()
+    # TSMV_DIST_BACKEND=gloo lets the N > 1 path run with several ranks on one
+    # GPU (logic check only; NCCL refuses two ranks on one device)
+    local = local % max(1, torch.cuda.device_count())
     if world > 1:
         import torch.distributed as dist
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        be = os.environ.get("TSMV_DIST_BACKEND", "nccl")
+        if be == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(be)
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     from paper_conf_icpp_jisl0t022_b200 import tsmv
@@ -409,6 +429,9 @@ def run_tsmv(args):
     bfs = None
     if not args.no_bfs and world == 1:
         bfs = run_bfs(args, dev, flush, tsmv)
+    elif not args.no_bfs:
+        del D, M
+        bfs = run_bfs_dist(args, dev, flush, rank, world)
     configs = None
     if not args.no_configs and world == 1:
         del M
@@ -422,7 +445,7 @@ def run_tsmv(args):
         mean_st = {kk: sum(s_[kk] for s_ in step_stats) / len(step_stats) for kk in step_stats[0]}
         line = {"metric": "spmspv_gflops", "value": round(value, 3), "unit": "GFLOP/s", "n_gpus": world,
                 "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms / args.steps, 5),
-                "higher_is_better": True, "scaling": "strong",
+                "higher_is_better": True, "scaling": args.scaling,
                 "vs_baseline": None, "dtype": args.dtype, "data": "synthetic (seeded R-MAT, seeded x)",
                 "config": workload_config(args), "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,
                 "gpu_launches": args.steps, "clocks": clk,
@@ -457,11 +480,66 @@ def run_bfs(args, dev, flush, tsmv):
                      "dirs": "".join({"push_csc": "C", "push_csr": "R", "pull_csc": "P"}.get(d, "?")
                                      for d in st["dirs"])})
     hm = len(runs) / sum(1.0 / r["gteps"] for r in runs if r["gteps"] > 0)
+    # min-id parents (MIN_SECOND semiring) of the last traversal, device time
+    parents = torch.empty(A.n, dtype=torch.int32, device=dev)
+    M.bfs_parents(levels, parents)
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    flush()
+    e0.record()
+    M.bfs_parents(levels, parents)
+    e1.record()
+    torch.cuda.synchronize()
+    par_ms = e0.elapsed_time(e1)
     M.close()
     return {"graph": f"rmat_s{args.bfs_scale}_ef16_sym", "nnz": info["nnz"], "gteps_hmean": round(hm, 3),
+            "parents_ms": round(par_ms, 4),
             "build_ms": round(info["build_ms"], 2), "build_wall_s": round(build_wall, 3),
             "edge_count": "sum of out-degrees of reached vertices (directed count of the symmetrised graph)",
             "runs": runs}
+
+
+def run_bfs_dist(args, dev, flush, rank, world):
+    """Row-block partitioned TileBFS on the symmetrised R-MAT: each
+    rank builds its nnz-balanced row block; one NCCL all-gather of the owned
+    frontier bitmaps + one all-reduce of (m_f, m_u) per level.  Time = max over
+    ranks of the CUDA-event time of the traversal; edges = sum of out-degrees of
+    the reached vertices (all ranks)."""
+    import torch.distributed as dist
+    from paper_conf_icpp_jisl0t022_b200 import dist as tdist
+    A = synth.rmat(args.bfs_scale, 16, seed=1, symmetrize=True, device=dev)
+    srcs = [0] + synth.sample_sources(A, max(0, args.bfs_sources - 1), seed=1)
+    splits = tdist.partition_rows(A.row_ptr, world)
+    Al = tdist.local_rows(A, splits, rank)
+    nnz = A.nnz
+    del A
+    t0 = time.perf_counter()
+    D = tdist.DistTiledMatrix(Al, splits, rank, world, dtype="pattern", device=dev.index,
+                              tile_dim=args.tile_dim, sparse_tile_max_nnz=args.thr)
+    build_wall = time.perf_counter() - t0
+    rowlen = (Al.row_ptr[1:] - Al.row_ptr[:-1]).to(torch.int64)
+    D.bfs(srcs[0])  # warm-up
+    runs = []
+    for s in srcs:
+        flush()
+        torch.cuda.synchronize()
+        dist.barrier()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        lv, nl = D.bfs(s)
+        e1.record()
+        torch.cuda.synchronize()
+        t = torch.tensor([e0.elapsed_time(e1)], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        red = torch.stack([(rowlen * (lv >= 0)).sum(), (lv >= 0).sum()]).to(torch.int64)
+        dist.all_reduce(red)
+        ms, edges = float(t), int(red[0])
+        runs.append({"source": int(s), "ms": round(ms, 4), "levels": int(nl), "edges": edges,
+                     "reached": int(red[1]), "gteps": round(edges / (ms * 1e-3) / 1e9, 3)})
+    hm = len(runs) / sum(1.0 / r["gteps"] for r in runs if r["gteps"] > 0)
+    return {"graph": f"rmat_s{args.bfs_scale}_ef16_sym", "nnz": nnz, "gteps_hmean": round(hm, 3),
+            "partition": f"row blocks x{world} (nnz-balanced)", "build_wall_s": round(build_wall, 3),
+            "edge_count": "sum of out-degrees of reached vertices (directed count of the symmetrised graph)",
+            "time": "CUDA events around the whole traversal, max over ranks", "runs": runs}
 
 
 def spmspv_gflops(M, A, dtype, density, flush, steps=5, warm=2):

@@ -187,6 +187,20 @@ tsmv_status tsmv_last_call_stats(tsmv_ctx *c, tsmv_call_stats *s);
 tsmv_status tsmv_bfs(tsmv_ctx *c, int64_t source, int32_t *levels, tsmv_bfs_stats *stats,
                      void *cuda_stream);
 
+/* BFS tree over the min-second semiring (the semiring the paper
+ * lists for BFS-type SpMSpV).  Given the levels of a
+ * finished tsmv_bfs on this ctx, writes
+ *   parents[v] = min { u : A[v][u] stored (edge u -> v) and levels[u] == levels[v] - 1 },
+ *   parents[source] = source, parents[v] = -1 when levels[v] == -1,
+ * i.e. what Alg 3 yields with x_j = j over MIN_SECOND: a unique,
+ * Graph500-valid tree.
+ *   levels  : int32[nrows] device, as written by tsmv_bfs (not modified).
+ *   parents : int32[nrows] device out, caller-owned.
+ * Enqueued on cuda_stream, not synchronised.  Single-GPU contexts with BFS
+ * structures only.  Errors: EINVAL (NULL, host pointers, distributed ctx, no
+ * BFS structures), ECUDA. */
+tsmv_status tsmv_bfs_parents(tsmv_ctx *c, const int32_t *levels, int32_t *parents, void *cuda_stream);
+
 /* ---- distributed TileBFS (row-block partition, Sec 8(e) of SURVEY / DESIGN.md) ----
  * Each rank owns global rows [row_splits[rank], row_splits[rank+1]).  Per level:
  *   tsmv_bfs_dist_expand  -> this rank's newly discovered owned vertices as a bitmap

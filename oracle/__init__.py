@@ -127,6 +127,17 @@ def bfs_alg3(C: CSC, source: int) -> np.ndarray:
     return levels[:C.n]
 
 
+def bfs_parents(C: CSC, source: int):
+    """Alg 3 over MIN_SECOND: (levels, min-id parents)."""
+    levels = np.zeros(max(C.n, 1), np.int32)
+    parents = np.zeros(max(C.n, 1), np.int32)
+    f = _L().oracle_bfs_parents
+    f.restype = ctypes.c_int
+    _chk(f(ctypes.c_int64(C.n), _p(C.col_ptr), _p(C.row_idx), ctypes.c_int64(source), _p(levels), _p(parents)),
+         "bfs_parents")
+    return levels[:C.n], parents[:C.n]
+
+
 def tile_vector(n, nt, x_idx, x_val):
     """Fig 3 tiled sparse vector: returns (x_ptr int64[ceil(n/nt)], x_tile float64)."""
     x_idx = _np(x_idx, np.int32)

@@ -241,6 +241,57 @@ __global__ void __launch_bounds__(256) k_pull_side(BfsTiles Q, BfsView B) {
         pull_side_vertex<NT>(Q, B, v);
 }
 
+// BFS parents over the min-second semiring:
+// parent[v] = min { u : edge u -> v (A[v][u] stored), levels[u] = levels[v] - 1 },
+// parent[source] = source, -1 if unreachable.  One warp per vertex: the lanes
+// walk v's row words in the row structure Q (tiles ascending by tile column, so
+// the first round of 32 tiles with a candidate holds the smallest one), then
+// v's side row, keeping the minimum.
+template <int NT>
+__global__ void __launch_bounds__(256) k_parents(BfsTiles Q, const int32_t *__restrict__ levels,
+                                                 int32_t *__restrict__ parents, long long m) {
+    using word_t = typename Tr<NT>::word_t;
+    const word_t *planes = (const word_t *)Q.planes;
+    const int lane = threadIdx.x & 31;
+    const long long warp = (blockIdx.x * (long long)blockDim.x + threadIdx.x) >> 5;
+    const long long nwarps = ((long long)gridDim.x * blockDim.x) >> 5;
+    for (long long v = warp; v < m; v += nwarps) {
+        const int L = levels[v];
+        if (L <= 0) {
+            if (lane == 0) parents[v] = (L == 0) ? (int32_t)v : -1;
+            continue;
+        }
+        const long long I = v / NT;
+        const int r = (int)(v % NT);
+        int best = INT_MAX;
+        const long long t0 = Q.ptr[I], t1 = Q.ptr[I + 1];
+        for (long long tb = t0; tb < t1 && best == INT_MAX; tb += 32) {
+            const long long t = tb + lane;
+            int cand = INT_MAX;
+            if (t < t1) {
+                word_t w = planes[(long long)r * Q.T + t];
+                const long long base = (long long)Q.trow[t] * NT;
+                while (w) {
+                    const int c = ffs_w(w);
+                    w &= w - 1;
+                    if (levels[base + c] == L - 1) {
+                        cand = (int)(base + c);
+                        break;
+                    }
+                }
+            }
+            best = __reduce_min_sync(0xffffffffu, cand);
+        }
+        int sb = best;
+        for (long long p = Q.sptr[v] + lane; p < Q.sptr[v + 1]; p += 32) {
+            const long long u = decode_row<NT>(Q.srow[p], Q.hot_list);
+            if (u < sb && levels[u] == L - 1) sb = (int)u;
+        }
+        sb = __reduce_min_sync(0xffffffffu, sb);
+        if (lane == 0) parents[v] = sb == INT_MAX ? -1 : sb;
+    }
+}
+
 __global__ void k_merge(const uint32_t *__restrict__ gathered, long long stride, int nranks,
                         const long long *__restrict__ splits, int self, uint32_t *__restrict__ Fn,
                         uint32_t *__restrict__ V) {
@@ -501,6 +552,27 @@ extern "C" tsmv_status tsmv_bfs(tsmv_ctx *c, int64_t source, int32_t *levels, ts
             stats->edges_traversed = edges;
             stats->ms = ms;
         }
+        return TSMV_OK;
+    } catch (const Err &e) {
+        return e.st;
+    }
+}
+
+extern "C" tsmv_status tsmv_bfs_parents(tsmv_ctx *c, const int32_t *levels, int32_t *parents, void *cuda_stream) {
+    try {
+        TSMV_REQUIRE(c != nullptr && levels != nullptr && parents != nullptr, "tsmv_bfs_parents: NULL argument");
+        bfs_check(c);
+        TSMV_REQUIRE(c->opt.nranks == 1, "tsmv_bfs_parents: single-GPU contexts only");
+        TSMV_REQUIRE(is_device_ptr(levels) && is_device_ptr(parents),
+                     "tsmv_bfs_parents: levels and parents must be device memory");
+        TSMV_CUDA(cudaSetDevice(c->device));
+        cudaStream_t st = (cudaStream_t)cuda_stream;
+        BfsTiles Q = bfs_tiles(*c->Q);
+        const int grid = grid_for(c->m * 32);
+        if (c->nt == 16) k_parents<16><<<grid, 256, 0, st>>>(Q, levels, parents, c->m);
+        else if (c->nt == 32) k_parents<32><<<grid, 256, 0, st>>>(Q, levels, parents, c->m);
+        else k_parents<64><<<grid, 256, 0, st>>>(Q, levels, parents, c->m);
+        TSMV_CUDA(cudaGetLastError());
         return TSMV_OK;
     } catch (const Err &e) {
         return e.st;

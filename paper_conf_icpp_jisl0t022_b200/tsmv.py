@@ -77,6 +77,7 @@ _SIGS = {
     "tsmv_get_timing": (ctypes.c_int, [_vp, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(_i64)]),
     "tsmv_last_call_stats": (ctypes.c_int, [_vp, ctypes.POINTER(tsmv_call_stats)]),
     "tsmv_bfs": (ctypes.c_int, [_vp, _i64, _vp, ctypes.POINTER(tsmv_bfs_stats), _vp]),
+    "tsmv_bfs_parents": (ctypes.c_int, [_vp, _vp, _vp, _vp]),
     "tsmv_bfs_dist_begin": (ctypes.c_int, [_vp, _i64, _vp, ctypes.POINTER(_i64), _vp]),
     "tsmv_bfs_dist_expand": (ctypes.c_int, [_vp, _i32, _vp, _vp]),
     "tsmv_bfs_dist_merge": (ctypes.c_int, [_vp, _vp, _i64, ctypes.POINTER(_i64), _vp]),
@@ -226,6 +227,13 @@ class TiledMatrix:
              "dirs": [DIR_NAMES.get(stats.dir_per_level[i], "?") for i in range(min(L, MAX_LEVELS))],
              "frontier": [stats.frontier_per_level[i] for i in range(min(L, MAX_LEVELS))]}
         return levels, d
+
+    def bfs_parents(self, levels: torch.Tensor, parents: Optional[torch.Tensor] = None, stream=None):
+        """Min-id BFS parents (min-second semiring) from the levels of a finished bfs()."""
+        if parents is None:
+            parents = torch.empty(self.m, dtype=torch.int32, device=self.device)
+        check(tsmv_bfs_parents(self.ctx, _ptr(levels), _ptr(parents), _stream(stream)), "tsmv_bfs_parents")
+        return parents
 
     # -- introspection -----------------------------------------------------------
     def info(self) -> dict:

@@ -119,3 +119,31 @@ def test_c3_rmat_s20_sym_directions(tsmv):
 def test_c3_rmat_s22_sym(tsmv):
     A = synth.rmat(22, 16, seed=1, symmetrize=True, device=DEV).to("cpu")
     _levels(tsmv, A, [0], dirs=[0])
+
+
+@pytest.mark.parametrize("nt", [16, 32, 64])
+@pytest.mark.parametrize("sym", [True, False])
+def test_bfs_parents_min_second(tsmv, nt, sym):
+    """tsmv_bfs_parents == oracle_bfs_parents (Alg 3 over MIN_SECOND), bit-exact."""
+    A = synth.rmat(12, 16, seed=3, symmetrize=sym)
+    C = oracle.csc_of(A)
+    M = tsmv.TiledMatrix.from_csr(A.to(DEV), dtype="pattern", tile_dim=nt)
+    for s in [0] + synth.sample_sources(A, 2, seed=4):
+        lv, _ = M.bfs(s)
+        par = M.bfs_parents(lv)
+        rl, rp = oracle.bfs_parents(C, s)
+        assert np.array_equal(lv.cpu().numpy(), rl)
+        got = par.cpu().numpy()
+        assert np.array_equal(got, rp), f"src={s}: {np.sum(got != rp)} parents differ"
+    M.close()
+
+
+def test_bfs_parents_grid_and_3d(tsmv):
+    for A in (synth.stencil2d(64, 64), synth.stencil3d(24), synth.banded(3000, 7)):
+        A = A.with_values(None)
+        M = tsmv.TiledMatrix.from_csr(A.to(DEV), dtype="pattern")
+        lv, _ = M.bfs(0)
+        got = M.bfs_parents(lv).cpu().numpy()
+        _, rp = oracle.bfs_parents(oracle.csc_of(A), 0)
+        assert np.array_equal(got, rp)
+        M.close()

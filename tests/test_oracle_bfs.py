@@ -102,3 +102,66 @@ def test_fig5_levels():
     lv = _levels_both(A, 0)
     for L, verts in enumerate(g["levels_sets"]):
         assert sorted(np.nonzero(lv == L)[0].tolist()) == verts
+
+
+# ---------------------------------------------------------------- min-id parents (NEXT-2)
+# oracle_bfs_parents follows Alg 3 over MIN_SECOND.
+# Pins: closed forms (path, 2D grid), a hand-worked diamond, and -- on R-MAT,
+# directed and symmetric -- the Graph500 parent rules plus minimality, checked
+# from the CSR rows with numpy (no oracle code involved).
+
+def _csr(n, edges):
+    """A[v][u] = 1 for every edge u -> v (column u holds u's out-neighbours)."""
+    r = np.array([v for u, v in edges], np.int64)
+    c = np.array([u for u, v in edges], np.int64)
+    M = sp.csr_matrix((np.ones(len(edges)), (r, c)), shape=(n, n))
+    M.sum_duplicates()
+    M.sort_indices()
+    return synth.CSR(n, n, _t(M.indptr, "int64"), _t(M.indices, "int32"), None, "toy")
+
+
+def _t(a, dt):
+    import torch
+    return torch.from_numpy(np.ascontiguousarray(a).astype(dt))
+
+
+def test_parents_path_closed_form():
+    n = 50
+    A = _csr(n, [(i, i + 1) for i in range(n - 1)])
+    lv, par = oracle.bfs_parents(oracle.csc_of(A), 0)
+    assert np.array_equal(lv, np.arange(n))
+    assert np.array_equal(par, np.r_[0, np.arange(n - 1)])
+
+
+def test_parents_diamond_hand_worked():
+    # 0 -> 2, 0 -> 1, 2 -> 3, 1 -> 3, 3 -> 4, 1 -> 4 ; 5 isolated
+    A = _csr(6, [(0, 2), (0, 1), (2, 3), (1, 3), (3, 4), (1, 4)])
+    lv, par = oracle.bfs_parents(oracle.csc_of(A), 0)
+    assert lv.tolist() == [0, 1, 1, 2, 2, -1]
+    # vertex 3: in-neighbours 1 and 2 on layer 1 -> 1; vertex 4: 1 (layer 1) beats 3 (layer 2)
+    assert par.tolist() == [0, 0, 0, 1, 1, -1]
+
+
+def test_parents_grid_closed_form():
+    A = synth.stencil2d(64, 64)
+    lv, par = oracle.bfs_parents(oracle.csc_of(A), 0)
+    v = np.arange(4096)
+    assert np.array_equal(lv, v // 64 + v % 64)
+    want = np.where(v >= 64, v - 64, v - 1)
+    want[0] = 0
+    assert np.array_equal(par, want)
+
+
+@pytest.mark.parametrize("sym", [True, False])
+def test_parents_graph500_rules_and_minimal(sym):
+    A = synth.rmat(10, 16, seed=5, symmetrize=sym)
+    C = oracle.csc_of(A)
+    for s in [0] + synth.sample_sources(A, 3, seed=2):
+        lv, par = oracle.bfs_parents(C, s)
+        assert np.array_equal(lv, oracle.bfs_queue(C, s))
+        rp, ci = A.row_ptr.numpy(), A.col_idx.numpy()
+        assert par[s] == s and np.all(par[lv < 0] == -1)
+        for v in np.nonzero(lv > 0)[0]:
+            ins = ci[rp[v]:rp[v + 1]]                      # u with A[v][u]: edges u -> v
+            ok = ins[lv[ins] == lv[v] - 1]
+            assert ok.size > 0 and par[v] == ok.min(), f"v={v}"

@@ -304,6 +304,7 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
     __shared__ long long s_hpre[MAXG + 1];
     __shared__ unsigned long long s_pc[KP];
     __shared__ long long s_pbase[KP], s_ex0[KP];
+    __shared__ int s_nd;  // dense bitmap words of the current C2 round
     __shared__ long long s_heavy[HEAVY_CAP][3];  // chunk-map runs too long for one thread: c0, c1, list | kind
     const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
     const int G = gridDim.x, b = blockIdx.x;
@@ -825,6 +826,10 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
     __syncthreads();
     const long long ycap = a.y_cap;
     const int nround = (int)((PS + PSR - 1) / PSR);
+    long long *s_dw = s_win;                                     // phase-B windows are free now
+    long long *s_dpos = s_winb;
+    unsigned *s_dbits = reinterpret_cast<unsigned *>(s_winx);
+    if (tid == 0) s_nd = 0;
     for (int rd = 0; rd < nround; ++rd) {
         const long long w = pw0 + (long long)rd * PSR + tp;
         CSTEP(0, 0);
@@ -876,37 +881,37 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
                 }
             }
         }
-        const long long wbase = w - lane;
+        // dense words (> SPW set rows) go to a CTA list and are emitted by all warps
+        // of the CTA, BATCH words per warp and round, lane l handling row l
+        // (coalesced acc loads and y stores): a dense stretch of y owned by a few
+        // threads of one piece is spread over the whole CTA
+        if (pc > SPW) {
+            const int q = atomicAdd(&s_nd, 1);
+            s_dw[q] = w;
+            s_dpos[q] = pos0;
+            s_dbits[q] = bits;
+        }
+        __syncthreads();
+        const int nd = s_nd;
         const unsigned lt = (1u << lane) - 1u;
-        unsigned todo = __ballot_sync(0xffffffffu, pc > SPW);
-        while (todo) {
-            int src[BATCH];
-            int nb = 0;
-#pragma unroll
-            for (int kk = 0; kk < BATCH; ++kk) {
-                src[kk] = 0;
-                if (todo) {
-                    src[kk] = __ffs(todo) - 1;
-                    todo &= todo - 1;
-                    nb = kk + 1;
-                }
-            }
-            unsigned wb[BATCH];
+        for (int q0 = wid * BATCH; q0 < nd; q0 += NWF * BATCH) {
+            long long wq[BATCH];
+            unsigned bq[BATCH];
             double v[BATCH];
             bool mine[BATCH];
 #pragma unroll
             for (int kk = 0; kk < BATCH; ++kk) {
-                wb[kk] = __shfl_sync(0xffffffffu, bits, src[kk]);
-                mine[kk] = kk < nb && ((wb[kk] >> lane) & 1u);
-                if (mine[kk]) v[kk] = __ldcg(&a.acc[(wbase + src[kk]) * 32 + lane]);
+                const int q = q0 + kk;
+                wq[kk] = q < nd ? s_dw[q] : 0;
+                bq[kk] = q < nd ? s_dbits[q] : 0u;
+                mine[kk] = (bq[kk] >> lane) & 1u;
+                if (mine[kk]) v[kk] = __ldcg(&a.acc[wq[kk] * 32 + lane]);
             }
-            CSTEP(3 + 2 * it, v[0] + v[BATCH - 1]);
 #pragma unroll
             for (int kk = 0; kk < BATCH; ++kk) {
-                const long long wp = __shfl_sync(0xffffffffu, pos0, src[kk]);
                 if (mine[kk]) {
-                    const long long row = (wbase + src[kk]) * 32 + lane;
-                    const long long pos = wp + __popc(wb[kk] & lt);
+                    const long long row = wq[kk] * 32 + lane;
+                    const long long pos = s_dpos[q0 + kk] + __popc(bq[kk] & lt);
                     a.acc[row] = __longlong_as_double((long long)EMPTY);
                     if (pos < ycap) {
                         a.y_idx[pos] = (int32_t)(row + a.row_begin);
@@ -919,9 +924,9 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
                     }
                 }
             }
-            CSTEP(4 + 2 * it, 0);
-            ++it;
         }
+        __syncthreads();
+        if (tid == 0) s_nd = 0;
     }
     if (b == 0 && tid == 0) {
         const long long yt = s_tot[0];

@@ -31,10 +31,17 @@ namespace {
 
 constexpr int FT = 1024;          // threads per CTA
 constexpr int NWF = FT / 32;      // warps per CTA
-constexpr int TL = 7;             // log2 tile items per warp task (phase B1)
+#ifndef TSMV_TL
+#define TSMV_TL 7
+#endif
+#ifndef TSMV_SL
+#define TSMV_SL 7
+#endif
+constexpr int TL = TSMV_TL;       // log2 tile items per warp task (phase B1)
 constexpr int UT = (1 << TL) / 32;
-constexpr int SL = 7;             // log2 side items per warp chunk
+constexpr int SL = TSMV_SL;       // log2 side items per warp chunk
 constexpr int US = (1 << SL) / 32;
+constexpr int WL = TL > SL ? TL : SL;  // log2 of the per-warp list windows (entries + 1)
 #ifndef TSMV_BATCH
 #define TSMV_BATCH 4
 #endif
@@ -287,7 +294,7 @@ __device__ __forceinline__ void grid_sync_f(unsigned long long *bar, unsigned lo
 template <class AV, class XV, int SR>
 __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
     constexpr int NT = 16, LOG = 4;
-    constexpr int WN = (1 << SL) + 1;
+    constexpr int WN = (1 << WL) + 1;
     __shared__ long long s_scan[8][NWF];
     extern __shared__ __align__(16) unsigned char s_dyn[];
     double *s_hacc = reinterpret_cast<double *>(s_dyn);                           // [HOT_SLOTS]
@@ -950,7 +957,7 @@ template <class AV, class XV> void *pick_sr_flat(int sr) {
 }
 void *pick_flat(bool f32, int sr) { return f32 ? pick_sr_flat<float, float>(sr) : pick_sr_flat<double, double>(sr); }
 
-constexpr size_t FLAT_DYN = HOT_SLOTS * 8 + (size_t)NWF * ((1 << SL) + 1) * 24 + HOT_SLOTS / 8;
+constexpr size_t FLAT_DYN = HOT_SLOTS * 8 + (size_t)NWF * ((1 << WL) + 1) * 24 + HOT_SLOTS / 8;
 
 void flat_set_smem() {
     static bool done = false;

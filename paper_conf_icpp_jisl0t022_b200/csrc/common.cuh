@@ -82,9 +82,29 @@ inline int idx_bytes(int nt) { return nt == 16 ? 1 : 2; }
 inline int word_bytes(int nt) { return nt / 8; }
 
 // ------------------------------------------------------------------ device memory
+// Owning device buffer (RAII: freed on scope exit, move-only), so that builder
+// temporaries can never outlive the call that made them.
 struct DevBuf {
     void *p = nullptr;
     size_t bytes = 0;
+    DevBuf() = default;
+    DevBuf(const DevBuf &) = delete;
+    DevBuf &operator=(const DevBuf &) = delete;
+    DevBuf(DevBuf &&o) noexcept : p(o.p), bytes(o.bytes) {
+        o.p = nullptr;
+        o.bytes = 0;
+    }
+    DevBuf &operator=(DevBuf &&o) noexcept {
+        if (this != &o) {
+            release();
+            p = o.p;
+            bytes = o.bytes;
+            o.p = nullptr;
+            o.bytes = 0;
+        }
+        return *this;
+    }
+    ~DevBuf() { release(); }
     void alloc(size_t b) {
         release();
         if (b == 0) b = 16;

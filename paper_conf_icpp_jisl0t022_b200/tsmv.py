@@ -156,9 +156,14 @@ class TiledMatrix:
         self.opts = default_options(**opts)
         self.device = torch.device("cuda", self.opts.device) if torch.cuda.is_available() else None
         ctx = _vp()
-        check(tsmv_create(ctypes.byref(ctx), self.m, self.n, _ptr(row_ptr) or row_ptr.data_ptr(),
-                          _ptr(col_idx), _ptr(values) if dtype != "pattern" else None,
-                          _DTYPES[dtype], ctypes.byref(self.opts)), "tsmv_create")
+        args = (self.m, self.n, _ptr(row_ptr) or row_ptr.data_ptr(), _ptr(col_idx),
+                _ptr(values) if dtype != "pattern" else None, _DTYPES[dtype], ctypes.byref(self.opts))
+        st = tsmv_create(ctypes.byref(ctx), *args)
+        if st == ENOMEM and self.device is not None:
+            # the library allocates with cudaMalloc: hand torch's cached blocks back and retry once
+            torch.cuda.empty_cache()
+            st = tsmv_create(ctypes.byref(ctx), *args)
+        check(st, "tsmv_create")
         self.ctx = ctx
         self.nnz = int(col_idx.numel())
 

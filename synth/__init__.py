@@ -106,14 +106,35 @@ class CSR:
             torch.arange(self.m, device=self.row_ptr.device, dtype=torch.int64), counts)
 
 
+_UNIQUE_MAX = 1 << 30   # torch.unique (CUB) refuses >= 2^31 elements
+
+
+def _unique_sorted(keys: torch.Tensor, lo: int, hi: int) -> torch.Tensor:
+    """Sorted distinct values of `keys` (all in [lo, hi)); large inputs are split
+    by value range (R-MAT scale 26 symmetrised has ~2^31 keys)."""
+    if keys.numel() <= _UNIQUE_MAX or hi - lo < 2:
+        return torch.unique(keys, sorted=True)
+    mid = (lo + hi) // 2
+    sel = keys < mid
+    left = keys[sel]
+    right = keys[~sel]
+    del sel, keys
+    a = _unique_sorted(left, lo, mid)
+    del left
+    b = _unique_sorted(right, mid, hi)
+    del right
+    return torch.cat([a, b])
+
+
 def csr_from_keys(keys: torch.Tensor, m: int, n: int, name: str = "") -> CSR:
     """keys = row*n + col, any order, duplicates allowed -> pattern CSR
     (duplicates coalesced, columns ascending)."""
-    keys = torch.unique(keys.to(torch.int64), sorted=True)
+    keys = _unique_sorted(keys.to(torch.int64), 0, m * n)
     rows = torch.div(keys, n, rounding_mode="floor")
     cols = (keys - rows * n).to(torch.int32)
+    del keys
     counts = torch.bincount(rows, minlength=m)
-    row_ptr = torch.zeros(m + 1, dtype=torch.int64, device=keys.device)
+    row_ptr = torch.zeros(m + 1, dtype=torch.int64, device=cols.device)
     row_ptr[1:] = torch.cumsum(counts, 0)
     return CSR(m, n, row_ptr, cols, None, name)
 

@@ -58,7 +58,8 @@ __global__ void __launch_bounds__(SCAN_BLOCK)
 k_fscan(const uint32_t *__restrict__ F, uint32_t *__restrict__ Fclear, long long nseg, long long NWpad,
         const long long *__restrict__ tptr, const long long *__restrict__ sptr, const int *__restrict__ outdeg,
         const int *__restrict__ indeg, long long row_begin, long long m_local, ListsView Lv,
-        Counters *__restrict__ cnt, Counters *__restrict__ hm, LBDesc<8> *__restrict__ desc, unsigned epoch) {
+        Counters *__restrict__ cnt, Counters *__restrict__ hm, LBDesc<8> *__restrict__ desc, unsigned epoch,
+        int write_lists) {
     using word_t = typename Tr<NT>::word_t;
     using BS = cub::BlockScan<Oct, SCAN_BLOCK>;
     __shared__ typename BS::TempStorage ts;
@@ -75,7 +76,56 @@ k_fscan(const uint32_t *__restrict__ F, uint32_t *__restrict__ Fclear, long long
     long long wt = 0;
     if (J < nseg) {
         bits = seg_bits<NT>(F, J);
-        if (bits) {
+        if constexpr (NT == 16) {
+            // the segment's 16 out-degrees, in-degrees and 17 side starts are
+            // contiguous: 4 + 4 + 9 independent 16-byte loads, one latency
+            if (bits) {
+                wt = tptr[J + 1] - tptr[J];
+                q.v[0] = wt > 0;
+                q.v[1] = wt;
+                q.v[4] = popc_w(bits);
+                const long long v0 = J * 16;
+                const int4 *od4 = reinterpret_cast<const int4 *>(outdeg + v0);
+                const longlong2 *sp2 = reinterpret_cast<const longlong2 *>(sptr + v0);
+                int od[16];
+                long long sp[18];
+#pragma unroll
+                for (int i = 0; i < 4; ++i) {
+                    const int4 t = __ldg(od4 + i);
+                    od[4 * i] = t.x, od[4 * i + 1] = t.y, od[4 * i + 2] = t.z, od[4 * i + 3] = t.w;
+                }
+#pragma unroll
+                for (int i = 0; i < 8; ++i) {
+                    const longlong2 t = __ldg(sp2 + i);
+                    sp[2 * i] = t.x, sp[2 * i + 1] = t.y;
+                }
+                sp[16] = __ldg(sptr + v0 + 16);
+                const long long lv0 = v0 - row_begin;
+                int id[16];
+                if (lv0 >= 0 && lv0 + 16 <= m_local) {
+                    const int4 *id4 = reinterpret_cast<const int4 *>(indeg + lv0);
+#pragma unroll
+                    for (int i = 0; i < 4; ++i) {
+                        const int4 t = __ldg(id4 + i);
+                        id[4 * i] = t.x, id[4 * i + 1] = t.y, id[4 * i + 2] = t.z, id[4 * i + 3] = t.w;
+                    }
+                } else {
+#pragma unroll
+                    for (int r = 0; r < 16; ++r)
+                        id[r] = (lv0 + r >= 0 && lv0 + r < m_local) ? __ldg(indeg + lv0 + r) : 0;
+                }
+#pragma unroll
+                for (int r = 0; r < 16; ++r) {
+                    if ((bits >> r) & 1u) {
+                        const long long ws = sp[r + 1] - sp[r];
+                        q.v[2] += ws > 0;
+                        q.v[3] += ws;
+                        q.v[5] += od[r];
+                        q.v[6] += id[r];
+                    }
+                }
+            }
+        } else if (bits) {
             wt = tptr[J + 1] - tptr[J];
             q.v[0] = wt > 0;
             q.v[1] = wt;
@@ -105,6 +155,49 @@ k_fscan(const uint32_t *__restrict__ F, uint32_t *__restrict__ Fclear, long long
             }
         }
     }
+    if (!write_lists) {
+        // statistics only: block reduction + one atomic per value and block; the
+        // last block publishes (no look-back chain across blocks)
+        __shared__ long long s_red[7];
+        __shared__ bool s_last;
+        if (threadIdx.x < 7) s_red[threadIdx.x] = 0;
+        __syncthreads();
+#pragma unroll
+        for (int i = 0; i < 7; ++i) {
+            long long x = q.v[i];
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1) x += __shfl_xor_sync(0xffffffffu, x, o);
+            if ((threadIdx.x & 31) == 0 && x) atomicAdd((unsigned long long *)&s_red[i], (unsigned long long)x);
+        }
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            long long *dst[7] = {&cnt->nLt, &cnt->Wt, &cnt->nLs, &cnt->Ws, &cnt->fsize, &cnt->mf, &cnt->din};
+            for (int i = 0; i < 7; ++i)
+                if (s_red[i]) atomicAdd((unsigned long long *)dst[i], (unsigned long long)s_red[i]);
+            __threadfence();
+            s_last = atomicAdd(&cnt->fscan_ticket, 1u) == gridDim.x - 1;
+        }
+        __syncthreads();
+        if (s_last && threadIdx.x == 0) {
+            __threadfence();
+            const long long nLt = __ldcg(&cnt->nLt), Wt = __ldcg(&cnt->Wt), nLs = __ldcg(&cnt->nLs),
+                            Ws = __ldcg(&cnt->Ws), fs = __ldcg(&cnt->fsize), mf = __ldcg(&cnt->mf),
+                            din = __ldcg(&cnt->din);
+            cnt->nCt = (Wt + CHUNK - 1) >> CHUNK_LOG;
+            cnt->nCs = (Ws + CHUNK - 1) >> CHUNK_LOG;
+            hm->fsize = fs;
+            hm->mf = mf;
+            hm->din = din;
+            hm->nLt = nLt;
+            hm->Wt = Wt;
+            hm->nLs = nLs;
+            hm->Ws = Ws;
+            cnt->chunk_next = 0;
+            cnt->bid_scan = 0;
+            cnt->fscan_ticket = 0;
+        }
+        return;
+    }
     Oct ex, agg;
     Oct zero;
 #pragma unroll
@@ -121,7 +214,7 @@ k_fscan(const uint32_t *__restrict__ F, uint32_t *__restrict__ Fclear, long long
     __syncthreads();
 #pragma unroll
     for (int i = 0; i < 8; ++i) ex.v[i] += s_pre[i];
-    if (bits && wt > 0) {
+    if (bits && wt > 0 && write_lists) {
         long long i = ex.v[0];
         Lv.Lt_seg[i] = J;
         Lv.Lt_mask[i] = (unsigned long long)bits;
@@ -129,7 +222,7 @@ k_fscan(const uint32_t *__restrict__ F, uint32_t *__restrict__ Fclear, long long
         Lv.Lt_wpre[i] = ex.v[1];
         write_chunks(Lv.Ct, ex.v[1], wt, (int)i);
     }
-    if (bits) {
+    if (bits && write_lists) {
         long long i = ex.v[2], w0 = ex.v[3];
         word_t b = bits;
         while (b) {
@@ -160,8 +253,10 @@ k_fscan(const uint32_t *__restrict__ F, uint32_t *__restrict__ Fclear, long long
         cnt->fsize = tot[4];
         cnt->mf = tot[5];
         cnt->din = tot[6];
-        Lv.Lt_wpre[tot[0]] = tot[1];
-        Lv.Ls_wpre[tot[2]] = tot[3];
+        if (write_lists) {
+            Lv.Lt_wpre[tot[0]] = tot[1];
+            Lv.Ls_wpre[tot[2]] = tot[3];
+        }
         hm->fsize = tot[4];
         hm->mf = tot[5];
         hm->din = tot[6];
@@ -338,14 +433,16 @@ struct BfsRunner {
         return B;
     }
 
-    template <int NT> void fscan(const uint32_t *F, uint32_t *Fclear) {
+    template <int NT> void fscan(const uint32_t *F, uint32_t *Fclear, bool lists) {
         long long nseg = c->nTC;
         int grid = (int)std::max<long long>(1, (nseg + SCAN_BLOCK - 1) / SCAN_BLOCK);
         c->epoch++;
+        if (!lists)  // the stats-only scan accumulates into zeroed counters {nLt..din}
+            TSMV_CUDA(cudaMemsetAsync(&c->counters.as<Counters>()->nLt, 0, 9 * sizeof(long long), st));
         k_fscan<NT><<<grid, SCAN_BLOCK, 0, st>>>(F, Fclear, nseg, NW, c->P.ptr.as<long long>(),
                                                  c->P.sptr.as<long long>(), c->outdeg.as<int>(), c->indeg.as<int>(),
                                                  c->row_begin, c->m, lists_view(c), c->counters.as<Counters>(),
-                                                 c->hcnt_dev, c->desc_bfs.as<LBDesc<8>>(), c->epoch);
+                                                 c->hcnt_dev, c->desc_bfs.as<LBDesc<8>>(), c->epoch, lists ? 1 : 0);
         TSMV_CUDA(cudaGetLastError());
     }
 
@@ -365,11 +462,14 @@ struct BfsRunner {
         TSMV_CUDA(cudaGetLastError());
     }
 
-    void do_fscan(const uint32_t *F, uint32_t *Fclear) {
+    // lists = false: statistics only (|F|, m_f, sum indeg, work totals), for the
+    // hybrid driver, whose next push level rebuilds its lists inside the
+    // persistent kernel
+    void do_fscan(const uint32_t *F, uint32_t *Fclear, bool lists = true) {
         switch (c->nt) {
-            case 16: fscan<16>(F, Fclear); break;
-            case 32: fscan<32>(F, Fclear); break;
-            default: fscan<64>(F, Fclear); break;
+            case 16: fscan<16>(F, Fclear, lists); break;
+            case 32: fscan<32>(F, Fclear, lists); break;
+            default: fscan<64>(F, Fclear, lists); break;
         }
     }
     void do_expand(int dir) {
@@ -462,7 +562,7 @@ extern "C" tsmv_status tsmv_bfs(tsmv_ctx *c, int64_t source, int32_t *levels, ts
                     c->bfs_level = (int)level;
                     c->fcur = (Fa == c->F0.as<uint32_t>()) ? 0 : 1;
                     R.do_expand(TSMV_DIR_PULL_CSC);
-                    R.do_fscan(Fb, Fa);  // next frontier lists + stats; clears Fa
+                    R.do_fscan(Fb, Fa, false);  // next frontier stats; clears Fa
                     TSMV_CUDA(cudaStreamSynchronize(st));
                     volatile Counters *h = c->hcnt;
                     const long long fsize = h->fsize, mf = h->mf, din = h->din;

@@ -349,7 +349,7 @@ void build_nt(TileSet &S, const int32_t *rows, const int32_t *cols, const V *val
     if (SN) k_side_split<<<grid_for(SN), 256, 0, st>>>(skey2.as<unsigned long long>(), SN, dimR,
                                                         S.srow.as<int32_t>(), scnt.as<int32_t>(), hot_map, NT);
     TSMV_CUDA(cudaGetLastError());
-    S.sptr.alloc((dimC + 1) * 8);
+    S.sptr.alloc(((dimC + 63) / 64 * 64 + 1) * 8);  // padded: whole-segment vector loads (k_fscan)
     counts_to_ptr(scnt.as<int32_t>(), dimC, S.sptr.as<int64_t>(), tmp, st);
     if (vals) S.sval.p = sval2.p, S.sval.bytes = sval2.bytes, sval2.p = nullptr, sval2.bytes = 0;
     TSMV_CUDA(cudaStreamSynchronize(st));
@@ -403,7 +403,7 @@ void prepare_csr(tsmv_ctx *c, const int64_t *row_ptr, const int32_t *col_idx, in
     bad.alloc(4);
     TSMV_CUDA(cudaMemsetAsync(bad.p, 0, 4, st));
     c->indeg.alloc(std::max<int64_t>(c->m, 1) * 4);
-    c->outdeg.alloc(std::max<int64_t>(c->n, 1) * 4);
+    c->outdeg.alloc(((std::max<int64_t>(c->n, 1) + 63) / 64 * 64) * 4);  // padded for segment vector loads
     TSMV_CUDA(cudaMemsetAsync(c->indeg.p, 0, c->indeg.bytes, st));
     TSMV_CUDA(cudaMemsetAsync(c->outdeg.p, 0, c->outdeg.bytes, st));
     if (c->m) k_validate_csr<<<grid_for(c->m), 256, 0, st>>>(row_ptr, col_idx, c->m, c->n, c->nnz, bad.as<int>(),

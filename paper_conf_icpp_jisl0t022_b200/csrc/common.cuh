@@ -181,6 +181,8 @@ struct Counters {
     unsigned long long resv_s;     // (entries << 37) | side work; reset at the end of each call
     unsigned long long nhits;      // flat SpMSpV: hit tiles appended in phase B1
     unsigned long long bfs_bars;   // fused BFS: grid barriers the last launch passed
+    unsigned int fscan_ticket;     // stats-only frontier scan: blocks done (last one publishes)
+    unsigned int pad2;
 };
 
 template <int K> struct LBDesc {

@@ -38,6 +38,7 @@ struct BfsTiles {
     const long long *sptr;
     const int *srow;
     const int32_t *hot_list;  // side rows of hot tile rows are encoded (TileSet::hot_list)
+    const unsigned long long *pmask;  // per group: planes with a nonzero (rows the tile part can discover)
 };
 
 inline BfsTiles bfs_tiles(const TileSet &S) {
@@ -51,6 +52,7 @@ inline BfsTiles bfs_tiles(const TileSet &S) {
     b.sptr = S.sptr.as<long long>();
     b.srow = S.srow.as<int>();
     b.hot_list = S.hot_list;
+    b.pmask = S.pmask.as<unsigned long long>();
     return b;
 }
 
@@ -111,7 +113,9 @@ __device__ __forceinline__ void pull_rowtile(const BfsTiles &Q, const BfsView &B
     using word_t = typename Tr<NT>::word_t;
     const word_t *planes = (const word_t *)Q.planes;
     const long long rb_seg = B.row_begin / NT;
-    word_t um = ~seg_bits<NT>(B.V, rb_seg + I);
+    // rows without in-edges in the tile part (isolated, or side-only) can never be
+    // found here: leave them out, or they would defeat the early exit every level
+    word_t um = ~seg_bits<NT>(B.V, rb_seg + I) & (word_t)Q.pmask[I];
     if (!um) return;
     word_t found = 0;
     const long long t0 = Q.ptr[I], t1 = Q.ptr[I + 1];
@@ -146,7 +150,7 @@ __device__ __forceinline__ void pull_rowtiles32(const BfsTiles &Q, const BfsView
     using word_t = typename Tr<NT>::word_t;
     const long long I = I0 + lane;
     bool open = false;
-    if (I < nTR) open = (word_t)~seg_bits<NT>(B.V, B.row_begin / NT + I) != 0 && Q.ptr[I + 1] > Q.ptr[I];
+    if (I < nTR) open = ((word_t)~seg_bits<NT>(B.V, B.row_begin / NT + I) & (word_t)Q.pmask[I]) != 0;
     unsigned todo = __ballot_sync(0xffffffffu, open);
     while (todo) {
         const int l = __ffs(todo) - 1;

@@ -177,6 +177,19 @@ template <class T> T read1(const T *dptr, cudaStream_t st) {
     return h;
 }
 
+// pmask[J] |= bit c for every plane c that is non-empty in a tile of group J
+template <int NT>
+__global__ void k_plane_occupancy(const typename Tr<NT>::word_t *__restrict__ planes, const int32_t *__restrict__ tgrp,
+                                  int64_t T, unsigned long long *__restrict__ pmask) {
+    for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < T; t += (int64_t)gridDim.x * blockDim.x) {
+        unsigned long long m = 0;
+#pragma unroll 4
+        for (int c = 0; c < NT; ++c)
+            if (planes[(int64_t)c * T + t]) m |= 1ull << c;
+        atomicOr(&pmask[tgrp[t]], m);
+    }
+}
+
 // counts (int32[n]) -> ptr (int64[n+1]) exclusive prefix
 void counts_to_ptr(const int32_t *cnt, int64_t n, int64_t *ptr, CubTemp &tmp, cudaStream_t st) {
     DevBuf wide;
@@ -313,6 +326,14 @@ void build_nt(TileSet &S, const int32_t *rows, const int32_t *cols, const V *val
     TSMV_CUDA(cudaMemcpyAsync(S.off.as<int64_t>() + T, &DN, 8, cudaMemcpyHostToDevice, st));
     S.ptr.alloc((S.nTC + 1) * 8);
     counts_to_ptr(colcnt.as<int32_t>(), S.nTC, S.ptr.as<int64_t>(), tmp, st);
+    if (want_planes) {
+        S.pmask.alloc(std::max<int64_t>(S.nTC, 1) * 8);
+        TSMV_CUDA(cudaMemsetAsync(S.pmask.p, 0, S.pmask.bytes, st));
+        if (T)
+            k_plane_occupancy<NT><<<grid_for(T), 256, 0, st>>>(S.planes.as<word_t>(), S.tgrp.as<int32_t>(), T,
+                                                               S.pmask.as<unsigned long long>());
+        TSMV_CUDA(cudaGetLastError());
+    }
     kout.release();
     vout.release();
     starts.release();

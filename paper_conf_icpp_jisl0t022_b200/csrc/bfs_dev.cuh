@@ -85,6 +85,32 @@ __device__ __forceinline__ void push_side_item(const BfsTiles &P, const BfsView 
     discover<NT>(B, v / NT, (word_t)1 << (v % NT));
 }
 
+// Rows r of `um` whose row word in tile t meets the frontier word f.  nt = 16:
+// all 16 candidate plane words are loaded at once (predicated, independent),
+// instead of one dependent loop trip per row.
+template <int NT>
+__device__ __forceinline__ typename Tr<NT>::word_t rows_hit(const typename Tr<NT>::word_t *planes, long long T,
+                                                            long long t, typename Tr<NT>::word_t um,
+                                                            typename Tr<NT>::word_t f) {
+    using word_t = typename Tr<NT>::word_t;
+    word_t res = 0;
+    if constexpr (NT == 16) {
+        word_t w[16];
+#pragma unroll
+        for (int r = 0; r < 16; ++r) w[r] = ((um >> r) & 1u) ? planes[(long long)r * T + t] : (word_t)0;
+#pragma unroll
+        for (int r = 0; r < 16; ++r)
+            if (w[r] & f) res |= (word_t)1 << r;
+    } else {
+        while (um) {
+            int r = ffs_w(um);
+            um &= um - 1;
+            if (planes[(long long)r * T + t] & f) res |= (word_t)1 << r;
+        }
+    }
+    return res;
+}
+
 // Push-CSR (Alg 6) tile item: tile t of the row structure Q; x word of its tile
 // column, row words of the still-unvisited rows.
 template <int NT>
@@ -97,12 +123,7 @@ __device__ __forceinline__ void push_csr_item(const BfsTiles &Q, const BfsView &
     long long Iseg = B.row_begin / NT + Q.tgrp[t];  // A's tile row (global segment)
     word_t um = ~seg_bits<NT>(B.V, Iseg);
     if (!um) return;
-    word_t res = 0;
-    while (um) {
-        int r = ffs_w(um);
-        um &= um - 1;
-        if (planes[(long long)r * Q.T + t] & f) res |= (word_t)1 << r;
-    }
+    const word_t res = rows_hit<NT>(planes, Q.T, t, um, f);
     if (res) discover<NT>(B, Iseg, res);
 }
 
@@ -124,14 +145,7 @@ __device__ __forceinline__ void pull_rowtile(const BfsTiles &Q, const BfsView &B
         word_t fl = 0;
         if (t < t1) {
             word_t f = seg_bits<NT>(B.F, Q.trow[t]);
-            if (f) {
-                word_t u = um;
-                while (u) {
-                    int r = ffs_w(u);
-                    u &= u - 1;
-                    if (planes[(long long)r * Q.T + t] & f) fl |= (word_t)1 << r;
-                }
-            }
+            if (f) fl = rows_hit<NT>(planes, Q.T, t, um, f);
         }
         fl = warp_or(fl);
         found |= fl;

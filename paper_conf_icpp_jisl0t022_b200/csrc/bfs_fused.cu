@@ -218,6 +218,49 @@ __device__ __forceinline__ void seg_counts(const BfsFusedArgs &a, const uint32_t
     using word_t = typename Tr<NT>::word_t;
     const word_t bits = seg_bits<NT>(F, J);
     if (!bits) return;
+    if constexpr (NT == 16) {
+        // 16 out-degrees, in-degrees and 17 side starts of the segment are
+        // contiguous (arrays padded to whole segments): vector loads, one latency
+        const long long wt = a.P.ptr[J + 1] - a.P.ptr[J];
+        v[0] += wt > 0;
+        v[1] += wt;
+        v[4] += popc_w(bits);
+        const long long v0 = J * 16;
+        int od[16], id[16];
+        long long sp[17];
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+            const int4 t = __ldg(reinterpret_cast<const int4 *>(a.outdeg + v0) + i);
+            od[4 * i] = t.x, od[4 * i + 1] = t.y, od[4 * i + 2] = t.z, od[4 * i + 3] = t.w;
+        }
+        if (v0 + 16 <= a.B.m_local) {
+#pragma unroll
+            for (int i = 0; i < 4; ++i) {
+                const int4 t = __ldg(reinterpret_cast<const int4 *>(a.indeg + v0) + i);
+                id[4 * i] = t.x, id[4 * i + 1] = t.y, id[4 * i + 2] = t.z, id[4 * i + 3] = t.w;
+            }
+        } else {
+#pragma unroll
+            for (int r = 0; r < 16; ++r) id[r] = v0 + r < a.B.m_local ? __ldg(a.indeg + v0 + r) : 0;
+        }
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+            const longlong2 t = __ldg(reinterpret_cast<const longlong2 *>(a.P.sptr + v0) + i);
+            sp[2 * i] = t.x, sp[2 * i + 1] = t.y;
+        }
+        sp[16] = __ldg(a.P.sptr + v0 + 16);
+#pragma unroll
+        for (int r = 0; r < 16; ++r) {
+            if ((bits >> r) & 1u) {
+                const long long ws = sp[r + 1] - sp[r];
+                v[2] += ws > 0;
+                v[3] += ws;
+                v[5] += od[r];
+                v[6] += id[r];
+            }
+        }
+        return;
+    }
     const long long wt = a.P.ptr[J + 1] - a.P.ptr[J];
     v[0] += wt > 0;
     v[1] += wt;

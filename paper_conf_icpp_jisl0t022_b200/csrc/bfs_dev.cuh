@@ -95,6 +95,14 @@ __device__ __forceinline__ typename Tr<NT>::word_t rows_hit(const typename Tr<NT
     using word_t = typename Tr<NT>::word_t;
     word_t res = 0;
     if constexpr (NT == 16) {
+        if (__popc((unsigned)um) <= 2) {  // few candidate rows (late pull levels): plain loop
+            while (um) {
+                const int r = ffs_w(um);
+                um &= um - 1;
+                if (planes[(long long)r * T + t] & f) res |= (word_t)1 << r;
+            }
+            return res;
+        }
         word_t w[16];
 #pragma unroll
         for (int r = 0; r < 16; ++r) w[r] = ((um >> r) & 1u) ? planes[(long long)r * T + t] : (word_t)0;
@@ -183,9 +191,21 @@ __device__ __forceinline__ void pull_side_vertex(const BfsTiles &Q, const BfsVie
     if ((B.V[g >> 5] >> (g & 31)) & 1u) return;
     long long p0 = Q.sptr[v], p1 = Q.sptr[v + 1];
     if (p0 == p1) return;
-    for (long long p = p0; p < p1; ++p) {
-        long long u = decode_row<NT>(Q.srow[p], Q.hot_list);
-        if ((B.F[u >> 5] >> (u & 31)) & 1u) {
+    // four in-neighbours per round: their ids, then their frontier bits, each
+    // step as independent loads (early exit between rounds)
+    for (long long p = p0; p < p1; p += 4) {
+        int sr[4];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) sr[j] = p + j < p1 ? Q.srow[p + j] : 0;
+        bool hit = false;
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+            if (p + j < p1) {
+                const long long u = decode_row<NT>(sr[j], Q.hot_list);
+                hit |= ((B.F[u >> 5] >> (u & 31)) & 1u) != 0;
+            }
+        }
+        if (hit) {
             discover<NT>(B, g / NT, (word_t)1 << (g % NT));
             break;
         }

@@ -321,19 +321,32 @@ __global__ void __launch_bounds__(256) k_push_csr(BfsTiles Q, BfsView B) {
         push_csr_item<NT>(Q, B, t);
 }
 
-template <int NT>
+// WIDE (late pull levels, few open rows): a warp tests the visited words of 32
+// row tiles at once and walks only the open ones; otherwise warp per row tile.
+template <int NT, bool WIDE>
 __global__ void __launch_bounds__(256) k_pull(BfsTiles Q, BfsView B, long long nTR_local) {
     const int lane = threadIdx.x & 31;
     const long long warp = (blockIdx.x * (long long)blockDim.x + threadIdx.x) >> 5;
     const long long nwarps = ((long long)gridDim.x * blockDim.x) >> 5;
-    for (long long I = warp; I < nTR_local; I += nwarps) pull_rowtile<NT>(Q, B, I, lane);
+    if constexpr (WIDE) {
+        for (long long I0 = warp * 32; I0 < nTR_local; I0 += nwarps * 32) pull_rowtiles32<NT>(Q, B, I0, nTR_local, lane);
+    } else {
+        for (long long I = warp; I < nTR_local; I += nwarps) pull_rowtile<NT>(Q, B, I, lane);
+    }
 }
 
-template <int NT>
+template <int NT, bool WIDE>
 __global__ void __launch_bounds__(256) k_pull_side(BfsTiles Q, BfsView B) {
-    for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < B.m_local;
-         v += (long long)gridDim.x * blockDim.x)
-        pull_side_vertex<NT>(Q, B, v);
+    if constexpr (WIDE) {  // thread per visited word: one load for 32 settled vertices
+        const long long w0 = B.row_begin / 32, nw = (B.m_local + 31) / 32;
+        for (long long w = blockIdx.x * (long long)blockDim.x + threadIdx.x; w < nw;
+             w += (long long)gridDim.x * blockDim.x)
+            pull_side_word<NT>(Q, B, w0 + w);
+    } else {
+        for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < B.m_local;
+             v += (long long)gridDim.x * blockDim.x)
+            pull_side_vertex<NT>(Q, B, v);
+    }
 }
 
 // BFS parents over the min-second semiring:
@@ -446,7 +459,7 @@ struct BfsRunner {
         TSMV_CUDA(cudaGetLastError());
     }
 
-    template <int NT> void expand(int dir) {
+    template <int NT> void expand(int dir, bool wide) {
         BfsView B = view();
         BfsTiles P = bfs_tiles(c->P), Q = bfs_tiles(*c->Q);
         if (dir == TSMV_DIR_PUSH_CSC) {
@@ -456,8 +469,13 @@ struct BfsRunner {
             if (Q.T) k_push_csr<NT><<<grid_for(Q.T), 256, 0, st>>>(Q, B);
         } else {
             long long nTRl = (c->m + NT - 1) / NT;
-            k_pull<NT><<<grid_for(nTRl * 32), 256, 0, st>>>(Q, B, nTRl);
-            k_pull_side<NT><<<grid_for(c->m), 256, 0, st>>>(Q, B);
+            if (wide) {
+                k_pull<NT, true><<<grid_for(nTRl), 256, 0, st>>>(Q, B, nTRl);
+                k_pull_side<NT, true><<<grid_for((c->m + 31) / 32), 256, 0, st>>>(Q, B);
+            } else {
+                k_pull<NT, false><<<grid_for(nTRl * 32), 256, 0, st>>>(Q, B, nTRl);
+                k_pull_side<NT, false><<<grid_for(c->m), 256, 0, st>>>(Q, B);
+            }
         }
         TSMV_CUDA(cudaGetLastError());
     }
@@ -472,11 +490,12 @@ struct BfsRunner {
             default: fscan<64>(F, Fclear, lists); break;
         }
     }
-    void do_expand(int dir) {
+    // wide: late Pull-CSC level (few unvisited edges left), see k_pull
+    void do_expand(int dir, bool wide = false) {
         switch (c->nt) {
-            case 16: expand<16>(dir); break;
-            case 32: expand<32>(dir); break;
-            default: expand<64>(dir); break;
+            case 16: expand<16>(dir, wide); break;
+            case 32: expand<32>(dir, wide); break;
+            default: expand<64>(dir, wide); break;
         }
     }
     void init(long long source) {
@@ -561,7 +580,7 @@ extern "C" tsmv_status tsmv_bfs(tsmv_ctx *c, int64_t source, int32_t *levels, ts
                 while (true) {
                     c->bfs_level = (int)level;
                     c->fcur = (Fa == c->F0.as<uint32_t>()) ? 0 : 1;
-                    R.do_expand(TSMV_DIR_PULL_CSC);
+                    R.do_expand(TSMV_DIR_PULL_CSC, mu * 4 < c->nnz);
                     R.do_fscan(Fb, Fa, false);  // next frontier stats; clears Fa
                     TSMV_CUDA(cudaStreamSynchronize(st));
                     volatile Counters *h = c->hcnt;

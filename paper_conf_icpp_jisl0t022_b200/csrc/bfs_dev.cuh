@@ -39,6 +39,7 @@ struct BfsTiles {
     const int *srow;
     const int32_t *hot_list;  // side rows of hot tile rows are encoded (TileSet::hot_list)
     const unsigned long long *pmask;  // per group: planes with a nonzero (rows the tile part can discover)
+    const uint32_t *smask;            // per 32 columns: side columns with a nonzero (rows the side part can discover)
 };
 
 inline BfsTiles bfs_tiles(const TileSet &S) {
@@ -53,6 +54,7 @@ inline BfsTiles bfs_tiles(const TileSet &S) {
     b.srow = S.srow.as<int>();
     b.hot_list = S.hot_list;
     b.pmask = S.pmask.as<unsigned long long>();
+    b.smask = S.smask.as<uint32_t>();
     return b;
 }
 
@@ -189,8 +191,8 @@ __device__ __forceinline__ void pull_side_vertex(const BfsTiles &Q, const BfsVie
     using word_t = typename Tr<NT>::word_t;
     long long g = B.row_begin + v;
     if ((B.V[g >> 5] >> (g & 31)) & 1u) return;
+    if (!((Q.smask[v >> 5] >> (v & 31)) & 1u)) return;  // no side in-edges
     long long p0 = Q.sptr[v], p1 = Q.sptr[v + 1];
-    if (p0 == p1) return;
     // four in-neighbours per round: their ids, then their frontier bits, each
     // step as independent loads (early exit between rounds)
     for (long long p = p0; p < p1; p += 4) {
@@ -218,7 +220,8 @@ __device__ __forceinline__ void pull_side_vertex(const BfsTiles &Q, const BfsVie
 // one by one: a fully visited word costs one load.
 template <int NT>
 __device__ __forceinline__ void pull_side_word(const BfsTiles &Q, const BfsView &B, long long w) {
-    uint32_t um = ~B.V[w];
+    const long long wl = w - B.row_begin / 32;  // local word (row_begin is a multiple of 64)
+    uint32_t um = ~B.V[w] & Q.smask[wl];
     while (um) {
         const int r = __ffs(um) - 1;
         um &= um - 1;

@@ -177,6 +177,17 @@ template <class T> T read1(const T *dptr, cudaStream_t st) {
     return h;
 }
 
+// smask word w: bit r set iff side column 32w + r is non-empty
+__global__ void k_side_occupancy(const int64_t *__restrict__ sptr, int64_t dimC, uint32_t *__restrict__ smask) {
+    for (int64_t w = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; w < (dimC + 31) / 32;
+         w += (int64_t)gridDim.x * blockDim.x) {
+        uint32_t m = 0;
+        for (int r = 0; r < 32 && w * 32 + r < dimC; ++r)
+            if (sptr[w * 32 + r + 1] > sptr[w * 32 + r]) m |= 1u << r;
+        smask[w] = m;
+    }
+}
+
 // pmask[J] |= bit c for every plane c that is non-empty in a tile of group J
 template <int NT>
 __global__ void k_plane_occupancy(const typename Tr<NT>::word_t *__restrict__ planes, const int32_t *__restrict__ tgrp,
@@ -372,6 +383,12 @@ void build_nt(TileSet &S, const int32_t *rows, const int32_t *cols, const V *val
     TSMV_CUDA(cudaGetLastError());
     S.sptr.alloc(((dimC + 63) / 64 * 64 + 1) * 8);  // padded: whole-segment vector loads (k_fscan)
     counts_to_ptr(scnt.as<int32_t>(), dimC, S.sptr.as<int64_t>(), tmp, st);
+    if (want_planes) {
+        const int64_t nw = (dimC + 31) / 32;
+        S.smask.alloc(std::max<int64_t>(nw, 1) * 4);
+        if (nw) k_side_occupancy<<<grid_for(nw), 256, 0, st>>>(S.sptr.as<int64_t>(), dimC, S.smask.as<uint32_t>());
+        TSMV_CUDA(cudaGetLastError());
+    }
     if (vals) S.sval.p = sval2.p, S.sval.bytes = sval2.bytes, sval2.p = nullptr, sval2.bytes = 0;
     TSMV_CUDA(cudaStreamSynchronize(st));
 }

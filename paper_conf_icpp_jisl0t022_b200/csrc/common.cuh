@@ -139,6 +139,7 @@ struct TileSet {
     DevBuf val;      // double/float[dense_nnz] (absent for pattern)
     DevBuf planes;   // word_t[NT][T]: plane c holds column word c of every tile (bit r = row r)
     DevBuf pmask;    // u64[nTC]: bit c = plane c non-empty in some tile of group J (pull: rows with tile in-edges)
+    DevBuf smask;    // u32[ceil(dimC/32)]: bit = side column non-empty (pull: rows with side in-edges)
     DevBuf desc;     // TileDesc[T]
     DevBuf cstart;   // cs_t[T][NT]: start of column c inside the tile's nonzeros (column-major)
     DevBuf rec;      // TileRec64[T] (nt = 16 only): descriptor + inline indices / column starts / values
@@ -153,10 +154,10 @@ struct TileSet {
     const int32_t *hot_list = nullptr;
     size_t bytes() const {
         return ptr.bytes + trow.bytes + tgrp.bytes + mask.bytes + off.bytes + idx.bytes + val.bytes +
-               planes.bytes + pmask.bytes + sptr.bytes + srow.bytes + sval.bytes + desc.bytes + cstart.bytes + rec.bytes + colinfo.bytes;
+               planes.bytes + pmask.bytes + smask.bytes + sptr.bytes + srow.bytes + sval.bytes + desc.bytes + cstart.bytes + rec.bytes + colinfo.bytes;
     }
     void release() {
-        for (DevBuf *b : {&ptr, &trow, &tgrp, &mask, &off, &idx, &val, &planes, &pmask, &sptr, &srow, &sval, &desc, &cstart, &rec, &colinfo})
+        for (DevBuf *b : {&ptr, &trow, &tgrp, &mask, &off, &idx, &val, &planes, &pmask, &smask, &sptr, &srow, &sval, &desc, &cstart, &rec, &colinfo})
             b->release();
     }
 };

@@ -20,7 +20,7 @@
 //     list window (start, x_j) is staged in shared memory;
 //   * chunks are dealt round-robin to warps (no work-queue atomics on one address);
 //   * compaction with one thread per bitmap word (loads of its set rows batched).
-// Phases: A | barrier | B (a3-a5) | barrier | C1 count | barrier | C2 write y.
+// Phases: A | barrier | B1 (a3, a5) -> B2 (a4, own hits, CTA barrier only) | barrier | C1 count | barrier | C2 write y.
 #include "device.cuh"
 #include <algorithm>
 #include <cstdlib>
@@ -307,8 +307,6 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
     __shared__ int s_err;
     __shared__ int s_nheavy;
     __shared__ int s_hcnt;
-    __shared__ long long s_nh;
-    __shared__ long long s_hpre[MAXG + 1];
     __shared__ unsigned long long s_pc[KP];
     __shared__ long long s_pbase[KP], s_ex0[KP];
     __shared__ int s_nd;  // dense bitmap words of the current C2 round
@@ -569,36 +567,11 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
                 if (hv[u]) a.L.hits[o++] = make_uint4((unsigned)tv[u], hv[u], (unsigned)Jv[u], 0u);
         }
     }
+    // B2 takes the hits of this CTA only: its list region is complete after this
+    // __syncthreads, so there is no grid barrier between B1 and B2 (a CTA whose
+    // B1 ends early starts multiplying at once)
     __syncthreads();
-    if (tid == 0) a.partials[b * 8 + 5] = s_hcnt;
-    grid_sync_f(&a.cnt->bar, target, tr ? tr + 3 : nullptr);
     if (stamp) ts[6] = globaltimer_ns();
-    // prefix of the per-CTA hit counts (hits of CTA g live at [g * RC, g * RC + count))
-    if (wid == 0) {
-        constexpr int PER = (MAXG + 31) / 32;
-        long long v[PER], run = 0;
-#pragma unroll
-        for (int i = 0; i < PER; ++i) {
-            const int g = lane * PER + i;
-            v[i] = g < G ? __ldcg(&a.partials[g * 8 + 5]) : 0;
-            run += v[i];
-        }
-        long long inc = run;
-#pragma unroll
-        for (int o2 = 1; o2 < 32; o2 <<= 1) {
-            const long long y = __shfl_up_sync(0xffffffffu, inc, o2);
-            if (lane >= o2) inc += y;
-        }
-        long long ex = inc - run;
-#pragma unroll
-        for (int i = 0; i < PER; ++i) {
-            const int g = lane * PER + i;
-            if (g <= G) s_hpre[g] = ex;
-            ex += v[i];
-        }
-        if (lane == 31) s_nh = inc;
-    }
-    __syncthreads();
 
     // ------------------------------------------------------------ phase B2 (a4)
     // lane = hit tile: one 64-byte record.  Tiles whose values are inline (and
@@ -606,23 +579,17 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
     // the other hit tiles of the warp are redistributed over the lanes (shuffles)
     // and read from the idx / val arrays.
     if (!err) {
-        const long long NH = s_nh;
+        const long long NH = s_hcnt;
         const AV *val = (const AV *)a.val;
         constexpr int INL = 32 / (int)sizeof(AV);
-        for (long long hb = ((long long)wid * G + b) * 32; hb < NH; hb += nwarps * 32) {
+        for (long long hb = (long long)wid * 32; hb < NH; hb += NWF * 32) {
             const long long h = hb + lane;
             unsigned hit = 0u;
             long long t = 0;
             int slot = 0;
             double xv0 = 0.0;
             if (h < NH) {
-                int lo = 0, hi = G - 1;  // CTA region holding hit h: last g with s_hpre[g] <= h
-                while (lo < hi) {
-                    const int mid = (lo + hi + 1) >> 1;
-                    if (s_hpre[mid] <= h) lo = mid;
-                    else hi = mid - 1;
-                }
-                const uint4 e = __ldcg(&a.L.hits[(long long)lo * RC + (h - s_hpre[lo])]);
+                const uint4 e = __ldcg(&a.L.hits[(long long)b * RC + h]);
                 t = e.x;
                 hit = e.y;
                 slot = (int)e.z;
@@ -1170,7 +1137,7 @@ void enqueue_spmspv_flat(tsmv_ctx *c, int sr, long long k, const int32_t *xi, co
     }
     cfg.attrs = at;
     TSMV_CUDA(cudaLaunchKernelExC(&cfg, pick_flat(f32, sr), args));
-    c->bar_base += 4ull * (unsigned long long)G;
+    c->bar_base += 3ull * (unsigned long long)G;
     c->last_blocks = G;
     if (c->timing) c->tcalls++;
 }

@@ -361,4 +361,7 @@ bool bfs_fused_launch(tsmv_ctx *c, long long source, cudaStream_t st, bool resum
 int choose_dir(const tsmv_options &o, long long n, long long fsize, long long mf, long long mu);
 // pointer classification
 bool is_device_ptr(const void *p);
+// device address of page-locked, mapped host memory (cudaHostAlloc / torch
+// pin_memory under UVA), or NULL for pageable / device memory
+void *mapped_device_ptr(const void *p);
 }  // namespace tsmv

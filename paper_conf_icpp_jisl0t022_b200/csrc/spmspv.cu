@@ -1014,6 +1014,35 @@ void stats_from_partials(tsmv_ctx *c, tsmv_call_stats *s) {
 
 using namespace tsmv;
 
+namespace tsmv {
+namespace {
+// y (device staging) -> caller's pinned host y, sized on the device by the
+// call's y_nnz (no host round trip between the multiply and the copy):
+// 16-byte stores where both sides are aligned, full PCIe write lines.
+__global__ void k_copy_y(const int32_t *__restrict__ yi, const void *__restrict__ yv, const long long *__restrict__ ynnz,
+                         long long ycap, int32_t *__restrict__ hyi, void *__restrict__ hyv, int vb) {
+    const long long n = min(*ynnz, ycap);
+    const long long tid = blockIdx.x * (long long)blockDim.x + threadIdx.x, nt = (long long)gridDim.x * blockDim.x;
+    if (hyi) {
+        const bool al = ((reinterpret_cast<uintptr_t>(hyi) & 15) == 0);
+        const long long nv = al ? n / 4 : 0;
+        for (long long i = tid; i < nv; i += nt)
+            reinterpret_cast<int4 *>(hyi)[i] = __ldcg(reinterpret_cast<const int4 *>(yi) + i);
+        for (long long i = nv * 4 + tid; i < n; i += nt) hyi[i] = yi[i];
+    }
+    if (hyv) {
+        const long long bytes = n * vb;
+        const bool al = ((reinterpret_cast<uintptr_t>(hyv) & 15) == 0);
+        const long long nv = al ? bytes / 16 : 0;
+        for (long long i = tid; i < nv; i += nt)
+            reinterpret_cast<int4 *>(hyv)[i] = __ldcg(reinterpret_cast<const int4 *>(yv) + i);
+        for (long long i = nv * 16 + tid; i < bytes; i += nt)
+            static_cast<char *>(hyv)[i] = static_cast<const char *>(yv)[i];
+    }
+}
+}  // namespace
+}  // namespace tsmv
+
 extern "C" tsmv_status tsmv_spmspv(tsmv_ctx *c, tsmv_semiring sr, int64_t x_nnz, const int32_t *x_idx,
                                    const void *x_val, int64_t y_cap, int32_t *y_idx, void *y_val, int64_t *y_nnz,
                                    void *cuda_stream) {
@@ -1035,17 +1064,27 @@ extern "C" tsmv_status tsmv_spmspv(tsmv_ctx *c, tsmv_semiring sr, int64_t x_nnz,
         const bool f32 = c->dtype == TSMV_F32;
         const size_t vb = f32 ? 4 : 8;
         // stage host inputs
+        // pinned (mapped) host x is read by the kernel in place (zero copy: phase A
+        // reads each entry once, coalesced); pageable host x is staged
         const int32_t *xi = x_idx;
         const void *xv = (sr == TSMV_OR_AND) ? nullptr : x_val;
         if (!is_device_ptr(xi)) {
-            c->stage_x_idx.ensure(x_nnz * 4);
-            TSMV_CUDA(cudaMemcpyAsync(c->stage_x_idx.p, xi, x_nnz * 4, cudaMemcpyHostToDevice, st));
-            xi = c->stage_x_idx.as<int32_t>();
+            if (const void *d = mapped_device_ptr(xi)) {
+                xi = static_cast<const int32_t *>(d);
+            } else {
+                c->stage_x_idx.ensure(x_nnz * 4);
+                TSMV_CUDA(cudaMemcpyAsync(c->stage_x_idx.p, xi, x_nnz * 4, cudaMemcpyHostToDevice, st));
+                xi = c->stage_x_idx.as<int32_t>();
+            }
         }
         if (xv && !is_device_ptr(xv)) {
-            c->stage_x_val.ensure(x_nnz * vb);
-            TSMV_CUDA(cudaMemcpyAsync(c->stage_x_val.p, xv, x_nnz * vb, cudaMemcpyHostToDevice, st));
-            xv = c->stage_x_val.p;
+            if (const void *d = mapped_device_ptr(xv)) {
+                xv = d;
+            } else {
+                c->stage_x_val.ensure(x_nnz * vb);
+                TSMV_CUDA(cudaMemcpyAsync(c->stage_x_val.p, xv, x_nnz * vb, cudaMemcpyHostToDevice, st));
+                xv = c->stage_x_val.p;
+            }
         }
         bool host_y = (y_cap > 0) && !is_device_ptr(y_idx);
         bool host_yv = (y_cap > 0) && sr != TSMV_OR_AND && y_val && !is_device_ptr(y_val);
@@ -1062,6 +1101,16 @@ extern "C" tsmv_status tsmv_spmspv(tsmv_ctx *c, tsmv_semiring sr, int64_t x_nnz,
             yv = c->stage_y_val.p;
         }
         enqueue_spmspv(c, sr, x_nnz, xi, xv, ycap_dev, yi, yv, nullptr, st);
+        // pinned (mapped) host y: copied by a kernel sized on the device, right
+        // behind the multiply, then ONE synchronisation for the whole call
+        void *myi = host_y ? mapped_device_ptr(y_idx) : nullptr;
+        void *myv = host_yv ? mapped_device_ptr(y_val) : nullptr;
+        const bool direct = (!host_y || myi) && (!host_yv || myv) && (host_y || host_yv);
+        if (direct) {
+            k_copy_y<<<c->sm_count * 4, 256, 0, st>>>(yi, yv, &c->counters.as<Counters>()->y_nnz, y_cap,
+                                                       static_cast<int32_t *>(myi), myv, (int)vb);
+            TSMV_CUDA(cudaGetLastError());
+        }
         TSMV_CUDA(cudaStreamSynchronize(st));
         volatile Counters *h = c->hcnt;
         int64_t ynnz = h->y_nnz;
@@ -1072,9 +1121,11 @@ extern "C" tsmv_status tsmv_spmspv(tsmv_ctx *c, tsmv_semiring sr, int64_t x_nnz,
             set_error("tsmv_spmspv: y_cap %lld < y_nnz %lld", (long long)y_cap, (long long)ynnz);
             return TSMV_ECAPACITY;
         }
-        if (host_y) TSMV_CUDA(cudaMemcpyAsync(y_idx, yi, ynnz * 4, cudaMemcpyDeviceToHost, st));
-        if (host_yv) TSMV_CUDA(cudaMemcpyAsync(y_val, yv, ynnz * vb, cudaMemcpyDeviceToHost, st));
-        if (host_y || host_yv) TSMV_CUDA(cudaStreamSynchronize(st));
+        if (!direct) {
+            if (host_y) TSMV_CUDA(cudaMemcpyAsync(y_idx, yi, ynnz * 4, cudaMemcpyDeviceToHost, st));
+            if (host_yv) TSMV_CUDA(cudaMemcpyAsync(y_val, yv, ynnz * vb, cudaMemcpyDeviceToHost, st));
+            if (host_y || host_yv) TSMV_CUDA(cudaStreamSynchronize(st));
+        }
         return TSMV_OK;
     } catch (const Err &e) {
         return e.st;

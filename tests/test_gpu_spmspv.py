@@ -197,3 +197,41 @@ def test_target_rmat_s22_full(tsmv):
     xi, xv = synth.sample_x(A.n, synth.density_k(A.n, 0.01), seed=1)
     yi, yv = M.spmspv(xi.to(DEV), xv.to(DEV))
     check_spmspv(C, yi, yv, xi, xv)
+
+
+@pytest.mark.parametrize("dtype", ["f64", "f32"])
+def test_pinned_host_buffers_zero_copy(dtype):
+    """Pinned host x is read in place by the kernel and pinned host y is filled by
+    the device-sized copy kernel; pageable host buffers go through staging.  All
+    three must equal the device-resident call: the index set exactly, the values to
+    the summation-order tolerance (fp64 atomics commit in any order; positive
+    values, no cancellation)."""
+    from paper_conf_icpp_jisl0t022_b200 import tsmv
+    A = synth.attach_values(synth.rmat(14, 16, seed=9), seed=2, dtype=dtype)
+    M = tsmv.TiledMatrix.from_csr(A.to(DEV), dtype=dtype)
+    xi, xv = synth.sample_x(A.n, synth.density_k(A.n, 0.02), seed=5, dtype=dtype)
+    di, dv = M.spmspv(xi.to(DEV), xv.to(DEV))
+    di, dv = di.cpu(), dv.cpu()
+    vt = dv.dtype
+    tol = 1e-12 if dtype == "f64" else 1e-6
+
+    def same(yi, yv):
+        return torch.equal(yi, di) and torch.allclose(yv, dv, rtol=tol, atol=0.0)
+
+    # pinned, 16-byte aligned
+    pi, pv = xi.pin_memory(), xv.pin_memory()
+    hyi, hyv = torch.empty(A.m, dtype=torch.int32).pin_memory(), torch.empty(A.m, dtype=vt).pin_memory()
+    yi, yv = M.spmspv(pi, pv, y_idx=hyi, y_val=hyv)
+    assert same(yi, yv)
+    # pinned but not 16-byte aligned outputs (offset views)
+    big_i, big_v = torch.empty(A.m + 3, dtype=torch.int32).pin_memory(), torch.empty(A.m + 3, dtype=vt).pin_memory()
+    yi, yv = M.spmspv(pi, pv, y_idx=big_i[1:], y_val=big_v[3:])
+    assert same(yi, yv)
+    # pageable
+    yi, yv = M.spmspv(xi.clone(), xv.clone(), y_idx=torch.empty(A.m, dtype=torch.int32),
+                      y_val=torch.empty(A.m, dtype=vt))
+    assert same(yi, yv)
+    # capacity error reports the size
+    with pytest.raises(tsmv.TsmvError):
+        M.spmspv(pi, pv, y_idx=hyi[:5], y_val=hyv[:5])
+    M.close()

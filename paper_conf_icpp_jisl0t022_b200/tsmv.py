@@ -117,10 +117,15 @@ def _ptr(t: Optional[torch.Tensor]):
     return t.data_ptr() if t.numel() else None
 
 
+_RAW_STREAM = getattr(torch._C, "_cuda_getCurrentRawStream", None)
+
+
 def _stream(stream=None):
     if stream is not None:
         return stream.cuda_stream if hasattr(stream, "cuda_stream") else int(stream)
     if torch.cuda.is_available():
+        if _RAW_STREAM is not None:  # the current stream's handle without building a Stream object
+            return _RAW_STREAM(torch.cuda.current_device())
         return torch.cuda.current_stream().cuda_stream
     return None
 
@@ -181,8 +186,9 @@ class TiledMatrix:
         length y_nnz (y_val None for or_and).  Tensors may live on the GPU or the host."""
         sr = _SEMIRINGS[semiring] if isinstance(semiring, str) else int(semiring)
         dev = x_idx.device
-        x_idx = x_idx.to(torch.int32).contiguous()
-        if x_val is not None:
+        if x_idx.dtype != torch.int32 or not x_idx.is_contiguous():
+            x_idx = x_idx.to(torch.int32).contiguous()
+        if x_val is not None and (x_val.dtype != self.vtype or not x_val.is_contiguous()):
             x_val = x_val.to(self.vtype).contiguous()
         if y_idx is None:
             y_idx = torch.empty(self.m, dtype=torch.int32, device=dev)

@@ -201,6 +201,29 @@ tsmv_status tsmv_bfs(tsmv_ctx *c, int64_t source, int32_t *levels, tsmv_bfs_stat
  * BFS structures), ECUDA. */
 tsmv_status tsmv_bfs_parents(tsmv_ctx *c, const int32_t *levels, int32_t *parents, void *cuda_stream);
 
+/* Multi-source TileBFS: Alg 3 from nsrc
+ * sources at once, the multiple-BFS workload of P:171-177.  One bit per source in
+ * 64-bit vertex words; every level is one bottom-up (Pull-CSC, Alg 7) pass for all
+ * sources over the row structure (tile row words gather the frontier words of
+ * the tile's column segment) and the side CSR.
+ *   nsrc    : 1..64.
+ *   sources : host int64[nsrc], each in [0, nrows) (repeats allowed).
+ *   levels  : device int32[nrows * nsrc], vertex-major: levels[v * nsrc + s] =
+ *             hop count of v from sources[s], -1 if unreachable (R15 per source).
+ *   stats   : host, may be NULL: nlevels = max over sources of the non-empty
+ *             levels, pairs_reached = sum over sources of reached vertices,
+ *             edges_traversed = sum over sources of R16, ms = device time.
+ * Single-GPU contexts with BFS structures and tile_dim 16 only (else EINVAL /
+ * EUNSUPPORTED).  Returns after the traversal (stream synchronised). */
+typedef struct {
+    int32_t nlevels;
+    int64_t pairs_reached;
+    int64_t edges_traversed;
+    double ms;
+} tsmv_msbfs_stats;
+tsmv_status tsmv_msbfs(tsmv_ctx *c, int32_t nsrc, const int64_t *sources, int32_t *levels,
+                       tsmv_msbfs_stats *stats, void *cuda_stream);
+
 /* ---- distributed TileBFS (row-block partition, Sec 8(e) of SURVEY / DESIGN.md) ----
  * Each rank owns global rows [row_splits[rank], row_splits[rank+1]).  Per level:
  *   tsmv_bfs_dist_expand  -> this rank's newly discovered owned vertices as a bitmap

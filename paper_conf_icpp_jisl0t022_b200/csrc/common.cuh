@@ -323,6 +323,10 @@ struct tsmv_ctx {
     tsmv::DevBuf lwork;        // int32[n]: push work of vertex u = tiles of its tile column + its side nonzeros
     tsmv::DevBuf bq0, bq1;     // int32[n]: frontier vertex lists, ping-pong by level parity
     tsmv::DevBuf lslots;       // long long[3][4]: {|F|, m_f, sum indeg, max lwork} of levels L, L+1, L+2
+    // multi-source BFS (msbfs.cu), allocated on first use
+    tsmv::DevBuf ms_V, ms_F0, ms_F1, ms_N;  // u64[m]: one bit per source
+    tsmv::DevBuf ms_seg0, ms_seg1;          // u32: 1 bit per 16-vertex segment holding frontier vertices
+    tsmv::DevBuf ms_src, ms_out;
     void *trace = nullptr;         // tsmv_set_trace (device, u64[tsmv_trace_words])
 };
 

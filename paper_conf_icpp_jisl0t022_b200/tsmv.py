@@ -58,6 +58,11 @@ class tsmv_info(ctypes.Structure):
                 ("bytes_workspace", ctypes.c_int64), ("build_ms", ctypes.c_double)]
 
 
+class tsmv_msbfs_stats(ctypes.Structure):
+    _fields_ = [("nlevels", ctypes.c_int32), ("pairs_reached", ctypes.c_int64), ("edges_traversed", ctypes.c_int64),
+                ("ms", ctypes.c_double)]
+
+
 class tsmv_bfs_stats(ctypes.Structure):
     _fields_ = [("nlevels", ctypes.c_int32), ("reached", ctypes.c_int64), ("edges_traversed", ctypes.c_int64),
                 ("ms", ctypes.c_double), ("dir_per_level", ctypes.c_int32 * MAX_LEVELS),
@@ -78,6 +83,7 @@ _SIGS = {
     "tsmv_last_call_stats": (ctypes.c_int, [_vp, ctypes.POINTER(tsmv_call_stats)]),
     "tsmv_bfs": (ctypes.c_int, [_vp, _i64, _vp, ctypes.POINTER(tsmv_bfs_stats), _vp]),
     "tsmv_bfs_parents": (ctypes.c_int, [_vp, _vp, _vp, _vp]),
+    "tsmv_msbfs": (ctypes.c_int, [_vp, _i32, _vp, _vp, ctypes.POINTER(tsmv_msbfs_stats), _vp]),
     "tsmv_bfs_dist_begin": (ctypes.c_int, [_vp, _i64, _vp, ctypes.POINTER(_i64), _vp]),
     "tsmv_bfs_dist_expand": (ctypes.c_int, [_vp, _i32, _vp, _vp]),
     "tsmv_bfs_dist_merge": (ctypes.c_int, [_vp, _vp, _i64, ctypes.POINTER(_i64), _vp]),
@@ -245,6 +251,18 @@ class TiledMatrix:
             parents = torch.empty(self.m, dtype=torch.int32, device=self.device)
         check(tsmv_bfs_parents(self.ctx, _ptr(levels), _ptr(parents), _stream(stream)), "tsmv_bfs_parents")
         return parents
+
+    def msbfs(self, sources, levels: Optional[torch.Tensor] = None, stream=None):
+        """Multi-source TileBFS from up to 64 sources at once.  Returns (levels
+        int32[m, nsrc] on the device, vertex-major, -1 = unreachable; stats)."""
+        src = torch.as_tensor(list(sources), dtype=torch.int64)
+        ns = int(src.numel())
+        if levels is None:
+            levels = torch.empty(self.m, ns, dtype=torch.int32, device=self.device)
+        st = tsmv_msbfs_stats()
+        check(tsmv_msbfs(self.ctx, ns, src.data_ptr(), _ptr(levels), ctypes.byref(st), _stream(stream)), "tsmv_msbfs")
+        return levels, {"nlevels": st.nlevels, "pairs_reached": st.pairs_reached,
+                        "edges_traversed": st.edges_traversed, "ms": st.ms}
 
     # -- introspection -----------------------------------------------------------
     def info(self) -> dict:

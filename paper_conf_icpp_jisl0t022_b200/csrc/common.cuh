@@ -327,6 +327,9 @@ struct tsmv_ctx {
     tsmv::DevBuf ms_V, ms_F0, ms_F1, ms_N;  // u64[m]: one bit per source
     tsmv::DevBuf ms_seg0, ms_seg1;          // u32: 1 bit per 16-vertex segment holding frontier vertices
     tsmv::DevBuf ms_src, ms_out;
+    tsmv::DevBuf ms_rowneed;                // u16 per row tile: rows still missing some source
+    tsmv::DevBuf ms_heavy;                  // int32: side vertices with > MS_HEAVY in-neighbours
+    int ms_nheavy = 0;
     void *trace = nullptr;         // tsmv_set_trace (device, u64[tsmv_trace_words])
 };
 

@@ -45,32 +45,36 @@ __global__ void k_ms_init(const long long *__restrict__ src, int nsrc, u64 *__re
     levels[v * nsrc + s] = 0;
 }
 
-// tile part of one bottom-up level (nt = 16)
-__global__ void __launch_bounds__(MSB) k_ms_pull_tiles(BfsTiles Q, const u64 *__restrict__ V, const u64 *__restrict__ F,
-                                                       const uint32_t *__restrict__ seg, u64 *__restrict__ N,
-                                                       long long m, long long nTR, u64 all) {
+// tile part of one bottom-up level (nt = 16), load-balanced over TILES: lane =
+// tile t (tiles are sorted by row tile I = tgrp[t]).  For the rows of I that
+// still miss some source (rowneed[I]) the row word (plane r) of t names the
+// in-neighbours c in column segment J = trow[t]; their frontier words are ORed
+// (one 128-byte line per tile).  Lanes holding the same row tile are merged by
+// a segmented OR over the warp, and the segment head ORs the result into N.
+__global__ void __launch_bounds__(MSB) k_ms_pull_tiles(BfsTiles Q, const u64 *__restrict__ F,
+                                                       const uint32_t *__restrict__ seg,
+                                                       const uint16_t *__restrict__ rowneed, u64 *__restrict__ N) {
     const int lane = threadIdx.x & 31;
     const long long warp = (blockIdx.x * (long long)blockDim.x + threadIdx.x) >> 5;
     const long long nwarps = ((long long)gridDim.x * blockDim.x) >> 5;
     const uint16_t *planes = (const uint16_t *)Q.planes;
-    for (long long I = warp; I < nTR; I += nwarps) {
-        const long long v0 = I * 16;
-        const u64 need = (lane < 16 && v0 + lane < m) ? (all & ~V[v0 + lane]) : 0ull;
-        const unsigned rows = __ballot_sync(0xffffffffu, need != 0ull) & 0xffffu & (unsigned)Q.pmask[I];
-        if (!rows) continue;
+    for (long long tb = warp * 32; tb < Q.T; tb += nwarps * 32) {
+        const long long t = tb + lane;
+        long long I = -1;
+        unsigned rn = 0;
         u64 acc[16];
 #pragma unroll
         for (int r = 0; r < 16; ++r) acc[r] = 0ull;
-        const long long t0 = Q.ptr[I], t1 = Q.ptr[I + 1];
-        for (long long tb = t0; tb < t1; tb += 32) {
-            const long long t = tb + lane;
-            if (t < t1) {
+        if (t < Q.T) {
+            I = Q.tgrp[t];
+            rn = rowneed[I];
+            if (rn) {
                 const long long J = Q.trow[t];
                 if ((seg[J >> 5] >> (J & 31)) & 1u) {
                     const u64 *Fs = F + J * 16;
 #pragma unroll
                     for (int r = 0; r < 16; ++r) {
-                        if ((rows >> r) & 1u) {
+                        if ((rn >> r) & 1u) {
                             unsigned w = planes[(long long)r * Q.T + t];
                             while (w) {
                                 const int c = __ffs(w) - 1;
@@ -82,70 +86,141 @@ __global__ void __launch_bounds__(MSB) k_ms_pull_tiles(BfsTiles Q, const u64 *__
                 }
             }
         }
-        u64 mine = 0ull;
+        // segmented OR over lanes with the same row tile (contiguous lanes)
+        const unsigned same = __match_any_sync(0xffffffffu, I);
+        const int last = 31 - __clz(same);
+        bool any = false;
 #pragma unroll
         for (int r = 0; r < 16; ++r) {
-            if ((rows >> r) & 1u) {  // uniform over the warp
-                const u64 x = warp_or64(acc[r]);
-                if (lane == r) mine = x;
+#pragma unroll
+            for (int d = 1; d < 32; d <<= 1) {
+                const u64 y = __shfl_down_sync(0xffffffffu, acc[r], d);
+                if (lane + d <= last) acc[r] |= y;
             }
+            any |= acc[r] != 0ull;
         }
-        if (lane < 16 && ((rows >> lane) & 1u)) N[v0 + lane] = mine & need;
+        const bool head = I >= 0 && (lane == 0 || ((same >> (lane - 1)) & 1u) == 0u);
+        if (head && any) {
+#pragma unroll
+            for (int r = 0; r < 16; ++r)
+                if (acc[r]) atomicOr(&N[I * 16 + r], acc[r]);
+        }
     }
 }
 
-// side part: in-neighbours u of v in the side CSR of Q
+// side part: in-neighbours u of v in the side CSR of Q.  Vertices with at most
+// MS_HEAVY side in-neighbours: thread per vertex, stop once every missing source
+// is found; heavier ones (power-law hubs) go to k_ms_pull_side_heavy.
+constexpr int MS_HEAVY = 64;
+
 template <int NT>
 __global__ void __launch_bounds__(MSB) k_ms_pull_side(BfsTiles Q, const u64 *__restrict__ V, const u64 *__restrict__ F,
                                                       u64 *__restrict__ N, long long m, u64 all) {
     for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < m; v += (long long)gridDim.x * blockDim.x) {
         if (!((Q.smask[v >> 5] >> (v & 31)) & 1u)) continue;
+        const long long p0 = Q.sptr[v], p1 = Q.sptr[v + 1];
+        if (p1 - p0 > MS_HEAVY) continue;
         const u64 need = all & ~V[v] & ~N[v];
         if (!need) continue;
         u64 acc = 0ull;
-        const long long p1 = Q.sptr[v + 1];
-        for (long long p = Q.sptr[v]; p < p1; ++p) {
-            acc |= F[decode_row<NT>(Q.srow[p], Q.hot_list)];
+        for (long long p = p0; p < p1; p += 4) {
+            int sr[4];
+#pragma unroll
+            for (int j = 0; j < 4; ++j) sr[j] = p + j < p1 ? Q.srow[p + j] : -1;
+#pragma unroll
+            for (int j = 0; j < 4; ++j)
+                if (p + j < p1) acc |= F[decode_row<NT>(sr[j], Q.hot_list)];
             if ((acc & need) == need) break;
         }
         if (acc & need) N[v] |= acc & need;
     }
 }
 
-// new = N & ~V; V |= new; next frontier = new; levels; counts
+template <int NT>
+__global__ void __launch_bounds__(MSB) k_ms_pull_side_heavy(BfsTiles Q, const u64 *__restrict__ V,
+                                                            const u64 *__restrict__ F, u64 *__restrict__ N,
+                                                            const int *__restrict__ heavy, int nheavy, u64 all) {
+    const int lane = threadIdx.x & 31;
+    const long long warp = (blockIdx.x * (long long)blockDim.x + threadIdx.x) >> 5;
+    const long long nwarps = ((long long)gridDim.x * blockDim.x) >> 5;
+    for (long long i = warp; i < nheavy; i += nwarps) {
+        const long long v = heavy[i];
+        const u64 need = all & ~V[v] & ~N[v];
+        if (!need) continue;
+        const long long p0 = Q.sptr[v], p1 = Q.sptr[v + 1];
+        u64 acc = 0ull;
+        for (long long pb = p0; pb < p1; pb += 32) {
+            if (pb + lane < p1) acc |= F[decode_row<NT>(Q.srow[pb + lane], Q.hot_list)];
+            const u64 w = warp_or64(acc);
+            if ((w & need) == need) {
+                acc = w;
+                break;
+            }
+            acc = w;
+        }
+        if (lane == 0 && (acc & need)) N[v] |= acc & need;
+    }
+}
+
+// side vertices with more than MS_HEAVY in-neighbours (built once per context)
+__global__ void k_ms_heavy_list(const long long *__restrict__ sptr, long long m, int *__restrict__ heavy,
+                                unsigned *__restrict__ nheavy) {
+    for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < m; v += (long long)gridDim.x * blockDim.x)
+        if (sptr[v + 1] - sptr[v] > MS_HEAVY) heavy[atomicAdd(nheavy, 1u)] = (int)v;
+}
+
+// new = N & ~V; V |= new; next frontier = new; levels; counts; rowneed[I] =
+// rows of row tile I still missing some source (a warp covers 32 consecutive
+// vertices = two row tiles)
 __global__ void __launch_bounds__(MSB) k_ms_update(u64 *__restrict__ V, u64 *__restrict__ N, u64 *__restrict__ Fn,
-                                                   uint32_t *__restrict__ segn, int32_t *__restrict__ levels,
-                                                   const int *__restrict__ outdeg, long long m, int nsrc, int level,
+                                                   uint32_t *__restrict__ segn, uint16_t *__restrict__ rowneed,
+                                                   int32_t *__restrict__ levels, const int *__restrict__ outdeg,
+                                                   long long m, int nsrc, int level, u64 all,
                                                    unsigned long long *__restrict__ out) {
+    const int lane = threadIdx.x & 31;
+    const long long warp = (blockIdx.x * (long long)blockDim.x + threadIdx.x) >> 5;
+    const long long nwarps = ((long long)gridDim.x * blockDim.x) >> 5;
     unsigned long long cnt = 0, edges = 0;
-    for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < m; v += (long long)gridDim.x * blockDim.x) {
-        const u64 n = N[v];
-        u64 nw = 0ull;
-        if (n) {
-            nw = n & ~V[v];
-            N[v] = 0ull;
-            if (nw) {
-                V[v] |= nw;
-                atomicOr(&segn[(v >> 4) >> 5], 1u << ((v >> 4) & 31));
-                const int pc = __popcll(nw);
-                cnt += pc;
-                edges += (unsigned long long)pc * (unsigned long long)outdeg[v];
-                u64 b = nw;
-                while (b) {
-                    const int s = __ffsll((long long)b) - 1;
-                    b &= b - 1;
-                    levels[v * nsrc + s] = level + 1;
+    for (long long base = warp * 32; base < m; base += nwarps * 32) {
+        const long long v = base + lane;
+        bool need = false;
+        if (v < m) {
+            const u64 n = N[v];
+            u64 vis = V[v];
+            u64 nw = 0ull;
+            if (n) {
+                nw = n & ~vis;
+                N[v] = 0ull;
+                if (nw) {
+                    vis |= nw;
+                    V[v] = vis;
+                    atomicOr(&segn[(v >> 4) >> 5], 1u << ((v >> 4) & 31));
+                    const int pc = __popcll(nw);
+                    cnt += pc;
+                    edges += (unsigned long long)pc * (unsigned long long)outdeg[v];
+                    u64 b = nw;
+                    while (b) {
+                        const int s = __ffsll((long long)b) - 1;
+                        b &= b - 1;
+                        levels[v * nsrc + s] = level + 1;
+                    }
                 }
             }
+            Fn[v] = nw;
+            need = (all & ~vis) != 0ull;
         }
-        Fn[v] = nw;
+        const unsigned bal = __ballot_sync(0xffffffffu, need);
+        if (lane == 0) {
+            rowneed[base >> 4] = (uint16_t)(bal & 0xffffu);
+            if (base + 16 < m) rowneed[(base >> 4) + 1] = (uint16_t)(bal >> 16);
+        }
     }
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) {
         cnt += __shfl_xor_sync(0xffffffffu, cnt, o);
         edges += __shfl_xor_sync(0xffffffffu, edges, o);
     }
-    if ((threadIdx.x & 31) == 0 && cnt) {
+    if (lane == 0 && cnt) {
         atomicAdd(&out[0], cnt);
         atomicAdd(&out[1], edges);
     }
@@ -193,6 +268,20 @@ extern "C" tsmv_status tsmv_msbfs(tsmv_ctx *c, int32_t nsrc, const int64_t *sour
         c->ms_seg1.ensure(nsw * 4);
         c->ms_src.ensure(64 * 8);
         c->ms_out.ensure(2 * 8);
+        c->ms_rowneed.ensure(((m + 15) / 16 + 1) * 2);
+        if (!c->ms_heavy.p) {  // side vertices with many in-neighbours, once per context
+            c->ms_heavy.alloc(std::max<long long>(m, 1) * 4);
+            DevBuf cntb;
+            cntb.alloc(4);
+            TSMV_CUDA(cudaMemsetAsync(cntb.p, 0, 4, st));
+            k_ms_heavy_list<<<grid_ms(m, c->sm_count * 8), MSB, 0, st>>>(c->Q->sptr.as<long long>(), m,
+                                                                          c->ms_heavy.as<int>(), cntb.as<unsigned>());
+            TSMV_CUDA(cudaGetLastError());
+            unsigned h = 0;
+            TSMV_CUDA(cudaMemcpyAsync(&h, cntb.p, 4, cudaMemcpyDeviceToHost, st));
+            TSMV_CUDA(cudaStreamSynchronize(st));
+            c->ms_nheavy = (int)h;
+        }
         u64 *V = c->ms_V.as<u64>(), *Fa = c->ms_F0.as<u64>(), *Fb = c->ms_F1.as<u64>(), *N = c->ms_N.as<u64>();
         uint32_t *sa = c->ms_seg0.as<uint32_t>(), *sb = c->ms_seg1.as<uint32_t>();
         unsigned long long *out = c->ms_out.as<unsigned long long>();
@@ -204,23 +293,27 @@ extern "C" tsmv_status tsmv_msbfs(tsmv_ctx *c, int32_t nsrc, const int64_t *sour
         TSMV_CUDA(cudaMemsetAsync(N, 0, m * 8, st));
         TSMV_CUDA(cudaMemsetAsync(sa, 0, nsw * 4, st));
         TSMV_CUDA(cudaMemsetAsync(levels, 0xff, (size_t)m * nsrc * 4, st));
+        TSMV_CUDA(cudaMemsetAsync(c->ms_rowneed.p, 0xff, c->ms_rowneed.bytes, st));  // level 0: every row may need
         TSMV_CUDA(cudaMemsetAsync(out, 0, 16, st));
         k_ms_init<<<1, 64, 0, st>>>(c->ms_src.as<long long>(), nsrc, V, Fa, sa, levels);
         k_ms_src_edges<<<1, 64, 0, st>>>(c->ms_src.as<long long>(), nsrc, c->outdeg.as<int>(), out);
         TSMV_CUDA(cudaGetLastError());
         BfsTiles Q = bfs_tiles(*c->Q);
-        const long long nTR = (m + 15) / 16;
         const int gmax = c->sm_count * 8;
         long long pairs = nsrc, edges = 0;
         int L = 0;
         std::vector<unsigned long long> h(2);
         while (true) {
             TSMV_CUDA(cudaMemsetAsync(sb, 0, nsw * 4, st));
-            k_ms_pull_tiles<<<grid_ms(nTR * 32, gmax), MSB, 0, st>>>(Q, V, Fa, sa, N, m, nTR, all);
+            uint16_t *rn = c->ms_rowneed.as<uint16_t>();
+            if (Q.T) k_ms_pull_tiles<<<grid_ms(Q.T, gmax), MSB, 0, st>>>(Q, Fa, sa, rn, N);
             k_ms_pull_side<16><<<grid_ms(m, gmax), MSB, 0, st>>>(Q, V, Fa, N, m, all);
+            if (c->ms_nheavy)
+                k_ms_pull_side_heavy<16><<<grid_ms((long long)c->ms_nheavy * 32, gmax), MSB, 0, st>>>(
+                    Q, V, Fa, N, c->ms_heavy.as<int>(), c->ms_nheavy, all);
             TSMV_CUDA(cudaMemsetAsync(out, 0, 8, st));  // new pairs of this level (edges keep accumulating)
-            k_ms_update<<<grid_ms(m, gmax), MSB, 0, st>>>(V, N, Fb, sb, levels, c->outdeg.as<int>(), m, nsrc, L,
-                                                          out);
+            k_ms_update<<<grid_ms(m, gmax), MSB, 0, st>>>(V, N, Fb, sb, rn, levels, c->outdeg.as<int>(), m, nsrc, L,
+                                                          all, out);
             TSMV_CUDA(cudaGetLastError());
             TSMV_CUDA(cudaMemcpyAsync(h.data(), out, 16, cudaMemcpyDeviceToHost, st));
             TSMV_CUDA(cudaStreamSynchronize(st));

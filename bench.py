@@ -490,9 +490,19 @@ def run_bfs(args, dev, flush, tsmv):
     e1.record()
     torch.cuda.synchronize()
     par_ms = e0.elapsed_time(e1)
+    # multi-source TileBFS (NEXT-3): 64 sources (vertex 0 + 63 hash-ordered)
+    ms_src = [0] + synth.sample_sources(A, 63, seed=2)
+    mlv, _ = M.msbfs(ms_src)
+    flush()
+    torch.cuda.synchronize()
+    mlv, mst = M.msbfs(ms_src, levels=mlv)
+    del mlv
+    msbfs = {"sources": len(ms_src), "ms": round(mst["ms"], 4), "levels": mst["nlevels"],
+             "pairs_reached": mst["pairs_reached"], "edges": mst["edges_traversed"],
+             "gteps": round(mst["edges_traversed"] / (mst["ms"] * 1e-3) / 1e9, 3)}
     M.close()
     return {"graph": f"rmat_s{args.bfs_scale}_ef16_sym", "nnz": info["nnz"], "gteps_hmean": round(hm, 3),
-            "parents_ms": round(par_ms, 4),
+            "parents_ms": round(par_ms, 4), "msbfs_64": msbfs,
             "build_ms": round(info["build_ms"], 2), "build_wall_s": round(build_wall, 3),
             "edge_count": "sum of out-degrees of reached vertices (directed count of the symmetrised graph)",
             "runs": runs}

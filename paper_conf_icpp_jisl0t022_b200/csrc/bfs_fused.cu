@@ -38,6 +38,8 @@ namespace {
 constexpr int BFB = 512;  // threads per CTA
 constexpr int LIST_MAXW = 512;   // list levels only while every frontier vertex has <= this much push work
 constexpr int QCAP = 2048;       // per-CTA shared-memory queue of discovered vertices
+constexpr int SOLO_QS = 2048;    // solo levels: frontier lists in shared memory
+constexpr int SOLO_ROUNDS = 4;   // solo while |F| x group size <= SOLO_ROUNDS x BFB
 
 struct BfsFusedArgs {
     BfsTiles P, Q;
@@ -61,8 +63,14 @@ struct BfsFusedArgs {
     // list-driven push levels
     const int *lwork;
     int *bq0, *bq1;
-    long long *lslots;   // [3][4]
-    int use_list;
+    long long *lslots;   // [3][4] slots, [12..15] profiling, [16] solo release flag, [17..20] solo state
+    int use_list, use_solo;
+};
+
+struct SoloShared {
+    int cnt, pad;
+    unsigned long long mf, din;
+    int maxw, pad2;
 };
 
 struct ListShared {
@@ -278,10 +286,136 @@ __device__ __forceinline__ void seg_counts(const BfsFusedArgs &a, const uint32_t
     }
 }
 
+// Solo levels (session 3): while the frontier is small (|F| x G <= SOLO_ROUNDS x
+// BFB), CTA 0 alone runs the list levels with the vertex lists in shared memory
+// and __syncthreads instead of grid barriers; the other CTAs wait on a release
+// flag.  A level is then: list entry (smem) -> column ranges -> plane words ->
+// atomicOr V -> smem queue -> degrees of the new vertices (~4 dependent L2
+// accesses instead of ~7 plus a grid barrier).  On exit the next frontier is
+// left in the global list and its counter slot, exactly as a grid list level
+// leaves it.  Entry: level L already counted (mu, reached, edges, dir_out).
 template <int NT>
+__device__ void solo_levels(const BfsFusedArgs &a, BfsView &B, int &level, long long &mu, long long &reached,
+                            long long &edges, long long fsize, long long maxw, int (*q)[SOLO_QS], SoloShared &ss,
+                            int tid) {
+    using word_t = typename Tr<NT>::word_t;
+    const word_t *planes = (const word_t *)a.P.planes;
+    {
+        const int *Qc = (level & 1) ? a.bq1 : a.bq0;
+        for (int i = tid; i < fsize; i += BFB) q[0][i] = __ldcg(&Qc[i]);
+    }
+    int cur = 0;
+    long long n = fsize;
+    int G = 1;
+    while (G < maxw && G < 32) G <<= 1;
+    while (true) {
+        B.level = level;
+        int *Qn = (level & 1) ? a.bq0 : a.bq1;  // list of level + 1 (overflow beyond SOLO_QS)
+        if (tid == 0) {
+            ss.cnt = 0;
+            ss.mf = 0;
+            ss.din = 0;
+            ss.maxw = 0;
+        }
+        __syncthreads();
+        const int gl = tid % G;
+        for (long long i = tid / G; i < n; i += BFB / G) {
+            const long long u = q[cur][i];
+            const long long J = u / NT;
+            const int c = (int)(u % NT);
+            const long long t0 = a.P.ptr[J], ntl = a.P.ptr[J + 1] - t0;
+            const long long s0 = a.P.sptr[u], ns = a.P.sptr[u + 1] - s0;
+            for (long long k = gl; k < ntl + ns; k += G) {
+                long long gseg;
+                word_t bits;
+                if (k < ntl) {
+                    const long long t = t0 + k;
+                    bits = planes[(long long)c * a.P.T + t];
+                    gseg = a.P.trow[t];
+                } else {
+                    const long long v = decode_row<NT>(a.P.srow[s0 + (k - ntl)], a.P.hot_list);
+                    bits = (word_t)1 << (v % NT);
+                    gseg = v / NT;
+                }
+                if (!bits) continue;
+                const word_t old = seg_or<NT>(B.V, gseg, bits);
+                word_t nw = bits & ~old;
+                if (!nw) continue;
+                int p = atomicAdd(&ss.cnt, popc_w(nw));
+                while (nw) {
+                    const int r = ffs_w(nw);
+                    nw &= nw - 1;
+                    const long long v = gseg * NT + r;
+                    B.levels[v] = level + 1;
+                    if (p < SOLO_QS) q[cur ^ 1][p] = (int)v;
+                    else Qn[p] = (int)v;
+                    ++p;
+                }
+            }
+        }
+        __syncthreads();
+        const long long n2 = ss.cnt;
+        {
+            unsigned long long mf = 0, din = 0;
+            int mx = 0;
+            for (long long i = tid; i < n2; i += BFB) {
+                const int v = i < SOLO_QS ? q[cur ^ 1][i] : __ldcg(&Qn[i]);
+                mf += (unsigned long long)a.outdeg[v];
+                din += (unsigned long long)a.indeg[v];
+                mx = max(mx, a.lwork[v]);
+            }
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1) {
+                mf += __shfl_xor_sync(0xffffffffu, mf, o);
+                din += __shfl_xor_sync(0xffffffffu, din, o);
+                mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+            }
+            if ((tid & 31) == 0 && (mf | din | (unsigned long long)mx)) {
+                atomicAdd(&ss.mf, mf);
+                atomicAdd(&ss.din, din);
+                atomicMax(&ss.maxw, mx);
+            }
+        }
+        __syncthreads();
+        ++level;
+        const long long mf2 = (long long)ss.mf, din2 = (long long)ss.din, mx2 = ss.maxw;
+        const int dir2 = n2 > 0 ? choose_dir_dev(a.force, a.alpha, a.dens, B.n, n2, mf2, mu - din2) : 0;
+        int G2 = 1;
+        while (G2 < mx2 && G2 < 32) G2 <<= 1;
+        const bool cont = n2 > 0 && dir2 == TSMV_DIR_PUSH_CSC && mx2 <= LIST_MAXW && n2 <= SOLO_QS &&
+                          n2 * G2 <= SOLO_ROUNDS * BFB && level < a.max_levels;
+        if (!cont) {
+            // leave frontier `level` in the global list + its slot, slot level+1 zeroed
+            int *Qg = (level & 1) ? a.bq1 : a.bq0;
+            for (long long i = tid; i < min(n2, (long long)SOLO_QS); i += BFB) Qg[i] = q[cur ^ 1][i];
+            if (tid == 0) {
+                long long *sl = a.lslots + (level % 3) * 4, *sn = a.lslots + ((level + 1) % 3) * 4;
+                sl[0] = n2;
+                sl[1] = mf2;
+                sl[2] = din2;
+                sl[3] = mx2;
+                sn[0] = sn[1] = sn[2] = sn[3] = 0;
+            }
+            __syncthreads();
+            return;
+        }
+        mu -= din2;
+        reached += n2;
+        edges += mf2;
+        if (tid == 0) {
+            a.dir_out[level] = dir2;
+            a.front_out[level] = n2;
+        }
+        cur ^= 1;
+        n = n2;
+        G = G2;
+    }
+}
+
 #ifndef TSMV_BFS_MINB
 #define TSMV_BFS_MINB 1
 #endif
+template <int NT>
 __global__ void __launch_bounds__(BFB, TSMV_BFS_MINB) k_bfs_fused(BfsFusedArgs a) {
     using word_t = typename Tr<NT>::word_t;
     constexpr int NWP = BFB / 32;
@@ -297,6 +431,9 @@ __global__ void __launch_bounds__(BFB, TSMV_BFS_MINB) k_bfs_fused(BfsFusedArgs a
     uint32_t *Fa = B.F, *Fb = B.Fn;
 
     __shared__ ListShared sh;
+    __shared__ int s_soloq[2][SOLO_QS];
+    __shared__ SoloShared s_solo;
+    unsigned long long solo_n = 0;  // solo episodes of this launch (same in every CTA)
     int mode_list = a.use_list && !a.resume;
 
     // ---- init: V = padding bits + source, F0 = {source} (scan mode) or the
@@ -372,6 +509,39 @@ __global__ void __launch_bounds__(BFB, TSMV_BFS_MINB) k_bfs_fused(BfsFusedArgs a
             long long *slot_n = a.lslots + ((level + 1) % 3) * 4;
             int G = 1;
             while (G < maxw && G < 32) G <<= 1;
+            if (a.use_solo && fsize <= SOLO_QS && fsize * G <= SOLO_ROUNDS * BFB) {
+                // small frontier: CTA 0 runs the next levels alone (solo_levels)
+                ++solo_n;
+                if (b == 0) {
+                    solo_levels<NT>(a, B, level, mu, reached, edges, fsize, maxw, s_soloq, s_solo, tid);
+                    if (tid == 0) {
+                        a.lslots[17] = level;
+                        a.lslots[18] = mu;
+                        a.lslots[19] = reached;
+                        a.lslots[20] = edges;
+                        __threadfence();
+                        atomicExch((unsigned long long *)&a.lslots[16], solo_n);
+                    }
+                    __syncthreads();
+                } else {
+                    if (tid == 0) {
+                        while (ld_acquire_u64((const unsigned long long *)&a.lslots[16]) < solo_n) __nanosleep(256);
+                        __threadfence();
+                    }
+                    __syncthreads();
+                    level = (int)__ldcg(&a.lslots[17]);
+                    mu = __ldcg(&a.lslots[18]);
+                    reached = __ldcg(&a.lslots[19]);
+                    edges = __ldcg(&a.lslots[20]);
+                }
+                if (b == 0 && tid == 0) {
+                    const unsigned long long t = globaltimer_ns();
+                    t_e += t - tq;
+                    tq = t;
+                }
+                --level;  // the loop increment brings it back
+                continue;
+            }
 #ifdef TSMV_LIST_PROF
             unsigned long long tl0 = 0, tl1 = 0, tl2 = 0;
             if (b == 0 && tid == 0) tl0 = globaltimer_ns();
@@ -617,7 +787,7 @@ void bfs_list_init(tsmv_ctx *c, cudaStream_t st) {
     c->lwork.alloc(std::max<int64_t>(c->n, 1) * 4);
     c->bq0.alloc(std::max<int64_t>(c->n, 1) * 4);
     c->bq1.alloc(std::max<int64_t>(c->n, 1) * 4);
-    c->lslots.alloc(16 * 8);
+    c->lslots.alloc(24 * 8);
     TSMV_CUDA(cudaMemsetAsync(c->lslots.p, 0, c->lslots.bytes, st));
     const long long n = c->n;
     const int grid = (int)std::max<long long>(1, std::min<long long>((n + 255) / 256, 148LL * 16));
@@ -685,6 +855,8 @@ bool bfs_fused_launch(tsmv_ctx *c, long long source, cudaStream_t st, bool resum
     a.bq1 = c->bq1.as<int>();
     a.lslots = c->lslots.as<long long>();
     a.use_list = (c->lwork.p != nullptr && !getenv("TSMV_BFS_NO_LIST")) ? 1 : 0;
+    a.use_solo = a.use_list && !getenv("TSMV_BFS_NO_SOLO") ? 1 : 0;
+    if (a.use_solo) TSMV_CUDA(cudaMemsetAsync(c->lslots.as<long long>() + 16, 0, 8, st));  // release flag
     void *args[] = {&a};
     void *f = c->nt == 16 ? (void *)k_bfs_fused<16> : c->nt == 32 ? (void *)k_bfs_fused<32> : (void *)k_bfs_fused<64>;
     const int G = c->bfs_blocks;

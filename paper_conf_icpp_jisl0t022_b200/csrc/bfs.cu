@@ -269,6 +269,102 @@ k_fscan(const uint32_t *__restrict__ F, uint32_t *__restrict__ Fclear, long long
     }
 }
 
+// Statistics-only frontier scan for nt = 16 (hybrid driver after a host pull
+// level): thread per HALF segment (8 vertices: 2 + 2 + 4.5 vector loads), grid-
+// stride, block reduction + one atomic per value and block, the last block
+// publishes; half the registers of k_fscan's whole-segment path, so twice the
+// resident threads and no waves.
+__global__ void __launch_bounds__(256) k_fstats16(const uint32_t *__restrict__ F, uint32_t *__restrict__ Fclear,
+                                                  long long nseg, const long long *__restrict__ tptr,
+                                                  const long long *__restrict__ sptr, const int *__restrict__ outdeg,
+                                                  const int *__restrict__ indeg, long long row_begin,
+                                                  long long m_local, Counters *__restrict__ cnt,
+                                                  Counters *__restrict__ hm) {
+    long long q[7] = {0, 0, 0, 0, 0, 0, 0};
+    const long long nh = nseg * 2;
+    for (long long hs = blockIdx.x * (long long)blockDim.x + threadIdx.x; hs < nh;
+         hs += (long long)gridDim.x * blockDim.x) {
+        const long long J = hs >> 1;
+        const int h = (int)(hs & 1);
+        const uint32_t w = F[J >> 1];
+        const unsigned bits8 = (w >> (((J & 1) << 4) + (h << 3))) & 0xffu;
+        if (h == 0 && Fclear && (J & 1) == 0) Fclear[J >> 1] = 0u;
+        if (!bits8) continue;
+        if (h == 0 || !((w >> ((J & 1) << 4)) & 0xffu)) {
+            // tile work of the segment, counted once: by the low half, or by the
+            // high half when the low half is empty
+            const long long wt = tptr[J + 1] - tptr[J];
+            q[0] += wt > 0;
+            q[1] += wt;
+        }
+        const long long v0 = J * 16 + h * 8;
+        int od[8], id[8];
+        long long sp[9];
+        const int4 o0 = __ldg(reinterpret_cast<const int4 *>(outdeg + v0)),
+                   o1 = __ldg(reinterpret_cast<const int4 *>(outdeg + v0) + 1);
+        od[0] = o0.x, od[1] = o0.y, od[2] = o0.z, od[3] = o0.w, od[4] = o1.x, od[5] = o1.y, od[6] = o1.z, od[7] = o1.w;
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+            const longlong2 t = __ldg(reinterpret_cast<const longlong2 *>(sptr + v0) + i);
+            sp[2 * i] = t.x, sp[2 * i + 1] = t.y;
+        }
+        sp[8] = __ldg(sptr + v0 + 8);
+        const long long lv0 = v0 - row_begin;
+        if (lv0 >= 0 && lv0 + 8 <= m_local) {
+            const int4 i0 = __ldg(reinterpret_cast<const int4 *>(indeg + lv0)),
+                       i1 = __ldg(reinterpret_cast<const int4 *>(indeg + lv0) + 1);
+            id[0] = i0.x, id[1] = i0.y, id[2] = i0.z, id[3] = i0.w, id[4] = i1.x, id[5] = i1.y, id[6] = i1.z,
+            id[7] = i1.w;
+        } else {
+#pragma unroll
+            for (int r = 0; r < 8; ++r) id[r] = (lv0 + r >= 0 && lv0 + r < m_local) ? __ldg(indeg + lv0 + r) : 0;
+        }
+        q[4] += __popc(bits8);
+#pragma unroll
+        for (int r = 0; r < 8; ++r) {
+            if ((bits8 >> r) & 1u) {
+                const long long ws = sp[r + 1] - sp[r];
+                q[2] += ws > 0;
+                q[3] += ws;
+                q[5] += od[r];
+                q[6] += id[r];
+            }
+        }
+    }
+    __shared__ unsigned long long s_red[7];
+    __shared__ bool s_last;
+    if (threadIdx.x < 7) s_red[threadIdx.x] = 0;
+    __syncthreads();
+#pragma unroll
+    for (int i = 0; i < 7; ++i) {
+        long long x = q[i];
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) x += __shfl_xor_sync(0xffffffffu, x, o);
+        if ((threadIdx.x & 31) == 0 && x) atomicAdd(&s_red[i], (unsigned long long)x);
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        long long *dst[7] = {&cnt->nLt, &cnt->Wt, &cnt->nLs, &cnt->Ws, &cnt->fsize, &cnt->mf, &cnt->din};
+        for (int i = 0; i < 7; ++i)
+            if (s_red[i]) atomicAdd((unsigned long long *)dst[i], s_red[i]);
+        __threadfence();
+        s_last = atomicAdd(&cnt->fscan_ticket, 1u) == gridDim.x - 1;
+    }
+    __syncthreads();
+    if (s_last && threadIdx.x == 0) {
+        __threadfence();
+        hm->fsize = __ldcg(&cnt->fsize);
+        hm->mf = __ldcg(&cnt->mf);
+        hm->din = __ldcg(&cnt->din);
+        hm->nLt = __ldcg(&cnt->nLt);
+        hm->Wt = __ldcg(&cnt->Wt);
+        hm->nLs = __ldcg(&cnt->nLs);
+        hm->Ws = __ldcg(&cnt->Ws);
+        cnt->chunk_next = 0;
+        cnt->fscan_ticket = 0;
+    }
+}
+
 // Push (vector-driven): tile chunks (Push-CSC, Alg 5) and side chunks.
 template <int NT, bool DO_TILES>
 __global__ void __launch_bounds__(256)
@@ -452,6 +548,20 @@ struct BfsRunner {
         c->epoch++;
         if (!lists)  // the stats-only scan accumulates into zeroed counters {nLt..din}
             TSMV_CUDA(cudaMemsetAsync(&c->counters.as<Counters>()->nLt, 0, 9 * sizeof(long long), st));
+        if (!lists && NT == 16) {
+            int bps = 0;
+            if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_fstats16, 256, 0) != cudaSuccess || bps < 1) {
+                cudaGetLastError();
+                bps = 1;
+            }
+            const int g = (int)std::max<long long>(
+                1, std::min<long long>((nseg * 2 + 255) / 256, (long long)c->sm_count * bps));
+            k_fstats16<<<g, 256, 0, st>>>(F, Fclear, nseg, c->P.ptr.as<long long>(), c->P.sptr.as<long long>(),
+                                          c->outdeg.as<int>(), c->indeg.as<int>(), c->row_begin, c->m,
+                                          c->counters.as<Counters>(), c->hcnt_dev);
+            TSMV_CUDA(cudaGetLastError());
+            return;
+        }
         k_fscan<NT><<<grid, SCAN_BLOCK, 0, st>>>(F, Fclear, nseg, NW, c->P.ptr.as<long long>(),
                                                  c->P.sptr.as<long long>(), c->outdeg.as<int>(), c->indeg.as<int>(),
                                                  c->row_begin, c->m, lists_view(c), c->counters.as<Counters>(),

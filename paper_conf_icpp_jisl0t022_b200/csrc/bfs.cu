@@ -699,7 +699,9 @@ extern "C" tsmv_status tsmv_bfs(tsmv_ctx *c, int64_t source, int32_t *levels, ts
                     ++level;
                     if (fsize == 0 || level >= TSMV_MAX_LEVELS) break;
                     const int dir = choose_dir(c->opt, c->n, fsize, mf, mu - din);
-                    if (dir != TSMV_DIR_PULL_CSC) break;  // resume the fused kernel at `level`
+                    // resume the fused kernel at `level` for push levels and for the late
+                    // (wide) pull levels, which it runs in place without host round trips
+                    if (dir != TSMV_DIR_PULL_CSC || (!getenv("TSMV_BFS_HOST_WIDE") && (mu - din) * 4 < c->nnz)) break;
                     mu -= din;
                     reached += fsize;
                     edges += mf;

@@ -65,6 +65,7 @@ struct BfsFusedArgs {
     int *bq0, *bq1;
     long long *lslots;   // [3][4] slots, [12..15] profiling, [16] solo release flag, [17..20] solo state
     int use_list, use_solo;
+    int wide_in_kernel;       // pull levels with m_u < nnz / 4 stay in the kernel (wide pull)
 };
 
 struct SoloShared {
@@ -645,10 +646,11 @@ __global__ void __launch_bounds__(BFB, TSMV_BFS_MINB) k_bfs_fused(BfsFusedArgs a
             a.dir_out[level] = dir;
             a.front_out[level] = fsize;
         }
-        // Pull levels go back to the host's high-occupancy kernels unless few
-        // edges are left unvisited (m_u <= 16 per thread of this grid: small
-        // graphs, the tail of a high-diameter traversal)
-        if (dir == TSMV_DIR_PULL_CSC && a.stop_on_pull && mu > 16 * gthreads) {
+        // Dense pull levels go back to the host's high-occupancy kernels; pull
+        // levels with few unvisited edges (m_u <= 16 per thread of this grid, or
+        // m_u < nnz / 4: late R-MAT levels, small graphs, the tail of a
+        // high-diameter traversal) run here with the wide row-tile test
+        if (dir == TSMV_DIR_PULL_CSC && a.stop_on_pull && mu > 16 * gthreads && (!a.wide_in_kernel || mu * 4 >= a.nnz)) {
             stopped = 1;  // uniform across CTAs: same totals, same decision
             break;
         }
@@ -856,6 +858,7 @@ bool bfs_fused_launch(tsmv_ctx *c, long long source, cudaStream_t st, bool resum
     a.lslots = c->lslots.as<long long>();
     a.use_list = (c->lwork.p != nullptr && !getenv("TSMV_BFS_NO_LIST")) ? 1 : 0;
     a.use_solo = a.use_list && !getenv("TSMV_BFS_NO_SOLO") ? 1 : 0;
+    a.wide_in_kernel = getenv("TSMV_BFS_HOST_WIDE") ? 0 : 1;
     if (a.use_solo) TSMV_CUDA(cudaMemsetAsync(c->lslots.as<long long>() + 16, 0, 8, st));  // release flag
     void *args[] = {&a};
     void *f = c->nt == 16 ? (void *)k_bfs_fused<16> : c->nt == 32 ? (void *)k_bfs_fused<32> : (void *)k_bfs_fused<64>;

@@ -87,3 +87,25 @@ def test_t_rmat_s22_fp32_and_semirings(tsmv):
     yi, yv = M.spmspv(xi.to(DEV), xv.to(DEV), semiring="min_second")
     check_spmspv(C, yi, yv, xi, xv, semiring=oracle.MIN_SECOND, dtype="f32")
     M.close()
+
+
+def test_c3_rmat_s22_parents_and_multisource(tsmv):
+    """C3 at full size: min-id BFS parents (MIN_SECOND, NEXT-2) against the oracle's
+    Alg 3 over MIN_SECOND, and the 64-source TileBFS (NEXT-3) against the queue BFS
+    on sampled source columns, in the launch configuration bench.py times."""
+    A = synth.rmat(22, 16, seed=1, symmetrize=True, device=DEV)
+    M = tsmv.TiledMatrix.from_csr(A, dtype="pattern")
+    Ah = A.to("cpu")
+    C = oracle.csc_of(Ah)
+    lv, _ = M.bfs(0)
+    par = M.bfs_parents(lv).cpu().numpy()
+    rl, rp = oracle.bfs_parents(C, 0)
+    assert np.array_equal(lv.cpu().numpy(), rl)
+    assert np.array_equal(par, rp)
+    src = [0] + synth.sample_sources(Ah, 63, seed=2)
+    mlv, st = M.msbfs(src)
+    got = mlv.cpu().numpy()
+    for i in (0, 17, 63):
+        assert np.array_equal(got[:, i], oracle.bfs_queue(C, src[i])), f"source column {i}"
+    assert st["pairs_reached"] == int((got >= 0).sum())
+    M.close()

@@ -609,6 +609,20 @@ def run_configs(args, dev, flush, tsmv):
         c2[dt] = [spmspv_gflops(M, A, dt, d, flush) for d in (0.0001, 0.001, 0.01, 0.1)]
         M.close()
     res["C2_rmat_s20_sweep"] = c2
+    # Graph500-style relabelled R-MAT s22 (hubs spread over the id space): SpMSpV at
+    # 1 % (directed, fp64) and TileBFS (symmetrised), to show the numbers above are
+    # not an artefact of the unpermuted generator's hub locality
+    A = synth.attach_values(synth.rmat(22, 16, seed=1, device=dev, permute=True), seed=1)
+    M = tsmv.TiledMatrix.from_csr(A, build_bfs=0)
+    sp = spmspv_gflops(M, A, "f64", 0.01, flush)
+    M.close()
+    del A
+    A = synth.rmat(22, 16, seed=1, symmetrize=True, device=dev, permute=True)
+    M = tsmv.TiledMatrix.from_csr(A, dtype="pattern")
+    res["rmat_s22_permuted"] = {"spmspv_f64_1pct": sp,
+                                "bfs": bfs_gteps(M, A, flush, [synth.sample_sources(A, 1, seed=1)[0]])}
+    M.close()
+    del A
     # C4: 3D 7-point 256^3 and banded (2^20, b = 64): TileBFS + SpMSpV at 1 %
     for name, A in (("C4_stencil3d_256", synth.stencil3d(256, device=dev)),
                     ("C4_banded_2e20_b64", synth.banded(1 << 20, 64, device=dev))):

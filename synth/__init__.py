@@ -30,6 +30,7 @@ S_XVAL = 4
 S_AVAL = 5
 S_UNIF = 6
 S_SRC = 7
+S_PERM = 8   # .. 10: vertex permutation rounds
 
 
 def _s64(c: int) -> int:
@@ -159,8 +160,22 @@ def attach_values(A: CSR, seed: int = 1, dtype: str = "f64", integer: bool = Fal
 
 # --------------------------------------------------------------------------- matrices
 
+def permute_bits(v: torch.Tensor, bits: int, seed: int = 1) -> torch.Tensor:
+    """A seeded bijection of [0, 2^bits): three rounds of (x * odd) mod 2^bits and
+    x ^= x >> ceil(bits/2) (each invertible on bits-bit integers)."""
+    mask = (1 << bits) - 1
+    x = v.to(torch.int64) & mask
+    sh = max(1, (bits + 1) // 2)
+    for rnd in range(3):
+        odd = (_key(seed, S_PERM + rnd) | 1) & 0x7FFFFFFFFFFF
+        x = (x * odd) & mask
+        x = x ^ (x >> sh)
+    return x
+
+
 def rmat(scale: int, edgefactor: int = 16, a: float = 0.57, b: float = 0.19, c: float = 0.19,
-         seed: int = 1, symmetrize: bool = False, device="cpu", chunk: int = 1 << 24) -> CSR:
+         seed: int = 1, symmetrize: bool = False, device="cpu", chunk: int = 1 << 24,
+         permute: bool = False) -> CSR:
     """R-MAT / Kronecker power-law graph (Graph500 parameters by default), no
     vertex permutation, duplicate edges coalesced.  Edge j->i is stored as A[i, j]
     ... here we simply store generated tuple (r, c) as A[r, c]; with
@@ -181,12 +196,16 @@ def rmat(scale: int, edgefactor: int = 16, a: float = 0.57, b: float = 0.19, c: 
             cb = ((u >= ta) & (u < tab)) | (u >= tabc)
             r |= rb.to(torch.int64) << lvl
             cc |= cb.to(torch.int64) << lvl
+        if permute:  # Graph500-style vertex relabelling: hubs no longer sit at low ids
+            r = permute_bits(r, scale, seed)
+            cc = permute_bits(cc, scale, seed)
         parts.append(r * n + cc)
         if symmetrize:
             parts.append(cc * n + r)
     keys = torch.cat(parts)
     del parts
-    return csr_from_keys(keys, n, n, f"rmat_s{scale}_ef{edgefactor}{'_sym' if symmetrize else ''}")
+    return csr_from_keys(keys, n, n, f"rmat_s{scale}_ef{edgefactor}{'_sym' if symmetrize else ''}"
+                         f"{'_perm' if permute else ''}")
 
 
 def stencil2d(nx: int, ny: int, device="cpu") -> CSR:

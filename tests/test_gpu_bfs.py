@@ -147,3 +147,21 @@ def test_bfs_parents_grid_and_3d(tsmv):
         _, rp = oracle.bfs_parents(oracle.csc_of(A), 0)
         assert np.array_equal(got, rp)
         M.close()
+
+
+def test_permuted_rmat(tsmv):
+    """Graph500-style relabelled R-MAT (hubs spread over the id space): levels,
+    parents and multi-source levels still equal the oracle."""
+    A = synth.rmat(12, 16, seed=6, symmetrize=True, permute=True)
+    C = oracle.csc_of(A)
+    M = tsmv.TiledMatrix.from_csr(A.to(DEV), dtype="pattern")
+    src = synth.sample_sources(A, 3, seed=1)
+    for s in src:
+        lv, _ = M.bfs(s)
+        assert np.array_equal(lv.cpu().numpy(), oracle.bfs_queue(C, s))
+        _, rp = oracle.bfs_parents(C, s)
+        assert np.array_equal(M.bfs_parents(lv).cpu().numpy(), rp)
+    mlv, _ = M.msbfs(src)
+    for i, s in enumerate(src):
+        assert np.array_equal(mlv[:, i].cpu().numpy(), oracle.bfs_queue(C, s))
+    M.close()

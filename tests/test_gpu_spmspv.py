@@ -235,3 +235,14 @@ def test_pinned_host_buffers_zero_copy(dtype):
     with pytest.raises(tsmv.TsmvError):
         M.spmspv(pi, pv, y_idx=hyi[:5], y_val=hyv[:5])
     M.close()
+
+
+def test_permuted_rmat_spmspv(tsmv):
+    A = synth.attach_values(synth.rmat(13, 16, seed=8, permute=True), seed=3)
+    C = oracle.csc_of(A)
+    M = tsmv.TiledMatrix.from_csr(A.to(DEV))
+    for d in (0.001, 0.01, 0.1):
+        xi, xv = synth.sample_x(A.n, synth.density_k(A.n, d), seed=4)
+        yi, yv = M.spmspv(xi.to(DEV), xv.to(DEV))
+        check_spmspv(C, yi, yv, xi, xv, Cabs=abs_csc(C))
+    M.close()

@@ -496,6 +496,151 @@ __global__ void __launch_bounds__(256) k_parents(BfsTiles Q, const int32_t *__re
     }
 }
 
+// nt = 16 parents in two passes.  Tile part: warp per row tile I (16 rows at
+// once); lanes walk the tiles of the group in ascending tile-column order, every
+// lane loads the 16 row words of its tile (predicated, one round) and keeps,
+// per row, the first in-neighbour c (ascending) at the previous level; a warp
+// min per row over the first round of 32 tiles with any candidate gives the
+// row's smallest tile-part parent.  Side part: thread per vertex (warp per
+// vertex above 64 side in-neighbours), minimum over the side row.
+__global__ void __launch_bounds__(256) k_parents_tiles16(BfsTiles Q, const int32_t *__restrict__ levels,
+                                                         int32_t *__restrict__ parents, long long m, long long nTR) {
+    const uint16_t *planes = (const uint16_t *)Q.planes;
+    const int lane = threadIdx.x & 31;
+    const long long warp = (blockIdx.x * (long long)blockDim.x + threadIdx.x) >> 5;
+    const long long nwarps = ((long long)gridDim.x * blockDim.x) >> 5;
+    for (long long I = warp; I < nTR; I += nwarps) {
+        const long long v0 = I * 16;
+        const int L = (lane < 16 && v0 + lane < m) ? levels[v0 + lane] : -1;
+        // rows that need a parent: level > 0 (lane r holds row r's level)
+        unsigned need = __ballot_sync(0xffffffffu, L > 0) & 0xffffu;
+        int lvl[16];
+#pragma unroll
+        for (int r = 0; r < 16; ++r) lvl[r] = __shfl_sync(0xffffffffu, L, r);
+        int best[16];
+#pragma unroll
+        for (int r = 0; r < 16; ++r) best[r] = INT_MAX;
+        const long long t0 = Q.ptr[I], t1 = Q.ptr[I + 1];
+        for (long long tb = t0; tb < t1 && need; tb += 32) {
+            const long long t = tb + lane;
+            int cand[16];
+#pragma unroll
+            for (int r = 0; r < 16; ++r) cand[r] = INT_MAX;
+            if (t < t1) {
+                const long long base = (long long)Q.trow[t] * 16;
+                unsigned w[16];
+#pragma unroll
+                for (int r = 0; r < 16; ++r) w[r] = ((need >> r) & 1u) ? planes[(long long)r * Q.T + t] : 0u;
+#pragma unroll
+                for (int r = 0; r < 16; ++r) {
+                    unsigned x = w[r];
+                    while (x) {
+                        const int c = __ffs(x) - 1;
+                        x &= x - 1;
+                        if (levels[base + c] == lvl[r] - 1) {
+                            cand[r] = (int)(base + c);
+                            break;
+                        }
+                    }
+                }
+            }
+            unsigned found = 0;
+#pragma unroll
+            for (int r = 0; r < 16; ++r) {
+                if ((need >> r) & 1u) {  // uniform
+                    const int mn = __reduce_min_sync(0xffffffffu, cand[r]);
+                    if (mn != INT_MAX) {
+                        best[r] = mn;
+                        found |= 1u << r;
+                    }
+                }
+            }
+            need &= ~found;  // rows with a tile-part parent in this round are done
+        }
+        if (lane < 16 && v0 + lane < m) {
+            int bl = INT_MAX;
+#pragma unroll
+            for (int r = 0; r < 16; ++r)
+                if (r == lane) bl = best[r];
+            parents[v0 + lane] = L == 0 ? (int32_t)(v0 + lane) : (L < 0 ? -1 : bl);
+        }
+    }
+}
+
+template <int NT, bool WARP>
+__global__ void __launch_bounds__(256) k_parents_side(BfsTiles Q, const int32_t *__restrict__ levels,
+                                                      int32_t *__restrict__ parents, long long m) {
+    const int lane = threadIdx.x & 31;
+    const long long tid = blockIdx.x * (long long)blockDim.x + threadIdx.x;
+    const long long nt = (long long)gridDim.x * blockDim.x;
+    const long long first = WARP ? (tid >> 5) : tid, stride = WARP ? (nt >> 5) : nt;
+    for (long long v = first; v < m; v += stride) {
+        if (!((Q.smask[v >> 5] >> (v & 31)) & 1u)) continue;
+        const long long p0 = Q.sptr[v], p1 = Q.sptr[v + 1];
+        if ((p1 - p0 > 64) != WARP) continue;
+        const int L = levels[v];
+        if (L <= 0) continue;
+        int cur = parents[v];
+        int sb = cur;
+        if (WARP) {
+            for (long long p = p0 + lane; p < p1; p += 32) {
+                const long long u = decode_row<NT>(Q.srow[p], Q.hot_list);
+                if (u < sb && levels[u] == L - 1) sb = (int)u;
+            }
+            sb = __reduce_min_sync(0xffffffffu, sb);
+            if (lane == 0 && sb < cur) parents[v] = sb;
+        } else {
+            for (long long p = p0; p < p1; ++p) {
+                const long long u = decode_row<NT>(Q.srow[p], Q.hot_list);
+                if (u < sb && levels[u] == L - 1) sb = (int)u;
+            }
+            if (sb < cur) parents[v] = sb;
+        }
+    }
+}
+
+// heavy side rows (> 64 in-neighbours, power-law hubs) in chunks of 256
+// entries, one warp per chunk, combined with atomicMin
+constexpr int PAR_CHUNK = 256;
+__global__ void k_par_chunk_count(const long long *__restrict__ sptr, long long m, int *__restrict__ cnt) {
+    for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < m; v += (long long)gridDim.x * blockDim.x) {
+        const long long len = sptr[v + 1] - sptr[v];
+        cnt[v] = len > 64 ? (int)((len + PAR_CHUNK - 1) / PAR_CHUNK) : 0;
+    }
+}
+__global__ void k_par_chunk_fill(const long long *__restrict__ sptr, long long m, const long long *__restrict__ off,
+                                 const int *__restrict__ cnt, long long *__restrict__ chunks) {
+    for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < m; v += (long long)gridDim.x * blockDim.x)
+        for (int i = 0; i < cnt[v]; ++i) chunks[off[v] + i] = (v << 24) | (long long)i;  // v < 2^39, chunk < 2^24
+}
+template <int NT>
+__global__ void __launch_bounds__(256) k_parents_chunks(BfsTiles Q, const int32_t *__restrict__ levels,
+                                                        int32_t *__restrict__ parents, const long long *__restrict__ chunks,
+                                                        long long nchunks) {
+    const int lane = threadIdx.x & 31;
+    const long long warp = (blockIdx.x * (long long)blockDim.x + threadIdx.x) >> 5;
+    const long long nwarps = ((long long)gridDim.x * blockDim.x) >> 5;
+    for (long long q = warp; q < nchunks; q += nwarps) {
+        const long long e = chunks[q];
+        const long long v = e >> 24, i = e & 0xffffff;
+        const int L = levels[v];
+        if (L <= 0) continue;
+        const long long p0 = Q.sptr[v] + i * PAR_CHUNK, p1 = min(Q.sptr[v + 1], p0 + PAR_CHUNK);
+        int sb = INT_MAX;
+        for (long long p = p0 + lane; p < p1; p += 32) {
+            const long long u = decode_row<NT>(Q.srow[p], Q.hot_list);
+            if (u < sb && levels[u] == L - 1) sb = (int)u;
+        }
+        sb = __reduce_min_sync(0xffffffffu, sb);
+        if (lane == 0 && sb != INT_MAX) atomicMin(&parents[v], sb);
+    }
+}
+
+__global__ void k_parents_fix(int32_t *__restrict__ parents, long long m) {
+    for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < m; v += (long long)gridDim.x * blockDim.x)
+        if (parents[v] == INT_MAX) parents[v] = -1;
+}
+
 __global__ void k_merge(const uint32_t *__restrict__ gathered, long long stride, int nranks,
                         const long long *__restrict__ splits, int self, uint32_t *__restrict__ Fn,
                         uint32_t *__restrict__ V) {
@@ -800,8 +945,36 @@ extern "C" tsmv_status tsmv_bfs_parents(tsmv_ctx *c, const int32_t *levels, int3
         cudaStream_t st = (cudaStream_t)cuda_stream;
         BfsTiles Q = bfs_tiles(*c->Q);
         const int grid = grid_for(c->m * 32);
-        if (c->nt == 16) k_parents<16><<<grid, 256, 0, st>>>(Q, levels, parents, c->m);
-        else if (c->nt == 32) k_parents<32><<<grid, 256, 0, st>>>(Q, levels, parents, c->m);
+        if (c->nt == 16) {
+            const long long nTR = (c->m + 15) / 16;
+            k_parents_tiles16<<<grid_for(nTR * 32), 256, 0, st>>>(Q, levels, parents, c->m, nTR);
+            k_parents_side<16, false><<<grid_for(c->m), 256, 0, st>>>(Q, levels, parents, c->m);
+            if (!c->par_chunks.p) {  // chunk list of the heavy side rows, once per context
+                DevBuf cnt, off;
+                cnt.alloc(std::max<long long>(c->m, 1) * 4);
+                k_par_chunk_count<<<grid_for(c->m), 256, 0, st>>>(c->Q->sptr.as<long long>(), c->m, cnt.as<int>());
+                std::vector<int> hc(c->m);
+                TSMV_CUDA(cudaMemcpyAsync(hc.data(), cnt.p, c->m * 4, cudaMemcpyDeviceToHost, st));
+                TSMV_CUDA(cudaStreamSynchronize(st));
+                std::vector<long long> ho(c->m);
+                long long tot = 0;
+                for (long long v = 0; v < c->m; ++v) {
+                    ho[v] = tot;
+                    tot += hc[v];
+                }
+                off.alloc(std::max<long long>(c->m, 1) * 8);
+                TSMV_CUDA(cudaMemcpyAsync(off.p, ho.data(), c->m * 8, cudaMemcpyHostToDevice, st));
+                c->par_chunks.alloc(std::max<long long>(tot, 1) * 8);
+                k_par_chunk_fill<<<grid_for(c->m), 256, 0, st>>>(c->Q->sptr.as<long long>(), c->m, off.as<long long>(),
+                                                                 cnt.as<int>(), c->par_chunks.as<long long>());
+                TSMV_CUDA(cudaStreamSynchronize(st));
+                c->par_nchunks = tot;
+            }
+            if (c->par_nchunks)
+                k_parents_chunks<16><<<grid_for(c->par_nchunks * 32), 256, 0, st>>>(
+                    Q, levels, parents, c->par_chunks.as<long long>(), c->par_nchunks);
+            k_parents_fix<<<grid_for(c->m), 256, 0, st>>>(parents, c->m);
+        } else if (c->nt == 32) k_parents<32><<<grid, 256, 0, st>>>(Q, levels, parents, c->m);
         else k_parents<64><<<grid, 256, 0, st>>>(Q, levels, parents, c->m);
         TSMV_CUDA(cudaGetLastError());
         return TSMV_OK;

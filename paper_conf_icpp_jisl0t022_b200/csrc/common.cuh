@@ -330,6 +330,8 @@ struct tsmv_ctx {
     tsmv::DevBuf ms_rowneed;                // u16 per row tile: rows still missing some source
     tsmv::DevBuf ms_heavy;                  // int32: side vertices with > MS_HEAVY in-neighbours
     int ms_nheavy = 0;
+    tsmv::DevBuf par_chunks;                // BFS parents: (vertex << 24 | chunk) of heavy side rows
+    long long par_nchunks = 0;
     void *trace = nullptr;         // tsmv_set_trace (device, u64[tsmv_trace_words])
 };
 

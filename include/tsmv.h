@@ -240,6 +240,10 @@ tsmv_status tsmv_msbfs(tsmv_ctx *c, int32_t nsrc, const int64_t *sources, int32_
  * int32[local rows].  All ranks make the same calls in the same order. */
 tsmv_status tsmv_bfs_dist_begin(tsmv_ctx *c, int64_t source, int32_t *levels, int64_t *out_stats,
                                 void *cuda_stream);
+/* dir: TSMV_DIR_PUSH_CSC .. TSMV_DIR_PULL_CSC, optionally | TSMV_DIST_WIDE: a hint
+ * for a late Pull-CSC level (few unvisited edges left: m_u < nnz / 4), which then
+ * tests 32 row tiles' visited words per warp; the result is the same. */
+#define TSMV_DIST_WIDE 0x100
 tsmv_status tsmv_bfs_dist_expand(tsmv_ctx *c, int32_t dir, uint32_t *owned_words_out, void *cuda_stream);
 tsmv_status tsmv_bfs_dist_merge(tsmv_ctx *c, const uint32_t *gathered, int64_t stride_words,
                                 int64_t *out_stats, void *cuda_stream);

@@ -1018,11 +1018,13 @@ extern "C" tsmv_status tsmv_bfs_dist_begin(tsmv_ctx *c, int64_t source, int32_t 
 extern "C" tsmv_status tsmv_bfs_dist_expand(tsmv_ctx *c, int32_t dir, uint32_t *owned_words_out, void *cuda_stream) {
     try {
         TSMV_REQUIRE(c && owned_words_out, "tsmv_bfs_dist_expand: NULL argument");
+        const bool wide = (dir & TSMV_DIST_WIDE) != 0;
+        dir &= ~TSMV_DIST_WIDE;
         TSMV_REQUIRE(dir >= 1 && dir <= 3, "tsmv_bfs_dist_expand: dir must be concrete (1..3)");
         TSMV_CUDA(cudaSetDevice(c->device));
         cudaStream_t st = (cudaStream_t)cuda_stream;
         BfsRunner R{c, st, (long long)(c->V.bytes / 4)};
-        R.do_expand(dir);
+        R.do_expand(dir, wide && dir == TSMV_DIR_PULL_CSC);
         uint32_t *Fnext = (c->fcur == 0 ? c->F1 : c->F0).as<uint32_t>();
         TSMV_CUDA(cudaMemcpyAsync(owned_words_out, Fnext + (c->row_begin >> 5), tsmv_owned_words(c) * 4,
                                   cudaMemcpyDeviceToDevice, st));

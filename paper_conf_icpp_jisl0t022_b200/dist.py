@@ -92,7 +92,9 @@ def bfs_loop(engine, source: int, group=None) -> int:
         red = torch.tensor([mf, mu], dtype=torch.int64, device=dev)
         dist.all_reduce(red, group=group)
         d = engine.choose(engine.n, f, int(red[0]), int(red[1]))
-        owned = engine.expand(d)
+        # late pull levels (few unvisited edges) take the wide row-tile test
+        wide = getattr(engine, "nnz_total", 0) > 0 and int(red[1]) * 4 < engine.nnz_total
+        owned = engine.expand(d, wide=wide)
         gathered = exchange_frontier(owned, engine.stride, group)
         f, mf, mu = engine.merge(gathered, engine.stride)
         levels += 1
@@ -118,6 +120,14 @@ class DistTiledMatrix:
         self.owned = torch.zeros(max(1, (self.m_local + 31) // 32), dtype=torch.int32, device=self.device)
         self.levels = torch.empty(max(1, self.m_local), dtype=torch.int32, device=self.device)
         self._stats = (torch.zeros(3, dtype=torch.int64))
+        # global nnz (one all-reduce at construction): the late-pull hint of bfs_loop;
+        # 0 (no hint) when there is no process group (simulated ranks)
+        self.nnz_total = 0
+        if dist.is_available() and dist.is_initialized():
+            tot = torch.tensor([int(A_local.nnz)], dtype=torch.int64,
+                               device=self.device if dist.get_backend(group) == "nccl" else "cpu")
+            dist.all_reduce(tot, group=group)
+            self.nnz_total = int(tot)
 
     # ---- SpMSpV: x entries are distributed by owner (x_idx in this rank's row range)
     def spmspv(self, x_idx_owned: torch.Tensor, x_val_owned: Optional[torch.Tensor], semiring="plus_times"):
@@ -139,8 +149,9 @@ class DistTiledMatrix:
                         "tsmv_bfs_dist_begin")
         return st[0], st[1], st[2]
 
-    def expand(self, d):
-        self.tsmv.check(self.tsmv.tsmv_bfs_dist_expand(self.M.ctx, int(d), self.owned.data_ptr(),
+    def expand(self, d, wide=False):
+        d = int(d) | (self.tsmv.DIST_WIDE if wide else 0)
+        self.tsmv.check(self.tsmv.tsmv_bfs_dist_expand(self.M.ctx, d, self.owned.data_ptr(),
                                                        torch.cuda.current_stream().cuda_stream),
                         "tsmv_bfs_dist_expand")
         return self.owned

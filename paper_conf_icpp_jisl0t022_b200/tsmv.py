@@ -26,6 +26,7 @@ _lib = ctypes.CDLL(LIB_PATH)
 
 # --------------------------------------------------------------------------- ABI types
 OK, EINVAL, ENOMEM, ECUDA, ENCCL, ECAPACITY, EUNSUPPORTED = range(7)
+DIST_WIDE = 0x100   # tsmv_bfs_dist_expand hint for late pull levels (TSMV_DIST_WIDE)
 F64, F32, PATTERN = 0, 1, 2
 PLUS_TIMES, OR_AND, MIN_SECOND = 0, 1, 2
 DIR_AUTO, DIR_PUSH_CSC, DIR_PUSH_CSR, DIR_PULL_CSC = 0, 1, 2, 3

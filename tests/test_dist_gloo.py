@@ -98,7 +98,7 @@ class NumpyEngine:
         self.L = 0
         return self._stats()
 
-    def expand(self, d):
+    def expand(self, d, wide=False):  # wide: late-pull hint (no effect on results)
         y = (self.B @ self.F.astype(np.float64)) > 0
         new = y & ~self.V[self.r0:self.r1]
         return _pack_words(new)

@@ -32,7 +32,8 @@ def _sim_bfs(engines, source):
         mf = sum(s[1] for s in st)
         mu = sum(s[2] for s in st)
         d = engines[0].choose(engines[0].n, st[0][0], mf, mu)
-        owned = [e.expand(d).clone() for e in engines]
+        nnz = sum(e.M.nnz for e in engines)
+        owned = [e.expand(d, wide=mu * 4 < nnz).clone() for e in engines]   # late-pull hint as bfs_loop
         stride = engines[0].stride
         gathered = torch.zeros(len(engines) * stride, dtype=torch.int32, device=DEV)
         for p, o in enumerate(owned):

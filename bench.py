@@ -51,6 +51,8 @@ def parse():
     p.add_argument("--thr", type=int, default=2)
     p.add_argument("--bfs-scale", type=int, default=22)
     p.add_argument("--bfs-sources", type=int, default=4)
+    p.add_argument("--bfs-thr", type=int, default=8,
+                   help="very-sparse-tile threshold of the TileBFS contexts (DESIGN.md R25; SpMSpV keeps --thr)")
     p.add_argument("--no-bfs", action="store_true")
     p.add_argument("--no-cpu", action="store_true")
     p.add_argument("--cpu-seconds", type=float, default=12.0)
@@ -463,7 +465,7 @@ def run_bfs(args, dev, flush, tsmv):
     """TileBFS GTEPS on the symmetrised R-MAT (BASELINE config 3 shape)."""
     A = synth.rmat(args.bfs_scale, 16, seed=1, symmetrize=True, device=dev)
     t0 = time.perf_counter()
-    M = tsmv.TiledMatrix.from_csr(A, dtype="pattern", tile_dim=args.tile_dim, sparse_tile_max_nnz=args.thr)
+    M = tsmv.TiledMatrix.from_csr(A, dtype="pattern", tile_dim=args.tile_dim, sparse_tile_max_nnz=args.bfs_thr)
     build_wall = time.perf_counter() - t0
     info = M.info()
     srcs = [0] + synth.sample_sources(A, max(0, args.bfs_sources - 1), seed=1)
@@ -501,7 +503,8 @@ def run_bfs(args, dev, flush, tsmv):
              "pairs_reached": mst["pairs_reached"], "edges": mst["edges_traversed"],
              "gteps": round(mst["edges_traversed"] / (mst["ms"] * 1e-3) / 1e9, 3)}
     M.close()
-    return {"graph": f"rmat_s{args.bfs_scale}_ef16_sym", "nnz": info["nnz"], "gteps_hmean": round(hm, 3),
+    return {"graph": f"rmat_s{args.bfs_scale}_ef16_sym", "sparse_tile_max_nnz": args.bfs_thr,
+            "nnz": info["nnz"], "gteps_hmean": round(hm, 3),
             "parents_ms": round(par_ms, 4), "msbfs_64": msbfs,
             "build_ms": round(info["build_ms"], 2), "build_wall_s": round(build_wall, 3),
             "edge_count": "sum of out-degrees of reached vertices (directed count of the symmetrised graph)",
@@ -524,7 +527,7 @@ def run_bfs_dist(args, dev, flush, rank, world):
     del A
     t0 = time.perf_counter()
     D = tdist.DistTiledMatrix(Al, splits, rank, world, dtype="pattern", device=dev.index,
-                              tile_dim=args.tile_dim, sparse_tile_max_nnz=args.thr)
+                              tile_dim=args.tile_dim, sparse_tile_max_nnz=args.bfs_thr)
     build_wall = time.perf_counter() - t0
     rowlen = (Al.row_ptr[1:] - Al.row_ptr[:-1]).to(torch.int64)
     D.bfs(srcs[0])  # warm-up
@@ -618,7 +621,7 @@ def run_configs(args, dev, flush, tsmv):
     M.close()
     del A
     A = synth.rmat(22, 16, seed=1, symmetrize=True, device=dev, permute=True)
-    M = tsmv.TiledMatrix.from_csr(A, dtype="pattern")
+    M = tsmv.TiledMatrix.from_csr(A, dtype="pattern", sparse_tile_max_nnz=args.bfs_thr)
     res["rmat_s22_permuted"] = {"spmspv_f64_1pct": sp,
                                 "bfs": bfs_gteps(M, A, flush, [synth.sample_sources(A, 1, seed=1)[0]])}
     M.close()

@@ -13,7 +13,7 @@ elif name.startswith("grid3d"):
 else:
     n, b = name[4:].split("_")
     A = synth.banded(1 << int(n), int(b), device=dev).with_values(None)
-M = tsmv.TiledMatrix.from_csr(A, dtype="pattern")
+M = tsmv.TiledMatrix.from_csr(A, dtype="pattern", sparse_tile_max_nnz=int(os.environ.get("THR", "2")))
 src = int(sys.argv[2]) if len(sys.argv) > 2 else 0
 lv = torch.empty(A.n, dtype=torch.int32, device=dev)
 M.bfs(src, levels=lv)

@@ -577,7 +577,7 @@ __global__ void __launch_bounds__(256) k_parents_side(BfsTiles Q, const int32_t 
     for (long long v = first; v < m; v += stride) {
         if (!((Q.smask[v >> 5] >> (v & 31)) & 1u)) continue;
         const long long p0 = Q.sptr[v], p1 = Q.sptr[v + 1];
-        if ((p1 - p0 > 64) != WARP) continue;
+        if ((p1 - p0 > 32) != WARP) continue;
         const int L = levels[v];
         if (L <= 0) continue;
         int cur = parents[v];
@@ -590,9 +590,16 @@ __global__ void __launch_bounds__(256) k_parents_side(BfsTiles Q, const int32_t 
             sb = __reduce_min_sync(0xffffffffu, sb);
             if (lane == 0 && sb < cur) parents[v] = sb;
         } else {
-            for (long long p = p0; p < p1; ++p) {
-                const long long u = decode_row<NT>(Q.srow[p], Q.hot_list);
-                if (u < sb && levels[u] == L - 1) sb = (int)u;
+            for (long long p = p0; p < p1; p += 4) {  // 4 in-neighbours, then their levels, per round
+                long long u[4];
+#pragma unroll
+                for (int j = 0; j < 4; ++j) u[j] = p + j < p1 ? decode_row<NT>(Q.srow[p + j], Q.hot_list) : -1;
+                int lv[4];
+#pragma unroll
+                for (int j = 0; j < 4; ++j) lv[j] = (u[j] >= 0 && u[j] < sb) ? levels[u[j]] : -2;
+#pragma unroll
+                for (int j = 0; j < 4; ++j)
+                    if (lv[j] == L - 1 && u[j] < sb) sb = (int)u[j];
             }
             if (sb < cur) parents[v] = sb;
         }
@@ -605,7 +612,7 @@ constexpr int PAR_CHUNK = 256;
 __global__ void k_par_chunk_count(const long long *__restrict__ sptr, long long m, int *__restrict__ cnt) {
     for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < m; v += (long long)gridDim.x * blockDim.x) {
         const long long len = sptr[v + 1] - sptr[v];
-        cnt[v] = len > 64 ? (int)((len + PAR_CHUNK - 1) / PAR_CHUNK) : 0;
+        cnt[v] = len > 32 ? (int)((len + PAR_CHUNK - 1) / PAR_CHUNK) : 0;
     }
 }
 __global__ void k_par_chunk_fill(const long long *__restrict__ sptr, long long m, const long long *__restrict__ off,

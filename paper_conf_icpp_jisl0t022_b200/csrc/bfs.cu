@@ -821,7 +821,10 @@ extern "C" tsmv_status tsmv_bfs(tsmv_ctx *c, int64_t source, int32_t *levels, ts
                 long long L, mu2, r2, e2;
                 int cur;
                 const bool stopped = bfs_fused_launch(c, source, st, resume, level, Fa, Fb, mu, reached, edges,
-                                                      stop_on_pull, TSMV_MAX_LEVELS, L, mu2, r2, e2, cur);
+                                                      stop_on_pull,
+                                                      getenv("TSMV_BFS_MAXLV") ? atoi(getenv("TSMV_BFS_MAXLV"))
+                                                                               : TSMV_MAX_LEVELS,
+                                                      L, mu2, r2, e2, cur);
                 if (getenv("TSMV_BFS_PHASES")) {
                     long long fl = 0;
                     if (c->lslots.p) {

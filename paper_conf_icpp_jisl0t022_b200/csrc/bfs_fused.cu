@@ -37,7 +37,10 @@ namespace {
 
 constexpr int BFB = 512;  // threads per CTA
 constexpr int LIST_MAXW = 512;   // list levels only while every frontier vertex has <= this much push work
-constexpr int QCAP = 2048;       // per-CTA shared-memory queue of discovered vertices
+#ifndef TSMV_QCAP
+#define TSMV_QCAP 2048
+#endif
+constexpr int QCAP = TSMV_QCAP;  // per-CTA shared-memory queue of discovered vertices
 constexpr int SOLO_QS = 2048;    // solo levels: frontier lists in shared memory
 constexpr int SOLO_ROUNDS = 4;   // solo while |F| x group size <= SOLO_ROUNDS x BFB
 

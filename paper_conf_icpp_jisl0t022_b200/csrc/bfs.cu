@@ -944,6 +944,32 @@ extern "C" tsmv_status tsmv_bfs(tsmv_ctx *c, int64_t source, int32_t *levels, ts
     }
 }
 
+// Chunk list (vertex << 24 | chunk of 256 entries) of the side rows of Q with
+// more than 32 entries (power-law hubs), built once per context; used by the
+// parents and multi-source BFS kernels.
+void tsmv::heavy_side_chunks(tsmv_ctx *c, cudaStream_t st) {
+    if (c->par_chunks.p) return;
+    DevBuf cnt, off;
+    cnt.alloc(std::max<long long>(c->m, 1) * 4);
+    k_par_chunk_count<<<grid_for(c->m), 256, 0, st>>>(c->Q->sptr.as<long long>(), c->m, cnt.as<int>());
+    std::vector<int> hc(c->m);
+    TSMV_CUDA(cudaMemcpyAsync(hc.data(), cnt.p, c->m * 4, cudaMemcpyDeviceToHost, st));
+    TSMV_CUDA(cudaStreamSynchronize(st));
+    std::vector<long long> ho(c->m);
+    long long tot = 0;
+    for (long long v = 0; v < c->m; ++v) {
+        ho[v] = tot;
+        tot += hc[v];
+    }
+    off.alloc(std::max<long long>(c->m, 1) * 8);
+    TSMV_CUDA(cudaMemcpyAsync(off.p, ho.data(), c->m * 8, cudaMemcpyHostToDevice, st));
+    c->par_chunks.alloc(std::max<long long>(tot, 1) * 8);
+    k_par_chunk_fill<<<grid_for(c->m), 256, 0, st>>>(c->Q->sptr.as<long long>(), c->m, off.as<long long>(),
+                                                     cnt.as<int>(), c->par_chunks.as<long long>());
+    TSMV_CUDA(cudaStreamSynchronize(st));
+    c->par_nchunks = tot;
+}
+
 extern "C" tsmv_status tsmv_bfs_parents(tsmv_ctx *c, const int32_t *levels, int32_t *parents, void *cuda_stream) {
     try {
         TSMV_REQUIRE(c != nullptr && levels != nullptr && parents != nullptr, "tsmv_bfs_parents: NULL argument");
@@ -959,27 +985,7 @@ extern "C" tsmv_status tsmv_bfs_parents(tsmv_ctx *c, const int32_t *levels, int3
             const long long nTR = (c->m + 15) / 16;
             k_parents_tiles16<<<grid_for(nTR * 32), 256, 0, st>>>(Q, levels, parents, c->m, nTR);
             k_parents_side<16, false><<<grid_for(c->m), 256, 0, st>>>(Q, levels, parents, c->m);
-            if (!c->par_chunks.p) {  // chunk list of the heavy side rows, once per context
-                DevBuf cnt, off;
-                cnt.alloc(std::max<long long>(c->m, 1) * 4);
-                k_par_chunk_count<<<grid_for(c->m), 256, 0, st>>>(c->Q->sptr.as<long long>(), c->m, cnt.as<int>());
-                std::vector<int> hc(c->m);
-                TSMV_CUDA(cudaMemcpyAsync(hc.data(), cnt.p, c->m * 4, cudaMemcpyDeviceToHost, st));
-                TSMV_CUDA(cudaStreamSynchronize(st));
-                std::vector<long long> ho(c->m);
-                long long tot = 0;
-                for (long long v = 0; v < c->m; ++v) {
-                    ho[v] = tot;
-                    tot += hc[v];
-                }
-                off.alloc(std::max<long long>(c->m, 1) * 8);
-                TSMV_CUDA(cudaMemcpyAsync(off.p, ho.data(), c->m * 8, cudaMemcpyHostToDevice, st));
-                c->par_chunks.alloc(std::max<long long>(tot, 1) * 8);
-                k_par_chunk_fill<<<grid_for(c->m), 256, 0, st>>>(c->Q->sptr.as<long long>(), c->m, off.as<long long>(),
-                                                                 cnt.as<int>(), c->par_chunks.as<long long>());
-                TSMV_CUDA(cudaStreamSynchronize(st));
-                c->par_nchunks = tot;
-            }
+            heavy_side_chunks(c, st);
             if (c->par_nchunks)
                 k_parents_chunks<16><<<grid_for(c->par_nchunks * 32), 256, 0, st>>>(
                     Q, levels, parents, c->par_chunks.as<long long>(), c->par_nchunks);

@@ -328,8 +328,6 @@ struct tsmv_ctx {
     tsmv::DevBuf ms_seg0, ms_seg1;          // u32: 1 bit per 16-vertex segment holding frontier vertices
     tsmv::DevBuf ms_src, ms_out;
     tsmv::DevBuf ms_rowneed;                // u16 per row tile: rows still missing some source
-    tsmv::DevBuf ms_heavy;                  // int32: side vertices with > MS_HEAVY in-neighbours
-    int ms_nheavy = 0;
     tsmv::DevBuf par_chunks;                // BFS parents: (vertex << 24 | chunk) of heavy side rows
     long long par_nchunks = 0;
     void *trace = nullptr;         // tsmv_set_trace (device, u64[tsmv_trace_words])
@@ -362,6 +360,7 @@ void enqueue_spmspv_flat(tsmv_ctx *c, int sr, long long k, const int32_t *xi, co
 // bfs_fused.cu
 int bfs_fused_occupancy(int nt);
 void bfs_list_init(tsmv_ctx *c, cudaStream_t st);
+void heavy_side_chunks(tsmv_ctx *c, cudaStream_t st);  // bfs.cu: chunks of side rows > 32 entries
 bool bfs_fused_launch(tsmv_ctx *c, long long source, cudaStream_t st, bool resume, long long level0, uint32_t *Fa,
                       uint32_t *Fb, long long mu, long long reached, long long edges, bool stop_on_pull,
                       long long max_levels, long long &level_out, long long &mu_out, long long &reached_out,

@@ -110,8 +110,8 @@ __global__ void __launch_bounds__(MSB) k_ms_pull_tiles(BfsTiles Q, const u64 *__
 
 // side part: in-neighbours u of v in the side CSR of Q.  Vertices with at most
 // MS_HEAVY side in-neighbours: thread per vertex, stop once every missing source
-// is found; heavier ones (power-law hubs) go to k_ms_pull_side_heavy.
-constexpr int MS_HEAVY = 64;
+// is found; heavier ones (power-law hubs) go to k_ms_pull_side_chunks.
+constexpr int MS_HEAVY = 32;  // = the chunk threshold of heavy_side_chunks
 
 template <int NT>
 __global__ void __launch_bounds__(MSB) k_ms_pull_side(BfsTiles Q, const u64 *__restrict__ V, const u64 *__restrict__ F,
@@ -136,38 +136,33 @@ __global__ void __launch_bounds__(MSB) k_ms_pull_side(BfsTiles Q, const u64 *__r
     }
 }
 
+// heavy side rows in 256-entry chunks (heavy_side_chunks), one warp per chunk,
+// merged into N with atomicOr; a chunk stops early once its rows cover every
+// source the vertex still misses
 template <int NT>
-__global__ void __launch_bounds__(MSB) k_ms_pull_side_heavy(BfsTiles Q, const u64 *__restrict__ V,
-                                                            const u64 *__restrict__ F, u64 *__restrict__ N,
-                                                            const int *__restrict__ heavy, int nheavy, u64 all) {
+__global__ void __launch_bounds__(MSB) k_ms_pull_side_chunks(BfsTiles Q, const u64 *__restrict__ V,
+                                                             const u64 *__restrict__ F, u64 *__restrict__ N,
+                                                             const long long *__restrict__ chunks, long long nchunks,
+                                                             u64 all) {
     const int lane = threadIdx.x & 31;
     const long long warp = (blockIdx.x * (long long)blockDim.x + threadIdx.x) >> 5;
     const long long nwarps = ((long long)gridDim.x * blockDim.x) >> 5;
-    for (long long i = warp; i < nheavy; i += nwarps) {
-        const long long v = heavy[i];
-        const u64 need = all & ~V[v] & ~N[v];
+    for (long long q = warp; q < nchunks; q += nwarps) {
+        const long long e = chunks[q];
+        const long long v = e >> 24, i = e & 0xffffff;
+        const u64 need = all & ~V[v];
         if (!need) continue;
-        const long long p0 = Q.sptr[v], p1 = Q.sptr[v + 1];
+        const long long p0 = Q.sptr[v] + i * 256, p1 = min(Q.sptr[v + 1], p0 + 256);
         u64 acc = 0ull;
         for (long long pb = p0; pb < p1; pb += 32) {
             if (pb + lane < p1) acc |= F[decode_row<NT>(Q.srow[pb + lane], Q.hot_list)];
-            const u64 w = warp_or64(acc);
-            if ((w & need) == need) {
-                acc = w;
-                break;
-            }
-            acc = w;
+            acc = warp_or64(acc);
+            if ((acc & need) == need) break;
         }
-        if (lane == 0 && (acc & need)) N[v] |= acc & need;
+        if (lane == 0 && (acc & need)) atomicOr(&N[v], acc & need);
     }
 }
 
-// side vertices with more than MS_HEAVY in-neighbours (built once per context)
-__global__ void k_ms_heavy_list(const long long *__restrict__ sptr, long long m, int *__restrict__ heavy,
-                                unsigned *__restrict__ nheavy) {
-    for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < m; v += (long long)gridDim.x * blockDim.x)
-        if (sptr[v + 1] - sptr[v] > MS_HEAVY) heavy[atomicAdd(nheavy, 1u)] = (int)v;
-}
 
 // new = N & ~V; V |= new; next frontier = new; levels; counts; rowneed[I] =
 // rows of row tile I still missing some source (a warp covers 32 consecutive
@@ -184,6 +179,7 @@ __global__ void __launch_bounds__(MSB) k_ms_update(u64 *__restrict__ V, u64 *__r
     for (long long base = warp * 32; base < m; base += nwarps * 32) {
         const long long v = base + lane;
         bool need = false;
+        u64 newbits = 0ull;
         if (v < m) {
             const u64 n = N[v];
             u64 vis = V[v];
@@ -198,16 +194,22 @@ __global__ void __launch_bounds__(MSB) k_ms_update(u64 *__restrict__ V, u64 *__r
                     const int pc = __popcll(nw);
                     cnt += pc;
                     edges += (unsigned long long)pc * (unsigned long long)outdeg[v];
-                    u64 b = nw;
-                    while (b) {
-                        const int s = __ffsll((long long)b) - 1;
-                        b &= b - 1;
-                        levels[v * nsrc + s] = level + 1;
-                    }
                 }
             }
             Fn[v] = nw;
             need = (all & ~vis) != 0ull;
+            newbits = nw;
+        }
+        // levels of the new (vertex, source) pairs: the warp writes one vertex row
+        // (nsrc int32) at a time, lane l taking sources l and l + 32
+        unsigned todo = __ballot_sync(0xffffffffu, newbits != 0ull);
+        while (todo) {
+            const int src_lane = __ffs(todo) - 1;
+            todo &= todo - 1;
+            const u64 nb = __shfl_sync(0xffffffffu, newbits, src_lane);
+            const long long row = (base + src_lane) * nsrc;
+            if ((nb >> lane) & 1ull) levels[row + lane] = level + 1;
+            if (lane + 32 < nsrc && ((nb >> (lane + 32)) & 1ull)) levels[row + lane + 32] = level + 1;
         }
         const unsigned bal = __ballot_sync(0xffffffffu, need);
         if (lane == 0) {
@@ -269,19 +271,7 @@ extern "C" tsmv_status tsmv_msbfs(tsmv_ctx *c, int32_t nsrc, const int64_t *sour
         c->ms_src.ensure(64 * 8);
         c->ms_out.ensure(2 * 8);
         c->ms_rowneed.ensure(((m + 15) / 16 + 1) * 2);
-        if (!c->ms_heavy.p) {  // side vertices with many in-neighbours, once per context
-            c->ms_heavy.alloc(std::max<long long>(m, 1) * 4);
-            DevBuf cntb;
-            cntb.alloc(4);
-            TSMV_CUDA(cudaMemsetAsync(cntb.p, 0, 4, st));
-            k_ms_heavy_list<<<grid_ms(m, c->sm_count * 8), MSB, 0, st>>>(c->Q->sptr.as<long long>(), m,
-                                                                          c->ms_heavy.as<int>(), cntb.as<unsigned>());
-            TSMV_CUDA(cudaGetLastError());
-            unsigned h = 0;
-            TSMV_CUDA(cudaMemcpyAsync(&h, cntb.p, 4, cudaMemcpyDeviceToHost, st));
-            TSMV_CUDA(cudaStreamSynchronize(st));
-            c->ms_nheavy = (int)h;
-        }
+        heavy_side_chunks(c, st);
         u64 *V = c->ms_V.as<u64>(), *Fa = c->ms_F0.as<u64>(), *Fb = c->ms_F1.as<u64>(), *N = c->ms_N.as<u64>();
         uint32_t *sa = c->ms_seg0.as<uint32_t>(), *sb = c->ms_seg1.as<uint32_t>();
         unsigned long long *out = c->ms_out.as<unsigned long long>();
@@ -308,9 +298,9 @@ extern "C" tsmv_status tsmv_msbfs(tsmv_ctx *c, int32_t nsrc, const int64_t *sour
             uint16_t *rn = c->ms_rowneed.as<uint16_t>();
             if (Q.T) k_ms_pull_tiles<<<grid_ms(Q.T, gmax), MSB, 0, st>>>(Q, Fa, sa, rn, N);
             k_ms_pull_side<16><<<grid_ms(m, gmax), MSB, 0, st>>>(Q, V, Fa, N, m, all);
-            if (c->ms_nheavy)
-                k_ms_pull_side_heavy<16><<<grid_ms((long long)c->ms_nheavy * 32, gmax), MSB, 0, st>>>(
-                    Q, V, Fa, N, c->ms_heavy.as<int>(), c->ms_nheavy, all);
+            if (c->par_nchunks)
+                k_ms_pull_side_chunks<16><<<grid_ms(c->par_nchunks * 32, gmax), MSB, 0, st>>>(
+                    Q, V, Fa, N, c->par_chunks.as<long long>(), c->par_nchunks, all);
             TSMV_CUDA(cudaMemsetAsync(out, 0, 8, st));  // new pairs of this level (edges keep accumulating)
             k_ms_update<<<grid_ms(m, gmax), MSB, 0, st>>>(V, N, Fb, sb, rn, levels, c->outdeg.as<int>(), m, nsrc, L,
                                                           all, out);

@@ -245,6 +245,9 @@ tsmv_status tsmv_bfs_dist_begin(tsmv_ctx *c, int64_t source, int32_t *levels, in
  * tests 32 row tiles' visited words per warp; the result is the same. */
 #define TSMV_DIST_WIDE 0x100
 tsmv_status tsmv_bfs_dist_expand(tsmv_ctx *c, int32_t dir, uint32_t *owned_words_out, void *cuda_stream);
+/* merge: out_stats may be host memory (the call synchronises, as begin does) or
+ * device memory (int64[3] written on the stream, no synchronisation: the caller
+ * all-reduces m_f / m_u on the device and reads the level's result once). */
 tsmv_status tsmv_bfs_dist_merge(tsmv_ctx *c, const uint32_t *gathered, int64_t stride_words,
                                 int64_t *out_stats, void *cuda_stream);
 /* Words of this rank's owned segment = ceil((row_splits[r+1]-row_splits[r])/32). */

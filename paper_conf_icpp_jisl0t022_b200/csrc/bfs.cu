@@ -648,6 +648,15 @@ __global__ void k_parents_fix(int32_t *__restrict__ parents, long long m) {
         if (parents[v] == INT_MAX) parents[v] = -1;
 }
 
+// distributed merge with device statistics: {|F| (global), m_f local, m_u local}
+__global__ void k_dist_stats(const Counters *__restrict__ cnt, long long *__restrict__ mu, int64_t *__restrict__ out) {
+    const long long m = *mu - cnt->din;
+    *mu = m;
+    out[0] = cnt->fsize;
+    out[1] = cnt->mf;
+    out[2] = m;
+}
+
 __global__ void k_merge(const uint32_t *__restrict__ gathered, long long stride, int nranks,
                         const long long *__restrict__ splits, int self, uint32_t *__restrict__ Fn,
                         uint32_t *__restrict__ V) {
@@ -1022,6 +1031,9 @@ extern "C" tsmv_status tsmv_bfs_dist_begin(tsmv_ctx *c, int64_t source, int32_t 
         TSMV_CUDA(cudaStreamSynchronize(st));
         volatile Counters *h = c->hcnt;
         c->m_u_local = c->nnz - h->din;
+        c->mu_dev.ensure(8);
+        TSMV_CUDA(cudaMemcpyAsync(c->mu_dev.p, &c->m_u_local, 8, cudaMemcpyHostToDevice, st));
+        TSMV_CUDA(cudaStreamSynchronize(st));
         out_stats[0] = h->fsize;
         out_stats[1] = h->mf;
         out_stats[2] = c->m_u_local;
@@ -1067,11 +1079,20 @@ extern "C" tsmv_status tsmv_bfs_dist_merge(tsmv_ctx *c, const uint32_t *gathered
             TSMV_CUDA(cudaGetLastError());
         }
         R.do_fscan(Fnext, Fcur);
+        c->fcur ^= 1;
+        c->bfs_level += 1;
+        if (is_device_ptr(out_stats)) {
+            // device statistics: no synchronisation here (the caller all-reduces
+            // them on the device and reads the result once per level)
+            k_dist_stats<<<1, 1, 0, st>>>(c->counters.as<Counters>(), c->mu_dev.as<long long>(), out_stats);
+            TSMV_CUDA(cudaGetLastError());
+            return TSMV_OK;
+        }
         TSMV_CUDA(cudaStreamSynchronize(st));
         volatile Counters *h = c->hcnt;
         c->m_u_local -= h->din;
-        c->fcur ^= 1;
-        c->bfs_level += 1;
+        TSMV_CUDA(cudaMemcpyAsync(c->mu_dev.p, &c->m_u_local, 8, cudaMemcpyHostToDevice, st));
+        TSMV_CUDA(cudaStreamSynchronize(st));
         out_stats[0] = h->fsize;
         out_stats[1] = h->mf;
         out_stats[2] = c->m_u_local;

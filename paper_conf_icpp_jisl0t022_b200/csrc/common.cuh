@@ -328,6 +328,7 @@ struct tsmv_ctx {
     tsmv::DevBuf ms_seg0, ms_seg1;          // u32: 1 bit per 16-vertex segment holding frontier vertices
     tsmv::DevBuf ms_src, ms_out;
     tsmv::DevBuf ms_rowneed;                // u16 per row tile: rows still missing some source
+    tsmv::DevBuf mu_dev;                    // distributed BFS: m_u of this rank on the device
     tsmv::DevBuf par_chunks;                // BFS parents: (vertex << 24 | chunk) of heavy side rows
     long long par_nchunks = 0;
     void *trace = nullptr;         // tsmv_set_trace (device, u64[tsmv_trace_words])

@@ -18,6 +18,7 @@ replicated visited bitmap, the frontier scan) runs in libtsmv.so.
 """
 from __future__ import annotations
 
+import ctypes
 from typing import List, Optional, Sequence
 
 import torch
@@ -87,16 +88,27 @@ def bfs_loop(engine, source: int, group=None) -> int:
     stride (padded words), n, choose(n, |F|, m_f, m_u).  Returns the number of levels."""
     dev = engine.device
     f, mf, mu = engine.begin(source)
+    red = torch.tensor([mf, mu], dtype=torch.int64, device=dev)
+    dist.all_reduce(red, group=group)
+    gmf, gmu = (int(x) for x in red.tolist())
     levels = 0
     while f > 0:
-        red = torch.tensor([mf, mu], dtype=torch.int64, device=dev)
-        dist.all_reduce(red, group=group)
-        d = engine.choose(engine.n, f, int(red[0]), int(red[1]))
+        d = engine.choose(engine.n, f, gmf, gmu)
         # late pull levels (few unvisited edges) take the wide row-tile test
-        wide = getattr(engine, "nnz_total", 0) > 0 and int(red[1]) * 4 < engine.nnz_total
+        wide = getattr(engine, "nnz_total", 0) > 0 and gmu * 4 < engine.nnz_total
         owned = engine.expand(d, wide=wide)
         gathered = exchange_frontier(owned, engine.stride, group)
-        f, mf, mu = engine.merge(gathered, engine.stride)
+        if hasattr(engine, "merge_dev"):
+            # statistics stay on the device: one all-reduce, one read per level
+            st = engine.merge_dev(gathered, engine.stride)
+            red = st[1:3].clone()
+            dist.all_reduce(red, group=group)
+            f, gmf, gmu = (int(x) for x in torch.cat([st[:1], red]).tolist())
+        else:
+            f, mf, mu = engine.merge(gathered, engine.stride)
+            red = torch.tensor([mf, mu], dtype=torch.int64, device=dev)
+            dist.all_reduce(red, group=group)
+            gmf, gmu = (int(x) for x in red.tolist())
         levels += 1
     return levels
 
@@ -120,6 +132,7 @@ class DistTiledMatrix:
         self.owned = torch.zeros(max(1, (self.m_local + 31) // 32), dtype=torch.int32, device=self.device)
         self.levels = torch.empty(max(1, self.m_local), dtype=torch.int32, device=self.device)
         self._stats = (torch.zeros(3, dtype=torch.int64))
+        self._stats_dev = torch.zeros(3, dtype=torch.int64, device=self.device)
         # global nnz (one all-reduce at construction): the late-pull hint of bfs_loop;
         # 0 (no hint) when there is no process group (simulated ranks)
         self.nnz_total = 0
@@ -163,6 +176,15 @@ class DistTiledMatrix:
                                                       torch.cuda.current_stream().cuda_stream),
                         "tsmv_bfs_dist_merge")
         return st[0], st[1], st[2]
+
+    def merge_dev(self, gathered, stride):
+        """merge() with the statistics left on the device (int64[3], no sync)."""
+        self.tsmv.check(self.tsmv.tsmv_bfs_dist_merge(self.M.ctx, gathered.data_ptr(), int(stride),
+                                                      ctypes.cast(self._stats_dev.data_ptr(),
+                                                                  ctypes.POINTER(ctypes.c_int64)),
+                                                      torch.cuda.current_stream().cuda_stream),
+                        "tsmv_bfs_dist_merge")
+        return self._stats_dev
 
     def bfs(self, source: int):
         nl = bfs_loop(self, source, self.group)

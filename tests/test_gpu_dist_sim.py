@@ -25,7 +25,7 @@ def _ranks(A, P, dtype="pattern", **opts):
     return splits, engines
 
 
-def _sim_bfs(engines, source):
+def _sim_bfs(engines, source, dev_stats=False):
     st = [e.begin(source) for e in engines]
     while st[0][0] > 0:
         assert len({s[0] for s in st}) == 1          # |F| identical on every rank
@@ -38,7 +38,10 @@ def _sim_bfs(engines, source):
         gathered = torch.zeros(len(engines) * stride, dtype=torch.int32, device=DEV)
         for p, o in enumerate(owned):
             gathered[p * stride:p * stride + o.numel()] = o
-        st = [e.merge(gathered, stride) for e in engines]
+        if dev_stats:   # merge with device statistics (tsmv_bfs_dist_merge, device out_stats)
+            st = [tuple(int(x) for x in e.merge_dev(gathered, stride).clone().cpu()) for e in engines]
+        else:
+            st = [e.merge(gathered, stride) for e in engines]
     return np.concatenate([e.levels[:e.m_local].cpu().numpy() for e in engines])
 
 
@@ -74,3 +77,14 @@ def test_sim_ranks_spmspv(P):
     ri, rv = oracle.spmspv(C, xi.numpy(), xv.numpy())
     assert np.array_equal(np.concatenate(ys_i), ri)      # global row ids, ascending across ranks
     assert np.array_equal(np.concatenate(ys_v), rv)
+
+
+@pytest.mark.parametrize("P", [2, 3])
+def test_sim_ranks_bfs_device_stats(P):
+    """The device-statistics merge gives the same levels (and |F| on every rank)."""
+    A = synth.rmat(12, 16, seed=11, symmetrize=True)
+    C = oracle.csc_of(A)
+    _, engines = _ranks(A, P)
+    for s in [0] + synth.sample_sources(A, 2, seed=5):
+        got = _sim_bfs(engines, s, dev_stats=True)
+        assert np.array_equal(got, oracle.bfs_queue(C, s))

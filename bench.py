@@ -336,7 +336,7 @@ def run_tsmv(args):
         else:
             lo, hi = D.splits[rank], D.splits[rank + 1]
             own = (xi >= lo) & (xi < hi)
-            D.spmspv(xi[own], xv[own])
+            D.spmspv_async(xi[own], xv[own], y_idx, y_val, y_nnz)
 
     for s in range(args.warmup):
         flush()

@@ -150,6 +150,17 @@ class DistTiledMatrix:
             return xi, xv
         return self.M.spmspv(xi, xv, semiring=semiring)
 
+    def spmspv_async(self, x_idx_owned: torch.Tensor, x_val_owned: Optional[torch.Tensor], y_idx: torch.Tensor,
+                     y_val: Optional[torch.Tensor], y_nnz: torch.Tensor, semiring="plus_times"):
+        """spmspv() without the final synchronisation: y for the owned rows and its
+        size (int64[1] on the device) are written on the current stream."""
+        xi = allgather_varlen(x_idx_owned.to(torch.int32), self.group)
+        xv = None if x_val_owned is None else allgather_varlen(x_val_owned, self.group)
+        if xi.numel() == 0:
+            y_nnz.zero_()
+            return
+        self.M.spmspv_async(xi, xv, y_idx, y_val, y_nnz, semiring=semiring)
+
     # ---- BFS engine interface
     def choose(self, n, f, mf, mu):
         return self.tsmv.choose_dir(n, f, mf, mu, self.M.opts)

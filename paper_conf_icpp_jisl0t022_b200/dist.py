@@ -55,13 +55,21 @@ def local_rows(A, splits: Sequence[int], rank: int):
     return synth.CSR(r1 - r0, A.n, rp - base, cols, vals, f"{A.name}[{r0}:{r1}]")
 
 
-def allgather_varlen(t: torch.Tensor, group=None) -> torch.Tensor:
-    """Concatenation, in rank order, of a 1-D tensor of per-rank length."""
+def allgather_sizes(count: int, device, group=None) -> List[int]:
+    """Per-rank element counts (one all-gather, one host read)."""
     world = dist.get_world_size(group)
-    n = torch.tensor([t.numel()], dtype=torch.int64, device=t.device)
-    sizes = [torch.zeros_like(n) for _ in range(world)]
-    dist.all_gather(sizes, n, group=group)
-    sizes = [int(s) for s in sizes]
+    n = torch.tensor([count], dtype=torch.int64, device=device)
+    out = torch.empty(world, dtype=torch.int64, device=device)
+    dist.all_gather_into_tensor(out, n, group=group)
+    return out.tolist()
+
+
+def allgather_varlen(t: torch.Tensor, group=None, sizes: Optional[List[int]] = None) -> torch.Tensor:
+    """Concatenation, in rank order, of a 1-D tensor of per-rank length (`sizes`,
+    if the caller already exchanged them)."""
+    world = dist.get_world_size(group)
+    if sizes is None:
+        sizes = allgather_sizes(t.numel(), t.device, group)
     mx = max(sizes) if sizes else 0
     pad = torch.zeros(max(mx, 1), dtype=t.dtype, device=t.device)
     pad[:t.numel()] = t
@@ -144,8 +152,9 @@ class DistTiledMatrix:
 
     # ---- SpMSpV: x entries are distributed by owner (x_idx in this rank's row range)
     def spmspv(self, x_idx_owned: torch.Tensor, x_val_owned: Optional[torch.Tensor], semiring="plus_times"):
-        xi = allgather_varlen(x_idx_owned.to(torch.int32), self.group)
-        xv = None if x_val_owned is None else allgather_varlen(x_val_owned, self.group)
+        sizes = allgather_sizes(x_idx_owned.numel(), x_idx_owned.device, self.group)
+        xi = allgather_varlen(x_idx_owned.to(torch.int32), self.group, sizes)
+        xv = None if x_val_owned is None else allgather_varlen(x_val_owned, self.group, sizes)
         if xi.numel() == 0:
             return xi, xv
         return self.M.spmspv(xi, xv, semiring=semiring)
@@ -154,8 +163,9 @@ class DistTiledMatrix:
                      y_val: Optional[torch.Tensor], y_nnz: torch.Tensor, semiring="plus_times"):
         """spmspv() without the final synchronisation: y for the owned rows and its
         size (int64[1] on the device) are written on the current stream."""
-        xi = allgather_varlen(x_idx_owned.to(torch.int32), self.group)
-        xv = None if x_val_owned is None else allgather_varlen(x_val_owned, self.group)
+        sizes = allgather_sizes(x_idx_owned.numel(), x_idx_owned.device, self.group)
+        xi = allgather_varlen(x_idx_owned.to(torch.int32), self.group, sizes)
+        xv = None if x_val_owned is None else allgather_varlen(x_val_owned, self.group, sizes)
         if xi.numel() == 0:
             y_nnz.zero_()
             return

@@ -222,7 +222,7 @@ struct FlatLists {
     DevBuf s_beg, s_wpre, s_x;        // per x entry with side work: first side nonzero, prefix, x_j
     DevBuf Ct, Cs;                    // chunk -> first list entry
     DevBuf hits;                      // uint4 {tile, hit columns, segment slot, 0} per hit tile
-    DevBuf pcnt;                      // long long[G * KP]: set bits per touched-bitmap piece
+    DevBuf pcnt;                      // u32[2][MAXG * KP]: touched rows per bitmap piece (2 buffers)
     size_t bytes() const {
         return t_beg.bytes + t_wpre.bytes + t_xm.bytes + t_J.bytes + t_xv.bytes + s_beg.bytes + s_wpre.bytes + s_x.bytes +
                Ct.bytes + Cs.bytes + hits.bytes;
@@ -313,6 +313,7 @@ struct tsmv_ctx {
     int fused_blocks = 0, fused_threads = 1024;
     bool use_flat = false;         // SpMSpV through the flat kernel (nt = 16), decided at create
     int flat_blocks = 0;           // CTAs of the flat SpMSpV kernel (1024 threads, 1 per SM)
+    long long flat_calls = 0;      // flat SpMSpV launches so far (piece-count buffer parity)
     int last_blocks = 0;           // CTAs of the last SpMSpV launch (partials / acct rows)
     tsmv::DevBuf partials;         // long long[fused_blocks][8]
     long long last_x_nnz = 0;

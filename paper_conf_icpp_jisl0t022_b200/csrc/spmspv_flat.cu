@@ -20,7 +20,9 @@
 //     list window (start, x_j) is staged in shared memory;
 //   * chunks are dealt round-robin to warps (no work-queue atomics on one address);
 //   * compaction with one thread per bitmap word (loads of its set rows batched).
-// Phases: A | barrier | B1 (a3, a5) -> B2 (a4, own hits, CTA barrier only) | barrier | C1 count | barrier | C2 write y.
+// Phases: A | barrier | B1 (a3, a5) -> B2 (a4, own hits, CTA barrier only) | barrier | C write y.
+// The touched rows of every bitmap piece are counted at their first touch in B,
+// so C needs no counting pass and no barrier of its own (round 2).
 #include "device.cuh"
 #include <algorithm>
 #include <cstdlib>
@@ -76,6 +78,10 @@ struct FlatArgs {
     void *y_val;
     long long y_cap;
     long long *ynnz_dev;
+    unsigned *pc;       // touched rows per bitmap piece, this call (zero on entry)
+    unsigned *pc_next;  // the other buffer: zeroed here for the next call
+    int ps_log;         // a piece is 2^ps_log bitmap words
+    int n_pieces;
     Counters *cnt;
     Counters *hm;
     unsigned long long bar_base;
@@ -91,25 +97,32 @@ struct FlatArgs {
 // times, fp64), and LLONG_MIN is the identity of a signed max, to which the
 // min-second keys are mapped (k' = ~ord_key(x) ^ 2^63 keeps the order).  The old
 // value returned by the atomic tells whether this contribution is the first to
-// its row, and only that one sets the row's touched bit (one RED.OR per output
-// row instead of one per contribution).  A row whose contributions are all -0.0
-// returns "first" more than once, which only repeats an idempotent OR.
+// its row; only that one sets the row's touched bit and counts the row in its
+// bitmap piece (one RED.OR + one RED.ADD per output row instead of one per
+// contribution).  The detection is exact: a zero product is added as +0.0, so
+// after its first contribution a row never holds -0.0 again (x + (-x) = +0.0
+// under round-to-nearest); Boolean rows are claimed with an exchange; a min key
+// never equals EMPTY (it would need an all-ones order key, i.e. a NaN x).
 constexpr unsigned long long EMPTY = 0x8000000000000000ull;
 
+__device__ __forceinline__ double prod_nz(double a, double x) {
+    const double v = a * x;
+    return v == 0.0 ? 0.0 : v;  // -0.0 -> +0.0
+}
 template <int SR>
 __device__ __forceinline__ bool acc_first(double *acc, long long row, double a, double x) {
     if constexpr (SR == TSMV_PLUS_TIMES) {
-        return (unsigned long long)__double_as_longlong(atomicAdd(&acc[row], a * x)) == EMPTY;
+        return (unsigned long long)__double_as_longlong(atomicAdd(&acc[row], prod_nz(a, x))) == EMPTY;
     } else if constexpr (SR == TSMV_MIN_SECOND) {
         const long long k = (long long)(~ord_key(x) ^ EMPTY);
         return (unsigned long long)atomicMax((long long *)&acc[row], k) == EMPTY;
     } else {
-        return true;
+        return atomicExch((unsigned long long *)&acc[row], 0ull) == EMPTY;
     }
 }
 template <int SR>
 __device__ __forceinline__ void acc_shared(double *s, int slot, double a, double x) {
-    if constexpr (SR == TSMV_PLUS_TIMES) atomicAdd(&s[slot], a * x);
+    if constexpr (SR == TSMV_PLUS_TIMES) atomicAdd(&s[slot], prod_nz(a, x));
     else if constexpr (SR == TSMV_MIN_SECOND) atomicMax((long long *)&s[slot], (long long)(~ord_key(x) ^ EMPTY));
 }
 
@@ -126,31 +139,15 @@ __device__ __forceinline__ long long contribute(const FlatArgs &a, double *s_hac
     }
     return acc_first<SR>(a.acc, rc, av, xv) ? rc : -1;
 }
-__device__ __forceinline__ void touch(uint32_t *rowbits, long long row) {
-    if (row >= 0) atomicOr(&rowbits[row >> 5], 1u << (row & 31));
+// first touch of `row` (>= 0; -1 = none): its bit, and its piece's count in the
+// CTA's shared-memory counters (added to the global ones once, at the end of B)
+__device__ __forceinline__ void touch(const FlatArgs &a, unsigned *s_pc, long long row) {
+    if (row >= 0) {
+        atomicOr(&a.rowbits[row >> 5], 1u << (row & 31));
+        atomicAdd(&s_pc[(row >> 5) >> a.ps_log], 1u);
+    }
 }
 
-#ifdef TSMV_FLAT_STEPS
-// development: stamp step k of warp 0 of CTA 0 once the value `dep` (produced by
-// the step's loads) is available
-#define FSTEP(k, dep)                                                                              \
-    do {                                                                                           \
-        if (a.trace && b == 0 && wid == 0 && lane == 0) {                                          \
-            if ((long long)(dep) == 0x5eed5eed5eedll) a.trace[2000] = 1;                          \
-            a.trace[148 * 12 + (k)] = globaltimer_ns();                                            \
-        }                                                                                          \
-    } while (0)
-#define CSTEP(k, dep)                                                                              \
-    do {                                                                                           \
-        if (a.trace && b == 1 && wid == 0 && lane == 0 && (k) < 16) {                              \
-            if ((long long)(dep) == 0x5eed5eed5eedll) a.trace[2000] = 1;                          \
-            a.trace[148 * 12 + 16 + (k)] = globaltimer_ns();                                       \
-        }                                                                                          \
-    } while (0)
-#else
-#define FSTEP(k, dep) ((void)0)
-#define CSTEP(k, dep) ((void)0)
-#endif
 
 constexpr int HEAVY_CAP = 128;
 constexpr int MAXG = 256;  // max CTAs of the flat kernel (one per SM)
@@ -302,12 +299,12 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
     long long *s_winb = s_win + NWF * WN;                                         // [NWF][WN]
     double *s_winx = reinterpret_cast<double *>(s_winb + NWF * WN);               // [NWF][WN]
     uint32_t *s_hbits = reinterpret_cast<uint32_t *>(s_winx + NWF * WN);          // [HOT_SLOTS/32]
+    unsigned *s_pcnt = s_hbits + HOT_SLOTS / 32;                                  // [MAXG * KP]
     __shared__ long long s_base[4], s_tot[4];
     __shared__ long long s_acct[NWF][4];
     __shared__ int s_err;
     __shared__ int s_nheavy;
     __shared__ int s_hcnt;
-    __shared__ unsigned long long s_pc[KP];
     __shared__ long long s_pbase[KP], s_ex0[KP];
     __shared__ int s_nd;  // dense bitmap words of the current C2 round
     __shared__ long long s_heavy[HEAVY_CAP][3];  // chunk-map runs too long for one thread: c0, c1, list | kind
@@ -322,10 +319,12 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
     const int n_slots = a.n_hot * NT;
     for (int i = tid; i < n_slots; i += FT) s_hacc[i] = __longlong_as_double((long long)EMPTY);
     for (int i = tid; i < (n_slots + 31) / 32; i += FT) s_hbits[i] = 0u;
+    for (int i = tid; i < a.n_pieces; i += FT) s_pcnt[i] = 0u;
     if (tid == 0) {
         s_nheavy = 0;
         s_hcnt = 0;
     }
+    if (tid < KP && b + tid * G < a.n_pieces) a.pc_next[b + tid * G] = 0u;
 
     // ------------------------------------------------------------ phase A (a2)
     // CTA b owns x entries [e0, e1); thread tid a contiguous run of them.
@@ -461,9 +460,7 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
             for (int u = 0; u < UT; ++u) hv[u] = 0u;
             if (task < nTT) {
                 const long long base = task << TL;
-                FSTEP(0, 0);
                 const long long s0 = __ldcg(&a.L.Ct[task]);
-                FSTEP(1, s0);
 #pragma unroll
                 for (int q0 = 0; q0 <= (1 << TL); q0 += 32) {
                     const int qx = q0 + lane;
@@ -479,7 +476,6 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
                     }
                 }
                 __syncwarp();
-                FSTEP(2, win[0]);
                 ChunkMap<TL> cm;
                 cm.build(win, base, lane);
                 unsigned xm[UT];
@@ -495,7 +491,6 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
                 }
 #pragma unroll
                 for (int u = 0; u < UT; ++u) hv[u] = xm[u] ? ((unsigned)__ldg(&a.mask[tv[u]]) & xm[u]) : 0u;
-                FSTEP(3, hv[0] + hv[UT - 1]);
                 __syncwarp();
             } else if (task < ntask) {
                 const long long c2 = task - nTT;
@@ -543,7 +538,7 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
                 for (int u = 0; u < US; ++u)
                     fr[u] = ok[u] ? contribute<SR>(a, s_hacc, s_hbits, (long long)row[u], av[u], xv[u]) : -1;
 #pragma unroll
-                for (int u = 0; u < US; ++u) touch(a.rowbits, fr[u]);
+                for (int u = 0; u < US; ++u) touch(a, s_pcnt, fr[u]);
                 __syncwarp();
             }
             // append this round's hits: warp offsets in shared memory, one global
@@ -596,7 +591,6 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
                 // x value of the first hit column, fetched beside the tile record
                 xv0 = __ldcg(&a.L.t_xv[(long long)slot * NT + (__ffs(hit) - 1)]);
             }
-            FSTEP(4, hit);
             unsigned off = 0, nnz = 0;
             int trow = 0;
             uint4 bb = make_uint4(0, 0, 0, 0);
@@ -644,7 +638,7 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
                             }
                         }
 #pragma unroll
-                        for (int j = 0; j < 4; ++j) touch(a.rowbits, fr[j]);
+                        for (int j = 0; j < 4; ++j) touch(a, s_pcnt, fr[j]);
                     }
                 } else {
                     useful = rec_useful(bb, hit, (int)nnz);
@@ -657,7 +651,6 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
                 if (lane >= o) incl += v;
             }
             const int total = __shfl_sync(0xffffffffu, incl, 31);
-            FSTEP(5, total);
             n_mac += useful;
             n_ind += useful;
             long long frp = -1, frq = -1;
@@ -690,14 +683,13 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
                     const double av = val ? (double)__ldg(&val[pos]) : 1.0;
                     const double xv = __ldcg(&a.L.t_xv[(long long)ss * NT + c]);
                     const long long rc = trs >= 0 ? (long long)trs * NT + rr : ~((long long)(~trs) * NT + rr);
-                    FSTEP(6, av + xv + rc);
                     frp = contribute<SR>(a, s_hacc, s_hbits, rc, av, xv);
                 }
-                touch(a.rowbits, frq);  // previous round's result: its atomic had a round to return
+                touch(a, s_pcnt, frq);  // previous round's result: its atomic had a round to return
                 frq = frp;
                 frp = -1;
             }
-            touch(a.rowbits, frq);
+            touch(a, s_pcnt, frq);
         }
     }
 #pragma unroll
@@ -738,57 +730,54 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
                 else if constexpr (SR == TSMV_MIN_SECOND)
                     first = (unsigned long long)atomicMax((long long *)&a.acc[row],
                                                           (long long)__double_as_longlong(s_hacc[sl])) == EMPTY;
+                else
+                    first = atomicExch((unsigned long long *)&a.acc[row], 0ull) == EMPTY;
                 if (first) fr[i] = row;
             }
         }
 #pragma unroll
-        for (int i = 0; i < FQ; ++i) touch(a.rowbits, fr[i]);
+        for (int i = 0; i < FQ; ++i) touch(a, s_pcnt, fr[i]);
     }
     if (tid < 4) {
         long long sum = 0;
         for (int w = 0; w < NWF; ++w) sum += s_acct[w][tid];
         a.acct[b * 4 + tid] = sum;
     }
+    __syncthreads();
+    for (int q = tid; q < a.n_pieces; q += FT)
+        if (s_pcnt[q]) atomicAdd(&a.pc[q], s_pcnt[q]);
     grid_sync_f(&a.cnt->bar, target, tr ? tr + 5 : nullptr);
     if (stamp) ts[3] = globaltimer_ns();
 
     // ------------------------------------------------------------ phase C (a6)
-    // The touched bitmap is cut into G*KP pieces of PS words; CTA b owns pieces
-    // b, b + G, ..., so a dense stretch of y (power-law rows) is spread over KP
-    // CTAs.  C1 counts each piece, C2 emits y at the piece's global offset.  A
-    // round covers PSR words of each of the CTA's pieces (thread tid: piece
-    // tid / PSR), so one block scan per round serves all pieces.
+    // The touched bitmap is cut into pieces of PS = 2^ps_log words (at most G*KP of
+    // them); CTA b owns pieces b, b + G, ..., so a dense stretch of y (power-law
+    // rows) is spread over KP CTAs.  The rows of every piece were counted at their
+    // first touch (touch()), so each CTA scans the piece counts and emits its
+    // pieces at their global offsets.  A round covers PSR words of each of the
+    // CTA's pieces (thread tid: piece tid / PSR), so one block scan per round
+    // serves all pieces.
     constexpr int PSR = FT / KP;
-    const long long PS = ((a.W + (long long)G * KP - 1) / ((long long)G * KP) + 31) & ~31ll;
+    const long long PS = 1ll << a.ps_log;
     const int kp = tid / PSR, tp = tid % PSR;
     const long long pw0 = ((long long)b + (long long)kp * G) * PS;
     const long long pw1 = min(a.W, pw0 + PS);
-    if (tid < KP) s_pc[tid] = 0;
-    __syncthreads();
-    {
-        long long mycnt = 0;
-        for (long long w = pw0 + tp; w < pw1; w += PSR) mycnt += __popc(__ldcg(&a.rowbits[w]));
-#pragma unroll
-        for (int o = 16; o > 0; o >>= 1) mycnt += __shfl_xor_sync(0xffffffffu, mycnt, o);
-        if (lane == 0 && mycnt) atomicAdd(&s_pc[kp], (unsigned long long)mycnt);
-    }
-    __syncthreads();
-    if (tid < KP) a.L.pcnt[b + tid * G] = (long long)s_pc[tid];
-    grid_sync_f(&a.cnt->bar, target, tr ? tr + 7 : nullptr);
     if (stamp) ts[4] = globaltimer_ns();
     {
-        // exclusive prefix of all G*KP piece counts (every CTA, in shared memory)
-        const int NP = G * KP;
+        // exclusive prefix of all piece counts (every CTA, in shared memory)
+        const int NP = a.n_pieces;
         constexpr int PPT = (MAXG * KP + FT - 1) / FT;
         long long v[PPT], run = 0;
 #pragma unroll
         for (int i = 0; i < PPT; ++i) {
             const int q = tid * PPT + i;
-            v[i] = q < NP ? __ldcg(&a.L.pcnt[q]) : 0;
+            v[i] = q < NP ? (long long)__ldcg(&a.pc[q]) : 0;
             run += v[i];
         }
         long long ex, tt;
         block_scan<1, FT>(&run, &ex, &tt, s_scan);
+        if (tid < KP) s_pbase[tid] = 0;
+        __syncthreads();
 #pragma unroll
         for (int i = 0; i < PPT; ++i) {
             const int q = tid * PPT + i;
@@ -806,9 +795,7 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
     if (tid == 0) s_nd = 0;
     for (int rd = 0; rd < nround; ++rd) {
         const long long w = pw0 + (long long)rd * PSR + tp;
-        CSTEP(0, 0);
         const unsigned bits = w < pw1 ? __ldcg(&a.rowbits[w]) : 0u;
-        CSTEP(1, bits);
         long long c = __popc(bits), exw, rtot;
         block_scan<1, FT>(&c, &exw, &rtot, s_scan);
         if (tp == 0) s_ex0[kp] = exw;
@@ -818,7 +805,6 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
         const long long pos0 = s_pbase[kp] + exw - seg0;
         __syncthreads();
         if (tp == 0) s_pbase[kp] += segsum;
-        CSTEP(2, exw);
         int it = 0;
         if (bits) a.rowbits[w] = 0u;
         // sparse words (<= SPW set rows) are emitted by their own thread, all in one
@@ -924,7 +910,7 @@ template <class AV, class XV> void *pick_sr_flat(int sr) {
 }
 void *pick_flat(bool f32, int sr) { return f32 ? pick_sr_flat<float, float>(sr) : pick_sr_flat<double, double>(sr); }
 
-constexpr size_t FLAT_DYN = HOT_SLOTS * 8 + (size_t)NWF * ((1 << WL) + 1) * 24 + HOT_SLOTS / 8;
+constexpr size_t FLAT_DYN = HOT_SLOTS * 8 + (size_t)NWF * ((1 << WL) + 1) * 24 + HOT_SLOTS / 8 + MAXG * KP * 4;
 
 void flat_set_smem() {
     static bool done = false;
@@ -1052,7 +1038,8 @@ void ensure_flat_lists(tsmv_ctx *c, int64_t k) {
         F.Ct.alloc(((c->P.T >> TL) + 2) * 4);
         F.Cs.alloc(((c->P.side_nnz >> SL) + 2) * 4);
         F.hits.alloc((size_t)(c->P.T + 128ll * (c->flat_blocks + 2)) * 16);
-        F.pcnt.alloc((size_t)MAXG * KP * 8);
+        F.pcnt.alloc((size_t)2 * MAXG * KP * 4);  // u32[2][MAXG * KP]: piece counts, double-buffered
+        TSMV_CUDA(cudaMemset(F.pcnt.p, 0, F.pcnt.bytes));
     }
 }
 
@@ -1106,6 +1093,19 @@ void enqueue_spmspv_flat(tsmv_ctx *c, int sr, long long k, const int32_t *xi, co
     a.y_val = (sr == TSMV_OR_AND) ? nullptr : yv;
     a.y_cap = ycap;
     a.ynnz_dev = ynnz_dev;
+    {
+        // pieces of 2^ps_log bitmap words, at most G * KP of them (phase C)
+        const long long per = (a.W + (long long)c->flat_blocks * KP - 1) / ((long long)c->flat_blocks * KP);
+        int lg = 5;
+        while ((1ll << lg) < per) ++lg;
+        a.ps_log = lg;
+        a.n_pieces = (int)((a.W + (1ll << lg) - 1) >> lg);
+        unsigned *pc = c->FL.pcnt.as<unsigned>();
+        const int cur = (int)(c->flat_calls & 1);
+        a.pc = pc + (size_t)cur * MAXG * KP;
+        a.pc_next = pc + (size_t)(1 - cur) * MAXG * KP;
+        c->flat_calls++;
+    }
     a.cnt = c->counters.as<Counters>();
     a.hm = c->hcnt_dev;
     a.bar_base = c->bar_base;
@@ -1137,7 +1137,7 @@ void enqueue_spmspv_flat(tsmv_ctx *c, int sr, long long k, const int32_t *xi, co
     }
     cfg.attrs = at;
     TSMV_CUDA(cudaLaunchKernelExC(&cfg, pick_flat(f32, sr), args));
-    c->bar_base += 3ull * (unsigned long long)G;
+    c->bar_base += 2ull * (unsigned long long)G;
     c->last_blocks = G;
     if (c->timing) c->tcalls++;
 }

@@ -105,6 +105,10 @@ typedef struct {
     double build_ms;            /* device time of tsmv_create's builder */
 } tsmv_info;
 
+/* Size of the per-level arrays of tsmv_bfs_stats.  It is NOT a traversal limit:
+ * a traversal with more levels runs to completion (every level written to
+ * `levels`); only the first TSMV_MAX_LEVELS entries of the per-level arrays are
+ * filled. */
 #define TSMV_MAX_LEVELS 65536
 typedef struct {
     int32_t nlevels;                 /* number of non-empty levels (source level counts) */
@@ -113,6 +117,11 @@ typedef struct {
     double ms;                       /* device time source-init -> last level */
     int32_t dir_per_level[TSMV_MAX_LEVELS];       /* tsmv_dir used to expand level L */
     int64_t frontier_per_level[TSMV_MAX_LEVELS];  /* |F| of level L */
+    float level_ms[TSMV_MAX_LEVELS];              /* device time of level L: from the decision
+                                                     to expand L (%globaltimer) to the decision
+                                                     for L + 1 (the last level: to the end);
+                                                     the paper's per-level analysis, Fig 10
+                                                      */
 } tsmv_bfs_stats;
 
 /* Fill *opt with the defaults documented above.  Never fails for non-NULL opt. */

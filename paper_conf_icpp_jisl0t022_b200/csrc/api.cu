@@ -106,7 +106,7 @@ static void destroy_impl(tsmv_ctx *c) {
     c->Qown.release();
     for (DevBuf *b : {&c->outdeg, &c->indeg, &c->acc, &c->rowbits, &c->desc_compact, &c->counters, &c->stage_x_idx,
                       &c->stage_x_val, &c->stage_y_idx, &c->stage_y_val, &c->stage_levels, &c->V, &c->F0, &c->F1,
-                      &c->desc_bfs, &c->splits_dev, &c->xdense, &c->acct, &c->tring, &c->partials, &c->hot_list, &c->bfs_dirs, &c->bfs_front, &c->lwork, &c->bq0,
+                      &c->desc_bfs, &c->splits_dev, &c->xdense, &c->acct, &c->tring, &c->partials, &c->hot_list, &c->bfs_dirs, &c->bfs_front, &c->bfs_tlv, &c->lwork, &c->bq0,
                       &c->bq1, &c->lslots})
         b->release();
     c->L.release();
@@ -285,6 +285,7 @@ extern "C" tsmv_status tsmv_create(tsmv_ctx **out, int64_t nrows, int64_t ncols,
             c->bfs_blocks = c->sm_count * std::min(bo, 2);
             c->bfs_dirs.alloc(TSMV_MAX_LEVELS * 4);
             c->bfs_front.alloc(TSMV_MAX_LEVELS * 8);
+            c->bfs_tlv.alloc((TSMV_MAX_LEVELS + 1) * 8);
             bfs_list_init(c, st);
         }
         c->partials.alloc((size_t)std::max({c->fused_blocks, c->bfs_blocks, c->flat_blocks}) * 8 * 8);

@@ -36,6 +36,10 @@ struct OctSum {
     }
 };
 
+// per-level device time (tsmv_bfs_stats::level_ms): %globaltimer of a level the
+// host runs itself, and of the end of the traversal
+__global__ void k_stamp(unsigned long long *t) { *t = globaltimer_ns(); }
+
 __global__ void k_bfs_init(BfsView B, long long NW, long long source) {
     long long tid = blockIdx.x * (long long)blockDim.x + threadIdx.x;
     long long stride = (long long)gridDim.x * blockDim.x;
@@ -802,6 +806,15 @@ static void bfs_prepare_levels(tsmv_ctx *c, int32_t *levels, bool &host_levels) 
     }
 }
 
+// level_ms[L] = time from level L's expansion decision to level L+1's (the last
+// level: to the end of the traversal), from the stamps in c->bfs_tlv
+static void level_times(tsmv_ctx *c, tsmv_bfs_stats *stats, long long nl, bool has_end) {
+    std::vector<unsigned long long> t(nl + 1, 0);
+    TSMV_CUDA(cudaMemcpy(t.data(), c->bfs_tlv.p, (nl + (has_end ? 1 : 0)) * 8, cudaMemcpyDeviceToHost));
+    for (long long L = 0; L < nl; ++L)
+        stats->level_ms[L] = (L + 1 < nl || has_end) && t[L + 1] >= t[L] ? (float)((t[L + 1] - t[L]) * 1e-6) : 0.f;
+}
+
 extern "C" tsmv_status tsmv_bfs(tsmv_ctx *c, int64_t source, int32_t *levels, tsmv_bfs_stats *stats,
                                 void *cuda_stream) {
     try {
@@ -824,16 +837,13 @@ extern "C" tsmv_status tsmv_bfs(tsmv_ctx *c, int64_t source, int32_t *levels, ts
             long long level = 0, mu = c->nnz, reached = 0, edges = 0;
             bool resume = false;
             BfsRunner R{c, st, (long long)(c->V.bytes / 4)};
-            std::vector<int> hdir;
-            std::vector<long long> hfront;
+            const long long maxlv = getenv("TSMV_BFS_MAXLV") ? atoll(getenv("TSMV_BFS_MAXLV")) : (1ll << 40);
+            unsigned long long *tlv = c->bfs_tlv.as<unsigned long long>();
             while (true) {
                 long long L, mu2, r2, e2;
                 int cur;
                 const bool stopped = bfs_fused_launch(c, source, st, resume, level, Fa, Fb, mu, reached, edges,
-                                                      stop_on_pull,
-                                                      getenv("TSMV_BFS_MAXLV") ? atoi(getenv("TSMV_BFS_MAXLV"))
-                                                                               : TSMV_MAX_LEVELS,
-                                                      L, mu2, r2, e2, cur);
+                                                      stop_on_pull, maxlv, L, mu2, r2, e2, cur);
                 if (getenv("TSMV_BFS_PHASES")) {
                     long long fl = 0;
                     if (c->lslots.p) {
@@ -861,7 +871,7 @@ extern "C" tsmv_status tsmv_bfs(tsmv_ctx *c, int64_t source, int32_t *levels, ts
                     const long long fsize = h->fsize, mf = h->mf, din = h->din;
                     std::swap(Fa, Fb);
                     ++level;
-                    if (fsize == 0 || level >= TSMV_MAX_LEVELS) break;
+                    if (fsize == 0 || level >= maxlv) break;
                     const int dir = choose_dir(c->opt, c->n, fsize, mf, mu - din);
                     // resume the fused kernel at `level` for push levels and for the late
                     // (wide) pull levels, which it runs in place without host round trips
@@ -869,18 +879,18 @@ extern "C" tsmv_status tsmv_bfs(tsmv_ctx *c, int64_t source, int32_t *levels, ts
                     mu -= din;
                     reached += fsize;
                     edges += mf;
-                    hdir.resize(level + 1, 0);
-                    hfront.resize(level + 1, 0);
-                    hdir[level] = dir;
-                    hfront[level] = fsize;
-                    int dd = dir;
-                    long long ff = fsize;
-                    TSMV_CUDA(cudaMemcpy(c->bfs_dirs.as<int>() + level, &dd, 4, cudaMemcpyHostToDevice));
-                    TSMV_CUDA(cudaMemcpy(c->bfs_front.as<long long>() + level, &ff, 8, cudaMemcpyHostToDevice));
+                    if (level < TSMV_MAX_LEVELS) {
+                        int dd = dir;
+                        long long ff = fsize;
+                        TSMV_CUDA(cudaMemcpy(c->bfs_dirs.as<int>() + level, &dd, 4, cudaMemcpyHostToDevice));
+                        TSMV_CUDA(cudaMemcpy(c->bfs_front.as<long long>() + level, &ff, 8, cudaMemcpyHostToDevice));
+                        k_stamp<<<1, 1, 0, st>>>(tlv + level);
+                    }
                 }
-                if (c->hcnt->fsize == 0 || level >= TSMV_MAX_LEVELS) break;
+                if (c->hcnt->fsize == 0 || level >= maxlv) break;
                 resume = true;
             }
+            if (level <= TSMV_MAX_LEVELS) k_stamp<<<1, 1, 0, st>>>(tlv + level);
             TSMV_CUDA(cudaEventRecord(c->ev1, st));
             if (host_levels) TSMV_CUDA(cudaMemcpyAsync(levels, c->levels_dev, c->m * 4, cudaMemcpyDeviceToHost, st));
             TSMV_CUDA(cudaStreamSynchronize(st));
@@ -892,8 +902,9 @@ extern "C" tsmv_status tsmv_bfs(tsmv_ctx *c, int64_t source, int32_t *levels, ts
                 if (nl > 0) {
                     TSMV_CUDA(cudaMemcpy(stats->dir_per_level, c->bfs_dirs.p, nl * 4, cudaMemcpyDeviceToHost));
                     TSMV_CUDA(cudaMemcpy(stats->frontier_per_level, c->bfs_front.p, nl * 8, cudaMemcpyDeviceToHost));
+                    level_times(c, stats, nl, level <= TSMV_MAX_LEVELS);
                 }
-                stats->nlevels = (int32_t)nl;
+                stats->nlevels = (int32_t)std::min<long long>(level, INT32_MAX);
                 stats->reached = reached;
                 stats->edges_traversed = edges;
                 stats->ms = ms;
@@ -913,12 +924,14 @@ extern "C" tsmv_status tsmv_bfs(tsmv_ctx *c, int64_t source, int32_t *levels, ts
         long long reached = 0, edges = 0;
         int L = 0;
         if (stats) stats->nlevels = 0;
+        unsigned long long *tlv = c->bfs_tlv.as<unsigned long long>();
         while (fsize > 0) {
             int dir = choose_dir(c->opt, c->n, fsize, mf, mu);
             if (stats && L < TSMV_MAX_LEVELS) {
                 stats->dir_per_level[L] = dir;
                 stats->frontier_per_level[L] = fsize;
             }
+            if (L < TSMV_MAX_LEVELS) k_stamp<<<1, 1, 0, st>>>(tlv + L);
             reached += fsize;
             edges += mf;
             c->bfs_level = L;
@@ -933,6 +946,7 @@ extern "C" tsmv_status tsmv_bfs(tsmv_ctx *c, int64_t source, int32_t *levels, ts
             c->fcur ^= 1;
             ++L;
         }
+        if (L <= TSMV_MAX_LEVELS) k_stamp<<<1, 1, 0, st>>>(tlv + L);
         TSMV_CUDA(cudaEventRecord(c->ev1, st));
         // leave F clean for the next traversal
         TSMV_CUDA(cudaMemsetAsync(c->F0.p, 0, c->F0.bytes, st));
@@ -943,6 +957,7 @@ extern "C" tsmv_status tsmv_bfs(tsmv_ctx *c, int64_t source, int32_t *levels, ts
             float ms = 0;
             TSMV_CUDA(cudaEventElapsedTime(&ms, c->ev0, c->ev1));
             stats->nlevels = L;
+            if (L > 0) level_times(c, stats, std::min<long long>(L, TSMV_MAX_LEVELS), L <= TSMV_MAX_LEVELS);
             stats->reached = reached;
             stats->edges_traversed = edges;
             stats->ms = ms;

@@ -52,8 +52,9 @@ struct BfsFusedArgs {
     long long *partials;  // [G][8]
     Counters *cnt;
     Counters *hm;         // mapped: fsize (levels), reached, edges
-    int *dir_out;         // [max_levels]
-    long long *front_out; // [max_levels]
+    int *dir_out;         // [TSMV_MAX_LEVELS] direction of level L (stats; written for L < TSMV_MAX_LEVELS)
+    long long *front_out; // [TSMV_MAX_LEVELS] |F| of level L
+    unsigned long long *tlv_out;  // [TSMV_MAX_LEVELS + 1] %globaltimer when level L's expansion is decided
     long long source, nnz, nseg, NW, nTR_local, max_levels;
     double alpha, dens;
     int force;
@@ -406,9 +407,10 @@ __device__ void solo_levels(const BfsFusedArgs &a, BfsView &B, int &level, long 
         mu -= din2;
         reached += n2;
         edges += mf2;
-        if (tid == 0) {
+        if (tid == 0 && level < TSMV_MAX_LEVELS) {
             a.dir_out[level] = dir2;
             a.front_out[level] = n2;
+            a.tlv_out[level] = globaltimer_ns();
         }
         cur ^= 1;
         n = n2;
@@ -492,9 +494,10 @@ __global__ void __launch_bounds__(BFB, TSMV_BFS_MINB) k_bfs_fused(BfsFusedArgs a
             reached += fsize;
             edges += mf;
             const int dir = choose_dir_dev(a.force, a.alpha, a.dens, B.n, fsize, mf, mu);
-            if (b == 0 && tid == 0) {
+            if (b == 0 && tid == 0 && level < TSMV_MAX_LEVELS) {
                 a.dir_out[level] = dir;
                 a.front_out[level] = fsize;
+                a.tlv_out[level] = globaltimer_ns();
             }
             const int *Qc = (level & 1) ? a.bq1 : a.bq0;
             if (dir != TSMV_DIR_PUSH_CSC || maxw > LIST_MAXW) {
@@ -645,9 +648,10 @@ __global__ void __launch_bounds__(BFB, TSMV_BFS_MINB) k_bfs_fused(BfsFusedArgs a
         }
         redo = false;
         const int dir = choose_dir_dev(a.force, a.alpha, a.dens, B.n, fsize, mf, mu);
-        if (b == 0 && tid == 0) {
+        if (b == 0 && tid == 0 && level < TSMV_MAX_LEVELS) {
             a.dir_out[level] = dir;
             a.front_out[level] = fsize;
+            a.tlv_out[level] = globaltimer_ns();
         }
         // Dense pull levels go back to the host's high-occupancy kernels; pull
         // levels with few unvisited edges (m_u <= 16 per thread of this grid, or
@@ -839,6 +843,7 @@ bool bfs_fused_launch(tsmv_ctx *c, long long source, cudaStream_t st, bool resum
     a.hm = c->hcnt_dev;
     a.dir_out = c->bfs_dirs.as<int>();
     a.front_out = c->bfs_front.as<long long>();
+    a.tlv_out = c->bfs_tlv.as<unsigned long long>();
     a.source = source;
     a.nnz = c->nnz;
     a.nseg = c->nTC;

@@ -320,6 +320,7 @@ struct tsmv_ctx {
     int bfs_blocks = 0;            // CTAs of the fused BFS kernel
     long long bfs_last_levels = 0;
     tsmv::DevBuf bfs_dirs, bfs_front;  // per-level direction / frontier size (device)
+    tsmv::DevBuf bfs_tlv;              // u64[TSMV_MAX_LEVELS + 1]: %globaltimer at each level's decision
     // list-driven push levels of the fused BFS kernel
     tsmv::DevBuf lwork;        // int32[n]: push work of vertex u = tiles of its tile column + its side nonzeros
     tsmv::DevBuf bq0, bq1;     // int32[n]: frontier vertex lists, ping-pong by level parity

@@ -67,7 +67,7 @@ class tsmv_msbfs_stats(ctypes.Structure):
 class tsmv_bfs_stats(ctypes.Structure):
     _fields_ = [("nlevels", ctypes.c_int32), ("reached", ctypes.c_int64), ("edges_traversed", ctypes.c_int64),
                 ("ms", ctypes.c_double), ("dir_per_level", ctypes.c_int32 * MAX_LEVELS),
-                ("frontier_per_level", ctypes.c_int64 * MAX_LEVELS)]
+                ("frontier_per_level", ctypes.c_int64 * MAX_LEVELS), ("level_ms", ctypes.c_float * MAX_LEVELS)]
 
 
 _vp, _i64, _i32 = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int32
@@ -243,7 +243,8 @@ class TiledMatrix:
         L = stats.nlevels
         d = {"nlevels": L, "reached": stats.reached, "edges_traversed": stats.edges_traversed, "ms": stats.ms,
              "dirs": [DIR_NAMES.get(stats.dir_per_level[i], "?") for i in range(min(L, MAX_LEVELS))],
-             "frontier": [stats.frontier_per_level[i] for i in range(min(L, MAX_LEVELS))]}
+             "frontier": [stats.frontier_per_level[i] for i in range(min(L, MAX_LEVELS))],
+             "level_ms": [stats.level_ms[i] for i in range(min(L, MAX_LEVELS))]}
         return levels, d
 
     def bfs_parents(self, levels: torch.Tensor, parents: Optional[torch.Tensor] = None, stream=None):

@@ -165,3 +165,37 @@ def test_permuted_rmat(tsmv):
     for i, s in enumerate(src):
         assert np.array_equal(mlv[:, i].cpu().numpy(), oracle.bfs_queue(C, s))
     M.close()
+
+
+@pytest.mark.parametrize("env", [None, "TSMV_BFS_HOSTLOOP"])
+def test_path_longer_than_stats_arrays(tsmv, env):
+    """A traversal with more levels than TSMV_MAX_LEVELS (the size of the stats
+    arrays) runs to completion: path graph (band b = 1) of 70,000 vertices,
+    level(v) = v (the fused loop used to stop at 65,536 levels)."""
+    n = 70_000
+    A = synth.banded(n, 1)
+    if env:
+        os.environ[env] = "1"
+    try:
+        M = tsmv.TiledMatrix.from_csr(A.to(DEV), dtype="pattern")
+        lv, st = M.bfs(0)
+    finally:
+        if env:
+            os.environ.pop(env)
+    assert np.array_equal(lv.cpu().numpy(), np.arange(n, dtype=np.int32))
+    assert st["nlevels"] == n and st["reached"] == n
+    assert len(st["dirs"]) == tsmv.MAX_LEVELS
+    M.close()
+
+
+def test_level_times(tsmv):
+    """Per-level device times (Fig 10 analysis): one entry per level,
+    non-negative, summing to about the traversal time."""
+    A = synth.rmat(16, 16, seed=1, symmetrize=True, device=DEV)
+    M = tsmv.TiledMatrix.from_csr(A, dtype="pattern")
+    for s in [0] + synth.sample_sources(A.to("cpu"), 2, seed=3):
+        _, st = M.bfs(s)
+        t = st["level_ms"]
+        assert len(t) == st["nlevels"] and all(x >= 0 for x in t)
+        assert 0.5 * st["ms"] <= sum(t) <= 1.05 * st["ms"] + 0.01, (sum(t), st["ms"])
+    M.close()

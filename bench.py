@@ -38,7 +38,7 @@ import synth  # noqa: E402
 FALLBACK_HBM = 6650.0  # GB/s, B200_PROFILING.md fallback
 
 
-def parse():
+def parse(argv=None):
     p = argparse.ArgumentParser()
     p.add_argument("--gpus", type=int, default=1)
     p.add_argument("--steps", type=int, default=30)
@@ -50,7 +50,10 @@ def parse():
     p.add_argument("--tile-dim", type=int, default=16)
     p.add_argument("--thr", type=int, default=2)
     p.add_argument("--bfs-scale", type=int, default=22)
-    p.add_argument("--bfs-sources", type=int, default=4)
+    p.add_argument("--bfs-sources", type=int, default=16,
+                   help="C3: vertex 0 + (N-1) hash-ordered non-isolated sources (SURVEY §8(d) step 4)")
+    p.add_argument("--bfs26-sources", type=int, default=8, help="C5 on one GPU: vertex 0 + 7 sources")
+    p.add_argument("--no-bfs26", action="store_true", help="skip the R-MAT s26 TileBFS block (C5 at N=1)")
     p.add_argument("--bfs-thr", type=int, default=8,
                    help="very-sparse-tile threshold of the TileBFS contexts (DESIGN.md R25; SpMSpV keeps --thr)")
     p.add_argument("--no-bfs", action="store_true")
@@ -60,7 +63,7 @@ def parse():
     p.add_argument("--scaling", default="weak", choices=["weak", "strong"],
                    help="weak (default): at N ranks the R-MAT scales grow by log2 N, so the nonzeros "
                         "per GPU stay fixed; strong: the same matrix at every N")
-    a = p.parse_args()
+    a = p.parse_args(argv)
     world = int(os.environ.get("WORLD_SIZE", "1"))
     a.base_scale, a.base_bfs_scale = a.scale, a.bfs_scale
     if a.scaling == "weak" and world > 1:
@@ -264,20 +267,32 @@ def call_bytes_v6(st, k, sv, nt, m):
 
 
 def random_access(kms, nt):
-    """The kernel's DRAM read sectors (ncu, profiles/flat_traffic.json) per second of
-    its device time, next to the measured ceiling of cold random sector reads
-    (profiles/random_access_ceiling.json): the irregular path is bound by random
-    sector rate long before streaming bandwidth."""
+    """The kernel's DRAM read sectors (ncu capture, profiles/r02_flat_traffic.json)
+    per second of its device time, next to the measured rate of cold random
+    sector reads (profiles/r02_random_ceiling.json, scripts/micro/randbw2.cu):
+    context for the HBM fraction, not a replacement of it."""
     try:
-        t = json.load(open(os.path.join(ROOT, "profiles", "flat_traffic.json" if nt == 16 else "fused_traffic.json")))
-        c = json.load(open(os.path.join(ROOT, "profiles", "random_access_ceiling.json")))
+        t = json.load(open(os.path.join(ROOT, "profiles", "r02_flat_traffic.json" if nt == 16 else "fused_traffic.json")))
+        c = json.load(open(os.path.join(ROOT, "profiles", "r02_random_ceiling.json")))
         sec = t.get("dram_sectors_read") or t["dram_bytes_per_launch"] / 32
         ach = sec / (kms * 1e-3) / 1e9
-        ceil = c["footprint_1GiB_G_req_per_s"]
+        ceil = c["G_sectors_per_s"]
         return {"dram_sectors_per_launch (ncu)": int(sec), "achieved_G_sectors_per_s": round(ach, 2),
-                "ceiling_G_random_sectors_per_s": ceil, "frac": round(ach / ceil, 4)}
+                "random_sector_rate_G_per_s": ceil, "rate_source": c.get("how"), "frac": round(ach / ceil, 4)}
     except Exception:
         return None
+
+
+def traffic_of(nt):
+    """DRAM bytes (read + write) per launch of the SpMSpV kernel at T from the ncu
+    --set full capture committed under profiles/ (not measured in this run)."""
+    name = "r02_flat_traffic.json" if nt == 16 else "fused_traffic.json"
+    path = os.path.join(ROOT, "profiles", name)
+    try:
+        d = json.load(open(path))
+        return d.get("dram_bytes_per_launch"), f"profiles/{name}: {d.get('how', 'ncu --set full capture')}"
+    except Exception:
+        return None, None
 
 
 def survey_bytes(st, k, sv, nt, macs):
@@ -366,12 +381,17 @@ def run_tsmv(args):
         svy_bytes += survey_bytes(st, k, sv, args.tile_dim, macs)
         step_stats.append(st)
     torch.cuda.synchronize()
+    M_parity = None
+    if world == 1:
+        nlast = int(y_nnz.item())
+        M_parity = (xs[args.warmup + args.steps - 1], (y_idx[:nlast].clone(), y_val[:nlast].clone()))
     if world > 1:
         torch.distributed.barrier()
     kt, ncalls = M.get_timing()
     M.set_timing(False)
     clk = clocks.stop() if clocks else None
-    ms = sum(e0.elapsed_time(e1) for e0, e1 in ev)
+    step_ms = [e0.elapsed_time(e1) for e0, e1 in ev]
+    ms = sum(step_ms)
     if world > 1:
         import torch.distributed as dist
         t = torch.tensor([ms], dtype=torch.float64, device=dev)
@@ -380,31 +400,32 @@ def run_tsmv(args):
         flops = sum(flops_of(colcnt, xs[args.warmup + i][0]) for i in range(args.steps))
     value = flops / (ms * 1e-3) / 1e9
 
-    # roofline of the dominant (only) kernel: one k_spmspv_fused launch per call,
-    # algorithmic bytes / its CUDA-event duration
+    # roofline of the dominant (only) kernel: one cooperative launch per call.
+    # achieved = SURVEY §8(d) B_alg of the call (computed per sample from the
+    # call's counters, survey_bytes) / its CUDA-event duration
     kms = ms / args.steps
-    achieved = (kexp_bytes / args.steps) / (kms * 1e-3) / 1e9
-    traffic = None
-    tpath = os.path.join(ROOT, "profiles", "flat_traffic.json" if args.tile_dim == 16 else "fused_traffic.json")
-    if os.path.exists(tpath):
-        try:
-            traffic = json.load(open(tpath)).get("dram_bytes_per_launch")
-        except Exception:
-            traffic = None
+    achieved = (svy_bytes / args.steps) / (kms * 1e-3) / 1e9
+    traffic, tsrc = traffic_of(args.tile_dim)
     n_ = max(ncalls, 1)
     roof = {"bound": "hbm", "achieved": round(achieved, 2), "peak": peak, "unit": "GB/s",
-            "frac": round(achieved / peak, 4), "traffic": traffic,
+            "frac": round(achieved / peak, 4), "traffic": traffic, "traffic_source": tsrc,
             "kernel": ("k_spmspv_flat" if args.tile_dim == 16 else "k_spmspv_fused") + " (the whole call is one cooperative launch)",
             "peak_source": peak_src,
-            "algorithmic_bytes_per_launch": int(kexp_bytes / args.steps),
+            "B_alg_bytes_per_launch": int(svy_bytes / args.steps),
+            "B_alg_definition": "SURVEY §8(d): tile descriptor (4+8+nt/8 B) per tile in a hit tile column + "
+                                "(value + index) per useful tile nonzero + 16 B side col_ptr pair per x entry + "
+                                "(4 + value) per useful side nonzero + read x + write y",
             "kernel_ms_per_launch": round(kms, 5),
+            "ms_per_launch_median": round(statistics.median(step_ms), 5),
+            "ms_per_launch_min": round(min(step_ms), 5),
             "phase_ms_per_launch (globaltimer, CTA 0)": {
                 "A_x_tiling": round(kt[0] / n_, 5), "B_intersect_multiply": round(kt[1] / n_, 5),
                 "C_compact": round(kt[2] / n_, 5), "whole": round(kt[3] / n_, 5)},
-            "random_access": random_access(kms, args.tile_dim),
-            "survey_B_alg": {"bytes": int(svy_bytes / args.steps),
-                             "achieved_GBps": round(svy_bytes / (ms * 1e-3) / 1e9, 2),
-                             "frac": round(svy_bytes / (ms * 1e-3) / 1e9 / peak, 4)}}
+            "layout_bytes": {"bytes_per_launch": int(kexp_bytes / args.steps),
+                             "what": "every byte of this build's own layout one call touches (64-B tile records, "
+                                     "list entries, chunk maps, bitmap passes): DESIGN.md §6",
+                             "frac": round(kexp_bytes / (ms * 1e-3) / 1e9 / peak, 4)},
+            "random_access": random_access(kms, args.tile_dim)}
 
     # e2e through the public synchronous API with pinned host buffers (N = 1)
     e2e = None
@@ -438,10 +459,14 @@ def run_tsmv(args):
     if not args.no_configs and world == 1:
         del M
         configs = run_configs(args, dev, flush, tsmv)
+    bfs26 = None
+    if world == 1 and not args.no_bfs and not args.no_bfs26:
+        torch.cuda.empty_cache()
+        bfs26 = run_bfs26(args, dev, flush, tsmv)
 
-    cpu = None
+    cpu = cpu_omp_line = parity = None
     if rank == 0 and world == 1 and not args.no_cpu:
-        cpu = cpu_baseline(args, A, colcnt, xs)
+        cpu, cpu_omp_line, parity = cpu_baseline(args, A, colcnt, xs, M_parity)
 
     if rank == 0:
         mean_st = {kk: sum(s_[kk] for s_ in step_stats) / len(step_stats) for kk in step_stats[0]}
@@ -449,13 +474,14 @@ def run_tsmv(args):
                 "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms / args.steps, 5),
                 "higher_is_better": True, "scaling": args.scaling,
                 "vs_baseline": None, "dtype": args.dtype, "data": "synthetic (seeded R-MAT, seeded x)",
-                "config": workload_config(args), "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,
+                "config": workload_config(args), "roofline": roof, "cpu_baseline": cpu, "cpu_openmp": cpu_omp_line,
+                "parity": parity, "e2e": e2e,
                 "gpu_launches": args.steps, "clocks": clk,
                 "per_step": {"k": k, "mean_flops": int(flops / args.steps),
                              **{kk: round(v, 1) for kk, v in mean_st.items() if kk != "x_nnz"}},
                 "format": {kk: info[kk] for kk in ("nnz", "n_tiles", "n_dense_tiles", "dense_nnz", "side_nnz",
                                                    "build_ms", "bytes_spmspv")},
-                "bfs": bfs, "configs": configs}
+                "bfs": bfs, "bfs_s26": bfs26, "configs": configs}
         print(json.dumps(line), flush=True)
     if world > 1:
         torch.distributed.destroy_process_group()
@@ -468,20 +494,32 @@ def run_bfs(args, dev, flush, tsmv):
     M = tsmv.TiledMatrix.from_csr(A, dtype="pattern", tile_dim=args.tile_dim, sparse_tile_max_nnz=args.bfs_thr)
     build_wall = time.perf_counter() - t0
     info = M.info()
-    srcs = [0] + synth.sample_sources(A, max(0, args.bfs_sources - 1), seed=1)
+    srcs = bfs_sources(A, args.bfs_sources)
     levels = torch.empty(A.n, dtype=torch.int32, device=dev)
     M.bfs(srcs[0], levels=levels)  # warm-up
-    runs = []
+    deg, loops = degrees_and_loops(A)
+    runs, lv0 = [], None
     for s in srcs:
         flush()
         torch.cuda.synchronize()
         _, st = M.bfs(s, levels=levels)
-        runs.append({"source": int(s), "ms": round(st["ms"], 4), "levels": st["nlevels"],
-                     "edges": st["edges_traversed"], "reached": st["reached"],
-                     "gteps": round(st["edges_traversed"] / (st["ms"] * 1e-3) / 1e9, 3),
-                     "dirs": "".join({"push_csc": "C", "push_csr": "R", "pull_csc": "P"}.get(d, "?")
-                                     for d in st["dirs"])})
+        runs.append(bfs_run_line(s, st, levels, deg, loops))
+        if lv0 is None:
+            lv0 = levels.clone()
+            lvl_ms = [round(x, 4) for x in st["level_ms"]]
     hm = len(runs) / sum(1.0 / r["gteps"] for r in runs if r["gteps"] > 0)
+    hm500 = len(runs) / sum(1.0 / r["gteps_graph500"] for r in runs if r["gteps_graph500"] > 0)
+    bpar = None
+    if not args.no_cpu:
+        # parity of the timed traversal from vertex 0 against the oracle's queue BFS
+        import numpy as np
+
+        import oracle
+        C = oracle.csc_of(A.to("cpu"))
+        ref = oracle.bfs_queue(C, srcs[0])
+        bpar = {"ok": bool(np.array_equal(lv0.cpu().numpy(), ref)),
+                "checked": f"levels of the timed traversal from {srcs[0]} == oracle.bfs_queue (every vertex)"}
+        del C
     # min-id parents (MIN_SECOND semiring) of the last traversal, device time
     parents = torch.empty(A.n, dtype=torch.int32, device=dev)
     M.bfs_parents(levels, parents)
@@ -504,11 +542,72 @@ def run_bfs(args, dev, flush, tsmv):
              "gteps": round(mst["edges_traversed"] / (mst["ms"] * 1e-3) / 1e9, 3)}
     M.close()
     return {"graph": f"rmat_s{args.bfs_scale}_ef16_sym", "sparse_tile_max_nnz": args.bfs_thr,
-            "nnz": info["nnz"], "gteps_hmean": round(hm, 3),
-            "parents_ms": round(par_ms, 4), "msbfs_64": msbfs,
+            "nnz": info["nnz"], "sources": len(runs), "gteps_hmean": round(hm, 3),
+            "gteps_graph500_hmean": round(hm500, 3),
+            "parents_ms": round(par_ms, 4), "msbfs_64": msbfs, "parity": bpar,
+            "level_ms_source0": lvl_ms,
             "build_ms": round(info["build_ms"], 2), "build_wall_s": round(build_wall, 3),
-            "edge_count": "sum of out-degrees of reached vertices (directed count of the symmetrised graph)",
-            "runs": runs}
+            "edge_count": EDGE_COUNT, "runs": runs}
+
+
+EDGE_COUNT = ("gteps: edges = sum of out-degrees of reached vertices (R16, directed count of the "
+              "symmetrised graph); gteps_graph500: undirected edges of the traversed component "
+              "((sum of degrees + self loops) / 2, Graph500 TEPS)")
+
+
+def bfs_sources(A, count):
+    """Vertex 0 plus hash-ordered non-isolated sources (seed 1): SURVEY §8(d) step 4."""
+    return [0] + synth.sample_sources(A, max(0, count - 1), seed=1)
+
+
+def degrees_and_loops(A):
+    rp = A.row_ptr
+    deg = (rp[1:] - rp[:-1]).to(torch.int64)
+    rows = torch.repeat_interleave(torch.arange(A.m, device=rp.device), deg)
+    loops = torch.zeros(A.m, dtype=torch.int64, device=rp.device)
+    sl = rows[A.col_idx.long() == rows]
+    loops[sl] = 1
+    del rows
+    return deg, loops
+
+
+def bfs_run_line(s, st, levels, deg, loops):
+    r = levels >= 0
+    und = int((deg[r].sum() + loops[r].sum()) // 2)
+    ms = st["ms"]
+    return {"source": int(s), "ms": round(ms, 4), "levels": st["nlevels"],
+            "edges": st["edges_traversed"], "edges_graph500": und, "reached": st["reached"],
+            "gteps": round(st["edges_traversed"] / (ms * 1e-3) / 1e9, 3),
+            "gteps_graph500": round(und / (ms * 1e-3) / 1e9, 3),
+            "dirs": "".join({"push_csc": "C", "push_csr": "R", "pull_csc": "P"}.get(d, "?") for d in st["dirs"])}
+
+
+def run_bfs26(args, dev, flush, tsmv):
+    """C5 on one GPU: TileBFS on the symmetrised R-MAT s26 (2.1 G nonzeros, int64
+    offsets), vertex 0 + 7 sources, the bench's BFS context settings."""
+    t0 = time.perf_counter()
+    A = synth.rmat(26, 16, seed=1, symmetrize=True, device=dev)
+    gen = time.perf_counter() - t0
+    torch.cuda.empty_cache()
+    M = tsmv.TiledMatrix.from_csr(A, dtype="pattern", tile_dim=args.tile_dim, sparse_tile_max_nnz=args.bfs_thr)
+    info = M.info()
+    srcs = bfs_sources(A, args.bfs26_sources)
+    deg, loops = degrees_and_loops(A)
+    levels = torch.empty(A.n, dtype=torch.int32, device=dev)
+    M.bfs(srcs[0], levels=levels)
+    runs = []
+    for s in srcs:
+        flush()
+        torch.cuda.synchronize()
+        _, st = M.bfs(s, levels=levels)
+        runs.append(bfs_run_line(s, st, levels, deg, loops))
+    M.close()
+    hm = len(runs) / sum(1.0 / r["gteps"] for r in runs if r["gteps"] > 0)
+    hm500 = len(runs) / sum(1.0 / r["gteps_graph500"] for r in runs if r["gteps_graph500"] > 0)
+    return {"graph": "rmat_s26_ef16_sym", "nnz": A.nnz, "sparse_tile_max_nnz": args.bfs_thr,
+            "sources": len(runs), "gteps_hmean": round(hm, 3), "gteps_graph500_hmean": round(hm500, 3),
+            "gen_s": round(gen, 2), "build_ms": round(info["build_ms"], 2), "edge_count": EDGE_COUNT,
+            "parity": "tests/test_gpu_bench_configs.py::test_c5_s26 (levels from vertex 0 vs oracle)", "runs": runs}
 
 
 def run_bfs_dist(args, dev, flush, rank, world):
@@ -637,24 +736,57 @@ def run_configs(args, dev, flush, tsmv):
     return res
 
 
-def cpu_baseline(args, A, colcnt, xs):
-    """The oracle as it stands on the host, bounded to ~cpu_seconds of CPU work."""
+def cpu_baseline(args, A, colcnt, xs, parity_y):
+    """(1) The oracle as it stands on the host (1 core), bounded to ~cpu_seconds of
+    CPU work; (2) the OpenMP speed baseline (cpu_omp/: SpMSpV-bucket column merge)
+    on all host cores over the same samples; (3) parity of one timed step: y of
+    the last timed sample from the CUDA path against the oracle (index set
+    bit-exact, values within 1e-12 * sum_j |a_ij x_j|)."""
+    import numpy as np
+
+    import cpu_omp
     import oracle
     Ac = A.to("cpu")
     C = oracle.csc_of(Ac)
     flops, t = 0, 0.0
     used = 0
+    cc = colcnt.cpu()
     for xi, xv in xs:
         xi_c, xv_c = xi.cpu(), xv.cpu()
         t0 = time.perf_counter()
         oracle.spmspv(C, xi_c, xv_c)
         t += time.perf_counter() - t0
-        flops += flops_of(colcnt.cpu(), xi_c)
+        flops += flops_of(cc, xi_c)
         used += 1
         if t > args.cpu_seconds:
             break
-    return {"value": round(flops / t / 1e9, 5), "unit": "GFLOP/s", "cores": 1, "kind": "oracle",
-            "sample": f"{used} x samples (k={xs[0][0].numel()}) of the same workload, oracle CSC built once untimed"}
+    cpu = {"value": round(flops / t / 1e9, 5), "unit": "GFLOP/s", "cores": 1, "kind": "oracle",
+           "sample": f"{used} x samples (k={xs[0][0].numel()}) of the same workload, oracle CSC built once untimed",
+           "nproc": os.cpu_count(), "cpu_model": cpu_omp.cpu_model()}
+    Co = cpu_omp.csc_of(Ac)
+    nth = cpu_omp.threads()
+    fo, to = 0, 0.0
+    for xi, xv in xs[:used]:
+        xi_c, xv_c = xi.cpu().numpy(), xv.cpu().numpy()
+        t0 = time.perf_counter()
+        cpu_omp.spmspv(Co, xi_c, xv_c, nthreads=nth)
+        to += time.perf_counter() - t0
+        fo += flops_of(cc, torch.from_numpy(xi_c))
+    omp = {"value": round(fo / to / 1e9, 5), "unit": "GFLOP/s", "cores": nth, "kind": "openmp (cpu_omp/)",
+           "sample": f"the same {used} samples", "cpu_model": cpu_omp.cpu_model(), "nproc": os.cpu_count()}
+    parity = None
+    if parity_y is not None:
+        (pxi, pxv), (yi, yv) = parity_y
+        ri, rv = oracle.spmspv(C, pxi.cpu().numpy(), pxv.cpu().numpy())
+        Ca = oracle.CSC(C.m, C.n, C.col_ptr, C.row_idx, np.abs(C.val))
+        _, mag = oracle.spmspv(Ca, pxi.cpu().numpy(), np.abs(pxv.cpu().numpy()))
+        gi, gv = yi.cpu().numpy(), yv.cpu().numpy()
+        same = gi.shape == ri.shape and bool(np.array_equal(gi, ri))
+        ok = same and bool(np.all(np.abs(gv - rv) <= 1e-12 * mag))
+        parity = {"ok": ok, "checked": "y of the last timed step vs oracle.spmspv: index set bit-exact, "
+                                       "|y - y_ref| <= 1e-12 * sum_j |a_ij x_j|",
+                  "y_nnz": int(gi.size), "y_nnz_oracle": int(ri.size)}
+    return cpu, omp, parity
 
 
 def main():

@@ -69,6 +69,7 @@ struct BfsFusedArgs {
     int *bq0, *bq1;
     long long *lslots;   // [3][4] slots, [12..15] profiling, [16] solo release flag, [17..20] solo state
     int use_list, use_solo;
+    int qcap;                 // usable entries of the shared-memory queue (<= QCAP; TSMV_BFS_QCAP tests the overflow path)
     int wide_in_kernel;       // pull levels with m_u < nnz / 4 stay in the kernel (wide pull)
 };
 
@@ -100,7 +101,7 @@ __device__ __forceinline__ void discover_list(const BfsFusedArgs &a, const BfsVi
         nw &= nw - 1;
         const long long v = gseg * NT + r;
         B.levels[v] = B.level + 1;
-        if (p < QCAP) {
+        if (p < a.qcap) {
             sh.q[p] = (int)v;
         } else {  // queue full: straight to the global list and counters
             const unsigned long long gp = atomicAdd((unsigned long long *)&slot_n[0], 1ull);
@@ -118,7 +119,7 @@ __device__ __forceinline__ void discover_list(const BfsFusedArgs &a, const BfsVi
 __device__ __forceinline__ void list_flush(const BfsFusedArgs &a, ListShared &sh, int *Qn, long long *slot_n,
                                            int tid, int lane) {
     __syncthreads();
-    const int qn = min(sh.qn, QCAP);
+    const int qn = min(sh.qn, a.qcap);
     if (qn == 0) return;  // uniform: no __syncthreads skipped by part of the CTA
     if (tid == 0) sh.base = (int)atomicAdd((unsigned long long *)&slot_n[0], (unsigned long long)qn);
     __syncthreads();
@@ -867,6 +868,7 @@ bool bfs_fused_launch(tsmv_ctx *c, long long source, cudaStream_t st, bool resum
     a.use_list = (c->lwork.p != nullptr && !getenv("TSMV_BFS_NO_LIST")) ? 1 : 0;
     a.use_solo = a.use_list && !getenv("TSMV_BFS_NO_SOLO") ? 1 : 0;
     a.wide_in_kernel = getenv("TSMV_BFS_HOST_WIDE") ? 0 : 1;
+    a.qcap = getenv("TSMV_BFS_QCAP") ? std::max(1, std::min(QCAP, atoi(getenv("TSMV_BFS_QCAP")))) : QCAP;
     if (a.use_solo) TSMV_CUDA(cudaMemsetAsync(c->lslots.as<long long>() + 16, 0, 8, st));  // release flag
     void *args[] = {&a};
     void *f = c->nt == 16 ? (void *)k_bfs_fused<16> : c->nt == 32 ? (void *)k_bfs_fused<32> : (void *)k_bfs_fused<64>;

@@ -6,8 +6,8 @@ configuration bench.py uses: parity against closed forms and the oracle.
   C3  TileBFS on R-MAT s22 (push/pull switching)          (here: every source level-exact)
   C4  3D 7-point 256^3 and banded (2^20, b=64): TileBFS levels == closed forms (every vertex),
       SpMSpV at 1 % == oracle (every entry)
-  C5  R-MAT s26 row blocks: not at full size on one GPU; the partitioned path is covered
-      by test_gpu_dist_sim.py (simulated ranks) and test_dist_gloo.py (CPU, gloo)."""
+  C5  R-MAT s26 on one GPU at full size: test_gpu_bench_configs.py::test_c5_s26; the
+      partitioned path: test_gpu_dist_sim.py (simulated ranks), test_dist_gloo.py (CPU, gloo)."""
 import numpy as np
 import pytest
 import torch
@@ -90,9 +90,11 @@ def test_t_rmat_s22_fp32_and_semirings(tsmv):
 
 
 def test_c3_rmat_s22_parents_and_multisource(tsmv):
-    """C3 at full size: min-id BFS parents (MIN_SECOND, NEXT-2) against the oracle's
-    Alg 3 over MIN_SECOND, and the 64-source TileBFS (NEXT-3) against the queue BFS
-    on sampled source columns, in the launch configuration bench.py times."""
+    """C3 at full size with the library default threshold (thr = 2): min-id BFS
+    parents (MIN_SECOND, NEXT-2) against the oracle's Alg 3 over MIN_SECOND, and
+    the 64-source TileBFS (NEXT-3) against the queue BFS on sampled source
+    columns.  The bench's own contexts (thr = 8, all sources, all 64 columns) are
+    checked in test_gpu_bench_configs.py."""
     A = synth.rmat(22, 16, seed=1, symmetrize=True, device=DEV)
     M = tsmv.TiledMatrix.from_csr(A, dtype="pattern")
     Ah = A.to("cpu")

@@ -385,6 +385,9 @@ __device__ void solo_levels(const BfsFusedArgs &a, BfsView &B, int &level, long 
         __syncthreads();
         ++level;
         const long long mf2 = (long long)ss.mf, din2 = (long long)ss.din, mx2 = ss.maxw;
+        // every thread has read the level's totals before thread 0 zeroes them for
+        // the next level (compute-sanitizer racecheck, round 2)
+        __syncthreads();
         const int dir2 = n2 > 0 ? choose_dir_dev(a.force, a.alpha, a.dens, B.n, n2, mf2, mu - din2) : 0;
         int G2 = 1;
         while (G2 < mx2 && G2 < 32) G2 <<= 1;

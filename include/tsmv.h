@@ -36,7 +36,7 @@ typedef enum {
     TSMV_EINVAL = 1,      /* bad argument (sizes, NULL, unsorted/duplicate x, source range) */
     TSMV_ENOMEM = 2,      /* device or host allocation failed */
     TSMV_ECUDA = 3,       /* a CUDA runtime error (message in tsmv_last_error) */
-    TSMV_ENCCL = 4,       /* reserved: collective failure (exchange is done by the caller) */
+    TSMV_ENCCL = 4,       /* NCCL unavailable or a collective failed (message in tsmv_last_error) */
     TSMV_ECAPACITY = 5,   /* y_cap < y_nnz: *y_nnz holds the required size */
     TSMV_EUNSUPPORTED = 6 /* valid request this build does not support */
 } tsmv_status;
@@ -74,6 +74,13 @@ typedef struct {
     int64_t row_begin;           /* global id of local row 0 (multiple of 64 when nranks > 1) */
     const int64_t *row_splits;   /* host, nranks+1 global row boundaries (NULL when nranks == 1);
                                     copied by tsmv_create */
+    const void *nccl_unique_id;  /* host, 128 bytes from tsmv_nccl_unique_id on one rank, the same on
+                                    every rank, or NULL.  When set, tsmv_create
+                                    creates the context's own NCCL communicator (collective over the
+                                    nranks ranks, each on its own GPU; nranks == 1 allowed) and
+                                    tsmv_bfs / tsmv_spmspv become collective calls that exchange the
+                                    frontier / x themselves.  When NULL with nranks > 1, the caller
+                                    drives the exchange with the tsmv_bfs_dist_* primitives. */
 } tsmv_options;
 
 /* Per-call counters of the last tsmv_spmspv (read from device on request). */
@@ -127,6 +134,13 @@ typedef struct {
 /* Fill *opt with the defaults documented above.  Never fails for non-NULL opt. */
 tsmv_status tsmv_default_options(tsmv_options *opt);
 
+/* Bootstrap of a distributed context: a new ncclUniqueId written
+ * to out128 (128 bytes, host).  Call on ONE rank and hand the bytes to the others
+ * (e.g. torch.distributed.broadcast_object_list), then every rank passes them as
+ * tsmv_options.nccl_unique_id to tsmv_create.  NCCL is loaded at run time
+ * (libnccl.so.2; TSMV_NCCL_LIB overrides).  Errors: EINVAL (NULL), ENCCL. */
+tsmv_status tsmv_nccl_unique_id(void *out128);
+
 /* Build the tiled representation of A (Sec 3.2.1; BFS bitmasks
  * Sec 3.2.3) on opt->device.
  *   nrows, ncols : local rows (rows of this rank's block) and global columns.
@@ -144,9 +158,15 @@ tsmv_status tsmv_create(tsmv_ctx **out, int64_t nrows, int64_t ncols, const int6
                         const tsmv_options *opt);
 
 /* y = A x over `sr` (Sec 3.3, Fig 4).
- *   x_nnz, x_idx, x_val : the sparse x; x_idx int32 STRICTLY ASCENDING global column
- *                  ids (R18), host or device; x_val double (F64/PATTERN) or float
- *                  (F32), host or device, may be NULL for OR_AND.
+ *   x_nnz, x_idx, x_val : the sparse x; x_idx int32 UNIQUE global column ids in any
+ *                  order (R21: ascending input takes the fast path; otherwise the
+ *                  call sorts x once on the device), host or device; x_val double
+ *                  (F64/PATTERN) or float (F32), host or device, may be NULL for OR_AND.
+ *                  Distributed context with a communicator (nccl_unique_id): a
+ *                  COLLECTIVE call; each rank passes the x entries it owns (indices
+ *                  in its row range [row_splits[rank], row_splits[rank+1]) of the
+ *                  square A, ascending), the call exchanges them (count all-gather +
+ *                  grouped broadcasts) and returns y for the rank's own rows.
  *   y_cap, y_idx, y_val : caller-owned outputs (host or device).  y_idx int32
  *                  ascending GLOBAL row ids; y_val same type as x_val (not written
  *                  for OR_AND; may then be NULL).  y_cap >= nrows always suffices.
@@ -186,8 +206,13 @@ int64_t tsmv_trace_words(const tsmv_ctx *c);
 tsmv_status tsmv_last_call_stats(tsmv_ctx *c, tsmv_call_stats *s);
 
 /* TileBFS from `source` (Alg 3 P:418-430 with the three kernels of Sec 3.4,
- * P:1417-1628).  Single-GPU contexts only (nranks == 1; distributed BFS uses
- * the tsmv_bfs_dist_* calls).  Requires a square A built with build_bfs.
+ * P:1417-1628).  Single-GPU contexts, and distributed contexts with their own
+ * communicator (nccl_unique_id): then a COLLECTIVE call (same source on every
+ * rank; levels = the rank's own rows; stats global and identical on every rank;
+ * one in-place broadcast of each rank's owned frontier words per level, the
+ * statistics computed from the replicated frontier, no reduction).  Distributed
+ * contexts without a communicator use the tsmv_bfs_dist_* calls.  Requires a
+ * square A built with build_bfs.
  *   levels : int32[nrows] host or device out: hop count from source, -1 if
  *            unreachable (R15).
  *   stats  : host, may be NULL.

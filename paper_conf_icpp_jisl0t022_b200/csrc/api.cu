@@ -5,6 +5,7 @@
 #include <algorithm>
 #include <cstdarg>
 #include <map>
+#include <mutex>
 #include <tuple>
 
 namespace tsmv {
@@ -54,6 +55,13 @@ int fused_occupancy(int nt, int dtype);
 // its lines in L2 across calls, so the first RED to a row does not fetch a zero
 // sector from HBM.  Device-wide set-aside (cudaLimitPersistingL2CacheSize) is
 // raised to the window size if the device allows it.  TSMV_NO_PERSIST=1 disables.
+// The device-wide set-aside is raised only while a context that uses it lives:
+// the first such context records the limit it found, the last one restores it
+// (and returns the persisting lines to normal), so the library leaves no L2
+// policy behind once every context is destroyed.
+static std::mutex g_persist_mu;
+static std::map<int, std::pair<int, size_t>> g_persist;  // device -> (contexts, limit found)
+
 static void setup_persistence(tsmv_ctx *c) {
     c->persist_bytes = 0;
     c->persist_ratio = 0.f;
@@ -66,15 +74,33 @@ static void setup_persistence(tsmv_ctx *c) {
     }
     if (max_persist <= 0 || max_win <= 0) return;
     const size_t want = std::min<size_t>(c->acc.bytes, (size_t)max_win);
+    std::lock_guard<std::mutex> lk(g_persist_mu);
     size_t cur = 0;
     cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize);
     const size_t setp = std::max(cur, std::min(want, (size_t)max_persist));
+    auto it = g_persist.find(c->device);
+    const size_t found = it == g_persist.end() ? cur : it->second.second;
     if (setp > cur && cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, setp) != cudaSuccess) {
         cudaGetLastError();
         return;
     }
+    g_persist[c->device] = {it == g_persist.end() ? 1 : it->second.first + 1, found};
     c->persist_bytes = want;
     c->persist_ratio = (float)std::min(1.0, (double)setp / (double)want);
+}
+
+static void release_persistence(tsmv_ctx *c) {
+    if (!c->persist_bytes) return;
+    std::lock_guard<std::mutex> lk(g_persist_mu);
+    auto it = g_persist.find(c->device);
+    if (it == g_persist.end()) return;
+    if (--it->second.first == 0) {
+        cudaCtxResetPersistingL2Cache();
+        cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, it->second.second);
+        cudaGetLastError();
+        g_persist.erase(it);
+    }
+    c->persist_bytes = 0;
 }
 }
 
@@ -102,6 +128,8 @@ static void destroy_impl(tsmv_ctx *c) {
     if (!c) return;
     cudaSetDevice(c->device);
     cudaDeviceSynchronize();
+    comm_destroy(c);
+    release_persistence(c);
     c->P.release();
     c->Qown.release();
     for (DevBuf *b : {&c->outdeg, &c->indeg, &c->acc, &c->rowbits, &c->desc_compact, &c->counters, &c->stage_x_idx,
@@ -146,7 +174,12 @@ extern "C" tsmv_status tsmv_create(tsmv_ctx **out, int64_t nrows, int64_t ncols,
         c->lognt = log2_nt(c->nt);
         c->m = nrows;
         c->n = ncols;
-        if (o.nranks > 1) {
+        if (o.nranks == 1 && o.nccl_unique_id) {
+            // a one-rank communicator (tests the collective path on one GPU)
+            TSMV_REQUIRE(o.row_begin == 0, "tsmv_create: row_begin must be 0 when nranks == 1");
+            c->row_splits = {0, nrows};
+            c->row_begin = 0;
+        } else if (o.nranks > 1) {
             TSMV_REQUIRE(o.row_splits != nullptr, "tsmv_create: nranks > 1 needs row_splits");
             c->row_splits.assign(o.row_splits, o.row_splits + o.nranks + 1);
             for (int p = 0; p <= o.nranks; ++p) {
@@ -264,6 +297,7 @@ extern "C" tsmv_status tsmv_create(tsmv_ctx **out, int64_t nrows, int64_t ncols,
             c->desc_bfs.alloc(bb * sizeof(LBDesc<8>));
             TSMV_CUDA(cudaMemsetAsync(c->desc_bfs.p, 0, c->desc_bfs.bytes, st));
         }
+        if (o.nccl_unique_id) comm_init(c, o.nccl_unique_id, st);
         if (o.nranks > 1) {
             c->splits_dev.alloc((o.nranks + 1) * 8);
             TSMV_CUDA(cudaMemcpyAsync(c->splits_dev.p, c->row_splits.data(), (o.nranks + 1) * 8,

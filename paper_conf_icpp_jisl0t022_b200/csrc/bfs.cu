@@ -707,6 +707,15 @@ struct BfsRunner {
         return B;
     }
 
+    // degree arrays of the frontier statistics: a context with its own
+    // communicator uses the replicated GLOBAL arrays (every rank then computes
+    // the same |F|, m_f and sum of in-degrees from the same frontier bitmap);
+    // otherwise its local ones (sum of in-degrees over its own rows only)
+    const int *odeg() const { return c->outdeg_g.p ? c->outdeg_g.as<int>() : c->outdeg.as<int>(); }
+    const int *ideg() const { return c->indeg_g.p ? c->indeg_g.as<int>() : c->indeg.as<int>(); }
+    long long irb() const { return c->indeg_g.p ? 0 : c->row_begin; }
+    long long iml() const { return c->indeg_g.p ? c->n : c->m; }
+
     template <int NT> void fscan(const uint32_t *F, uint32_t *Fclear, bool lists) {
         long long nseg = c->nTC;
         int grid = (int)std::max<long long>(1, (nseg + SCAN_BLOCK - 1) / SCAN_BLOCK);
@@ -722,14 +731,13 @@ struct BfsRunner {
             const int g = (int)std::max<long long>(
                 1, std::min<long long>((nseg * 2 + 255) / 256, (long long)c->sm_count * bps));
             k_fstats16<<<g, 256, 0, st>>>(F, Fclear, nseg, c->P.ptr.as<long long>(), c->P.sptr.as<long long>(),
-                                          c->outdeg.as<int>(), c->indeg.as<int>(), c->row_begin, c->m,
-                                          c->counters.as<Counters>(), c->hcnt_dev);
+                                          odeg(), ideg(), irb(), iml(), c->counters.as<Counters>(), c->hcnt_dev);
             TSMV_CUDA(cudaGetLastError());
             return;
         }
         k_fscan<NT><<<grid, SCAN_BLOCK, 0, st>>>(F, Fclear, nseg, NW, c->P.ptr.as<long long>(),
-                                                 c->P.sptr.as<long long>(), c->outdeg.as<int>(), c->indeg.as<int>(),
-                                                 c->row_begin, c->m, lists_view(c), c->counters.as<Counters>(),
+                                                 c->P.sptr.as<long long>(), odeg(), ideg(),
+                                                 irb(), iml(), lists_view(c), c->counters.as<Counters>(),
                                                  c->hcnt_dev, c->desc_bfs.as<LBDesc<8>>(), c->epoch, lists ? 1 : 0);
         TSMV_CUDA(cudaGetLastError());
     }
@@ -815,12 +823,93 @@ static void level_times(tsmv_ctx *c, tsmv_bfs_stats *stats, long long nl, bool h
         stats->level_ms[L] = (L + 1 < nl || has_end) && t[L + 1] >= t[L] ? (float)((t[L + 1] - t[L]) * 1e-6) : 0.f;
 }
 
+// Distributed TileBFS of a context with its own communicator:
+// Alg 3's level loop on every rank, one exchange per level.  The
+// frontier F and the visited bitmap V are replicated (n bits); each rank expands
+// the level into its OWNED rows with the level kernels (Push-CSC / Push-CSR /
+// Pull-CSC over its row block), the owned segments of the next frontier are
+// broadcast in place to every rank (comm_exchange_frontier), and the statistics
+// scan of the whole next frontier with the replicated global degree arrays gives
+// every rank the same |F|, m_f and m_u, hence the same direction decision and
+// termination, with no reduction.  One host synchronisation per level (the
+// statistics decide which kernels the host launches).
+static void bfs_distributed(tsmv_ctx *c, int64_t source, tsmv_bfs_stats *stats, cudaStream_t st) {
+    ensure_lists(c, c->n);
+    BfsRunner R{c, st, (long long)(c->V.bytes / 4)};
+    unsigned long long *tlv = c->bfs_tlv.as<unsigned long long>();
+    c->fcur = 0;
+    c->bfs_level = 0;
+    TSMV_CUDA(cudaEventRecord(c->ev0, st));
+    TSMV_CUDA(cudaMemsetAsync(c->F1.p, 0, c->F1.bytes, st));
+    R.init(source);
+    R.do_fscan(c->F0.as<uint32_t>(), nullptr);
+    TSMV_CUDA(cudaStreamSynchronize(st));
+    volatile Counters *h = c->hcnt;
+    long long fsize = h->fsize, mf = h->mf, mu = c->nnz_global - h->din;
+    long long reached = 0, edges = 0;
+    long long L = 0;
+    while (fsize > 0) {
+        const int dir = choose_dir(c->opt, c->n, fsize, mf, mu);
+        if (L < TSMV_MAX_LEVELS) {
+            if (stats) {
+                stats->dir_per_level[L] = dir;
+                stats->frontier_per_level[L] = fsize;
+            }
+            k_stamp<<<1, 1, 0, st>>>(tlv + L);
+        }
+        reached += fsize;
+        edges += mf;
+        c->bfs_level = (int)L;
+        R.do_expand(dir, dir == TSMV_DIR_PULL_CSC && mu * 4 < c->nnz_global);
+        uint32_t *Fcur = (c->fcur == 0 ? c->F0 : c->F1).as<uint32_t>();
+        uint32_t *Fnext = (c->fcur == 0 ? c->F1 : c->F0).as<uint32_t>();
+        comm_exchange_frontier(c, Fnext, c->V.as<uint32_t>(), (c->n + 31) / 32, st);
+        R.do_fscan(Fnext, Fcur);
+        TSMV_CUDA(cudaStreamSynchronize(st));
+        fsize = h->fsize;
+        mf = h->mf;
+        mu -= h->din;
+        c->fcur ^= 1;
+        ++L;
+    }
+    if (L <= TSMV_MAX_LEVELS) k_stamp<<<1, 1, 0, st>>>(tlv + L);
+    TSMV_CUDA(cudaEventRecord(c->ev1, st));
+    TSMV_CUDA(cudaMemsetAsync(c->F0.p, 0, c->F0.bytes, st));
+    TSMV_CUDA(cudaMemsetAsync(c->F1.p, 0, c->F1.bytes, st));
+    TSMV_CUDA(cudaStreamSynchronize(st));
+    c->bfs_last_levels = L;
+    if (stats) {
+        float ms = 0;
+        TSMV_CUDA(cudaEventElapsedTime(&ms, c->ev0, c->ev1));
+        stats->nlevels = (int32_t)std::min<long long>(L, INT32_MAX);
+        if (L > 0) level_times(c, stats, std::min<long long>(L, TSMV_MAX_LEVELS), L <= TSMV_MAX_LEVELS);
+        stats->reached = reached;
+        stats->edges_traversed = edges;
+        stats->ms = ms;
+    }
+}
+
 extern "C" tsmv_status tsmv_bfs(tsmv_ctx *c, int64_t source, int32_t *levels, tsmv_bfs_stats *stats,
                                 void *cuda_stream) {
     try {
         TSMV_REQUIRE(c != nullptr && levels != nullptr, "tsmv_bfs: NULL argument");
         bfs_check(c);
-        TSMV_REQUIRE(c->opt.nranks == 1, "tsmv_bfs: distributed contexts use tsmv_bfs_dist_*");
+        if (has_comm(c)) {
+            TSMV_REQUIRE(source >= 0 && source < c->n, "tsmv_bfs: source %lld out of range", (long long)source);
+            TSMV_CUDA(cudaSetDevice(c->device));
+            cudaStream_t st = (cudaStream_t)cuda_stream;
+            bool host_levels;
+            bfs_prepare_levels(c, levels, host_levels);
+            bfs_distributed(c, source, stats, st);
+            if (host_levels) {
+                TSMV_CUDA(cudaMemcpyAsync(levels, c->levels_dev, c->m * 4, cudaMemcpyDeviceToHost, st));
+                TSMV_CUDA(cudaStreamSynchronize(st));
+            }
+            return TSMV_OK;
+        }
+        TSMV_REQUIRE(c->opt.nranks == 1,
+                     "tsmv_bfs: a distributed context needs its own communicator (tsmv_options.nccl_unique_id) "
+                     "or the tsmv_bfs_dist_* calls");
         TSMV_REQUIRE(source >= 0 && source < c->n, "tsmv_bfs: source %lld out of range", (long long)source);
         TSMV_CUDA(cudaSetDevice(c->device));
         cudaStream_t st = (cudaStream_t)cuda_stream;

@@ -292,6 +292,7 @@ struct tsmv_ctx {
 
     // host staging
     tsmv::DevBuf stage_x_idx, stage_x_val, stage_y_idx, stage_y_val, stage_levels;
+    tsmv::DevBuf sort_x_idx, sort_x_val, sort_tmp;  // x sorted by tsmv_spmspv when not ascending (R21)
 
     // BFS state
     tsmv::DevBuf V, F0, F1;    // uint32[ceil(n/64)*2] visited, frontier ping-pong
@@ -334,6 +335,13 @@ struct tsmv_ctx {
     tsmv::DevBuf par_chunks;                // BFS parents: (vertex << 24 | chunk) of heavy side rows
     long long par_nchunks = 0;
     void *trace = nullptr;         // tsmv_set_trace (device, u64[tsmv_trace_words])
+    // distributed context with its own NCCL communicator (comm.cu)
+    void *nccl_comm = nullptr;     // ncclComm_t
+    tsmv::DevBuf outdeg_g;         // int32[n]: global column counts (all ranks' blocks)
+    tsmv::DevBuf indeg_g;          // int32[n]: global row counts
+    long long nnz_global = 0;
+    tsmv::DevBuf kcounts;          // int64[nranks + 1]: x counts of the ranks (SpMSpV exchange)
+    tsmv::DevBuf xg_idx, xg_val;   // the gathered global x
 };
 
 namespace tsmv {
@@ -368,6 +376,13 @@ bool bfs_fused_launch(tsmv_ctx *c, long long source, cudaStream_t st, bool resum
                       uint32_t *Fb, long long mu, long long reached, long long edges, bool stop_on_pull,
                       long long max_levels, long long &level_out, long long &mu_out, long long &reached_out,
                       long long &edges_out, int &cur_out);
+// comm.cu
+bool has_comm(const tsmv_ctx *c);
+void comm_init(tsmv_ctx *c, const void *unique_id, cudaStream_t st);
+void comm_destroy(tsmv_ctx *c);
+void comm_exchange_frontier(tsmv_ctx *c, uint32_t *F, uint32_t *V, long long nwords, cudaStream_t st);
+long long comm_gather_x(tsmv_ctx *c, long long k_local, const int32_t *x_idx, const void *x_val, size_t vb,
+                        const int32_t **xi_out, const void **xv_out, cudaStream_t st);
 // bfs.cu
 int choose_dir(const tsmv_options &o, long long n, long long fsize, long long mf, long long mu);
 // pointer classification

@@ -25,6 +25,7 @@
 //           handles bit l of each word, so a dense stretch of y costs one round
 //           of 32 parallel accumulator loads per word.  acc/bits cleared on read.
 #include "device.cuh"
+#include <cub/device/device_radix_sort.cuh>
 
 namespace tsmv {
 
@@ -1043,6 +1044,37 @@ __global__ void k_copy_y(const int32_t *__restrict__ yi, const void *__restrict_
 }  // namespace
 }  // namespace tsmv
 
+// Reading R21: x in any order of unique indices.  The kernels take ascending x
+// (segments are runs); an x they reject is sorted here once (CUB radix sort of
+// (index, value) pairs into ctx buffers) and the call is repeated; duplicates
+// or out-of-range indices are then still rejected (EINVAL).
+static void sort_x(tsmv_ctx *c, long long k, const int32_t *xi, const void *xv, size_t vb, const int32_t **xi_out,
+                   const void **xv_out, cudaStream_t st) {
+    c->sort_x_idx.ensure((size_t)k * 4);
+    if (xv) c->sort_x_val.ensure((size_t)k * vb);
+    int32_t *ko = c->sort_x_idx.as<int32_t>();
+    size_t tb = 0;
+    if (!xv) {
+        TSMV_CUDA(cub::DeviceRadixSort::SortKeys(nullptr, tb, xi, ko, (int)k, 0, 32, st));
+        c->sort_tmp.ensure(tb);
+        TSMV_CUDA(cub::DeviceRadixSort::SortKeys(c->sort_tmp.p, tb, xi, ko, (int)k, 0, 32, st));
+    } else if (vb == 8) {
+        const double *vi = static_cast<const double *>(xv);
+        double *vo = c->sort_x_val.as<double>();
+        TSMV_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tb, xi, ko, vi, vo, (int)k, 0, 32, st));
+        c->sort_tmp.ensure(tb);
+        TSMV_CUDA(cub::DeviceRadixSort::SortPairs(c->sort_tmp.p, tb, xi, ko, vi, vo, (int)k, 0, 32, st));
+    } else {
+        const float *vi = static_cast<const float *>(xv);
+        float *vo = c->sort_x_val.as<float>();
+        TSMV_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tb, xi, ko, vi, vo, (int)k, 0, 32, st));
+        c->sort_tmp.ensure(tb);
+        TSMV_CUDA(cub::DeviceRadixSort::SortPairs(c->sort_tmp.p, tb, xi, ko, vi, vo, (int)k, 0, 32, st));
+    }
+    *xi_out = ko;
+    *xv_out = xv ? c->sort_x_val.p : nullptr;
+}
+
 extern "C" tsmv_status tsmv_spmspv(tsmv_ctx *c, tsmv_semiring sr, int64_t x_nnz, const int32_t *x_idx,
                                    const void *x_val, int64_t y_cap, int32_t *y_idx, void *y_val, int64_t *y_nnz,
                                    void *cuda_stream) {
@@ -1060,7 +1092,7 @@ extern "C" tsmv_status tsmv_spmspv(tsmv_ctx *c, tsmv_semiring sr, int64_t x_nnz,
         cudaStream_t st = (cudaStream_t)cuda_stream;
         *y_nnz = 0;
         c->last_x_nnz = x_nnz;
-        if (x_nnz == 0) return TSMV_OK;
+        if (x_nnz == 0 && !has_comm(c)) return TSMV_OK;  // a collective call always takes part
         const bool f32 = c->dtype == TSMV_F32;
         const size_t vb = f32 ? 4 : 8;
         // stage host inputs
@@ -1068,8 +1100,9 @@ extern "C" tsmv_status tsmv_spmspv(tsmv_ctx *c, tsmv_semiring sr, int64_t x_nnz,
         // reads each entry once, coalesced); pageable host x is staged
         const int32_t *xi = x_idx;
         const void *xv = (sr == TSMV_OR_AND) ? nullptr : x_val;
+        // (a collective call hands x to NCCL: device memory only, so it is staged)
         if (!is_device_ptr(xi)) {
-            if (const void *d = mapped_device_ptr(xi)) {
+            if (const void *d = has_comm(c) ? nullptr : mapped_device_ptr(xi)) {
                 xi = static_cast<const int32_t *>(d);
             } else {
                 c->stage_x_idx.ensure(x_nnz * 4);
@@ -1078,13 +1111,19 @@ extern "C" tsmv_status tsmv_spmspv(tsmv_ctx *c, tsmv_semiring sr, int64_t x_nnz,
             }
         }
         if (xv && !is_device_ptr(xv)) {
-            if (const void *d = mapped_device_ptr(xv)) {
+            if (const void *d = has_comm(c) ? nullptr : mapped_device_ptr(xv)) {
                 xv = d;
             } else {
                 c->stage_x_val.ensure(x_nnz * vb);
                 TSMV_CUDA(cudaMemcpyAsync(c->stage_x_val.p, xv, x_nnz * vb, cudaMemcpyHostToDevice, st));
                 xv = c->stage_x_val.p;
             }
+        }
+        if (has_comm(c)) {
+            // distributed: x entries owned by the ranks -> one global ascending x
+            x_nnz = comm_gather_x(c, x_nnz, xi, xv, vb, &xi, &xv, st);
+            c->last_x_nnz = x_nnz;
+            if (x_nnz == 0) return TSMV_OK;
         }
         bool host_y = (y_cap > 0) && !is_device_ptr(y_idx);
         bool host_yv = (y_cap > 0) && sr != TSMV_OR_AND && y_val && !is_device_ptr(y_val);
@@ -1100,22 +1139,27 @@ extern "C" tsmv_status tsmv_spmspv(tsmv_ctx *c, tsmv_semiring sr, int64_t x_nnz,
             c->stage_y_val.ensure(std::max<int64_t>(ycap_dev, 1) * vb);
             yv = c->stage_y_val.p;
         }
-        enqueue_spmspv(c, sr, x_nnz, xi, xv, ycap_dev, yi, yv, nullptr, st);
         // pinned (mapped) host y: copied by a kernel sized on the device, right
         // behind the multiply, then ONE synchronisation for the whole call
         void *myi = host_y ? mapped_device_ptr(y_idx) : nullptr;
         void *myv = host_yv ? mapped_device_ptr(y_val) : nullptr;
         const bool direct = (!host_y || myi) && (!host_yv || myv) && (host_y || host_yv);
-        if (direct) {
-            k_copy_y<<<c->sm_count * 4, 256, 0, st>>>(yi, yv, &c->counters.as<Counters>()->y_nnz, y_cap,
-                                                       static_cast<int32_t *>(myi), myv, (int)vb);
-            TSMV_CUDA(cudaGetLastError());
-        }
-        TSMV_CUDA(cudaStreamSynchronize(st));
         volatile Counters *h = c->hcnt;
+        int err = 0;
+        for (int attempt = 0; attempt < 2; ++attempt) {
+            enqueue_spmspv(c, sr, x_nnz, xi, xv, ycap_dev, yi, yv, nullptr, st);
+            if (direct) {
+                k_copy_y<<<c->sm_count * 4, 256, 0, st>>>(yi, yv, &c->counters.as<Counters>()->y_nnz, y_cap,
+                                                           static_cast<int32_t *>(myi), myv, (int)vb);
+                TSMV_CUDA(cudaGetLastError());
+            }
+            TSMV_CUDA(cudaStreamSynchronize(st));
+            err = h->err;
+            if (!err || attempt) break;
+            sort_x(c, x_nnz, xi, xv, vb, &xi, &xv, st);  // R21: any order of unique indices
+        }
         int64_t ynnz = h->y_nnz;
-        int err = h->err;
-        TSMV_REQUIRE(err == 0, "tsmv_spmspv: x indices must be strictly ascending and in [0, %lld)", (long long)c->n);
+        TSMV_REQUIRE(err == 0, "tsmv_spmspv: x indices must be unique and in [0, %lld)", (long long)c->n);
         *y_nnz = ynnz;
         if (ynnz > y_cap) {
             set_error("tsmv_spmspv: y_cap %lld < y_nnz %lld", (long long)y_cap, (long long)ynnz);

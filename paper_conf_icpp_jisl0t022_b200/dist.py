@@ -1,4 +1,4 @@
-"""Row-block multi-GPU TileSpMSpV / TileBFS (SURVEY §8(e); DESIGN.md §Multi-GPU).
+"""Row-block multi-GPU TileSpMSpV / TileBFS (SURVEY §8(e); DESIGN.md §8).
 
 The paper is single-GPU; the partitioned path is this build's addition
 (BASELINE.json north_star item 4).  One process per GPU.  Rank p owns global
@@ -6,15 +6,17 @@ rows [splits[p], splits[p+1]) of A (contiguous, nnz-balanced, cut at multiples
 of 64 rows so tile rows and bitmap words never straddle ranks) in its own
 libtsmv context; columns stay global.
 
-Per iteration there is exactly one exchange, done with torch.distributed (NCCL
-over NVLink on the GPU box, gloo in the CPU tests):
-  * SpMSpV: all-gather of the owners' x entries (counts, then padded entries);
-    every rank then computes y for its own rows -- no reduction is needed;
-  * TileBFS: all-gather of each rank's newly discovered owned-vertex bitmap
-    segment (padded to the largest segment) + one all-reduce of two int64
-    (m_f, m_u) so that all ranks take the same push/pull decision.
-Everything else (the level kernels, the merge of the gathered frontier into the
-replicated visited bitmap, the frontier scan) runs in libtsmv.so.
+The product path is `DistMatrix`: this module only BOOTSTRAPS it (the row
+partition, and one ncclUniqueId from rank 0 shared over torch.distributed);
+the context then owns its NCCL communicator and `tsmv_bfs` / `tsmv_spmspv`
+are collective calls whose level loop and exchanges run inside libtsmv.so
+(comm.cu: in-place broadcasts of the owned frontier words per level; count
+all-gather + broadcasts of the owned x entries).
+
+`DistTiledMatrix` + `bfs_loop` keep the caller-driven form (the
+tsmv_bfs_dist_* primitives, exchange by torch.distributed or by concatenation):
+it runs where a communicator cannot (several simulated ranks on one GPU, the
+gloo CPU tests) and checks the partitioned kernels rank by rank.
 """
 from __future__ import annotations
 
@@ -38,21 +40,80 @@ def partition_rows(row_ptr: torch.Tensor, nranks: int, align: int = ALIGN) -> Li
     for p in range(1, nranks):
         target = (nnz * p + nranks - 1) // nranks
         r = int(torch.searchsorted(rp, torch.tensor(target, dtype=torch.int64), right=False))
-        r = min(m, ((r + align // 2) // align) * align)   # nearest multiple of `align`
+        # nearest multiple of `align`, never past the last aligned row (an interior
+        # split must stay a multiple of `align` even when m is not)
+        r = min((m // align) * align, ((r + align // 2) // align) * align)
         splits.append(max(r, splits[-1]))
     splits.append(m)
     return splits
 
 
-def local_rows(A, splits: Sequence[int], rank: int):
+class RowBlock:
+    """A CSR row block: m local rows, n global columns (row_ptr int64, col_idx int32)."""
+
+    def __init__(self, m, n, row_ptr, col_idx, values=None, name="block"):
+        self.m, self.n, self.row_ptr, self.col_idx, self.values, self.name = m, n, row_ptr, col_idx, values, name
+
+    @property
+    def nnz(self):
+        return int(self.col_idx.numel())
+
+    def to(self, device):
+        v = None if self.values is None else self.values.to(device)
+        return RowBlock(self.m, self.n, self.row_ptr.to(device), self.col_idx.to(device), v, self.name)
+
+    def with_values(self, values):
+        return RowBlock(self.m, self.n, self.row_ptr, self.col_idx, values, self.name)
+
+
+def local_rows(A, splits: Sequence[int], rank: int) -> RowBlock:
     """The CSR block of A holding rows [splits[rank], splits[rank+1]) (global columns)."""
-    import synth  # only for the CSR container type
     r0, r1 = int(splits[rank]), int(splits[rank + 1])
     rp = A.row_ptr[r0:r1 + 1]
     base = int(rp[0])
     cols = A.col_idx[base:int(rp[-1])]
     vals = None if A.values is None else A.values[base:int(rp[-1])]
-    return synth.CSR(r1 - r0, A.n, rp - base, cols, vals, f"{A.name}[{r0}:{r1}]")
+    return RowBlock(r1 - r0, A.n, rp - base, cols, vals, f"{getattr(A, 'name', 'A')}[{r0}:{r1}]")
+
+
+def bootstrap_unique_id(group=None) -> bytes:
+    """One ncclUniqueId made by rank 0 and shared with every rank of `group` over
+    torch.distributed (object broadcast: works on gloo and NCCL groups)."""
+    from . import tsmv
+    obj = [tsmv.nccl_unique_id() if dist.get_rank(group) == 0 else None]
+    dist.broadcast_object_list(obj, src=dist.get_global_rank(group, 0) if group is not None else 0, group=group)
+    return obj[0]
+
+
+class DistMatrix:
+    """This rank's row block in a libtsmv context that owns its NCCL communicator:
+    bfs() and spmspv() are collective calls running entirely in the library."""
+
+    def __init__(self, A_local, splits: Sequence[int], rank: int, nranks: int, unique_id: bytes,
+                 dtype: Optional[str] = None, device: int = 0, **opts):
+        from . import tsmv
+        self.splits = [int(s) for s in splits]
+        self.rank, self.nranks = rank, nranks
+        self.m_local, self.n = A_local.m, A_local.n
+        self.device = torch.device("cuda", device)
+        kw = dict(rank=rank, nranks=nranks, nccl_unique_id=unique_id, build_bfs=1)
+        if nranks > 1:
+            kw["row_splits"] = self.splits
+        self.M = tsmv.TiledMatrix(A_local.m, A_local.n, A_local.row_ptr, A_local.col_idx, A_local.values,
+                                  dtype=dtype, device=device, **kw, **opts)
+
+    def bfs(self, source: int, levels: Optional[torch.Tensor] = None):
+        """Collective: levels of this rank's rows, global statistics."""
+        return self.M.bfs(source, levels=levels)
+
+    def spmspv(self, x_idx_owned: torch.Tensor, x_val_owned: Optional[torch.Tensor], semiring="plus_times",
+               y_idx: Optional[torch.Tensor] = None, y_val: Optional[torch.Tensor] = None):
+        """Collective: x entries owned by this rank (indices in its row range) in,
+        y of this rank's rows out."""
+        return self.M.spmspv(x_idx_owned, x_val_owned, semiring=semiring, y_idx=y_idx, y_val=y_val)
+
+    def close(self):
+        self.M.close()
 
 
 def allgather_sizes(count: int, device, group=None) -> List[int]:

@@ -41,7 +41,8 @@ class tsmv_options(ctypes.Structure):
                 ("sparse_tile_max_nnz", ctypes.c_int32), ("build_bfs", ctypes.c_int32),
                 ("push_csr_density", ctypes.c_double), ("pull_alpha", ctypes.c_double),
                 ("force_dir", ctypes.c_int32), ("rank", ctypes.c_int32), ("nranks", ctypes.c_int32),
-                ("row_begin", ctypes.c_int64), ("row_splits", ctypes.POINTER(ctypes.c_int64))]
+                ("row_begin", ctypes.c_int64), ("row_splits", ctypes.POINTER(ctypes.c_int64)),
+                ("nccl_unique_id", ctypes.c_void_p)]
 
 
 class tsmv_call_stats(ctypes.Structure):
@@ -73,6 +74,7 @@ class tsmv_bfs_stats(ctypes.Structure):
 _vp, _i64, _i32 = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int32
 _SIGS = {
     "tsmv_default_options": (ctypes.c_int, [ctypes.POINTER(tsmv_options)]),
+    "tsmv_nccl_unique_id": (ctypes.c_int, [_vp]),
     "tsmv_create": (ctypes.c_int, [ctypes.POINTER(_vp), _i64, _i64, _vp, _vp, _vp, ctypes.c_int,
                                    ctypes.POINTER(tsmv_options)]),
     "tsmv_spmspv": (ctypes.c_int, [_vp, ctypes.c_int, _i64, _vp, _vp, _i64, _vp, _vp, ctypes.POINTER(_i64), _vp]),
@@ -147,6 +149,10 @@ def default_options(**kw) -> tsmv_options:
             arr = (ctypes.c_int64 * len(v))(*[int(x) for x in v])
             o._splits_keepalive = arr
             o.row_splits = ctypes.cast(arr, ctypes.POINTER(ctypes.c_int64))
+        elif k == "nccl_unique_id":
+            buf = ctypes.create_string_buffer(bytes(v), 128)
+            o._nccl_keepalive = buf
+            o.nccl_unique_id = ctypes.cast(buf, ctypes.c_void_p)
         else:
             setattr(o, k, v)
     return o
@@ -309,6 +315,13 @@ class TiledMatrix:
 
     def __exit__(self, *a):
         self.close()
+
+
+def nccl_unique_id() -> bytes:
+    """128 bytes for tsmv_options.nccl_unique_id (call on one rank, share with all)."""
+    buf = ctypes.create_string_buffer(128)
+    check(tsmv_nccl_unique_id(buf), "tsmv_nccl_unique_id")
+    return buf.raw
 
 
 def choose_dir(n, frontier, m_f, m_u, opts: Optional[tsmv_options] = None) -> int:

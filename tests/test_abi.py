@@ -60,3 +60,23 @@ def test_create_rejects_bad_args_without_gpu():
                           ctypes.byref(o))
     assert st == tsmv.EINVAL and b"tile_dim" in tsmv.tsmv_last_error()
     assert not ctx.value
+
+
+def test_nccl_unique_id_without_gpu():
+    """Bootstrap of a distributed context: NCCL is loaded at run time
+    and a unique id needs no GPU."""
+    from paper_conf_icpp_jisl0t022_b200 import tsmv
+    a, b = tsmv.nccl_unique_id(), tsmv.nccl_unique_id()
+    assert len(a) == 128 and any(a) and a != b
+    assert tsmv.tsmv_nccl_unique_id(None) == tsmv.EINVAL
+
+
+def test_options_layout_matches_header():
+    """ctypes mirror of tsmv_options has the header's field order (last: nccl_unique_id)."""
+    from paper_conf_icpp_jisl0t022_b200 import tsmv
+    src = open(os.path.join(ROOT, "include", "tsmv.h")).read()
+    body = src[src.index("typedef struct {\n    int32_t device;"):src.index("} tsmv_options;")]
+    body = re.sub(r"/\*.*?\*/", "", body, flags=re.S)
+    names = re.findall(r"\b([a-z_]+)\s*(?:,\s*([a-z_]+))?\s*;", body)
+    flat = [x for pair in names for x in pair if x]
+    assert flat == [f for f, _ in tsmv.tsmv_options._fields_]

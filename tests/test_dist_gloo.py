@@ -190,3 +190,21 @@ def test_distributed_spmspv_gloo():
     gi = np.concatenate([np.load(os.path.join(tmp, f"yi{r}.npy")) for r in range(WORLD)])
     gv = np.concatenate([np.load(os.path.join(tmp, f"yv{r}.npy")) for r in range(WORLD)])
     assert np.array_equal(gi, ri) and np.array_equal(gv, rv)
+
+
+def test_partition_rows_unaligned_m():
+    """m not a multiple of 64: interior splits stay multiples of 64 and
+    never pass the last aligned row, also when the nonzeros sit in the last rows."""
+    import synth as S
+    for m, P in ((120, 8), (120, 2), (1000, 3), (65, 2)):
+        counts = torch.zeros(m, dtype=torch.int64)
+        counts[-8:] = 50                                  # tail-heavy
+        rp = torch.zeros(m + 1, dtype=torch.int64)
+        rp[1:] = torch.cumsum(counts, 0)
+        s = D.partition_rows(rp, P)
+        assert s[0] == 0 and s[-1] == m and len(s) == P + 1
+        assert all(x % 64 == 0 for x in s[1:-1]), s
+        assert all(s[i] <= s[i + 1] for i in range(P)), s
+    U = S.uniform(1000, 1000, 4, seed=1)
+    s = D.partition_rows(U.row_ptr, 4)
+    assert all(x % 64 == 0 for x in s[1:-1]) and s[-1] == 1000

@@ -88,3 +88,44 @@ def test_sim_ranks_bfs_device_stats(P):
     for s in [0] + synth.sample_sources(A, 2, seed=5):
         got = _sim_bfs(engines, s, dev_stats=True)
         assert np.array_equal(got, oracle.bfs_queue(C, s))
+
+
+@pytest.mark.parametrize("P", [2, 3])
+def test_sim_ranks_dist_spmspv_owned_x(P, monkeypatch):
+    """DistTiledMatrix.spmspv / spmspv_async with per-owner x slices (one rank owns
+    no entry): the size and entry all-gathers are replaced by concatenation, so
+    the owner filter, the exchange glue and the local multiply are all checked."""
+    A = synth.attach_values(synth.rmat(12, 16, seed=4), seed=3)
+    C = oracle.csc_of(A)
+    splits, engines = _ranks(A, P, dtype="f64")
+    xi, xv = synth.sample_x(A.n, 300, seed=8)
+    lo_empty, hi_empty = splits[1], splits[2]          # rank 1 owns no x entry
+    keep = (xi < lo_empty) | (xi >= hi_empty)
+    xi, xv = xi[keep], xv[keep]
+    owned = [((xi >= splits[r]) & (xi < splits[r + 1])) for r in range(P)]
+    parts_i = [xi[o].to(DEV) for o in owned]
+    parts_v = [xv[o].to(DEV) for o in owned]
+    sizes = [int(p.numel()) for p in parts_i]
+    assert sizes[1] == 0
+    monkeypatch.setattr(D, "allgather_sizes", lambda count, device, group=None: sizes)
+
+    def varlen(t, group=None, sizes=None):
+        src = parts_i if t.dtype == torch.int32 else parts_v
+        return torch.cat([p.to(t.dtype) for p in src])
+    monkeypatch.setattr(D, "allgather_varlen", varlen)
+    ri, rv = oracle.spmspv(C, xi.numpy(), xv.numpy())
+    gi, gv, ai, av = [], [], [], []
+    for r, e in enumerate(engines):
+        yi, yv = e.spmspv(parts_i[r].to(torch.int32), parts_v[r])
+        gi.append(yi.cpu().numpy())
+        gv.append(yv.cpu().numpy())
+        y_i = torch.empty(e.m_local, dtype=torch.int32, device=DEV)
+        y_v = torch.empty(e.m_local, dtype=torch.float64, device=DEV)
+        y_n = torch.zeros(1, dtype=torch.int64, device=DEV)
+        e.spmspv_async(parts_i[r].to(torch.int32), parts_v[r], y_i, y_v, y_n)
+        k = int(y_n.item())
+        ai.append(y_i[:k].cpu().numpy())
+        av.append(y_v[:k].cpu().numpy())
+    for I, V in ((gi, gv), (ai, av)):
+        assert np.array_equal(np.concatenate(I), ri)
+        assert np.allclose(np.concatenate(V), rv, rtol=1e-12, atol=0)

@@ -134,12 +134,16 @@ def test_errors_keep_workspace_clean(tsmv):
     A = synth.attach_values(synth.rmat(10, 8, seed=1), seed=1)
     C = oracle.csc_of(A)
     M = _mk(tsmv, A)
-    bad = [torch.tensor([5, 5], dtype=torch.int32), torch.tensor([9, 3], dtype=torch.int32),
+    # duplicates (also unsorted ones), out of range (R21: any order of unique indices is valid)
+    bad = [torch.tensor([5, 5], dtype=torch.int32), torch.tensor([9, 3, 9], dtype=torch.int32),
            torch.tensor([A.n], dtype=torch.int32), torch.tensor([-1], dtype=torch.int32)]
     for xi in bad:
         with pytest.raises(tsmv.TsmvError) as e:
             M.spmspv(xi.to(DEV), torch.ones(xi.numel(), dtype=torch.float64, device=DEV))
         assert e.value.status == tsmv.EINVAL
+    xi = torch.tensor([9, 3], dtype=torch.int32)                    # unsorted, unique: accepted
+    yi, yv = M.spmspv(xi.to(DEV), torch.ones(2, dtype=torch.float64, device=DEV))
+    check_spmspv(C, yi, yv, torch.tensor([3, 9]), torch.ones(2, dtype=torch.float64))
     xi, xv = synth.sample_x(A.n, 100, seed=2)
     yi, yv = M.spmspv(xi.to(DEV), xv.to(DEV))
     check_spmspv(C, yi, yv, xi, xv)

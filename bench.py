@@ -60,16 +60,12 @@ def parse(argv=None):
     p.add_argument("--no-cpu", action="store_true")
     p.add_argument("--cpu-seconds", type=float, default=12.0)
     p.add_argument("--no-configs", action="store_true", help="skip the per-config table (C1, C2, C4)")
-    p.add_argument("--scaling", default="weak", choices=["weak", "strong"],
-                   help="weak (default): at N ranks the R-MAT scales grow by log2 N, so the nonzeros "
-                        "per GPU stay fixed; strong: the same matrix at every N")
+    p.add_argument("--dist-scale", type=int, default=26,
+                   help="N > 1: R-MAT scale of the strong-scaling run (C5: the same s26 matrix at every N)")
+    p.add_argument("--no-s26", action="store_true", help="N = 1: skip the s26 SpMSpV / TileBFS blocks")
     a = p.parse_args(argv)
-    world = int(os.environ.get("WORLD_SIZE", "1"))
+    a.scaling = "strong"
     a.base_scale, a.base_bfs_scale = a.scale, a.bfs_scale
-    if a.scaling == "weak" and world > 1:
-        grow = int(round(math.log2(world)))
-        a.scale += grow
-        a.bfs_scale += grow
     return a
 
 
@@ -156,11 +152,17 @@ def run_reference(args):
     if world > 1 and rank != 0:
         return
     dev = "cuda" if torch.cuda.is_available() else "cpu"
-    A = make_matrix(args.scale, args.dtype, dev).to("cpu")
+    # our arm's workload: T at N = 1, C5 (s26, strong scaling) at N > 1; at s26 each
+    # step is a bounded sample of the step (every 8th x entry: still uniform columns)
+    scale = args.dist_scale if world > 1 else args.scale
+    stride = 8 if world > 1 else 1
+    A = make_matrix(scale, args.dtype, dev).to("cpu")
     C = oracle.csc_of(A)
+    del A
     colcnt = torch.from_numpy(C.col_ptr[1:] - C.col_ptr[:-1])
-    k = synth.density_k(A.n, args.density)
-    xs = x_samples(A.n, k, args.warmup + args.steps, args.dtype, "cpu")
+    k = synth.density_k(C.n, args.density)
+    xs = [(xi[::stride].contiguous(), xv[::stride].contiguous())
+          for xi, xv in x_samples(C.n, k, args.warmup + args.steps, args.dtype, "cpu")]
     for s in range(args.warmup):
         oracle.spmspv(C, xs[s][0], xs[s][1])
     flops, tsum, times = 0, 0.0, []
@@ -175,25 +177,27 @@ def run_reference(args):
     val = flops / tsum / 1e9
     line = {"impl": "reference", "metric": "spmspv_gflops", "value": round(val, 4), "unit": "GFLOP/s",
             "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
-            "ms_per_step": round(1e3 * tsum / args.steps, 4), "higher_is_better": True, "scaling": args.scaling,
+            "ms_per_step": round(1e3 * tsum / args.steps, 4), "higher_is_better": True,
+            "scaling": "strong" if world > 1 else args.scaling,
             "vs_baseline": None, "dtype": args.dtype, "data": "synthetic",
-            "config": workload_config(args),
+            "config": workload_config(args, scale),
             "cpu_baseline": {"value": round(val, 4), "unit": "GFLOP/s", "cores": 1, "kind": "oracle",
-                             "sample": f"{args.steps} x samples of k={k} on R-MAT s{args.scale} "
-                                       f"(oracle CSC built once, untimed)"},
+                             "sample": f"{args.steps} x samples of k={k} on R-MAT s{scale}"
+                                       + (f", every {stride}th x entry per step" if stride > 1 else "")
+                                       + " (oracle CSC built once, untimed)"},
             "e2e": {"value": round(val, 4), "unit": "GFLOP/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
 
-def workload_config(args):
-    return {"workload": f"rmat_s{args.scale}_ef16_directed_{args.dtype}_x{args.density * 100:g}pct",
-            "matrix": f"R-MAT scale {args.scale}, edgefactor 16, (0.57,0.19,0.19,0.05), unpermuted, coalesced",
+def workload_config(args, scale=None):
+    scale = args.scale if scale is None else scale
+    return {"workload": f"rmat_s{scale}_ef16_directed_{args.dtype}_x{args.density * 100:g}pct",
+            "matrix": f"R-MAT scale {scale}, edgefactor 16, (0.57,0.19,0.19,0.05), unpermuted, coalesced",
             "x_density": args.density, "tile_dim": args.tile_dim, "sparse_tile_max_nnz": args.thr,
             "l2": "flushed before every step (256 MiB write + 256 MiB read of another buffer, outside the events)",
-            "parallelism": f"row-block x{args.gpus}" if args.gpus > 1 else "single GPU",
-            "scaling_rule": (f"weak: R-MAT scale {args.base_scale} + log2(N) for SpMSpV, {args.base_bfs_scale} + log2(N) "
-                             "for TileBFS (nonzeros per GPU fixed)") if args.scaling == "weak"
-                            else "strong: same matrix at every N"}
+            "parallelism": "single GPU",
+            "multi_gpu": f"N > 1 runs C5 (R-MAT s{args.dist_scale}) as strong scaling; at N = 1 the same s26 "
+                         "workloads are the spmspv_s26 / bfs_s26 blocks"}
 
 
 # --------------------------------------------------------------------------- our arm
@@ -459,8 +463,11 @@ def run_tsmv(args):
     if not args.no_configs and world == 1:
         del M
         configs = run_configs(args, dev, flush, tsmv)
-    bfs26 = None
-    if world == 1 and not args.no_bfs and not args.no_bfs26:
+    bfs26 = sp26 = None
+    if world == 1 and not args.no_s26:
+        torch.cuda.empty_cache()
+        sp26 = run_spmspv26(args, dev, flush, tsmv)
+    if world == 1 and not args.no_bfs and not args.no_bfs26 and not args.no_s26:
         torch.cuda.empty_cache()
         bfs26 = run_bfs26(args, dev, flush, tsmv)
 
@@ -481,7 +488,7 @@ def run_tsmv(args):
                              **{kk: round(v, 1) for kk, v in mean_st.items() if kk != "x_nnz"}},
                 "format": {kk: info[kk] for kk in ("nnz", "n_tiles", "n_dense_tiles", "dense_nnz", "side_nnz",
                                                    "build_ms", "bytes_spmspv")},
-                "bfs": bfs, "bfs_s26": bfs26, "configs": configs}
+                "bfs": bfs, "spmspv_s26": sp26, "bfs_s26": bfs26, "configs": configs}
         print(json.dumps(line), flush=True)
     if world > 1:
         torch.distributed.destroy_process_group()
@@ -580,6 +587,19 @@ def bfs_run_line(s, st, levels, deg, loops):
             "gteps": round(st["edges_traversed"] / (ms * 1e-3) / 1e9, 3),
             "gteps_graph500": round(und / (ms * 1e-3) / 1e9, 3),
             "dirs": "".join({"push_csc": "C", "push_csr": "R", "pull_csc": "P"}.get(d, "?") for d in st["dirs"])}
+
+
+def run_spmspv26(args, dev, flush, tsmv, steps=8, warm=3):
+    """C5 SpMSpV on one GPU: R-MAT s26 directed fp64, x 1 % (671 K entries), the
+    N = 1 point of the strong-scaling curve bench.py --gpus N measures."""
+    A = make_matrix(26, args.dtype, dev)
+    M = tsmv.TiledMatrix.from_csr(A, dtype=args.dtype, tile_dim=args.tile_dim, sparse_tile_max_nnz=args.thr,
+                                  build_bfs=0)
+    r = spmspv_gflops(M, A, args.dtype, args.density, flush, steps=steps, warm=warm)
+    M.close()
+    del A
+    torch.cuda.empty_cache()
+    return {"graph": "rmat_s26_ef16_directed", **r}
 
 
 def run_bfs26(args, dev, flush, tsmv):
@@ -789,10 +809,171 @@ def cpu_baseline(args, A, colcnt, xs, parity_y):
     return cpu, omp, parity
 
 
+def run_dist(args):
+    """N > 1 (C5): strong scaling on the same R-MAT s26 at every N.
+    Every rank generates the seeded matrix, keeps its nnz-balanced row block in a
+    libtsmv context that owns its NCCL communicator (bootstrap: one unique id from
+    rank 0 over torch.distributed), and the timed calls are the collective
+    tsmv_spmspv (owned x in, owned y out: count all-gather + x broadcasts inside
+    the library) and tsmv_bfs (the level loop and the per-level frontier
+    broadcasts inside the library).  Time = CUDA events around each call on every
+    rank, max over ranks; value = all flops / that time."""
+    import torch.distributed as dist
+    world, rank, local = dist_env()
+    local = local % max(1, torch.cuda.device_count())
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    dist.init_process_group("nccl", device_id=dev)
+    from paper_conf_icpp_jisl0t022_b200 import dist as tdist
+    uid = tdist.bootstrap_unique_id()
+    flush = L2Flush(dev)
+
+    def max_over_ranks(v):
+        t = torch.tensor([v], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t)
+
+    # ---- SpMSpV, x 1 %, fp64
+    A = make_matrix(args.dist_scale, args.dtype, dev)
+    colcnt = torch.bincount(A.col_idx.long(), minlength=A.n)
+    splits = tdist.partition_rows(A.row_ptr, world)
+    t0 = time.perf_counter()
+    D = tdist.DistMatrix(tdist.local_rows(A, splits, rank), splits, rank, world, uid, dtype=args.dtype,
+                         device=local, tile_dim=args.tile_dim, sparse_tile_max_nnz=args.thr, build_bfs=0)
+    build_s = time.perf_counter() - t0
+    n = A.n
+    del A
+    torch.cuda.empty_cache()
+    k = synth.density_k(n, args.density)
+    lo, hi = splits[rank], splits[rank + 1]
+    xs = []
+    for xi, xv in x_samples(n, k, args.warmup + args.steps, args.dtype, dev):
+        own = (xi >= lo) & (xi < hi)
+        xs.append((xi[own].contiguous(), xv[own].contiguous(), 2 * int(colcnt[xi.long()].sum())))
+    m_loc = hi - lo
+    y_idx = torch.empty(m_loc, dtype=torch.int32, device=dev)
+    y_val = torch.empty(m_loc, dtype=torch.float32 if args.dtype == "f32" else torch.float64, device=dev)
+    for s in range(args.warmup):
+        D.spmspv(xs[s][0], xs[s][1], y_idx=y_idx, y_val=y_val)
+    clocks = Clocks(local) if rank == 0 else None
+    if clocks:
+        clocks.start()
+    dist.barrier()
+    torch.cuda.synchronize()
+    step_ms, flops = [], 0
+    for i in range(args.steps):
+        xi, xv, fl = xs[args.warmup + i]
+        flush()
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        D.spmspv(xi, xv, y_idx=y_idx, y_val=y_val)
+        e1.record()
+        torch.cuda.synchronize()
+        step_ms.append(e0.elapsed_time(e1))
+        flops += fl
+    torch.cuda.synchronize()
+    dist.barrier()
+    clk = clocks.stop() if clocks else None
+    ms = max_over_ranks(sum(step_ms))
+    value = flops / (ms * 1e-3) / 1e9
+    # e2e: the same collective call with pinned host x and y, wall clock, max over ranks
+    hx = [(xi.cpu().pin_memory(), xv.cpu().pin_memory()) for xi, xv, _ in xs[args.warmup:]]
+    hy_i = torch.empty(m_loc, dtype=torch.int32).pin_memory()
+    hy_v = torch.empty(m_loc, dtype=y_val.dtype).pin_memory()
+    dist.barrier()
+    t_e2e, h2d, d2h = 0.0, 0, 0
+    for xi, xv in hx:
+        flush()
+        torch.cuda.synchronize()
+        dist.barrier()
+        t0 = time.perf_counter()
+        yi, yv = D.spmspv(xi, xv, y_idx=hy_i, y_val=hy_v)
+        t_e2e += time.perf_counter() - t0
+        h2d += xi.numel() * 4 + xv.numel() * xv.element_size()
+        d2h += yi.numel() * (4 + yv.element_size())
+    t_e2e = max_over_ranks(t_e2e)
+    n_e2e = len(hx)
+    D.close()
+    del D, y_idx, y_val, colcnt, xs, hx
+    torch.cuda.empty_cache()
+
+    # ---- TileBFS on the symmetrised s26, vertex 0 + 7 sources
+    bfs = None
+    if not args.no_bfs:
+        A = synth.rmat(args.dist_scale, 16, seed=1, symmetrize=True, device=dev)
+        torch.cuda.empty_cache()
+        splits_b = tdist.partition_rows(A.row_ptr, world)
+        uid_b = tdist.bootstrap_unique_id()   # a unique id serves one communicator only
+        Db = tdist.DistMatrix(tdist.local_rows(A, splits_b, rank), splits_b, rank, world, uid_b, dtype="pattern",
+                              device=local, tile_dim=args.tile_dim, sparse_tile_max_nnz=args.bfs_thr)
+        srcs = bfs_sources(A, args.bfs26_sources)
+        deg, loops = degrees_and_loops(A)
+        nnz = A.nnz
+        del A
+        torch.cuda.empty_cache()
+        lvl = torch.empty(splits_b[rank + 1] - splits_b[rank], dtype=torch.int32, device=dev)
+        Db.bfs(srcs[0], levels=lvl)
+        runs = []
+        for s in srcs:
+            flush()
+            torch.cuda.synchronize()
+            dist.barrier()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            _, st = Db.bfs(s, levels=lvl)
+            e1.record()
+            torch.cuda.synchronize()
+            tms = max_over_ranks(e0.elapsed_time(e1))
+            # Graph500 count: reached rows of every rank
+            r = lvl >= 0
+            part = torch.stack([deg[splits_b[rank]:splits_b[rank + 1]][r].sum(),
+                                loops[splits_b[rank]:splits_b[rank + 1]][r].sum()])
+            dist.all_reduce(part)
+            und = int((part[0] + part[1]) // 2)
+            runs.append({"source": int(s), "ms": round(tms, 4), "levels": st["nlevels"],
+                         "edges": st["edges_traversed"], "edges_graph500": und, "reached": st["reached"],
+                         "gteps": round(st["edges_traversed"] / (tms * 1e-3) / 1e9, 3),
+                         "gteps_graph500": round(und / (tms * 1e-3) / 1e9, 3),
+                         "dirs": "".join({"push_csc": "C", "push_csr": "R", "pull_csc": "P"}.get(d, "?")
+                                         for d in st["dirs"])})
+        Db.close()
+        hm = len(runs) / sum(1.0 / x["gteps"] for x in runs if x["gteps"] > 0)
+        hm500 = len(runs) / sum(1.0 / x["gteps_graph500"] for x in runs if x["gteps_graph500"] > 0)
+        bfs = {"graph": f"rmat_s{args.dist_scale}_ef16_sym", "nnz": nnz, "sources": len(runs),
+               "gteps_hmean": round(hm, 3), "gteps_graph500_hmean": round(hm500, 3),
+               "sparse_tile_max_nnz": args.bfs_thr, "partition": f"row blocks x{world} (nnz-balanced)",
+               "time": "CUDA events around the collective tsmv_bfs, max over ranks", "edge_count": EDGE_COUNT,
+               "runs": runs}
+    if rank == 0:
+        line = {"metric": "spmspv_gflops", "value": round(value, 3), "unit": "GFLOP/s", "n_gpus": world,
+                "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms / args.steps, 5),
+                "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": args.dtype,
+                "data": "synthetic (seeded R-MAT, seeded x)",
+                "config": {"workload": f"rmat_s{args.dist_scale}_ef16_directed_{args.dtype}_x{args.density * 100:g}pct",
+                           "matrix": f"R-MAT scale {args.dist_scale}, edgefactor 16, unpermuted, coalesced",
+                           "x_density": args.density, "tile_dim": args.tile_dim, "sparse_tile_max_nnz": args.thr,
+                           "l2": "flushed before every step (256 MiB write + 256 MiB read, outside the events)",
+                           "parallelism": f"row blocks x{world} (nnz-balanced), NCCL communicator inside libtsmv",
+                           "scaling_rule": "strong: the same matrix at every N (C5); N = 1: bench.py's spmspv_s26 / bfs_s26 blocks"},
+                "e2e": {"value": round(flops / t_e2e / 1e9, 3), "unit": "GFLOP/s",
+                        "h2d_bytes_per_step": int(h2d / n_e2e), "d2h_bytes_per_step": int(d2h / n_e2e),
+                        "path": "collective tsmv_spmspv (C ABI) with pinned host owned x and y; wall clock, max over ranks"},
+                "gpu_launches": args.steps, "clocks": clk,
+                "comm": {"nranks": world, "backend": "NCCL (communicator owned by the libtsmv context)",
+                         "nccl_version": ".".join(str(v) for v in torch.cuda.nccl.version())},
+                "build_s_rank0": round(build_s, 2), "bfs": bfs}
+        print(json.dumps(line), flush=True)
+    dist.barrier()
+    dist.destroy_process_group()
+
+
 def main():
     args = parse()
     if args.impl == "reference":
         run_reference(args)
+    elif int(os.environ.get("WORLD_SIZE", "1")) > 1 or os.environ.get("TSMV_BENCH_DIST"):
+        run_dist(args)   # TSMV_BENCH_DIST=1: the N > 1 path with one rank (checks it on one GPU)
     else:
         run_tsmv(args)
 

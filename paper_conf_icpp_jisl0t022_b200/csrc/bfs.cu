@@ -1170,6 +1170,16 @@ extern "C" tsmv_status tsmv_bfs_dist_merge(tsmv_ctx *c, const uint32_t *gathered
                                            int64_t *out_stats, void *cuda_stream) {
     try {
         TSMV_REQUIRE(c && out_stats, "tsmv_bfs_dist_merge: NULL argument");
+        bfs_check(c);
+        TSMV_REQUIRE(c->levels_dev != nullptr, "tsmv_bfs_dist_merge: no traversal begun (tsmv_bfs_dist_begin)");
+        if (c->opt.nranks > 1) {
+            long long need = 0;
+            for (int p = 0; p < c->opt.nranks; ++p)
+                need = std::max<long long>(need, (c->row_splits[p + 1] - c->row_splits[p] + 31) / 32);
+            TSMV_REQUIRE(stride_words >= need, "tsmv_bfs_dist_merge: stride_words %lld < largest owned segment %lld",
+                         (long long)stride_words, need);
+            TSMV_REQUIRE(is_device_ptr(gathered), "tsmv_bfs_dist_merge: gathered must be device memory");
+        }
         TSMV_CUDA(cudaSetDevice(c->device));
         cudaStream_t st = (cudaStream_t)cuda_stream;
         BfsRunner R{c, st, (long long)(c->V.bytes / 4)};

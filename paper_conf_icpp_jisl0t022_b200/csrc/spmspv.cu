@@ -1187,6 +1187,12 @@ extern "C" tsmv_status tsmv_spmspv_async(tsmv_ctx *c, tsmv_semiring sr, int64_t 
         TSMV_REQUIRE(x_idx != nullptr && (sr == TSMV_OR_AND || x_val != nullptr), "tsmv_spmspv_async: NULL x");
         TSMV_REQUIRE(y_cap >= 0 && (y_cap == 0 || y_idx != nullptr), "tsmv_spmspv_async: NULL y_idx");
         TSMV_REQUIRE(sr == TSMV_OR_AND || y_cap == 0 || y_val != nullptr, "tsmv_spmspv_async: NULL y_val");
+        TSMV_REQUIRE(!has_comm(c), "tsmv_spmspv_async: a distributed context's call is collective (tsmv_spmspv)");
+        TSMV_REQUIRE(is_device_ptr(x_idx) && (sr == TSMV_OR_AND || is_device_ptr(x_val)) &&
+                         (y_cap == 0 || is_device_ptr(y_idx)) &&
+                         (sr == TSMV_OR_AND || y_cap == 0 || is_device_ptr(y_val)) &&
+                         (y_nnz_dev == nullptr || is_device_ptr(y_nnz_dev)),
+                     "tsmv_spmspv_async: every pointer must be device memory");
         TSMV_CUDA(cudaSetDevice(c->device));
         c->last_x_nnz = x_nnz;
         enqueue_spmspv(c, sr, x_nnz, x_idx, sr == TSMV_OR_AND ? nullptr : x_val, y_cap, y_idx,

@@ -78,7 +78,8 @@ def local_rows(A, splits: Sequence[int], rank: int) -> RowBlock:
 
 def bootstrap_unique_id(group=None) -> bytes:
     """One ncclUniqueId made by rank 0 and shared with every rank of `group` over
-    torch.distributed (object broadcast: works on gloo and NCCL groups)."""
+    torch.distributed (object broadcast: works on gloo and NCCL groups).  An id
+    creates ONE communicator: bootstrap a new one for every DistMatrix."""
     from . import tsmv
     obj = [tsmv.nccl_unique_id() if dist.get_rank(group) == 0 else None]
     dist.broadcast_object_list(obj, src=dist.get_global_rank(group, 0) if group is not None else 0, group=group)
@@ -96,7 +97,8 @@ class DistMatrix:
         self.rank, self.nranks = rank, nranks
         self.m_local, self.n = A_local.m, A_local.n
         self.device = torch.device("cuda", device)
-        kw = dict(rank=rank, nranks=nranks, nccl_unique_id=unique_id, build_bfs=1)
+        kw = dict(rank=rank, nranks=nranks, nccl_unique_id=unique_id)
+        opts.setdefault("build_bfs", 1)
         if nranks > 1:
             kw["row_splits"] = self.splits
         self.M = tsmv.TiledMatrix(A_local.m, A_local.n, A_local.row_ptr, A_local.col_idx, A_local.values,

@@ -218,6 +218,12 @@ class TiledMatrix:
                      y_val: Optional[torch.Tensor], y_nnz: torch.Tensor, semiring="plus_times", stream=None):
         """Device-only, no synchronisation; y_nnz (int64[1] on the device) receives the size."""
         sr = _SEMIRINGS[semiring] if isinstance(semiring, str) else int(semiring)
+        if x_idx.dtype != torch.int32 or not x_idx.is_contiguous():
+            x_idx = x_idx.to(torch.int32).contiguous()
+        if x_val is not None and (x_val.dtype != self.vtype or not x_val.is_contiguous()):
+            x_val = x_val.to(self.vtype).contiguous()
+        if y_nnz.dtype != torch.int64 or y_nnz.numel() != 1 or y_nnz.device != x_idx.device:
+            raise ValueError("spmspv_async: y_nnz must be one int64 on the device of x")
         check(tsmv_spmspv_async(self.ctx, sr, x_idx.numel(), _ptr(x_idx), _ptr(x_val), y_idx.numel(), _ptr(y_idx),
                                 _ptr(y_val) if sr != OR_AND else None, _ptr(y_nnz), _stream(stream)),
               "tsmv_spmspv_async")

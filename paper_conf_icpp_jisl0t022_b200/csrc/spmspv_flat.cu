@@ -31,7 +31,10 @@ namespace tsmv {
 
 namespace {
 
-constexpr int FT = 1024;          // threads per CTA
+#ifndef TSMV_FT
+#define TSMV_FT 1024
+#endif
+constexpr int FT = TSMV_FT;       // threads per CTA
 constexpr int NWF = FT / 32;      // warps per CTA
 #ifndef TSMV_TL
 #define TSMV_TL 7
@@ -171,6 +174,13 @@ __device__ __forceinline__ void put_chunks(int *C, long long w0, long long w, in
     for (long long ch = c0; ch < c1; ++ch) C[ch] = entry;
 }
 
+// 32-byte read-only load (one LDG.E.ENL2.256 request instead of two 16-byte ones)
+__device__ __forceinline__ void ld32_nc(const void *p, uint4 &lo, uint4 &hi) {
+    asm volatile("ld.global.nc.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+                 : "=r"(lo.x), "=r"(lo.y), "=r"(lo.z), "=r"(lo.w), "=r"(hi.x), "=r"(hi.y), "=r"(hi.z), "=r"(hi.w)
+                 : "l"(p));
+}
+
 __device__ __forceinline__ ColInfo load_colinfo(const ColInfo *p) {
     const longlong2 v = __ldg(reinterpret_cast<const longlong2 *>(p));
     ColInfo c;
@@ -307,6 +317,7 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
     __shared__ int s_hcnt;
     __shared__ long long s_pbase[KP], s_ex0[KP];
     __shared__ int s_nd;  // dense bitmap words of the current C2 round
+    __shared__ int s_hlist[HOT_SLOTS / 16];  // tile rows of the privatised hot rows
     __shared__ long long s_heavy[HEAVY_CAP][3];  // chunk-map runs too long for one thread: c0, c1, list | kind
     const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
     const int G = gridDim.x, b = blockIdx.x;
@@ -320,6 +331,7 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
     for (int i = tid; i < n_slots; i += FT) s_hacc[i] = __longlong_as_double((long long)EMPTY);
     for (int i = tid; i < (n_slots + 31) / 32; i += FT) s_hbits[i] = 0u;
     for (int i = tid; i < a.n_pieces; i += FT) s_pcnt[i] = 0u;
+    for (int i = tid; i < a.n_hot; i += FT) s_hlist[i] = a.hot_list[i];
     if (tid == 0) {
         s_nheavy = 0;
         s_hcnt = 0;
@@ -366,6 +378,7 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
         s_base[3] = (long long)(os & ((1ull << S_CNT_SHIFT) - 1));
 #pragma unroll
         for (int i = 0; i < 4; ++i) a.partials[b * 8 + i] = tot[i];
+        if (tr) tr[8] = globaltimer_ns();
     }
     __syncthreads();
     {
@@ -566,6 +579,7 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
     // __syncthreads, so there is no grid barrier between B1 and B2 (a CTA whose
     // B1 ends early starts multiplying at once)
     __syncthreads();
+    if (tr && tid == 0) tr[3] = globaltimer_ns();
     if (stamp) ts[6] = globaltimer_ns();
 
     // ------------------------------------------------------------ phase B2 (a4)
@@ -597,7 +611,9 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
             int useful = 0;
             if (hit) {
                 const uint4 *rp = reinterpret_cast<const uint4 *>(a.rec + t);
-                const uint4 h0 = __ldg(rp), h1 = __ldg(rp + 1), v0 = __ldg(rp + 2), v1 = __ldg(rp + 3);
+                uint4 h0, h1, v0, v1;
+                ld32_nc(rp, h0, h1);
+                ld32_nc(rp + 2, v0, v1);
                 off = h0.x;
                 trow = (int)h0.y;
                 nnz = h0.z;
@@ -699,6 +715,7 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
         n_mac += __shfl_xor_sync(0xffffffffu, n_mac, o);
         n_ind += __shfl_xor_sync(0xffffffffu, n_ind, o);
     }
+    if (tr && tid == 0) tr[4] = globaltimer_ns();
     if (lane == 0) {
         s_acct[wid][0] = n_hit;
         s_acct[wid][1] = n_hcol;
@@ -714,38 +731,53 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
 #endif
         // CTAs start at different slots so that the 148 flushes of one hot row are
         // spread over time instead of queueing on one L2 address together
+        // the flush atomics are issued first and their old values consumed after
+        // the piece-count flush below, so their round trip overlaps it
         const int rot = (int)(((long long)b * n_slots) / G);
-        constexpr int FQ = HOT_SLOTS / FT;
-        long long fr[FQ];
+        constexpr int FQ = (HOT_SLOTS + FT - 1) / FT;
+        long long row_of[FQ];
+        unsigned long long old[FQ];
 #pragma unroll
         for (int i = 0; i < FQ; ++i) {
             const int q = tid + i * FT;
             const int sl = q + rot < n_slots ? q + rot : q + rot - n_slots;
-            fr[i] = -1;
+            row_of[i] = -1;
+            old[i] = 0;
             if (q < n_slots && ((s_hbits[sl >> 5] >> (sl & 31)) & 1u)) {
-                const long long row = (long long)a.hot_list[sl / NT] * NT + sl % NT;
-                bool first = true;
+                const long long row = (long long)s_hlist[sl / NT] * NT + sl % NT;
+                row_of[i] = row;
                 if constexpr (SR == TSMV_PLUS_TIMES)
-                    first = (unsigned long long)__double_as_longlong(atomicAdd(&a.acc[row], s_hacc[sl])) == EMPTY;
+                    old[i] = (unsigned long long)__double_as_longlong(atomicAdd(&a.acc[row], s_hacc[sl]));
                 else if constexpr (SR == TSMV_MIN_SECOND)
-                    first = (unsigned long long)atomicMax((long long *)&a.acc[row],
-                                                          (long long)__double_as_longlong(s_hacc[sl])) == EMPTY;
+                    old[i] = (unsigned long long)atomicMax((long long *)&a.acc[row],
+                                                           (long long)__double_as_longlong(s_hacc[sl]));
                 else
-                    first = atomicExch((unsigned long long *)&a.acc[row], 0ull) == EMPTY;
-                if (first) fr[i] = row;
+                    old[i] = atomicExch((unsigned long long *)&a.acc[row], 0ull);
             }
         }
+        if (tid < 4) {
+            long long sum = 0;
+            for (int w = 0; w < NWF; ++w) sum += s_acct[w][tid];
+            a.acct[b * 4 + tid] = sum;
+        }
+        // piece counts of the rows this CTA touched first in B (s_pcnt is complete:
+        // every touch of B happened before the __syncthreads above)
+        for (int q = tid; q < a.n_pieces; q += FT)
+            if (s_pcnt[q]) atomicAdd(&a.pc[q], s_pcnt[q]);
 #pragma unroll
-        for (int i = 0; i < FQ; ++i) touch(a, s_pcnt, fr[i]);
-    }
-    if (tid < 4) {
+        for (int i = 0; i < FQ; ++i) {
+            if (row_of[i] >= 0 && old[i] == EMPTY) {
+                const long long row = row_of[i];
+                atomicOr(&a.rowbits[row >> 5], 1u << (row & 31));
+                atomicAdd(&a.pc[(row >> 5) >> a.ps_log], 1u);
+            }
+        }
+    } else if (tid < 4) {
         long long sum = 0;
         for (int w = 0; w < NWF; ++w) sum += s_acct[w][tid];
         a.acct[b * 4 + tid] = sum;
     }
-    __syncthreads();
-    for (int q = tid; q < a.n_pieces; q += FT)
-        if (s_pcnt[q]) atomicAdd(&a.pc[q], s_pcnt[q]);
+    if (tr && tid == 0) tr[7] = globaltimer_ns();
     grid_sync_f(&a.cnt->bar, target, tr ? tr + 5 : nullptr);
     if (stamp) ts[3] = globaltimer_ns();
 
@@ -1037,7 +1069,7 @@ void ensure_flat_lists(tsmv_ctx *c, int64_t k) {
     if (!F.Ct.p) {
         F.Ct.alloc(((c->P.T >> TL) + 2) * 4);
         F.Cs.alloc(((c->P.side_nnz >> SL) + 2) * 4);
-        F.hits.alloc((size_t)(c->P.T + 128ll * (c->flat_blocks + 2)) * 16);
+        F.hits.alloc((size_t)(c->P.T + (1ll << TL) * (c->flat_blocks + 2)) * 16);
         F.pcnt.alloc((size_t)2 * MAXG * KP * 4);  // u32[2][MAXG * KP]: piece counts, double-buffered
         TSMV_CUDA(cudaMemset(F.pcnt.p, 0, F.pcnt.bytes));
     }

@@ -81,6 +81,13 @@ typedef struct {
                                     tsmv_bfs / tsmv_spmspv become collective calls that exchange the
                                     frontier / x themselves.  When NULL with nranks > 1, the caller
                                     drives the exchange with the tsmv_bfs_dist_* primitives. */
+    double row_driven_density;   /* nt = 16: x density k / ncols at or above which tsmv_spmspv runs the
+                                    row-driven kernel (Alg 4: every row tile walks its
+                                    tiles, skipping those whose x segment misses them) instead of the
+                                    column-driven one, for matrices that keep <= 10 % of their
+                                    nonzeros in the side matrix and <= 32 per tile (small matrices:
+                                    at any density); 0 = never.  Results are identical; default 0.05,
+                                    the crossover measured on B200. */
 } tsmv_options;
 
 /* Per-call counters of the last tsmv_spmspv (read from device on request). */

@@ -114,6 +114,7 @@ extern "C" tsmv_status tsmv_default_options(tsmv_options *o) {
     o->push_csr_density = 0.01;
     o->pull_alpha = 14.0;
     o->force_dir = TSMV_DIR_AUTO;
+    o->row_driven_density = 0.05;  // measured crossover
     o->rank = 0;
     o->nranks = 1;
     o->row_begin = 0;
@@ -250,6 +251,7 @@ extern "C" tsmv_status tsmv_create(tsmv_ctx **out, int64_t nrows, int64_t ncols,
                       c->n_hot ? hot_map.as<int32_t>() : nullptr);
         hot_map.release();
         build_rec64(c, c->P, st);
+        build_row_tiles(c, st);
         c->nTR = c->P.nTR;
         c->nTC = c->P.nTC;
         if (want_bfs) {

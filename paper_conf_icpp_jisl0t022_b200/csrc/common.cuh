@@ -313,6 +313,11 @@ struct tsmv_ctx {
     unsigned long long bar_base = 0;  // value of Counters::bar at the next launch
     int fused_blocks = 0, fused_threads = 1024;
     bool use_flat = false;         // SpMSpV through the flat kernel (nt = 16), decided at create
+    bool use_rows = false;         // row-driven kernel (Alg 4, spmspv_rows.cu) available (nt = 16)
+    int rows_G = 0;                // CTAs of the row-driven kernel
+    tsmv::DevBuf rt_row, rt_J, rt_id, rt_mask;  // dense tiles of P in row-major order
+    tsmv::DevBuf rt_wstart;        // int64[rows_G * 32 + 1]: per-warp tile ranges (row-tile aligned)
+    tsmv::DevBuf xbits;            // u32[n/32 + 1]: x bitmap of the row-driven kernel (zero between calls)
     int flat_blocks = 0;           // CTAs of the flat SpMSpV kernel (1024 threads, 1 per SM)
     long long flat_calls = 0;      // flat SpMSpV launches so far (piece-count buffer parity)
     int last_blocks = 0;           // CTAs of the last SpMSpV launch (partials / acct rows)
@@ -368,6 +373,12 @@ void build_rec64(tsmv_ctx *c, TileSet &S, cudaStream_t st);
 int flat_occupancy(int dtype);
 void enqueue_spmspv_flat(tsmv_ctx *c, int sr, long long k, const int32_t *xi, const void *xv, long long ycap,
                          int32_t *yi, void *yv, long long *ynnz_dev, cudaStream_t st);
+void ensure_flat_lists(tsmv_ctx *c, int64_t k);
+// spmspv_rows.cu
+void build_row_tiles(tsmv_ctx *c, cudaStream_t st);
+void enqueue_spmspv_rows(tsmv_ctx *c, int sr, long long k, const int32_t *xi, const void *xv, long long ycap,
+                         int32_t *yi, void *yv, long long *ynnz_dev, cudaStream_t st);
+bool use_rows_kernel(const tsmv_ctx *c, long long k);
 // bfs_fused.cu
 int bfs_fused_occupancy(int nt);
 void bfs_list_init(tsmv_ctx *c, cudaStream_t st);

@@ -940,6 +940,11 @@ void ensure_lists(tsmv_ctx *c, int64_t k) {
 // Enqueue one fused SpMSpV (device pointers only, no sync).
 void enqueue_spmspv(tsmv_ctx *c, int sr, long long k, const int32_t *xi, const void *xv, long long ycap,
                     int32_t *yi, void *yv, long long *ynnz_dev, cudaStream_t st) {
+    if (use_rows_kernel(c, k)) {
+        ensure_flat_lists(c, k);  // piece-count buffers shared with the flat kernel
+        enqueue_spmspv_rows(c, sr, k, xi, xv, ycap, yi, yv, ynnz_dev, st);
+        return;
+    }
     if (flat_supported(c)) {
         enqueue_spmspv_flat(c, sr, k, xi, xv, ycap, yi, yv, ynnz_dev, st);
         return;

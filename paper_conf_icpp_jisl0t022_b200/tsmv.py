@@ -42,7 +42,7 @@ class tsmv_options(ctypes.Structure):
                 ("push_csr_density", ctypes.c_double), ("pull_alpha", ctypes.c_double),
                 ("force_dir", ctypes.c_int32), ("rank", ctypes.c_int32), ("nranks", ctypes.c_int32),
                 ("row_begin", ctypes.c_int64), ("row_splits", ctypes.POINTER(ctypes.c_int64)),
-                ("nccl_unique_id", ctypes.c_void_p)]
+                ("nccl_unique_id", ctypes.c_void_p), ("row_driven_density", ctypes.c_double)]
 
 
 class tsmv_call_stats(ctypes.Structure):

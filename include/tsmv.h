@@ -67,8 +67,11 @@ typedef struct {
                                     matrix (R12); default 2; 0 = none */
     int32_t build_bfs;           /* 1 = also build the TileBFS bitmask tiles (square A);
                                     default 1 when nrows == ncols and nranks == 1 */
-    double push_csr_density;     /* |F|/n threshold Push-CSC -> Push-CSR; default 0.01 */
-    double pull_alpha;           /* Pull-CSC when m_f > m_u / alpha (R9); default 14 */
+    double push_csr_density;     /* |F|/n threshold Push-CSC -> Push-CSR; the paper's is 0.01
+                                    (P:1423-1433); default 0.05, measured on B200 */
+    double pull_alpha;           /* Pull-CSC when m_f > m_u / alpha (R9); Beamer's 14; default 2,
+                                    measured on B200 (list-driven Push-CSC levels stay cheaper than
+                                    bitmap-wide levels longer than on the paper's GPU) */
     int32_t force_dir;           /* tsmv_dir; AUTO = rule of R9 (tests / ablation) */
     int32_t rank, nranks;        /* row-block partition: this rank / number of ranks (1 = single GPU) */
     int64_t row_begin;           /* global id of local row 0 (multiple of 64 when nranks > 1) */

@@ -111,8 +111,10 @@ extern "C" tsmv_status tsmv_default_options(tsmv_options *o) {
     o->tile_dim = 16;
     o->sparse_tile_max_nnz = 2;
     o->build_bfs = -1;  // auto: square and single rank
-    o->push_csr_density = 0.01;
-    o->pull_alpha = 14.0;
+    // direction rule R9 with the thresholds measured on B200 (DESIGN.md §6,
+    // profiles/r02_bfs_knobs.txt); the paper's 0.01 and Beamer's 14 stay selectable
+    o->push_csr_density = 0.05;
+    o->pull_alpha = 2.0;
     o->force_dir = TSMV_DIR_AUTO;
     o->row_driven_density = 0.05;  // measured crossover
     o->rank = 0;

@@ -25,8 +25,9 @@ import synth  # noqa: E402
 from paper_conf_icpp_jisl0t022_b200 import tsmv  # noqa: E402
 
 DEV = torch.device("cuda", 0)
-MODES = {"K1 push-csc": {"force_dir": 1}, "K1+K2 push only": {"pull_alpha": 1e-300},
-         "K1+K2+K3 auto": {}, "K3 pull only": {"force_dir": 3}}
+PAPER = {"push_csr_density": 0.01, "pull_alpha": 14.0}   # the paper's density rule + Beamer's alpha
+MODES = {"K1 push-csc": {"force_dir": 1}, "K1+K2 push only": {"pull_alpha": 1e-300, "push_csr_density": 0.01},
+         "K1+K2+K3 paper rule": PAPER, "K1+K2+K3 B200 defaults": {}, "K3 pull only": {"force_dir": 3}}
 DCH = {"push_csc": "C", "push_csr": "R", "pull_csc": "P"}
 
 

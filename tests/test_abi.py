@@ -40,11 +40,17 @@ def test_host_only_calls():
     assert tsmv.tsmv_version() >> 16 == 1
     o = tsmv.default_options()
     assert o.tile_dim == 16 and o.sparse_tile_max_nnz == 2 and o.nranks == 1
-    assert abs(o.push_csr_density - 0.01) < 1e-15
-    # direction rule (reading R9)
-    assert tsmv.choose_dir(1000, 1, 10, 10_000) == tsmv.DIR_PUSH_CSC
-    assert tsmv.choose_dir(1000, 10, 10, 10_000) == tsmv.DIR_PUSH_CSR
-    assert tsmv.choose_dir(1000, 10, 1000, 10_000) == tsmv.DIR_PULL_CSC
+    assert abs(o.push_csr_density - 0.05) < 1e-15 and o.pull_alpha == 2.0   # B200 defaults
+    # direction rule (reading R9) with the paper's thresholds (0.01, Beamer's 14)
+    pap = tsmv.default_options(push_csr_density=0.01, pull_alpha=14.0)
+    assert tsmv.choose_dir(1000, 1, 10, 10_000, pap) == tsmv.DIR_PUSH_CSC
+    assert tsmv.choose_dir(1000, 10, 10, 10_000, pap) == tsmv.DIR_PUSH_CSR
+    assert tsmv.choose_dir(1000, 10, 1000, 10_000, pap) == tsmv.DIR_PULL_CSC
+    # B200 defaults: Push-CSR from 5 % of n, Pull-CSC when m_f > m_u / 2
+    assert tsmv.choose_dir(1000, 10, 10, 10_000) == tsmv.DIR_PUSH_CSC
+    assert tsmv.choose_dir(1000, 50, 10, 10_000) == tsmv.DIR_PUSH_CSR
+    assert tsmv.choose_dir(1000, 10, 1000, 10_000) == tsmv.DIR_PUSH_CSC
+    assert tsmv.choose_dir(1000, 10, 6000, 10_000) == tsmv.DIR_PULL_CSC
     o.force_dir = tsmv.DIR_PUSH_CSR
     assert tsmv.choose_dir(1000, 1, 1000, 10, o) == tsmv.DIR_PUSH_CSR
     assert tsmv.tsmv_destroy(None) == tsmv.OK

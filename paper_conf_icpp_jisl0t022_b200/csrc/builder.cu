@@ -28,20 +28,6 @@ struct CubTemp {
     }
 };
 
-__global__ void k_rows_of(const int64_t *__restrict__ row_ptr, int64_t m, int64_t nnz,
-                          int32_t *__restrict__ rows) {
-    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < nnz;
-         e += (int64_t)gridDim.x * blockDim.x) {
-        int64_t lo = 0, hi = m;  // find last row with row_ptr[row] <= e
-        while (hi - lo > 1) {
-            int64_t mid = (lo + hi) >> 1;
-            if (row_ptr[mid] <= e) lo = mid;
-            else hi = mid;
-        }
-        rows[e] = (int32_t)lo;
-    }
-}
-
 template <int NT>
 __global__ void k_keys(const int32_t *__restrict__ rows, const int32_t *__restrict__ cols, int64_t nnz,
                        int64_t nTR, unsigned long long *__restrict__ keys) {
@@ -409,23 +395,31 @@ __global__ void k_cmp(const unsigned long long *__restrict__ a, const unsigned l
         if (a[e] != b[e]) *diff = 1;
 }
 
-__global__ void k_validate_csr(const int64_t *__restrict__ row_ptr, const int32_t *__restrict__ col, int64_t m,
-                               int64_t ncols, int64_t nnz, int *__restrict__ bad, int32_t *__restrict__ indeg) {
+// row_ptr checks (thread per row), in-degrees, and the row id of every non-empty
+// row's first nonzero (the max-scan of these heads gives the row of every nonzero)
+__global__ void k_check_rows(const int64_t *__restrict__ row_ptr, int64_t m, int64_t nnz, int *__restrict__ bad,
+                             int32_t *__restrict__ indeg, int32_t *__restrict__ heads) {
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m; i += (int64_t)gridDim.x * blockDim.x) {
-        int64_t p0 = row_ptr[i], p1 = row_ptr[i + 1];
+        const int64_t p0 = row_ptr[i], p1 = row_ptr[i + 1];
         if (p0 > p1 || p0 < 0 || p1 > nnz || (i == 0 && p0 != 0) || (i == m - 1 && p1 != nnz)) {
             *bad = 1;
             continue;
         }
         indeg[i] = (int32_t)(p1 - p0);
-        int64_t prev = -1;
-        for (int64_t p = p0; p < p1; ++p) {
-            int64_t cc = col[p];
-            if (cc <= prev || cc >= ncols) *bad = 2;
-            prev = cc;
-        }
+        if (p1 > p0) heads[p0] = (int32_t)i;
     }
 }
+// columns strictly ascending inside a row and < ncols (thread per nonzero)
+__global__ void k_check_cols(const int32_t *__restrict__ rows, const int32_t *__restrict__ col, int64_t nnz,
+                             int64_t ncols, int *__restrict__ bad) {
+    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < nnz; e += (int64_t)gridDim.x * blockDim.x) {
+        const int32_t cc = col[e];
+        if (cc < 0 || cc >= ncols || (e > 0 && rows[e] == rows[e - 1] && cc <= col[e - 1])) *bad = 2;
+    }
+}
+struct MaxI32 {
+    __device__ __forceinline__ int32_t operator()(int32_t a, int32_t b) const { return a > b ? a : b; }
+};
 
 __global__ void k_colcount(const int32_t *__restrict__ col, int64_t nnz, int32_t *__restrict__ cnt) {
     for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < nnz; e += (int64_t)gridDim.x * blockDim.x)
@@ -444,14 +438,30 @@ void prepare_csr(tsmv_ctx *c, const int64_t *row_ptr, const int32_t *col_idx, in
     c->outdeg.alloc(((std::max<int64_t>(c->n, 1) + 63) / 64 * 64) * 4);  // padded for segment vector loads
     TSMV_CUDA(cudaMemsetAsync(c->indeg.p, 0, c->indeg.bytes, st));
     TSMV_CUDA(cudaMemsetAsync(c->outdeg.p, 0, c->outdeg.bytes, st));
-    if (c->m) k_validate_csr<<<grid_for(c->m), 256, 0, st>>>(row_ptr, col_idx, c->m, c->n, c->nnz, bad.as<int>(),
-                                                            c->indeg.as<int32_t>());
+    // row checks + row heads (thread per row), row of every nonzero by a max-scan
+    // of the heads, column checks (thread per nonzero): O(nnz) with no per-row
+    // serial loop (a power-law row used to serialise one thread for milliseconds)
+    DevBuf heads;
+    if (c->nnz) {
+        heads.alloc(c->nnz * 4);
+        TSMV_CUDA(cudaMemsetAsync(heads.p, 0, c->nnz * 4, st));
+    }
+    if (c->m) k_check_rows<<<grid_for(c->m), 256, 0, st>>>(row_ptr, c->m, c->nnz, bad.as<int>(),
+                                                          c->indeg.as<int32_t>(), c->nnz ? heads.as<int32_t>() : nullptr);
     TSMV_CUDA(cudaGetLastError());
     int b = read1(bad.as<int>(), st);
-    TSMV_REQUIRE(b == 0, b == 1 ? "tsmv_create: row_ptr not monotone / inconsistent with nnz"
-                                : "tsmv_create: column indices must be strictly ascending per row and < ncols");
+    TSMV_REQUIRE(b == 0, "tsmv_create: row_ptr not monotone / inconsistent with nnz");
     if (c->nnz) {
-        k_rows_of<<<grid_for(c->nnz), 256, 0, st>>>(row_ptr, c->m, c->nnz, rows);
+        size_t tb = 0;
+        TSMV_CUDA(cub::DeviceScan::InclusiveScan(nullptr, tb, heads.as<int32_t>(), rows, MaxI32(), c->nnz, st));
+        DevBuf tmp;
+        tmp.alloc(tb);
+        TSMV_CUDA(cub::DeviceScan::InclusiveScan(tmp.p, tb, heads.as<int32_t>(), rows, MaxI32(), c->nnz, st));
+        heads.release();
+        k_check_cols<<<grid_for(c->nnz), 256, 0, st>>>(rows, col_idx, c->nnz, c->n, bad.as<int>());
+        TSMV_CUDA(cudaGetLastError());
+        b = read1(bad.as<int>(), st);
+        TSMV_REQUIRE(b == 0, "tsmv_create: column indices must be strictly ascending per row and < ncols");
         k_colcount<<<grid_for(c->nnz), 256, 0, st>>>(col_idx, c->nnz, c->outdeg.as<int32_t>());
     }
     TSMV_CUDA(cudaGetLastError());

@@ -289,8 +289,9 @@ def random_access(kms, nt):
 
 def traffic_of(nt):
     """DRAM bytes (read + write) per launch of the SpMSpV kernel at T from the ncu
-    --set full capture committed under profiles/ (not measured in this run)."""
-    name = "r02_flat_traffic.json" if nt == 16 else "fused_traffic.json"
+    capture committed under profiles/ (taken under this bench's own L2-flush
+    protocol; not measured in this run)."""
+    name = "r02_flat_traffic_bench.json" if nt == 16 else "fused_traffic.json"
     path = os.path.join(ROOT, "profiles", name)
     try:
         d = json.load(open(path))

@@ -140,6 +140,12 @@ def _worker(rank, world, port, tmp, which):
                 np.save(os.path.join(tmp, f"lv{rank}_{s}.npy"), eng.levels)
             np.save(os.path.join(tmp, "srcs.npy"), np.array(srcs))
             np.save(os.path.join(tmp, "splits.npy"), np.array(splits))
+        elif which == "bootstrap":
+            # DistMatrix bootstrap: one NCCL unique id made on rank 0, shared over the group
+            uid = D.bootstrap_unique_id()
+            np.save(os.path.join(tmp, f"uid{rank}.npy"), np.frombuffer(uid, dtype=np.uint8))
+            uid2 = D.bootstrap_unique_id()
+            np.save(os.path.join(tmp, f"uidb{rank}.npy"), np.frombuffer(uid2, dtype=np.uint8))
         elif which == "spmspv":
             A = synth.attach_values(synth.rmat(10, 8, seed=2), seed=1, integer=True)
             splits = D.partition_rows(A.row_ptr, world)
@@ -180,6 +186,17 @@ def test_distributed_bfs_loop_gloo(which):
     for s in np.load(os.path.join(tmp, "srcs.npy")):
         got = np.concatenate([np.load(os.path.join(tmp, f"lv{r}_{s}.npy")) for r in range(WORLD)])
         assert np.array_equal(got, oracle.bfs_queue(C, int(s)))
+
+
+def test_bootstrap_unique_id_gloo():
+    """dist.bootstrap_unique_id: every rank gets rank 0's 128 bytes; a second call
+    (a second communicator) gets a new id."""
+    tmp = _run("bootstrap")
+    ids = [np.load(os.path.join(tmp, f"uid{r}.npy")) for r in range(WORLD)]
+    idsb = [np.load(os.path.join(tmp, f"uidb{r}.npy")) for r in range(WORLD)]
+    assert ids[0].size == 128 and ids[0].any()
+    assert all(np.array_equal(ids[0], x) for x in ids) and all(np.array_equal(idsb[0], x) for x in idsb)
+    assert not np.array_equal(ids[0], idsb[0])
 
 
 def test_distributed_spmspv_gloo():

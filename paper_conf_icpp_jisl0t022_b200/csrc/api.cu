@@ -144,6 +144,9 @@ static void destroy_impl(tsmv_ctx *c) {
     c->FL.release();
     if (c->hcnt) cudaFreeHost(c->hcnt);
     if (c->ev0) cudaEventDestroy(c->ev0);
+    if (c->ev_fork) cudaEventDestroy(c->ev_fork);
+    if (c->ev_join) cudaEventDestroy(c->ev_join);
+    if (c->aux_stream) cudaStreamDestroy(c->aux_stream);
     if (c->ev1) cudaEventDestroy(c->ev1);
     delete c;
 }
@@ -213,6 +216,9 @@ extern "C" tsmv_status tsmv_create(tsmv_ctx **out, int64_t nrows, int64_t ncols,
         TSMV_CUDA(cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking));
         TSMV_CUDA(cudaEventCreate(&c->ev0));
         TSMV_CUDA(cudaEventCreate(&c->ev1));
+        TSMV_CUDA(cudaStreamCreateWithFlags(&c->aux_stream, cudaStreamNonBlocking));
+        TSMV_CUDA(cudaEventCreateWithFlags(&c->ev_fork, cudaEventDisableTiming));
+        TSMV_CUDA(cudaEventCreateWithFlags(&c->ev_join, cudaEventDisableTiming));
         TSMV_CUDA(cudaEventRecord(c->ev0, st));
 
         // --- inputs on device

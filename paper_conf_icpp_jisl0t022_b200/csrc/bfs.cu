@@ -756,8 +756,20 @@ struct BfsRunner {
                 k_pull<NT, true><<<grid_for(nTRl), 256, 0, st>>>(Q, B, nTRl);
                 k_pull_side<NT, true><<<grid_for((c->m + 31) / 32), 256, 0, st>>>(Q, B);
             } else {
-                k_pull<NT, false><<<grid_for(nTRl * 32), 256, 0, st>>>(Q, B, nTRl);
-                k_pull_side<NT, false><<<grid_for(c->m), 256, 0, st>>>(Q, B);
+                // the tile part and the side part of a dense pull level are independent
+                // (both claim new vertices with atomics on V): the side kernel runs on
+                // the context's second stream, concurrently with the tile kernel
+                if (c->aux_stream) {
+                    TSMV_CUDA(cudaEventRecord(c->ev_fork, st));
+                    TSMV_CUDA(cudaStreamWaitEvent(c->aux_stream, c->ev_fork, 0));
+                    k_pull_side<NT, false><<<grid_for(c->m), 256, 0, c->aux_stream>>>(Q, B);
+                    TSMV_CUDA(cudaEventRecord(c->ev_join, c->aux_stream));
+                    k_pull<NT, false><<<grid_for(nTRl * 32), 256, 0, st>>>(Q, B, nTRl);
+                    TSMV_CUDA(cudaStreamWaitEvent(st, c->ev_join, 0));
+                } else {
+                    k_pull<NT, false><<<grid_for(nTRl * 32), 256, 0, st>>>(Q, B, nTRl);
+                    k_pull_side<NT, false><<<grid_for(c->m), 256, 0, st>>>(Q, B);
+                }
             }
         }
         TSMV_CUDA(cudaGetLastError());

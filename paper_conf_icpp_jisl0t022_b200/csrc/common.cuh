@@ -305,6 +305,8 @@ struct tsmv_ctx {
     long long cur_fsize = 0, cur_mf = 0;
 
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+    cudaStream_t aux_stream = nullptr;          // second stream of the dense pull level (bfs.cu)
+    cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
     // optional per-phase timing of tsmv_spmspv* (tsmv_set_timing): block 0 of the
     // fused kernel stamps %globaltimer at its phase boundaries into a ring
     bool timing = false;

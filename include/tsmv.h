@@ -268,20 +268,24 @@ typedef struct {
 tsmv_status tsmv_msbfs(tsmv_ctx *c, int32_t nsrc, const int64_t *sources, int32_t *levels,
                        tsmv_msbfs_stats *stats, void *cuda_stream);
 
-/* ---- distributed TileBFS (row-block partition, Sec 8(e) of SURVEY / DESIGN.md) ----
+/* ---- distributed TileBFS, caller-driven exchange (row-block partition, SURVEY
+ * §8(e) / DESIGN.md §8; contexts WITHOUT a communicator: simulated ranks, gloo) ----
  * Each rank owns global rows [row_splits[rank], row_splits[rank+1]).  Per level:
  *   tsmv_bfs_dist_expand  -> this rank's newly discovered owned vertices as a bitmap
  *                            segment (uint32 words, bit v%32 of word (v-row_begin)/32);
  *   caller all-gathers the segments (torch.distributed / NCCL), each padded to
  *   `stride_words` words, in rank order;
  *   tsmv_bfs_dist_merge   -> OR the gathered frontier into the replicated visited
- *                            bitmap, rebuild the frontier, return its size.
- * begin / merge return out_stats[3] = { |F| (global: same on every rank),
- * m_f local (sum over F of this block's column counts), m_u local (sum of the
- * in-degrees of this rank's unvisited rows) }; the caller all-reduces m_f and
- * m_u and passes tsmv_choose_dir(...) of the global numbers as `dir` (1..3) to
- * expand, so every rank takes the same decision.  levels: device memory,
- * int32[local rows].  All ranks make the same calls in the same order. */
+ *                            bitmap, clear the old frontier, return the statistics.
+ * (r2) begin / merge return this rank's SHARES out_stats[3] = { |F| of its own rows,
+ * m_f share (sum of the GLOBAL out-degrees of its frontier vertices), m_u local (sum
+ * of the in-degrees of its unvisited rows) }, computed over its own rows only
+ * (O(n / P) per level); the caller sums the three over the ranks and passes
+ * tsmv_choose_dir(...) of the sums as `dir` (1..3) to expand, so every rank takes
+ * the same decision.  The global out-degrees (column counts of all blocks) are set
+ * once with tsmv_bfs_dist_set_degrees (a one-rank context uses its own).  levels:
+ * device memory, int32[local rows].  All ranks make the same calls in the same order. */
+tsmv_status tsmv_bfs_dist_set_degrees(tsmv_ctx *c, const int32_t *outdeg_global /* int32[ncols], host or device */);
 tsmv_status tsmv_bfs_dist_begin(tsmv_ctx *c, int64_t source, int32_t *levels, int64_t *out_stats,
                                 void *cuda_stream);
 /* dir: TSMV_DIR_PUSH_CSC .. TSMV_DIR_PULL_CSC, optionally | TSMV_DIST_WIDE: a hint

@@ -297,7 +297,7 @@ extern "C" tsmv_status tsmv_create(tsmv_ctx **out, int64_t nrows, int64_t ncols,
         memset(c->hcnt, 0, sizeof(Counters));
         TSMV_CUDA(cudaHostGetDevicePointer((void **)&c->hcnt_dev, c->hcnt, 0));
         if (want_bfs) {
-            int64_t NWpad = ((ncols + 63) / 64) * 2;
+            int64_t NWpad = ((ncols + 127) / 128) * 4;  // whole 16-byte vectors (k_fscan)
             c->V.alloc(NWpad * 4);
             c->F0.alloc(NWpad * 4);
             c->F1.alloc(NWpad * 4);

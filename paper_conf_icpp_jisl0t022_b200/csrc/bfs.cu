@@ -56,108 +56,145 @@ __global__ void k_bfs_init(BfsView B, long long NW, long long source) {
         B.levels[v] = (v + B.row_begin == source) ? 0 : -1;
 }
 
-// Frontier scan: one thread per nt-segment of the (global) frontier bitmap F.
+// One nt-segment J of the frontier bitmap F: q.v[0..3] = list terms (segment
+// has tile work, its tile work, side columns with entries, their side work),
+// with `full` also q.v[4..6] = |F| bits, m_f, sum of in-degrees of local rows.
 template <int NT>
-__global__ void __launch_bounds__(SCAN_BLOCK)
-k_fscan(const uint32_t *__restrict__ F, uint32_t *__restrict__ Fclear, long long nseg, long long NWpad,
-        const long long *__restrict__ tptr, const long long *__restrict__ sptr, const int *__restrict__ outdeg,
-        const int *__restrict__ indeg, long long row_begin, long long m_local, ListsView Lv,
-        Counters *__restrict__ cnt, Counters *__restrict__ hm, LBDesc<8> *__restrict__ desc, unsigned epoch,
-        int write_lists) {
+__device__ __forceinline__ typename Tr<NT>::word_t
+scan_seg(const uint32_t *__restrict__ F, long long J, const long long *__restrict__ tptr,
+         const long long *__restrict__ sptr, const int *__restrict__ outdeg, const int *__restrict__ indeg,
+         long long row_begin, long long m_local, bool full, Oct &q, long long &wt) {
     using word_t = typename Tr<NT>::word_t;
-    using BS = cub::BlockScan<Oct, SCAN_BLOCK>;
-    __shared__ typename BS::TempStorage ts;
-    __shared__ unsigned s_bid;
-    __shared__ long long s_pre[8];
-    if (threadIdx.x == 0) s_bid = atomicAdd(&cnt->bid_scan, 1u);
-    __syncthreads();
-    const unsigned bid = s_bid;
-    const long long J = (long long)bid * SCAN_BLOCK + threadIdx.x;
-    Oct q;
 #pragma unroll
     for (int i = 0; i < 8; ++i) q.v[i] = 0;
-    word_t bits = 0;
-    long long wt = 0;
-    if (J < nseg) {
-        bits = seg_bits<NT>(F, J);
-        if constexpr (NT == 16) {
-            // the segment's 16 out-degrees, in-degrees and 17 side starts are
-            // contiguous: 4 + 4 + 9 independent 16-byte loads, one latency
-            if (bits) {
-                wt = tptr[J + 1] - tptr[J];
-                q.v[0] = wt > 0;
-                q.v[1] = wt;
-                q.v[4] = popc_w(bits);
-                const long long v0 = J * 16;
-                const int4 *od4 = reinterpret_cast<const int4 *>(outdeg + v0);
-                const longlong2 *sp2 = reinterpret_cast<const longlong2 *>(sptr + v0);
-                int od[16];
-                long long sp[18];
+    wt = 0;
+    const word_t bits = seg_bits<NT>(F, J);
+    if (!bits) return bits;
+    wt = tptr[J + 1] - tptr[J];
+    q.v[0] = wt > 0;
+    q.v[1] = wt;
+    if constexpr (NT == 16) {
+        // the segment's 16 out-degrees, in-degrees and 17 side starts are
+        // contiguous: 4 + 4 + 9 independent 16-byte loads, one latency
+        const long long v0 = J * 16;
+        const longlong2 *sp2 = reinterpret_cast<const longlong2 *>(sptr + v0);
+        long long sp[18];
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+            const longlong2 t = __ldg(sp2 + i);
+            sp[2 * i] = t.x, sp[2 * i + 1] = t.y;
+        }
+        sp[16] = __ldg(sptr + v0 + 16);
+        int od[16], id[16];
+#pragma unroll
+        for (int r = 0; r < 16; ++r) od[r] = id[r] = 0;
+        if (full) {
+            q.v[4] = popc_w(bits);
+            const int4 *od4 = reinterpret_cast<const int4 *>(outdeg + v0);
+#pragma unroll
+            for (int i = 0; i < 4; ++i) {
+                const int4 t = __ldg(od4 + i);
+                od[4 * i] = t.x, od[4 * i + 1] = t.y, od[4 * i + 2] = t.z, od[4 * i + 3] = t.w;
+            }
+            const long long lv0 = v0 - row_begin;
+            if (lv0 >= 0 && lv0 + 16 <= m_local) {
+                const int4 *id4 = reinterpret_cast<const int4 *>(indeg + lv0);
 #pragma unroll
                 for (int i = 0; i < 4; ++i) {
-                    const int4 t = __ldg(od4 + i);
-                    od[4 * i] = t.x, od[4 * i + 1] = t.y, od[4 * i + 2] = t.z, od[4 * i + 3] = t.w;
+                    const int4 t = __ldg(id4 + i);
+                    id[4 * i] = t.x, id[4 * i + 1] = t.y, id[4 * i + 2] = t.z, id[4 * i + 3] = t.w;
                 }
+            } else {
 #pragma unroll
-                for (int i = 0; i < 8; ++i) {
-                    const longlong2 t = __ldg(sp2 + i);
-                    sp[2 * i] = t.x, sp[2 * i + 1] = t.y;
-                }
-                sp[16] = __ldg(sptr + v0 + 16);
-                const long long lv0 = v0 - row_begin;
-                int id[16];
-                if (lv0 >= 0 && lv0 + 16 <= m_local) {
-                    const int4 *id4 = reinterpret_cast<const int4 *>(indeg + lv0);
-#pragma unroll
-                    for (int i = 0; i < 4; ++i) {
-                        const int4 t = __ldg(id4 + i);
-                        id[4 * i] = t.x, id[4 * i + 1] = t.y, id[4 * i + 2] = t.z, id[4 * i + 3] = t.w;
-                    }
-                } else {
-#pragma unroll
-                    for (int r = 0; r < 16; ++r)
-                        id[r] = (lv0 + r >= 0 && lv0 + r < m_local) ? __ldg(indeg + lv0 + r) : 0;
-                }
-#pragma unroll
-                for (int r = 0; r < 16; ++r) {
-                    if ((bits >> r) & 1u) {
-                        const long long ws = sp[r + 1] - sp[r];
-                        q.v[2] += ws > 0;
-                        q.v[3] += ws;
-                        q.v[5] += od[r];
-                        q.v[6] += id[r];
-                    }
-                }
+                for (int r = 0; r < 16; ++r)
+                    id[r] = (lv0 + r >= 0 && lv0 + r < m_local) ? __ldg(indeg + lv0 + r) : 0;
             }
-        } else if (bits) {
-            wt = tptr[J + 1] - tptr[J];
-            q.v[0] = wt > 0;
-            q.v[1] = wt;
-            word_t b = bits;
-            while (b) {
-                int r = ffs_w(b);
-                b &= b - 1;
-                long long v = J * NT + r;
-                long long ws = sptr[v + 1] - sptr[v];
+        }
+#pragma unroll
+        for (int r = 0; r < 16; ++r) {
+            if ((bits >> r) & 1u) {
+                const long long ws = sp[r + 1] - sp[r];
                 q.v[2] += ws > 0;
                 q.v[3] += ws;
+                q.v[5] += od[r];
+                q.v[6] += id[r];
+            }
+        }
+    } else {
+        word_t b = bits;
+        while (b) {
+            int r = ffs_w(b);
+            b &= b - 1;
+            long long v = J * NT + r;
+            long long ws = sptr[v + 1] - sptr[v];
+            q.v[2] += ws > 0;
+            q.v[3] += ws;
+            if (full) {
                 q.v[5] += outdeg[v];
                 long long lv = v - row_begin;
                 if (lv >= 0 && lv < m_local) q.v[6] += indeg[lv];
             }
-            q.v[4] = popc_w(bits);
         }
-        // clear the consumed frontier (the level that was just expanded)
-        if (Fclear) {
-            if constexpr (NT == 16) {
-                if ((J & 1) == 0) Fclear[J >> 1] = 0u;
-            } else if constexpr (NT == 32) {
-                Fclear[J] = 0u;
-            } else {
-                Fclear[2 * J] = 0u;
-                Fclear[2 * J + 1] = 0u;
+        if (full) q.v[4] = popc_w(bits);
+    }
+    return bits;
+}
+
+// Frontier scan over the nseg nt-segments of the (global) frontier bitmap F.
+// One wave of blocks, each owning a contiguous range of `tpb` super-tiles; a
+// super-tile is SCAN_BLOCK threads x SPT = 128/nt consecutive segments, one
+// 16-byte load of F per thread, so an empty stretch of the frontier costs one
+// coalesced read (r2: a block per 256 segments made a 4096-block look-back chain
+// at scale 24 -- 144 us for a one-vertex frontier):
+//   pass 1: per-segment terms of the whole range, block aggregate, clear Fclear;
+//   (statistics only: block reduction + atomics, the last block publishes)
+//   look-back for the range's exclusive prefix;
+//   pass 2: super-tiles with a frontier bit again, block-exclusive-scan of the
+//           four list terms + running offset, write the tile / side lists and
+//           chunk starts, each thread its SPT segments in order.
+template <int NT>
+__device__ __forceinline__ uint4 ld_f4(const uint32_t *__restrict__ F, long long w, long long nwpad) {
+    return w + 4 <= nwpad ? __ldg(reinterpret_cast<const uint4 *>(F + w)) : make_uint4(0u, 0u, 0u, 0u);
+}
+
+template <int NT>
+__global__ void __launch_bounds__(SCAN_BLOCK)
+k_fscan(const uint32_t *__restrict__ F, uint32_t *__restrict__ Fclear, long long nseg, long long tpb,
+        long long nwpad, const long long *__restrict__ tptr, const long long *__restrict__ sptr,
+        const int *__restrict__ outdeg, const int *__restrict__ indeg, long long row_begin, long long m_local,
+        ListsView Lv, Counters *__restrict__ cnt, Counters *__restrict__ hm, LBDesc<8> *__restrict__ desc,
+        unsigned epoch, int write_lists) {
+    using word_t = typename Tr<NT>::word_t;
+    constexpr int SPT = 128 / NT;
+    using BS = cub::BlockScan<Oct, SCAN_BLOCK>;
+    __shared__ typename BS::TempStorage ts;
+    __shared__ unsigned s_bid;
+    __shared__ long long s_pre[8], s_run[4];
+    if (threadIdx.x == 0) s_bid = atomicAdd(&cnt->bid_scan, 1u);
+    __syncthreads();
+    const unsigned bid = s_bid;
+    const long long nst = (nseg + (long long)SCAN_BLOCK * SPT - 1) / ((long long)SCAN_BLOCK * SPT);
+    const long long t0 = (long long)bid * tpb, t1 = min(nst, t0 + tpb);
+    Oct acc;
+#pragma unroll
+    for (int i = 0; i < 8; ++i) acc.v[i] = 0;
+    for (long long t = t0; t < t1; ++t) {
+        const long long u = t * SCAN_BLOCK + threadIdx.x;  // this thread's 16-byte unit
+        const uint4 f4 = ld_f4<NT>(F, u * 4, nwpad);
+        if (f4.x | f4.y | f4.z | f4.w) {
+#pragma unroll 1
+            for (int k = 0; k < SPT; ++k) {
+                const long long J = u * SPT + k;
+                if (J >= nseg) break;
+                Oct q;
+                long long wt;
+                scan_seg<NT>(F, J, tptr, sptr, outdeg, indeg, row_begin, m_local, true, q, wt);
+#pragma unroll
+                for (int i = 0; i < 8; ++i) acc.v[i] += q.v[i];
             }
         }
+        // clear the consumed frontier (the level that was just expanded)
+        if (Fclear && u * 4 + 4 <= nwpad) *reinterpret_cast<uint4 *>(Fclear + u * 4) = make_uint4(0u, 0u, 0u, 0u);
     }
     if (!write_lists) {
         // statistics only: block reduction + one atomic per value and block; the
@@ -168,7 +205,7 @@ k_fscan(const uint32_t *__restrict__ F, uint32_t *__restrict__ Fclear, long long
         __syncthreads();
 #pragma unroll
         for (int i = 0; i < 7; ++i) {
-            long long x = q.v[i];
+            long long x = acc.v[i];
 #pragma unroll
             for (int o = 16; o > 0; o >>= 1) x += __shfl_xor_sync(0xffffffffu, x, o);
             if ((threadIdx.x & 31) == 0 && x) atomicAdd((unsigned long long *)&s_red[i], (unsigned long long)x);
@@ -202,49 +239,84 @@ k_fscan(const uint32_t *__restrict__ F, uint32_t *__restrict__ Fclear, long long
         }
         return;
     }
-    Oct ex, agg;
-    Oct zero;
+    Oct zero, ex, agg;
 #pragma unroll
     for (int i = 0; i < 8; ++i) zero.v[i] = 0;
-    BS(ts).ExclusiveScan(q, ex, zero, OctSum(), agg);
+    BS(ts).ExclusiveScan(acc, ex, zero, OctSum(), agg);
     if (threadIdx.x < 32) {
         long long pre[8];
         lookback_warp<8>(desc, bid, epoch, agg.v, pre, threadIdx.x);
         if (threadIdx.x == 0) {
 #pragma unroll
             for (int i = 0; i < 8; ++i) s_pre[i] = pre[i];
+#pragma unroll
+            for (int i = 0; i < 4; ++i) s_run[i] = pre[i];
         }
     }
     __syncthreads();
+    for (long long t = t0; t < t1; ++t) {
+        const long long u = t * SCAN_BLOCK + threadIdx.x;
+        const uint4 f4 = ld_f4<NT>(F, u * 4, nwpad);
+        const bool any = (f4.x | f4.y | f4.z | f4.w) != 0u;
+        if (!__syncthreads_or(any)) continue;  // no frontier bit in this super-tile
+        Oct q;
 #pragma unroll
-    for (int i = 0; i < 8; ++i) ex.v[i] += s_pre[i];
-    if (bits && wt > 0 && write_lists) {
-        long long i = ex.v[0];
-        Lv.Lt_seg[i] = J;
-        Lv.Lt_mask[i] = (unsigned long long)bits;
-        Lv.Lt_tbeg[i] = tptr[J];
-        Lv.Lt_wpre[i] = ex.v[1];
-        write_chunks(Lv.Ct, ex.v[1], wt, (int)i);
-    }
-    if (bits && write_lists) {
-        long long i = ex.v[2], w0 = ex.v[3];
-        word_t b = bits;
-        while (b) {
-            int r = ffs_w(b);
-            b &= b - 1;
-            long long v = J * NT + r;
-            long long ws = sptr[v + 1] - sptr[v];
-            if (ws > 0) {
-                Lv.Ls_beg[i] = sptr[v];
-                Lv.Ls_wpre[i] = w0;
-                Lv.Ls_col[i] = (int)v;
-                write_chunks(Lv.Cs, w0, ws, (int)i);
-                ++i;
-                w0 += ws;
+        for (int i = 0; i < 8; ++i) q.v[i] = 0;
+        if (any) {
+#pragma unroll 1
+            for (int k = 0; k < SPT; ++k) {
+                const long long J = u * SPT + k;
+                if (J >= nseg) break;
+                Oct qk;
+                long long wt;
+                scan_seg<NT>(F, J, tptr, sptr, outdeg, indeg, row_begin, m_local, false, qk, wt);
+#pragma unroll
+                for (int i = 0; i < 4; ++i) q.v[i] += qk.v[i];
             }
         }
+        Oct tagg;
+        BS(ts).ExclusiveScan(q, ex, zero, OctSum(), tagg);
+        if (any) {
+            long long it = s_run[0] + ex.v[0], wp = s_run[1] + ex.v[1];
+            long long is = s_run[2] + ex.v[2], w0 = s_run[3] + ex.v[3];
+#pragma unroll 1
+            for (int k = 0; k < SPT; ++k) {
+                const long long J = u * SPT + k;
+                if (J >= nseg) break;
+                const word_t bits = seg_bits<NT>(F, J);
+                if (!bits) continue;
+                const long long wt = tptr[J + 1] - tptr[J];
+                if (wt > 0) {
+                    Lv.Lt_seg[it] = J;
+                    Lv.Lt_mask[it] = (unsigned long long)bits;
+                    Lv.Lt_tbeg[it] = tptr[J];
+                    Lv.Lt_wpre[it] = wp;
+                    write_chunks(Lv.Ct, wp, wt, (int)it);
+                    ++it;
+                    wp += wt;
+                }
+                word_t b = bits;
+                while (b) {
+                    int r = ffs_w(b);
+                    b &= b - 1;
+                    long long v = J * NT + r;
+                    long long ws = sptr[v + 1] - sptr[v];
+                    if (ws > 0) {
+                        Lv.Ls_beg[is] = sptr[v];
+                        Lv.Ls_wpre[is] = w0;
+                        Lv.Ls_col[is] = (int)v;
+                        write_chunks(Lv.Cs, w0, ws, (int)is);
+                        ++is;
+                        w0 += ws;
+                    }
+                }
+            }
+        }
+        __syncthreads();  // every thread has read s_run
+        if (threadIdx.x < 4) s_run[threadIdx.x] += tagg.v[threadIdx.x];
+        __syncthreads();
     }
-    if (bid == gridDim.x - 1 && threadIdx.x == SCAN_BLOCK - 1) {
+    if (bid == gridDim.x - 1 && threadIdx.x == 0) {
         long long tot[8];
 #pragma unroll
         for (int i = 0; i < 8; ++i) tot[i] = s_pre[i] + agg.v[i];
@@ -257,10 +329,8 @@ k_fscan(const uint32_t *__restrict__ F, uint32_t *__restrict__ Fclear, long long
         cnt->fsize = tot[4];
         cnt->mf = tot[5];
         cnt->din = tot[6];
-        if (write_lists) {
-            Lv.Lt_wpre[tot[0]] = tot[1];
-            Lv.Ls_wpre[tot[2]] = tot[3];
-        }
+        Lv.Lt_wpre[tot[0]] = tot[1];
+        Lv.Ls_wpre[tot[2]] = tot[3];
         hm->fsize = tot[4];
         hm->mf = tot[5];
         hm->din = tot[6];
@@ -652,12 +722,65 @@ __global__ void k_parents_fix(int32_t *__restrict__ parents, long long m) {
         if (parents[v] == INT_MAX) parents[v] = -1;
 }
 
-// distributed merge with device statistics: {|F| (global), m_f local, m_u local}
-__global__ void k_dist_stats(const Counters *__restrict__ cnt, long long *__restrict__ mu, int64_t *__restrict__ out) {
-    const long long m = *mu - cnt->din;
+
+// Statistics of this rank's share of the next frontier (distributed levels, r2):
+// over the owned words [w0, w1) of F: out[0] += |F_owned|, out[1] += sum of the
+// GLOBAL out-degrees of those vertices (m_f share), out[2] += sum of their
+// in-degrees (row counts of owned rows: the m_u decrement).  Every rank scans
+// only its own rows, O(n / P); the shares are summed over the ranks.
+__global__ void k_owned_stats(const uint32_t *__restrict__ F, long long w0, long long w1, long long row_begin,
+                              const int *__restrict__ outdeg_g, const int *__restrict__ indeg_local,
+                              unsigned long long *__restrict__ out) {
+    // a warp takes 32 consecutive words (one coalesced load), then walks them:
+    // for a non-zero word lane l tests bit l, so the degree loads of a word are
+    // one 128-byte line each (a thread-per-word bit loop serialised them)
+    const int lane = threadIdx.x & 31;
+    const long long nwarps = ((long long)gridDim.x * blockDim.x) >> 5;
+    unsigned long long q0 = 0, q1 = 0, q2 = 0;
+    for (long long wb = w0 + (((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5) * 32; wb < w1;
+         wb += nwarps * 32) {
+        const uint32_t mine = (wb + lane < w1) ? __ldg(F + wb + lane) : 0u;
+        unsigned nz = __ballot_sync(0xffffffffu, mine != 0u);
+        while (nz) {
+            const int j = __ffs(nz) - 1;
+            nz &= nz - 1;
+            const uint32_t b = __shfl_sync(0xffffffffu, mine, j);
+            if ((b >> lane) & 1u) {
+                const long long v = (wb + j) * 32 + lane;
+                ++q0;
+                q1 += (unsigned long long)__ldg(outdeg_g + v);
+                q2 += (unsigned long long)__ldg(indeg_local + (v - row_begin));
+            }
+        }
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        q0 += __shfl_xor_sync(0xffffffffu, q0, o);
+        q1 += __shfl_xor_sync(0xffffffffu, q1, o);
+        q2 += __shfl_xor_sync(0xffffffffu, q2, o);
+    }
+    if (lane == 0 && q0) {
+        atomicAdd(&out[0], q0);
+        atomicAdd(&out[1], q1);
+        atomicAdd(&out[2], q2);
+    }
+}
+// begin: shares of the source's frontier {source} (only its owner counts it)
+__global__ void k_source_stats(long long source, long long row_begin, long long m_local,
+                               const int *__restrict__ outdeg_g, const int *__restrict__ indeg_local,
+                               unsigned long long *__restrict__ out) {
+    const bool own = source >= row_begin && source < row_begin + m_local;
+    out[0] = own ? 1ull : 0ull;
+    out[1] = own ? (unsigned long long)outdeg_g[source] : 0ull;
+    out[2] = own ? (unsigned long long)indeg_local[source - row_begin] : 0ull;
+}
+// distributed merge with device statistics: {|F| share, m_f share, m_u local}
+__global__ void k_dist_stats2(const unsigned long long *__restrict__ dstats, long long *__restrict__ mu,
+                              int64_t *__restrict__ out) {
+    const long long m = *mu - (long long)dstats[2];
     *mu = m;
-    out[0] = cnt->fsize;
-    out[1] = cnt->mf;
+    out[0] = (long long)dstats[0];
+    out[1] = (long long)dstats[1];
     out[2] = m;
 }
 
@@ -718,7 +841,19 @@ struct BfsRunner {
 
     template <int NT> void fscan(const uint32_t *F, uint32_t *Fclear, bool lists) {
         long long nseg = c->nTC;
-        int grid = (int)std::max<long long>(1, (nseg + SCAN_BLOCK - 1) / SCAN_BLOCK);
+        // one wave: blocks x tiles-per-block cover the ceil(nseg / SCAN_BLOCK) tiles
+        static int bps_scan[3] = {0, 0, 0};
+        int &bps = bps_scan[NT == 16 ? 0 : NT == 32 ? 1 : 2];
+        if (bps == 0 && (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_fscan<NT>, SCAN_BLOCK, 0) !=
+                             cudaSuccess || bps < 1)) {
+            cudaGetLastError();
+            bps = 1;
+        }
+        const long long spt = 128 / NT;
+        const long long ntiles = std::max<long long>(1, (nseg + SCAN_BLOCK * spt - 1) / (SCAN_BLOCK * spt));
+        const long long cap = std::max<long long>(1, (long long)c->sm_count * bps);
+        const long long tpb = (ntiles + cap - 1) / cap;
+        const int grid = (int)((ntiles + tpb - 1) / tpb);
         c->epoch++;
         if (!lists)  // the stats-only scan accumulates into zeroed counters {nLt..din}
             TSMV_CUDA(cudaMemsetAsync(&c->counters.as<Counters>()->nLt, 0, 9 * sizeof(long long), st));
@@ -735,7 +870,8 @@ struct BfsRunner {
             TSMV_CUDA(cudaGetLastError());
             return;
         }
-        k_fscan<NT><<<grid, SCAN_BLOCK, 0, st>>>(F, Fclear, nseg, NW, c->P.ptr.as<long long>(),
+        k_fscan<NT><<<grid, SCAN_BLOCK, 0, st>>>(F, Fclear, nseg, tpb, (long long)(c->V.bytes / 4),
+                                                 c->P.ptr.as<long long>(),
                                                  c->P.sptr.as<long long>(), odeg(), ideg(),
                                                  irb(), iml(), lists_view(c), c->counters.as<Counters>(),
                                                  c->hcnt_dev, c->desc_bfs.as<LBDesc<8>>(), c->epoch, lists ? 1 : 0);
@@ -800,6 +936,23 @@ struct BfsRunner {
     }
 };
 
+// global out-degrees: set for a distributed context (communicator or
+// tsmv_bfs_dist_set_degrees); a one-rank context's own column counts are global
+static const int *out_degrees(const tsmv_ctx *c) {
+    return c->outdeg_g.p ? c->outdeg_g.as<int>() : c->outdeg.as<int>();
+}
+
+// this rank's words of the frontier bitmap and its statistics shares (dstats)
+static void owned_stats(tsmv_ctx *c, const uint32_t *F, cudaStream_t st) {
+    c->dstats.ensure(4 * 8);
+    TSMV_CUDA(cudaMemsetAsync(c->dstats.p, 0, 4 * 8, st));
+    const long long w0 = c->row_begin >> 5, w1 = (c->row_begin + c->m + 31) >> 5;
+    if (w1 > w0)
+        k_owned_stats<<<grid_for(w1 - w0, 256, c->sm_count * 8), 256, 0, st>>>(F, w0, w1, c->row_begin, out_degrees(c),
+                                                         c->indeg.as<int>(), c->dstats.as<unsigned long long>());
+    TSMV_CUDA(cudaGetLastError());
+}
+
 int choose_dir(const tsmv_options &o, long long n, long long fsize, long long mf, long long mu) {
     if (o.force_dir != TSMV_DIR_AUTO) return o.force_dir;
     // reading R9: Beamer-style edge test for pull, then the paper's 0.01 density rule
@@ -839,25 +992,35 @@ static void level_times(tsmv_ctx *c, tsmv_bfs_stats *stats, long long nl, bool h
 // Alg 3's level loop on every rank, one exchange per level.  The
 // frontier F and the visited bitmap V are replicated (n bits); each rank expands
 // the level into its OWNED rows with the level kernels (Push-CSC / Push-CSR /
-// Pull-CSC over its row block), the owned segments of the next frontier are
-// broadcast in place to every rank (comm_exchange_frontier), and the statistics
-// scan of the whole next frontier with the replicated global degree arrays gives
-// every rank the same |F|, m_f and m_u, hence the same direction decision and
-// termination, with no reduction.  One host synchronisation per level (the
-// statistics decide which kernels the host launches).
+// Pull-CSC over its row block; the push lists are built from the replicated
+// frontier on push levels only), computes the statistics shares of its owned
+// new vertices (count, sum of global out-degrees, sum of in-degrees: O(n / P)),
+// and one NCCL group broadcasts the owned frontier words in place and
+// all-gathers the shares; every rank sums the same shares, hence takes the same
+// direction decision and stops at the same level.  One host synchronisation per
+// level (the statistics choose the kernels).  Nothing per level is O(n) except
+// the OR of the frontier into V (n / 32 words) and the clearing of the old one.
 static void bfs_distributed(tsmv_ctx *c, int64_t source, tsmv_bfs_stats *stats, cudaStream_t st) {
     ensure_lists(c, c->n);
     BfsRunner R{c, st, (long long)(c->V.bytes / 4)};
     unsigned long long *tlv = c->bfs_tlv.as<unsigned long long>();
+    const int P = c->opt.nranks;
+    c->dstats_all.ensure((size_t)P * 4 * 8);
+    std::vector<unsigned long long> sh((size_t)P * 4);
     c->fcur = 0;
     c->bfs_level = 0;
     TSMV_CUDA(cudaEventRecord(c->ev0, st));
     TSMV_CUDA(cudaMemsetAsync(c->F1.p, 0, c->F1.bytes, st));
     R.init(source);
-    R.do_fscan(c->F0.as<uint32_t>(), nullptr);
-    TSMV_CUDA(cudaStreamSynchronize(st));
-    volatile Counters *h = c->hcnt;
-    long long fsize = h->fsize, mf = h->mf, mu = c->nnz_global - h->din;
+    long long fsize = 1, mf = 0, mu = c->nnz_global;
+    {
+        int od = 0, id = 0;
+        TSMV_CUDA(cudaMemcpyAsync(&od, c->outdeg_g.as<int>() + source, 4, cudaMemcpyDeviceToHost, st));
+        TSMV_CUDA(cudaMemcpyAsync(&id, c->indeg_g.as<int>() + source, 4, cudaMemcpyDeviceToHost, st));
+        TSMV_CUDA(cudaStreamSynchronize(st));
+        mf = od;
+        mu -= id;
+    }
     long long reached = 0, edges = 0;
     long long L = 0;
     while (fsize > 0) {
@@ -872,15 +1035,23 @@ static void bfs_distributed(tsmv_ctx *c, int64_t source, tsmv_bfs_stats *stats, 
         reached += fsize;
         edges += mf;
         c->bfs_level = (int)L;
-        R.do_expand(dir, dir == TSMV_DIR_PULL_CSC && mu * 4 < c->nnz_global);
         uint32_t *Fcur = (c->fcur == 0 ? c->F0 : c->F1).as<uint32_t>();
         uint32_t *Fnext = (c->fcur == 0 ? c->F1 : c->F0).as<uint32_t>();
-        comm_exchange_frontier(c, Fnext, c->V.as<uint32_t>(), (c->n + 31) / 32, st);
-        R.do_fscan(Fnext, Fcur);
+        if (dir != TSMV_DIR_PULL_CSC) R.do_fscan(Fcur, nullptr);  // push lists of the replicated frontier
+        R.do_expand(dir, dir == TSMV_DIR_PULL_CSC && mu * 4 < c->nnz_global);
+        owned_stats(c, Fnext, st);
+        comm_exchange_frontier(c, Fnext, c->V.as<uint32_t>(), (c->n + 31) / 32, c->dstats.p, c->dstats_all.p, st);
+        TSMV_CUDA(cudaMemsetAsync(Fcur, 0, ((c->n + 63) / 64) * 8, st));
+        TSMV_CUDA(cudaMemcpyAsync(sh.data(), c->dstats_all.p, sh.size() * 8, cudaMemcpyDeviceToHost, st));
         TSMV_CUDA(cudaStreamSynchronize(st));
-        fsize = h->fsize;
-        mf = h->mf;
-        mu -= h->din;
+        fsize = mf = 0;
+        long long din = 0;
+        for (int p = 0; p < P; ++p) {
+            fsize += (long long)sh[p * 4];
+            mf += (long long)sh[p * 4 + 1];
+            din += (long long)sh[p * 4 + 2];
+        }
+        mu -= din;
         c->fcur ^= 1;
         ++L;
     }
@@ -1127,6 +1298,37 @@ extern "C" tsmv_status tsmv_bfs_parents(tsmv_ctx *c, const int32_t *levels, int3
 // ----------------------------------------------------------------- distributed primitives
 extern "C" int64_t tsmv_owned_words(const tsmv_ctx *c) { return c ? (c->m + 31) / 32 : 0; }
 
+extern "C" tsmv_status tsmv_bfs_dist_set_degrees(tsmv_ctx *c, const int32_t *outdeg_global) {
+    try {
+        TSMV_REQUIRE(c && outdeg_global, "tsmv_bfs_dist_set_degrees: NULL argument");
+        TSMV_CUDA(cudaSetDevice(c->device));
+        c->outdeg_g.alloc(((std::max<int64_t>(c->n, 1) + 63) / 64 * 64) * 4);
+        TSMV_CUDA(cudaMemset(c->outdeg_g.p, 0, c->outdeg_g.bytes));
+        TSMV_CUDA(cudaMemcpy(c->outdeg_g.p, outdeg_global, c->n * 4, cudaMemcpyDefault));
+        return TSMV_OK;
+    } catch (const Err &e) {
+        return e.st;
+    }
+}
+
+static void dist_out(tsmv_ctx *c, int64_t *out_stats, cudaStream_t st) {
+    if (is_device_ptr(out_stats)) {
+        // device statistics: no synchronisation (the caller reduces them on the device)
+        k_dist_stats2<<<1, 1, 0, st>>>(c->dstats.as<unsigned long long>(), c->mu_dev.as<long long>(), out_stats);
+        TSMV_CUDA(cudaGetLastError());
+        return;
+    }
+    unsigned long long h[4];
+    TSMV_CUDA(cudaMemcpyAsync(h, c->dstats.p, 32, cudaMemcpyDeviceToHost, st));
+    TSMV_CUDA(cudaStreamSynchronize(st));
+    c->m_u_local -= (long long)h[2];
+    TSMV_CUDA(cudaMemcpyAsync(c->mu_dev.p, &c->m_u_local, 8, cudaMemcpyHostToDevice, st));
+    TSMV_CUDA(cudaStreamSynchronize(st));
+    out_stats[0] = (long long)h[0];
+    out_stats[1] = (long long)h[1];
+    out_stats[2] = c->m_u_local;
+}
+
 extern "C" tsmv_status tsmv_bfs_dist_begin(tsmv_ctx *c, int64_t source, int32_t *levels, int64_t *out_stats,
                                            void *cuda_stream) {
     try {
@@ -1134,6 +1336,8 @@ extern "C" tsmv_status tsmv_bfs_dist_begin(tsmv_ctx *c, int64_t source, int32_t 
         bfs_check(c);
         TSMV_REQUIRE(source >= 0 && source < c->n, "tsmv_bfs_dist_begin: source out of range");
         TSMV_REQUIRE(is_device_ptr(levels), "tsmv_bfs_dist_begin: levels must be device memory");
+        TSMV_REQUIRE(c->outdeg_g.p != nullptr || c->opt.nranks == 1,
+                     "tsmv_bfs_dist_begin: global out-degrees not set (tsmv_bfs_dist_set_degrees)");
         TSMV_CUDA(cudaSetDevice(c->device));
         cudaStream_t st = (cudaStream_t)cuda_stream;
         c->levels_dev = levels;
@@ -1143,16 +1347,14 @@ extern "C" tsmv_status tsmv_bfs_dist_begin(tsmv_ctx *c, int64_t source, int32_t 
         c->bfs_level = 0;
         TSMV_CUDA(cudaMemsetAsync(c->F1.p, 0, c->F1.bytes, st));
         R.init(source);
-        R.do_fscan(c->F0.as<uint32_t>(), nullptr);
-        TSMV_CUDA(cudaStreamSynchronize(st));
-        volatile Counters *h = c->hcnt;
-        c->m_u_local = c->nnz - h->din;
+        c->dstats.ensure(32);
+        k_source_stats<<<1, 1, 0, st>>>(source, c->row_begin, c->m, out_degrees(c), c->indeg.as<int>(),
+                                       c->dstats.as<unsigned long long>());
+        TSMV_CUDA(cudaGetLastError());
+        c->m_u_local = c->nnz;
         c->mu_dev.ensure(8);
         TSMV_CUDA(cudaMemcpyAsync(c->mu_dev.p, &c->m_u_local, 8, cudaMemcpyHostToDevice, st));
-        TSMV_CUDA(cudaStreamSynchronize(st));
-        out_stats[0] = h->fsize;
-        out_stats[1] = h->mf;
-        out_stats[2] = c->m_u_local;
+        dist_out(c, out_stats, st);
         return TSMV_OK;
     } catch (const Err &e) {
         return e.st;
@@ -1165,11 +1367,15 @@ extern "C" tsmv_status tsmv_bfs_dist_expand(tsmv_ctx *c, int32_t dir, uint32_t *
         const bool wide = (dir & TSMV_DIST_WIDE) != 0;
         dir &= ~TSMV_DIST_WIDE;
         TSMV_REQUIRE(dir >= 1 && dir <= 3, "tsmv_bfs_dist_expand: dir must be concrete (1..3)");
+        TSMV_REQUIRE(c->levels_dev != nullptr, "tsmv_bfs_dist_expand: no traversal begun (tsmv_bfs_dist_begin)");
         TSMV_CUDA(cudaSetDevice(c->device));
         cudaStream_t st = (cudaStream_t)cuda_stream;
         BfsRunner R{c, st, (long long)(c->V.bytes / 4)};
-        R.do_expand(dir, wide && dir == TSMV_DIR_PULL_CSC);
+        uint32_t *Fcur = (c->fcur == 0 ? c->F0 : c->F1).as<uint32_t>();
         uint32_t *Fnext = (c->fcur == 0 ? c->F1 : c->F0).as<uint32_t>();
+        if (dir != TSMV_DIR_PULL_CSC) R.do_fscan(Fcur, nullptr);  // push lists of the replicated frontier
+        R.do_expand(dir, wide && dir == TSMV_DIR_PULL_CSC);
+        owned_stats(c, Fnext, st);
         TSMV_CUDA(cudaMemcpyAsync(owned_words_out, Fnext + (c->row_begin >> 5), tsmv_owned_words(c) * 4,
                                   cudaMemcpyDeviceToDevice, st));
         return TSMV_OK;
@@ -1194,7 +1400,6 @@ extern "C" tsmv_status tsmv_bfs_dist_merge(tsmv_ctx *c, const uint32_t *gathered
         }
         TSMV_CUDA(cudaSetDevice(c->device));
         cudaStream_t st = (cudaStream_t)cuda_stream;
-        BfsRunner R{c, st, (long long)(c->V.bytes / 4)};
         uint32_t *Fcur = (c->fcur == 0 ? c->F0 : c->F1).as<uint32_t>();
         uint32_t *Fnext = (c->fcur == 0 ? c->F1 : c->F0).as<uint32_t>();
         if (c->opt.nranks > 1) {
@@ -1204,24 +1409,10 @@ extern "C" tsmv_status tsmv_bfs_dist_merge(tsmv_ctx *c, const uint32_t *gathered
                                                             c->V.as<uint32_t>());
             TSMV_CUDA(cudaGetLastError());
         }
-        R.do_fscan(Fnext, Fcur);
+        TSMV_CUDA(cudaMemsetAsync(Fcur, 0, ((c->n + 63) / 64) * 8, st));
         c->fcur ^= 1;
         c->bfs_level += 1;
-        if (is_device_ptr(out_stats)) {
-            // device statistics: no synchronisation here (the caller all-reduces
-            // them on the device and reads the result once per level)
-            k_dist_stats<<<1, 1, 0, st>>>(c->counters.as<Counters>(), c->mu_dev.as<long long>(), out_stats);
-            TSMV_CUDA(cudaGetLastError());
-            return TSMV_OK;
-        }
-        TSMV_CUDA(cudaStreamSynchronize(st));
-        volatile Counters *h = c->hcnt;
-        c->m_u_local -= h->din;
-        TSMV_CUDA(cudaMemcpyAsync(c->mu_dev.p, &c->m_u_local, 8, cudaMemcpyHostToDevice, st));
-        TSMV_CUDA(cudaStreamSynchronize(st));
-        out_stats[0] = h->fsize;
-        out_stats[1] = h->mf;
-        out_stats[2] = c->m_u_local;
+        dist_out(c, out_stats, st);
         return TSMV_OK;
     } catch (const Err &e) {
         return e.st;

@@ -147,9 +147,11 @@ void comm_destroy(tsmv_ctx *c) {
 }
 
 // Next frontier: every rank's owned words [row_splits[p] / 32, row_splits[p+1] / 32)
-// of F are broadcast in place from rank p (splits are multiples of 64 rows), then
-// the whole frontier is ORed into the replicated visited bitmap.
-void comm_exchange_frontier(tsmv_ctx *c, uint32_t *F, uint32_t *V, long long nwords, cudaStream_t st) {
+// of F are broadcast in place from rank p (splits are multiples of 64 rows), the
+// ranks' statistics shares (4 x u64) all-gathered in the same NCCL group, then the
+// whole frontier is ORed into the replicated visited bitmap.
+void comm_exchange_frontier(tsmv_ctx *c, uint32_t *F, uint32_t *V, long long nwords, const void *stats_send,
+                            void *stats_all, cudaStream_t st) {
     const NcclApi &N = nccl();
     ncclComm_t comm = static_cast<ncclComm_t>(c->nccl_comm);
     TSMV_NCCL(N.groupStart());
@@ -157,6 +159,8 @@ void comm_exchange_frontier(tsmv_ctx *c, uint32_t *F, uint32_t *V, long long nwo
         const long long w0 = c->row_splits[p] >> 5, w1 = (c->row_splits[p + 1] + 31) >> 5;
         if (w1 > w0) TSMV_NCCL(N.broadcast(F + w0, F + w0, (size_t)(w1 - w0), ncclUint32, p, comm, st));
     }
+    // every rank's statistics shares of the new frontier ride in the same group
+    if (stats_send) TSMV_NCCL(N.allGather(stats_send, stats_all, 4, ncclUint64, comm, st));
     TSMV_NCCL(N.groupEnd());
     k_or_words<<<grid_n(nwords), 256, 0, st>>>(V, F, nwords);
     TSMV_CUDA(cudaGetLastError());

@@ -339,6 +339,8 @@ struct tsmv_ctx {
     tsmv::DevBuf ms_src, ms_out;
     tsmv::DevBuf ms_rowneed;                // u16 per row tile: rows still missing some source
     tsmv::DevBuf mu_dev;                    // distributed BFS: m_u of this rank on the device
+    tsmv::DevBuf dstats;                    // distributed BFS: u64[4] statistics shares of the next frontier
+    tsmv::DevBuf dstats_all;                // distributed BFS: u64[nranks][4] gathered shares (comm path)
     tsmv::DevBuf par_chunks;                // BFS parents: (vertex << 24 | chunk) of heavy side rows
     long long par_nchunks = 0;
     void *trace = nullptr;         // tsmv_set_trace (device, u64[tsmv_trace_words])
@@ -393,7 +395,8 @@ bool bfs_fused_launch(tsmv_ctx *c, long long source, cudaStream_t st, bool resum
 bool has_comm(const tsmv_ctx *c);
 void comm_init(tsmv_ctx *c, const void *unique_id, cudaStream_t st);
 void comm_destroy(tsmv_ctx *c);
-void comm_exchange_frontier(tsmv_ctx *c, uint32_t *F, uint32_t *V, long long nwords, cudaStream_t st);
+void comm_exchange_frontier(tsmv_ctx *c, uint32_t *F, uint32_t *V, long long nwords, const void *stats_send,
+                            void *stats_all, cudaStream_t st);
 long long comm_gather_x(tsmv_ctx *c, long long k_local, const int32_t *x_idx, const void *x_val, size_t vb,
                         const int32_t **xi_out, const void **xv_out, cudaStream_t st);
 // bfs.cu

@@ -154,14 +154,15 @@ def exchange_frontier(owned_words: torch.Tensor, stride: int, group=None) -> tor
 
 def bfs_loop(engine, source: int, group=None) -> int:
     """Level-synchronous distributed TileBFS driver (Alg 3, one
-    exchange per level).  `engine` provides begin(source) -> (|F|, m_f, m_u) local,
-    expand(dir) -> owned words, merge(gathered, stride) -> (|F|, m_f, m_u),
-    stride (padded words), n, choose(n, |F|, m_f, m_u).  Returns the number of levels."""
+    exchange per level).  `engine` provides begin(source) -> this rank's shares
+    (|F|, m_f, m_u) of its own rows, expand(dir) -> owned words, merge(gathered,
+    stride) -> shares, stride (padded words), n, choose(n, |F|, m_f, m_u).  The three
+    shares are summed over the ranks (one all-reduce per level), so every rank
+    decides the direction on the same global numbers.  Returns the number of levels."""
     dev = engine.device
-    f, mf, mu = engine.begin(source)
-    red = torch.tensor([mf, mu], dtype=torch.int64, device=dev)
+    red = torch.tensor(list(engine.begin(source)), dtype=torch.int64, device=dev)
     dist.all_reduce(red, group=group)
-    gmf, gmu = (int(x) for x in red.tolist())
+    f, gmf, gmu = (int(x) for x in red.tolist())
     levels = 0
     while f > 0:
         d = engine.choose(engine.n, f, gmf, gmu)
@@ -171,15 +172,11 @@ def bfs_loop(engine, source: int, group=None) -> int:
         gathered = exchange_frontier(owned, engine.stride, group)
         if hasattr(engine, "merge_dev"):
             # statistics stay on the device: one all-reduce, one read per level
-            st = engine.merge_dev(gathered, engine.stride)
-            red = st[1:3].clone()
-            dist.all_reduce(red, group=group)
-            f, gmf, gmu = (int(x) for x in torch.cat([st[:1], red]).tolist())
+            red = engine.merge_dev(gathered, engine.stride).clone()
         else:
-            f, mf, mu = engine.merge(gathered, engine.stride)
-            red = torch.tensor([mf, mu], dtype=torch.int64, device=dev)
-            dist.all_reduce(red, group=group)
-            gmf, gmu = (int(x) for x in red.tolist())
+            red = torch.tensor(list(engine.merge(gathered, engine.stride)), dtype=torch.int64, device=dev)
+        dist.all_reduce(red, group=group)
+        f, gmf, gmu = (int(x) for x in red.tolist())
         levels += 1
     return levels
 
@@ -208,10 +205,29 @@ class DistTiledMatrix:
         # 0 (no hint) when there is no process group (simulated ranks)
         self.nnz_total = 0
         if dist.is_available() and dist.is_initialized():
-            tot = torch.tensor([int(A_local.nnz)], dtype=torch.int64,
-                               device=self.device if dist.get_backend(group) == "nccl" else "cpu")
+            on = self.device if dist.get_backend(group) == "nccl" else "cpu"
+            tot = torch.tensor([int(A_local.nnz)], dtype=torch.int64, device=on)
             dist.all_reduce(tot, group=group)
             self.nnz_total = int(tot)
+            # global out-degrees: the column counts of all row blocks (m_f of Alg 3's
+            # direction rule counts every block's edges of a frontier vertex)
+            deg = self.column_counts(A_local).to(on)
+            dist.all_reduce(deg, group=group)
+            self.set_degrees(deg)
+
+    @staticmethod
+    def column_counts(A_local) -> torch.Tensor:
+        """int32[n] column counts of this row block (host-side marshalling for
+        set_degrees; summed over the ranks they are the global out-degrees)."""
+        ci = A_local.col_idx.to(torch.int64)
+        return torch.bincount(ci, minlength=A_local.n).to(torch.int32)
+
+    def set_degrees(self, outdeg_global: torch.Tensor):
+        """Global out-degrees (int32[n]) for the direction statistics; set by the
+        constructor when a process group exists, by the caller for simulated ranks."""
+        d = outdeg_global.to(device=self.device, dtype=torch.int32).contiguous()
+        self.tsmv.check(self.tsmv.tsmv_bfs_dist_set_degrees(self.M.ctx, d.data_ptr()),
+                        "tsmv_bfs_dist_set_degrees")
 
     # ---- SpMSpV: x entries are distributed by owner (x_idx in this rank's row range)
     def spmspv(self, x_idx_owned: torch.Tensor, x_val_owned: Optional[torch.Tensor], semiring="plus_times"):

@@ -88,6 +88,7 @@ _SIGS = {
     "tsmv_bfs_parents": (ctypes.c_int, [_vp, _vp, _vp, _vp]),
     "tsmv_msbfs": (ctypes.c_int, [_vp, _i32, _vp, _vp, ctypes.POINTER(tsmv_msbfs_stats), _vp]),
     "tsmv_bfs_dist_begin": (ctypes.c_int, [_vp, _i64, _vp, ctypes.POINTER(_i64), _vp]),
+    "tsmv_bfs_dist_set_degrees": (ctypes.c_int, [_vp, _vp]),
     "tsmv_bfs_dist_expand": (ctypes.c_int, [_vp, _i32, _vp, _vp]),
     "tsmv_bfs_dist_merge": (ctypes.c_int, [_vp, _vp, _i64, ctypes.POINTER(_i64), _vp]),
     "tsmv_owned_words": (_i64, [_vp]),

@@ -73,7 +73,8 @@ class NumpyEngine:
         self.r0, self.r1 = splits[rank], splits[rank + 1]
         Al = D.local_rows(A, splits, rank)
         self.B = sp.csr_matrix((np.ones(Al.nnz), Al.col_idx.numpy(), Al.row_ptr.numpy()), shape=(Al.m, A.n))
-        self.outdeg = np.asarray(self.B.sum(axis=0)).ravel().astype(np.int64)
+        # global out-degrees (column counts of all blocks), as tsmv_bfs_dist_set_degrees
+        self.outdeg = np.bincount(A.col_idx.numpy(), minlength=A.n).astype(np.int64)
         self.indeg = np.diff(Al.row_ptr.numpy()).astype(np.int64)
         self.stride = max((splits[p + 1] - splits[p] + 31) // 32 for p in range(len(splits) - 1))
         self.device = torch.device("cpu")
@@ -85,8 +86,11 @@ class NumpyEngine:
         return self.tsmv.choose_dir(n, f, mf, mu)
 
     def _stats(self):
+        # this rank's shares over its own rows (the libtsmv r2 semantics); bfs_loop sums them
+        own_f = self.F[self.r0:self.r1]
         own_unvisited = ~self.V[self.r0:self.r1]
-        return int(self.F.sum()), int(self.outdeg[self.F].sum()), int(self.indeg[own_unvisited].sum())
+        return (int(own_f.sum()), int(self.outdeg[self.r0:self.r1][own_f].sum()),
+                int(self.indeg[own_unvisited].sum()))
 
     def begin(self, s):
         self.V = np.zeros(self.n, bool)

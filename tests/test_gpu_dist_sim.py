@@ -22,16 +22,39 @@ def _ranks(A, P, dtype="pattern", **opts):
         if dtype == "pattern":
             Al = Al.with_values(None)
         engines.append(D.DistTiledMatrix(Al, splits, r, P, dtype=dtype, **opts))
+    # no process group: the caller hands every rank the global out-degrees
+    deg = sum(D.DistTiledMatrix.column_counts(D.local_rows(A, splits, r)).to(torch.int64) for r in range(P))
+    for e in engines:
+        e.set_degrees(deg.to(torch.int32))
     return splits, engines
 
 
-def _sim_bfs(engines, source, dev_stats=False):
+def _level_stats(A, lv):
+    """(|F|, m_f, m_u) of every level from the oracle's levels: F = vertices of the
+    level, m_f = their out-degrees (column counts), m_u = in-degrees (row lengths)
+    of the vertices still unvisited after it (Alg 3's direction statistics)."""
+    outdeg = np.bincount(A.col_idx.numpy(), minlength=A.n)
+    indeg = np.diff(A.row_ptr.numpy())
+    out = []
+    for L in range(int(lv.max()) + 1):
+        fr = lv == L
+        unv = (lv < 0) | (lv > L)
+        out.append((int(fr.sum()), int(outdeg[fr].sum()), int(indeg[unv].sum())))
+    return out
+
+
+def _sim_bfs(engines, source, dev_stats=False, expect=None):
     st = [e.begin(source) for e in engines]
-    while st[0][0] > 0:
-        assert len({s[0] for s in st}) == 1          # |F| identical on every rank
+    level = 0
+    while sum(s[0] for s in st) > 0:
+        # every rank returns its shares over its own rows; the sums are the global numbers
+        f = sum(s[0] for s in st)
         mf = sum(s[1] for s in st)
         mu = sum(s[2] for s in st)
-        d = engines[0].choose(engines[0].n, st[0][0], mf, mu)
+        if expect is not None:
+            assert (f, mf, mu) == expect[level], level
+        level += 1
+        d = engines[0].choose(engines[0].n, f, mf, mu)
         nnz = sum(e.M.nnz for e in engines)
         owned = [e.expand(d, wide=mu * 4 < nnz).clone() for e in engines]   # late-pull hint as bfs_loop
         stride = engines[0].stride
@@ -52,7 +75,8 @@ def test_sim_ranks_bfs(P, sym):
     C = oracle.csc_of(A)
     _, engines = _ranks(A, P)
     for s in [0] + synth.sample_sources(A, 2, seed=2):
-        assert np.array_equal(_sim_bfs(engines, s), oracle.bfs_queue(C, s))
+        ref = oracle.bfs_queue(C, s)
+        assert np.array_equal(_sim_bfs(engines, s, expect=_level_stats(A, ref)), ref)
 
 
 @pytest.mark.parametrize("force", [1, 2, 3])

@@ -66,7 +66,9 @@ typedef struct {
     int32_t sparse_tile_max_nnz; /* tiles with <= this many nonzeros go to the side
                                     matrix (R12); default 2; 0 = none */
     int32_t build_bfs;           /* 1 = also build the TileBFS bitmask tiles (square A);
-                                    default 1 when nrows == ncols and nranks == 1 */
+                                    default 1 when nrows == ncols and nranks == 1;
+                                    2 = a 2D-partition block A_ij (any shape, nranks 1):
+                                    the structures serve tsmv_bfs2d_expand only */
     double push_csr_density;     /* |F|/n threshold Push-CSC -> Push-CSR; the paper's is 0.01
                                     (P:1423-1433); default 0.05, measured on B200 */
     double pull_alpha;           /* Pull-CSC when m_f > m_u / alpha (R9); Beamer's 14; default 2,
@@ -300,6 +302,53 @@ tsmv_status tsmv_bfs_dist_merge(tsmv_ctx *c, const uint32_t *gathered, int64_t s
                                 int64_t *out_stats, void *cuda_stream);
 /* Words of this rank's owned segment = ceil((row_splits[r+1]-row_splits[r])/32). */
 int64_t tsmv_owned_words(const tsmv_ctx *c);
+
+/* ---- 2D-partitioned TileBFS steps (Alg 3 P:418-430 with the
+ * OR-AND semiring of P:1373-1379; DESIGN.md §8 "2D") ----
+ * Rank (i, j) of a Pr x Pc grid holds A_ij = A[R_i, C_j] as an ordinary context
+ * (nranks = 1, local row ids 0..|R_i|-1, local column ids of C_j's padded column
+ * space).  A level: y = A_ij x_j by tsmv_spmspv(_async) with TSMV_OR_AND, then
+ *   tsmv_bfs2d_scatter : y's local row ids (y_idx[0 .. *y_nnz), device, *y_nnz on
+ *       the device, at most y_cap read) -> bitmap words[nwords] over R_i (zeroed
+ *       first; bit r % 32 of word r / 32); nwords >= ceil(rows / 32);
+ *   caller: all-to-all in processor row i of the words of each sub-piece R_ij';
+ *   tsmv_bfs2d_merge : OR of nseg partial bitmaps segs[p * stride_words + w] of this
+ *       rank's nverts = |R_ij| vertices; new = OR & ~visited; visited |= new;
+ *       levels[v] = level for new v; front_out[w] = new words; stats_dev (device
+ *       int64[3], no synchronisation) = { |new|, sum outdeg[v], sum indeg[v] } over
+ *       the new v (outdeg / indeg int32[nverts] of this rank's vertices, GLOBAL
+ *       degrees, may be NULL: sum 0) -- the shares of Alg 3's |F|, m_f and the m_u
+ *       decrement, summed over the ranks by the caller;
+ *   caller: all-gather in processor column j of the front words -> C_j's bitmap;
+ *   tsmv_bfs2d_list : bitmap words (nbits bits) -> ascending ids idx_out[0..count);
+ *       count_out host (the call synchronises the stream) or device.
+ * Direction-optimising levels (context built with build_bfs = 2) replace the
+ * SpMSpV + scatter by
+ *   tsmv_bfs2d_expand : dir 1..3 (| TSMV_DIST_WIDE for late pull levels), decided
+ *       by the caller from the summed statistics (tsmv_choose_dir); x_words = C_j's
+ *       frontier bitmap (ceil(ncols / 32) words), row_new (may be NULL) = R_i's
+ *       bitmap of the vertices found by the previous level (the processor-row
+ *       all-gather of the owners' front words) ORed into visited_rows first;
+ *       visited_rows = R_i's visited bitmap (ceil(nrows / 32) words; the pull level
+ *       tests and the discoveries update it); next_words = the partial bitmap of
+ *       R_i found by this block (zeroed first; the all-to-all send buffer);
+ *       levels_rows int32[nrows] scratch (discoveries write level + 1).
+ *       Push-CSC (Alg 5), Push-CSR (Alg 6) and Pull-CSC (Alg 7) run the level kernels
+ *       of the row-block path on the block's own tiles.
+ * All buffers are the caller's device memory; the context supplies the device, the
+ * stream's scratch (bfs2d_list) and the SM count.  Errors: EINVAL on NULL / host
+ * pointers or inconsistent sizes. */
+tsmv_status tsmv_bfs2d_scatter(tsmv_ctx *c, const int32_t *y_idx, const int64_t *y_nnz, int64_t y_cap,
+                               uint32_t *words, int64_t nwords, void *cuda_stream);
+tsmv_status tsmv_bfs2d_merge(tsmv_ctx *c, const uint32_t *segs, int32_t nseg, int64_t stride_words,
+                             int64_t nverts, uint32_t *visited, int32_t *levels, int32_t level,
+                             uint32_t *front_out, const int32_t *outdeg, const int32_t *indeg,
+                             int64_t *stats_dev, void *cuda_stream);
+tsmv_status tsmv_bfs2d_expand(tsmv_ctx *c, int32_t dir, const uint32_t *x_words, const uint32_t *row_new,
+                              uint32_t *visited_rows, uint32_t *next_words, int32_t *levels_rows,
+                              int32_t level, void *cuda_stream);
+tsmv_status tsmv_bfs2d_list(tsmv_ctx *c, const uint32_t *words, int64_t nbits, int32_t *idx_out,
+                            int64_t *count_out, void *cuda_stream);
 
 /* Direction rule of reading R9: PULL_CSC if m_f > m_u / pull_alpha,
  * else PUSH_CSR if frontier / n >= push_csr_density, else PUSH_CSC; force_dir wins

@@ -203,9 +203,12 @@ extern "C" tsmv_status tsmv_create(tsmv_ctx **out, int64_t nrows, int64_t ncols,
             c->row_begin = 0;
         }
         bool square_global = (o.nranks == 1) ? (nrows == ncols) : true;
+        const bool block2d = o.build_bfs == 2;
+        TSMV_REQUIRE(!block2d || o.nranks == 1, "tsmv_create: build_bfs = 2 (2D block) needs nranks == 1");
         bool want_bfs = o.build_bfs < 0 ? square_global : o.build_bfs != 0;
-        TSMV_REQUIRE(!want_bfs || square_global, "tsmv_create: build_bfs needs a square matrix");
-        c->opt.build_bfs = want_bfs ? 1 : 0;
+        TSMV_REQUIRE(!want_bfs || square_global || block2d, "tsmv_create: build_bfs needs a square matrix");
+        c->opt.build_bfs = block2d ? 2 : want_bfs ? 1 : 0;
+        c->bfs_block2d = block2d;
 
         TSMV_CUDA(cudaSetDevice(c->device));
         // device inputs may still be in flight on the caller's streams
@@ -263,7 +266,7 @@ extern "C" tsmv_status tsmv_create(tsmv_ctx **out, int64_t nrows, int64_t ncols,
         c->nTR = c->P.nTR;
         c->nTC = c->P.nTC;
         if (want_bfs) {
-            c->symmetric = (o.nranks == 1) && same_pattern_transposed(c, d_rows.as<int32_t>(), ci, nnz, st);
+            c->symmetric = (o.nranks == 1) && !block2d && same_pattern_transposed(c, d_rows.as<int32_t>(), ci, nnz, st);
             if (c->symmetric) {
                 c->Q = &c->P;
             } else {
@@ -323,7 +326,7 @@ extern "C" tsmv_status tsmv_create(tsmv_ctx **out, int64_t nrows, int64_t ncols,
             TSMV_REQUIRE(fl >= 1, "tsmv_create: flat SpMSpV kernel cannot be resident (occupancy 0)");
             c->flat_blocks = std::min(c->sm_count, 256);  // one 1024-thread CTA per SM (MAXG)
         }
-        if (want_bfs && o.nranks == 1) {
+        if (want_bfs && o.nranks == 1 && !block2d) {
             int bo = bfs_fused_occupancy(c->nt);
             TSMV_REQUIRE(bo >= 1, "tsmv_create: fused BFS kernel cannot be resident (occupancy 0)");
             c->bfs_blocks = c->sm_count * std::min(bo, 2);

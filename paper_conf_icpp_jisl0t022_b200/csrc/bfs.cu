@@ -784,6 +784,23 @@ __global__ void k_dist_stats2(const unsigned long long *__restrict__ dstats, lon
     out[2] = m;
 }
 
+// 2D block level prologue (tsmv_bfs2d_expand)
+__global__ void k_level2d_prep(uint32_t *__restrict__ V, const uint32_t *__restrict__ rnew, uint32_t *__restrict__ Fn,
+                               long long nwr, uint32_t *__restrict__ F, const uint32_t *__restrict__ x, long long nwx,
+                               long long nwpad) {
+    for (long long w = blockIdx.x * (long long)blockDim.x + threadIdx.x; w < max(nwr, nwpad);
+         w += (long long)gridDim.x * blockDim.x) {
+        if (w < nwr) {
+            if (rnew) {
+                const uint32_t b = rnew[w];
+                if (b) V[w] |= b;
+            }
+            Fn[w] = 0u;
+        }
+        if (w < nwpad) F[w] = w < nwx ? x[w] : 0u;
+    }
+}
+
 __global__ void k_merge(const uint32_t *__restrict__ gathered, long long stride, int nranks,
                         const long long *__restrict__ splits, int self, uint32_t *__restrict__ Fn,
                         uint32_t *__restrict__ V) {
@@ -816,8 +833,10 @@ struct BfsRunner {
     tsmv_ctx *c;
     cudaStream_t st;
     long long NW;
+    const BfsView *ov = nullptr;  // 2D block levels: caller-provided row / column bitmaps
 
     BfsView view() {
+        if (ov) return *ov;
         BfsView B;
         B.V = c->V.as<uint32_t>();
         B.F = (c->fcur == 0 ? c->F0 : c->F1).as<uint32_t>();
@@ -967,6 +986,7 @@ using namespace tsmv;
 
 static void bfs_check(tsmv_ctx *c) {
     TSMV_REQUIRE(c->bfs_built, "tsmv_bfs: context built without BFS structures (square A and build_bfs=1 needed)");
+    TSMV_REQUIRE(!c->bfs_block2d, "tsmv_bfs: a 2D block context (build_bfs = 2) serves tsmv_bfs2d_expand only");
 }
 
 static void bfs_prepare_levels(tsmv_ctx *c, int32_t *levels, bool &host_levels) {
@@ -1378,6 +1398,49 @@ extern "C" tsmv_status tsmv_bfs_dist_expand(tsmv_ctx *c, int32_t dir, uint32_t *
         owned_stats(c, Fnext, st);
         TSMV_CUDA(cudaMemcpyAsync(owned_words_out, Fnext + (c->row_begin >> 5), tsmv_owned_words(c) * 4,
                                   cudaMemcpyDeviceToDevice, st));
+        return TSMV_OK;
+    } catch (const Err &e) {
+        return e.st;
+    }
+}
+
+// 2D block level (bfs2d.cu's sequence, include/tsmv.h): the level kernels of the
+// row-block path on caller-provided row bitmaps (visited / next over R_i) and the
+// column frontier of C_j staged in F0 (zero-padded to whole 16-byte vectors)
+extern "C" tsmv_status tsmv_bfs2d_expand(tsmv_ctx *c, int32_t dir, const uint32_t *x_words, const uint32_t *row_new,
+                                         uint32_t *visited_rows, uint32_t *next_words, int32_t *levels_rows,
+                                         int32_t level, void *cuda_stream) {
+    try {
+        TSMV_REQUIRE(c && x_words && visited_rows && next_words && levels_rows, "tsmv_bfs2d_expand: NULL argument");
+        TSMV_REQUIRE(c->bfs_built && c->bfs_block2d, "tsmv_bfs2d_expand: context not built with build_bfs = 2");
+        const bool wide = (dir & TSMV_DIST_WIDE) != 0;
+        dir &= ~TSMV_DIST_WIDE;
+        TSMV_REQUIRE(dir >= 1 && dir <= 3, "tsmv_bfs2d_expand: dir must be concrete (1..3)");
+        TSMV_REQUIRE(is_device_ptr(x_words) && (!row_new || is_device_ptr(row_new)) && is_device_ptr(visited_rows) &&
+                         is_device_ptr(next_words) && is_device_ptr(levels_rows),
+                     "tsmv_bfs2d_expand: device memory expected");
+        TSMV_CUDA(cudaSetDevice(c->device));
+        cudaStream_t st = (cudaStream_t)cuda_stream;
+        const long long nwr = (c->m + 31) / 32, nwx = (c->n + 31) / 32, nwpad = (long long)(c->V.bytes / 4);
+        uint32_t *F = c->F0.as<uint32_t>();
+        // one launch: visited_rows |= row_new, next_words = 0, F0 = x (zero-padded)
+        k_level2d_prep<<<grid_for(std::max(nwr, nwpad)), 256, 0, st>>>(visited_rows, row_new, next_words, nwr, F,
+                                                                        x_words, nwx, nwpad);
+        TSMV_CUDA(cudaGetLastError());
+        ensure_lists(c, c->n);
+        BfsView B;
+        B.V = visited_rows;
+        B.F = F;
+        B.Fn = next_words;
+        B.levels = levels_rows;
+        B.row_begin = 0;
+        B.m_local = c->m;
+        B.n = c->n;
+        B.level = level;
+        BfsRunner R{c, st, nwpad};
+        R.ov = &B;
+        if (dir != TSMV_DIR_PULL_CSC) R.do_fscan(F, nullptr);
+        R.do_expand(dir, wide && dir == TSMV_DIR_PULL_CSC);
         return TSMV_OK;
     } catch (const Err &e) {
         return e.st;

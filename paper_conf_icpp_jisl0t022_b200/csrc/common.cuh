@@ -341,6 +341,8 @@ struct tsmv_ctx {
     tsmv::DevBuf mu_dev;                    // distributed BFS: m_u of this rank on the device
     tsmv::DevBuf dstats;                    // distributed BFS: u64[4] statistics shares of the next frontier
     tsmv::DevBuf dstats_all;                // distributed BFS: u64[nranks][4] gathered shares (comm path)
+    tsmv::DevBuf b2d_bsum, b2d_boff, b2d_total, b2d_temp;  // 2D BFS bitmap -> list scratch (bfs2d.cu)
+    bool bfs_block2d = false;               // build_bfs = 2: a 2D-partition block (bfs2d only)
     tsmv::DevBuf par_chunks;                // BFS parents: (vertex << 24 | chunk) of heavy side rows
     long long par_nchunks = 0;
     void *trace = nullptr;         // tsmv_set_trace (device, u64[tsmv_trace_words])

@@ -89,6 +89,10 @@ _SIGS = {
     "tsmv_msbfs": (ctypes.c_int, [_vp, _i32, _vp, _vp, ctypes.POINTER(tsmv_msbfs_stats), _vp]),
     "tsmv_bfs_dist_begin": (ctypes.c_int, [_vp, _i64, _vp, ctypes.POINTER(_i64), _vp]),
     "tsmv_bfs_dist_set_degrees": (ctypes.c_int, [_vp, _vp]),
+    "tsmv_bfs2d_scatter": (ctypes.c_int, [_vp, _vp, _vp, _i64, _vp, _i64, _vp]),
+    "tsmv_bfs2d_merge": (ctypes.c_int, [_vp, _vp, _i32, _i64, _i64, _vp, _vp, _i32, _vp, _vp, _vp, _vp, _vp]),
+    "tsmv_bfs2d_expand": (ctypes.c_int, [_vp, _i32, _vp, _vp, _vp, _vp, _vp, _i32, _vp]),
+    "tsmv_bfs2d_list": (ctypes.c_int, [_vp, _vp, _i64, _vp, _vp, _vp]),
     "tsmv_bfs_dist_expand": (ctypes.c_int, [_vp, _i32, _vp, _vp]),
     "tsmv_bfs_dist_merge": (ctypes.c_int, [_vp, _vp, _i64, ctypes.POINTER(_i64), _vp]),
     "tsmv_owned_words": (_i64, [_vp]),

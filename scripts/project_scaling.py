@@ -36,11 +36,12 @@ ap.add_argument("--nccl-us", type=float, default=20.0)
 ap.add_argument("--link-gbs", type=float, default=770.0)
 ap.add_argument("--sources", type=int, default=4)
 ap.add_argument("--thr", type=int, default=8)
+ap.add_argument("--permute", action="store_true")
 args = ap.parse_args()
 dev = torch.device("cuda", 0)
-A = synth.rmat(args.scale, 16, seed=1, symmetrize=True, device=dev)
+A = synth.rmat(args.scale, 16, seed=1, symmetrize=True, device=dev, permute=args.permute)
 srcs = [0] + synth.sample_sources(A, args.sources - 1, seed=1)
-out = {"graph": f"rmat_s{args.scale}_ef16_sym", "nnz": A.nnz, "assumptions": {
+out = {"graph": f"rmat_s{args.scale}_ef16_sym" + ("_permuted" if args.permute else ""), "nnz": A.nnz, "assumptions": {
     "nccl_latency_us_per_level": args.nccl_us, "link_GBps": args.link_gbs}, "runs": {}}
 
 # one-GPU fused traversal for reference

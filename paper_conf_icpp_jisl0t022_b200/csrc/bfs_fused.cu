@@ -41,8 +41,8 @@ constexpr int LIST_MAXW = 512;   // list levels only while every frontier vertex
 #define TSMV_QCAP 2048
 #endif
 constexpr int QCAP = TSMV_QCAP;  // per-CTA shared-memory queue of discovered vertices
-constexpr int SOLO_QS = 2048;    // solo levels: frontier lists in shared memory
-constexpr int SOLO_ROUNDS = 4;   // solo while |F| x group size <= SOLO_ROUNDS x BFB
+constexpr int SOLO_QS = BFB;     // solo levels: frontier records in shared memory (one per thread)
+constexpr int SOLO_ITEMS = 4 * BFB;  // solo while the level's push work <= 4 items per thread
 
 struct BfsFusedArgs {
     BfsTiles P, Q;
@@ -71,10 +71,17 @@ struct BfsFusedArgs {
     int use_list, use_solo;
     int qcap;                 // usable entries of the shared-memory queue (<= QCAP; TSMV_BFS_QCAP tests the overflow path)
     int wide_in_kernel;       // pull levels with m_u < nnz / 4 stay in the kernel (wide pull)
+    // r2: L2 warm-up of the push structures + degrees (graphs whose structures fit
+    // in half the L2): bulk L2 prefetches by every CTA before the first level, so the
+    // latency-bound list / solo levels of high-diameter graphs hit L2, not HBM
+    const void *pf_p[8];
+    long long pf_b[8];
+    int pf_n;
 };
+constexpr long long PF_CHUNK = 8192;
 
 struct SoloShared {
-    int cnt, pad;
+    int cnt, W;
     unsigned long long mf, din;
     int maxw, pad2;
 };
@@ -292,80 +299,179 @@ __device__ __forceinline__ void seg_counts(const BfsFusedArgs &a, const uint32_t
     }
 }
 
-// Solo levels (session 3): while the frontier is small (|F| x G <= SOLO_ROUNDS x
-// BFB), CTA 0 alone runs the list levels with the vertex lists in shared memory
-// and __syncthreads instead of grid barriers; the other CTAs wait on a release
-// flag.  A level is then: list entry (smem) -> column ranges -> plane words ->
-// atomicOr V -> smem queue -> degrees of the new vertices (~4 dependent L2
-// accesses instead of ~7 plus a grid barrier).  On exit the next frontier is
-// left in the global list and its counter slot, exactly as a grid list level
-// leaves it.  Entry: level L already counted (mu, reached, edges, dir_out).
+// Solo levels (session 3; r2 restructured): while the frontier is small, CTA 0
+// alone runs the list levels with the level in shared memory and __syncthreads
+// instead of grid barriers; the other CTAs wait on a release flag.  r2: a
+// frontier entry is a 16-byte record {v, tile start, side start, tile count,
+// side count} built when v is discovered, in the same pass (and the same memory
+// latency) as v's degrees, and the level's push work is flattened into an item
+// map (item -> entry), so a level is
+//   items (smem) -> up to 4 plane / side words per thread, loads issued together
+//   -> atomicOr V -> next ids (smem) -> __syncthreads
+//   -> per new vertex: degrees + column starts (one latency) -> records, block
+//      scan of the work, item map -> __syncthreads,
+// three dependent global round trips per level instead of seven.  On exit the
+// next frontier is left in the global list and its counter slot, exactly as a
+// grid list level leaves it.  Entry: level L already counted (mu, reached,
+// edges, dir_out); |F| <= SOLO_QS and |F| x max work <= SOLO_ITEMS.
+struct SoloRec {
+    int v;
+    unsigned t0, s0;              // tile / side starts (< 2^32: use_solo checks)
+    unsigned short ntl, ns;       // tile / side counts (<= LIST_MAXW)
+};
+struct SoloBuf {
+    SoloRec rec[SOLO_QS];
+    int pre[SOLO_QS];             // exclusive prefix of the entries' work
+    int nq[SOLO_QS];              // ids found by the level (next frontier)
+    unsigned long long part_mf[BFB / 32], part_din[BFB / 32];
+    int part_mx[BFB / 32];
+    unsigned short item[SOLO_ITEMS];
+    cub::BlockScan<int, BFB>::TempStorage scan;
+};
+
+// records + item map of the n <= SOLO_QS entries ids[0..n); with `stats` also the
+// level's degree sums (ss.mf, ss.din) and the maximum work (ss.maxw); ss.W = items
+template <int NT>
+__device__ void solo_records(const BfsFusedArgs &a, const int *ids, bool ids_global, long long n, SoloBuf &sb,
+                             SoloShared &ss, int tid, long long &out_mf, long long &out_din, long long &out_mx) {
+    int w = 0;
+    unsigned long long mf = 0, din = 0;
+    if (tid < n) {
+        const int v = ids_global ? __ldcg(&ids[tid]) : ids[tid];
+        const long long J = v / NT;
+        const long long t0 = a.P.ptr[J], t1 = a.P.ptr[J + 1];
+        const long long s0 = a.P.sptr[v], s1 = a.P.sptr[v + 1];
+        mf = (unsigned long long)a.outdeg[v];
+        din = (unsigned long long)a.indeg[v];
+        SoloRec r;
+        r.v = v;
+        r.t0 = (unsigned)t0;
+        r.s0 = (unsigned)s0;
+        r.ntl = (unsigned short)min(t1 - t0, 65535LL);
+        r.ns = (unsigned short)min(s1 - s0, 65535LL);
+        sb.rec[tid] = r;
+        w = (int)min((t1 - t0) + (s1 - s0), (long long)INT_MAX / 4);
+    }
+    {
+        // warp partials (no 64-bit shared atomics: they serialised the level)
+        int mx = w;
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) {
+            mf += __shfl_xor_sync(0xffffffffu, mf, o);
+            din += __shfl_xor_sync(0xffffffffu, din, o);
+            mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+        }
+        if ((tid & 31) == 0) {
+            sb.part_mf[tid >> 5] = mf;
+            sb.part_din[tid >> 5] = din;
+            sb.part_mx[tid >> 5] = mx;
+        }
+    }
+    int pre, tot;
+    cub::BlockScan<int, BFB>(sb.scan).ExclusiveSum(w, pre, tot);
+    if (tid < n) sb.pre[tid] = pre;
+    if (tot <= SOLO_ITEMS)
+        for (int k = 0; k < w; ++k) sb.item[pre + k] = (unsigned short)tid;
+    if (tid == 0) ss.W = tot;
+    __syncthreads();
+    // every thread sums the partials itself (broadcast reads, no further barrier)
+    unsigned long long smf = 0, sdin = 0;
+    int smx = 0;
+#pragma unroll
+    for (int i = 0; i < BFB / 32; ++i) {
+        smf += sb.part_mf[i];
+        sdin += sb.part_din[i];
+        smx = max(smx, sb.part_mx[i]);
+    }
+    out_mf = (long long)smf;
+    out_din = (long long)sdin;
+    out_mx = smx;
+}
+
 template <int NT>
 __device__ void solo_levels(const BfsFusedArgs &a, BfsView &B, int &level, long long &mu, long long &reached,
-                            long long &edges, long long fsize, long long maxw, int (*q)[SOLO_QS], SoloShared &ss,
-                            int tid) {
+                            long long &edges, long long fsize, SoloBuf &sb, SoloShared &ss, int tid) {
     using word_t = typename Tr<NT>::word_t;
     const word_t *planes = (const word_t *)a.P.planes;
-    {
-        const int *Qc = (level & 1) ? a.bq1 : a.bq0;
-        for (int i = tid; i < fsize; i += BFB) q[0][i] = __ldcg(&Qc[i]);
-    }
-    int cur = 0;
+    long long mf2, din2, mx2;
+    solo_records<NT>(a, (level & 1) ? a.bq1 : a.bq0, true, fsize, sb, ss, tid, mf2, din2, mx2);
     long long n = fsize;
-    int G = 1;
-    while (G < maxw && G < 32) G <<= 1;
+#ifdef TSMV_SOLO_PROF
+    long long pc[5] = {0, 0, 0, 0, 0}, nlev = 0, c0 = clock64(), c1;
+#define SOLO_T(i) (c1 = clock64(), pc[i] += c1 - c0, c0 = c1)
+#else
+#define SOLO_T(i)
+#endif
     while (true) {
         B.level = level;
         int *Qn = (level & 1) ? a.bq0 : a.bq1;  // list of level + 1 (overflow beyond SOLO_QS)
+        const int W = ss.W;
+        __syncthreads();  // every thread has read W before ss is reset
         if (tid == 0) {
             ss.cnt = 0;
             ss.mf = 0;
             ss.din = 0;
             ss.maxw = 0;
         }
-        __syncthreads();
-        const int gl = tid % G;
-        for (long long i = tid / G; i < n; i += BFB / G) {
-            const long long u = q[cur][i];
-            const long long J = u / NT;
-            const int c = (int)(u % NT);
-            const long long t0 = a.P.ptr[J], ntl = a.P.ptr[J + 1] - t0;
-            const long long s0 = a.P.sptr[u], ns = a.P.sptr[u + 1] - s0;
-            for (long long k = gl; k < ntl + ns; k += G) {
-                long long gseg;
-                word_t bits;
-                if (k < ntl) {
-                    const long long t = t0 + k;
-                    bits = planes[(long long)c * a.P.T + t];
-                    gseg = a.P.trow[t];
+        // ---- expand: item e = tid + k * BFB, k < 4 (W <= SOLO_ITEMS = 4 BFB)
+        word_t bits[4];
+        long long gseg[4];
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+            bits[k] = 0;
+            gseg[k] = 0;
+            const int e = tid + k * BFB;
+            if (e < W) {
+                const int i = sb.item[e];
+                const SoloRec r = sb.rec[i];
+                const int kk = e - sb.pre[i];
+                const int c = r.v % NT;
+                if (kk < r.ntl) {
+                    const long long t = (long long)r.t0 + kk;
+                    bits[k] = planes[(long long)c * a.P.T + t];
+                    gseg[k] = a.P.trow[t];
                 } else {
-                    const long long v = decode_row<NT>(a.P.srow[s0 + (k - ntl)], a.P.hot_list);
-                    bits = (word_t)1 << (v % NT);
-                    gseg = v / NT;
-                }
-                if (!bits) continue;
-                const word_t old = seg_or<NT>(B.V, gseg, bits);
-                word_t nw = bits & ~old;
-                if (!nw) continue;
-                int p = atomicAdd(&ss.cnt, popc_w(nw));
-                while (nw) {
-                    const int r = ffs_w(nw);
-                    nw &= nw - 1;
-                    const long long v = gseg * NT + r;
-                    B.levels[v] = level + 1;
-                    if (p < SOLO_QS) q[cur ^ 1][p] = (int)v;
-                    else Qn[p] = (int)v;
-                    ++p;
+                    const long long v = decode_row<NT>(a.P.srow[(long long)r.s0 + (kk - r.ntl)], a.P.hot_list);
+                    bits[k] = (word_t)1 << (v % NT);
+                    gseg[k] = v / NT;
                 }
             }
         }
+        __syncthreads();  // ss reset visible; records / items no longer read after the loads
+        SOLO_T(0);
+        // all of a thread's atomics first (independent round trips in flight
+        // together), then the discoveries
+        word_t olds[4];
+#pragma unroll
+        for (int k = 0; k < 4; ++k) olds[k] = bits[k] ? seg_or<NT>(B.V, gseg[k], bits[k]) : bits[k];
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+            word_t nw = bits[k] & ~olds[k];
+            if (!nw) continue;
+            int p = atomicAdd(&ss.cnt, popc_w(nw));
+            while (nw) {
+                const int r = ffs_w(nw);
+                nw &= nw - 1;
+                const long long v = gseg[k] * NT + r;
+                B.levels[v] = level + 1;
+                if (p < SOLO_QS) sb.nq[p] = (int)v;
+                else Qn[p] = (int)v;
+                ++p;
+            }
+        }
         __syncthreads();
+        SOLO_T(1);
         const long long n2 = ss.cnt;
-        {
+        ++level;
+        if (n2 <= SOLO_QS) {
+            // records of the next level (its degrees in the same pass)
+            solo_records<NT>(a, sb.nq, false, n2, sb, ss, tid, mf2, din2, mx2);
+            SOLO_T(2);
+        } else {
             unsigned long long mf = 0, din = 0;
             int mx = 0;
             for (long long i = tid; i < n2; i += BFB) {
-                const int v = i < SOLO_QS ? q[cur ^ 1][i] : __ldcg(&Qn[i]);
+                const int v = i < SOLO_QS ? sb.nq[i] : __ldcg(&Qn[i]);
                 mf += (unsigned long long)a.outdeg[v];
                 din += (unsigned long long)a.indeg[v];
                 mx = max(mx, a.lwork[v]);
@@ -381,22 +487,24 @@ __device__ void solo_levels(const BfsFusedArgs &a, BfsView &B, int &level, long 
                 atomicAdd(&ss.din, din);
                 atomicMax(&ss.maxw, mx);
             }
+            __syncthreads();
+            mf2 = (long long)ss.mf;
+            din2 = (long long)ss.din;
+            mx2 = ss.maxw;
         }
-        __syncthreads();
-        ++level;
-        const long long mf2 = (long long)ss.mf, din2 = (long long)ss.din, mx2 = ss.maxw;
-        // every thread has read the level's totals before thread 0 zeroes them for
-        // the next level (compute-sanitizer racecheck, round 2)
-        __syncthreads();
         const int dir2 = n2 > 0 ? choose_dir_dev(a.force, a.alpha, a.dens, B.n, n2, mf2, mu - din2) : 0;
-        int G2 = 1;
-        while (G2 < mx2 && G2 < 32) G2 <<= 1;
         const bool cont = n2 > 0 && dir2 == TSMV_DIR_PUSH_CSC && mx2 <= LIST_MAXW && n2 <= SOLO_QS &&
-                          n2 * G2 <= SOLO_ROUNDS * BFB && level < a.max_levels;
+                          ss.W <= SOLO_ITEMS && level < a.max_levels;
+        SOLO_T(3);
         if (!cont) {
+#ifdef TSMV_SOLO_PROF
+            if (tid == 0 && nlev > 100)
+                printf("solo %lld levels: cycles/level loads %lld atomics %lld records %lld decide %lld tail %lld\n",
+                       nlev, pc[0] / nlev, pc[1] / nlev, pc[2] / nlev, pc[3] / nlev, pc[4] / nlev);
+#endif
             // leave frontier `level` in the global list + its slot, slot level+1 zeroed
             int *Qg = (level & 1) ? a.bq1 : a.bq0;
-            for (long long i = tid; i < min(n2, (long long)SOLO_QS); i += BFB) Qg[i] = q[cur ^ 1][i];
+            for (long long i = tid; i < min(n2, (long long)SOLO_QS); i += BFB) Qg[i] = sb.nq[i];
             if (tid == 0) {
                 long long *sl = a.lslots + (level % 3) * 4, *sn = a.lslots + ((level + 1) % 3) * 4;
                 sl[0] = n2;
@@ -416,9 +524,11 @@ __device__ void solo_levels(const BfsFusedArgs &a, BfsView &B, int &level, long 
             a.front_out[level] = n2;
             a.tlv_out[level] = globaltimer_ns();
         }
-        cur ^= 1;
         n = n2;
-        G = G2;
+#ifdef TSMV_SOLO_PROF
+        ++nlev;
+#endif
+        SOLO_T(4);
     }
 }
 
@@ -441,7 +551,7 @@ __global__ void __launch_bounds__(BFB, TSMV_BFS_MINB) k_bfs_fused(BfsFusedArgs a
     uint32_t *Fa = B.F, *Fb = B.Fn;
 
     __shared__ ListShared sh;
-    __shared__ int s_soloq[2][SOLO_QS];
+    __shared__ SoloBuf s_solo_buf;
     __shared__ SoloShared s_solo;
     unsigned long long solo_n = 0;  // solo episodes of this launch (same in every CTA)
     int mode_list = a.use_list && !a.resume;
@@ -464,6 +574,15 @@ __global__ void __launch_bounds__(BFB, TSMV_BFS_MINB) k_bfs_fused(BfsFusedArgs a
         sh.maxw = 0;
         sh.mf = 0;
         sh.din = 0;
+    }
+    // L2 warm-up (fire and forget: the first levels do not wait for it)
+    for (int r = 0; r < a.pf_n; ++r) {
+        const char *base = (const char *)a.pf_p[r];
+        const long long nb = a.pf_b[r] & ~15LL;
+        for (long long ch = gtid; ch * PF_CHUNK < nb; ch += gthreads) {
+            const unsigned sz = (unsigned)min(PF_CHUNK, nb - ch * PF_CHUNK);
+            asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(base + ch * PF_CHUNK), "r"(sz) : "memory");
+        }
     }
     if (mode_list && b == 0 && tid == 0) {
         a.bq0[0] = (int)a.source;
@@ -520,11 +639,11 @@ __global__ void __launch_bounds__(BFB, TSMV_BFS_MINB) k_bfs_fused(BfsFusedArgs a
             long long *slot_n = a.lslots + ((level + 1) % 3) * 4;
             int G = 1;
             while (G < maxw && G < 32) G <<= 1;
-            if (a.use_solo && fsize <= SOLO_QS && fsize * G <= SOLO_ROUNDS * BFB) {
+            if (a.use_solo && fsize <= SOLO_QS && fsize * maxw <= SOLO_ITEMS) {
                 // small frontier: CTA 0 runs the next levels alone (solo_levels)
                 ++solo_n;
                 if (b == 0) {
-                    solo_levels<NT>(a, B, level, mu, reached, edges, fsize, maxw, s_soloq, s_solo, tid);
+                    solo_levels<NT>(a, B, level, mu, reached, edges, fsize, s_solo_buf, s_solo, tid);
                     if (tid == 0) {
                         a.lslots[17] = level;
                         a.lslots[18] = mu;
@@ -869,10 +988,30 @@ bool bfs_fused_launch(tsmv_ctx *c, long long source, cudaStream_t st, bool resum
     a.bq1 = c->bq1.as<int>();
     a.lslots = c->lslots.as<long long>();
     a.use_list = (c->lwork.p != nullptr && !getenv("TSMV_BFS_NO_LIST")) ? 1 : 0;
-    a.use_solo = a.use_list && !getenv("TSMV_BFS_NO_SOLO") ? 1 : 0;
+    // solo records hold 32-bit tile / side starts
+    a.use_solo = a.use_list && !getenv("TSMV_BFS_NO_SOLO") && c->P.T < (1LL << 32) && c->P.side_nnz < (1LL << 32)
+                     ? 1 : 0;
     a.wide_in_kernel = getenv("TSMV_BFS_HOST_WIDE") ? 0 : 1;
     a.qcap = getenv("TSMV_BFS_QCAP") ? std::max(1, std::min(QCAP, atoi(getenv("TSMV_BFS_QCAP")))) : QCAP;
     if (a.use_solo) TSMV_CUDA(cudaMemsetAsync(c->lslots.as<long long>() + 16, 0, 8, st));  // release flag
+    a.pf_n = 0;
+    {
+        const TileSet &P = c->P;
+        const DevBuf *bufs[8] = {&P.ptr, &P.sptr, &P.planes, &P.trow, &P.srow, &c->outdeg, &c->indeg, &c->lwork};
+        long long tot = 0;
+        for (const DevBuf *d : bufs) tot += (long long)d->bytes;
+        int l2 = 0;
+        cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, c->device);
+        const char *e = getenv("TSMV_BFS_L2PF");
+        const bool on = e ? atoi(e) != 0 : (!resume && a.use_list && tot <= (long long)l2 / 2);
+        if (on)
+            for (const DevBuf *d : bufs)
+                if (d->p && d->bytes >= 16) {
+                    a.pf_p[a.pf_n] = d->p;
+                    a.pf_b[a.pf_n] = (long long)d->bytes;
+                    ++a.pf_n;
+                }
+    }
     void *args[] = {&a};
     void *f = c->nt == 16 ? (void *)k_bfs_fused<16> : c->nt == 32 ? (void *)k_bfs_fused<32> : (void *)k_bfs_fused<64>;
     const int G = c->bfs_blocks;

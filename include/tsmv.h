@@ -93,6 +93,12 @@ typedef struct {
                                     nonzeros in the side matrix and <= 32 per tile (small matrices:
                                     at any density); 0 = never.  Results are identical; default 0.05,
                                     the crossover measured on B200. */
+    double pull_alpha_burst;     /* (r2) alpha used instead of pull_alpha on a level whose frontier
+                                    grew >= burst_growth x over the previous level's (the explosive
+                                    levels of low-diameter graphs, where Beamer's 14 pays: R-MAT s26
+                                    290 -> 387 GTEPS), R9'; default 14; 0 = off */
+    double burst_growth;         /* growth factor of that test; default 4 (grids and bands grow
+                                    < 4x per level and keep pull_alpha) */
 } tsmv_options;
 
 /* Per-call counters of the last tsmv_spmspv (read from device on request). */
@@ -204,6 +210,11 @@ tsmv_status tsmv_spmspv_async(tsmv_ctx *c, tsmv_semiring sr, int64_t x_nnz, cons
  * window; tsmv_get_timing waits for the events and returns the summed ms of
  * {x-scan, expand, compact, whole call} over the `calls` timed calls since. */
 tsmv_status tsmv_set_timing(tsmv_ctx *c, int32_t enable);
+
+/* Retune the TileBFS direction rule (reading R9) of a built context:
+ * the tsmv_options fields push_csr_density (> 0), pull_alpha (> 0) and force_dir
+ * (TSMV_DIR_AUTO .. TSMV_DIR_PULL_CSC) for the next traversals.  EINVAL on range. */
+tsmv_status tsmv_set_direction_rule(tsmv_ctx *c, double push_csr_density, double pull_alpha, int32_t force_dir);
 tsmv_status tsmv_get_timing(tsmv_ctx *c, double *ms_out4, int64_t *calls);
 
 /* Development trace of the multiply phase: when `device_buffer` (u64 words,
@@ -350,10 +361,13 @@ tsmv_status tsmv_bfs2d_expand(tsmv_ctx *c, int32_t dir, const uint32_t *x_words,
 tsmv_status tsmv_bfs2d_list(tsmv_ctx *c, const uint32_t *words, int64_t nbits, int32_t *idx_out,
                             int64_t *count_out, void *cuda_stream);
 
-/* Direction rule of reading R9: PULL_CSC if m_f > m_u / pull_alpha,
+/* Direction rule of reading R9: PULL_CSC if m_f > m_u / alpha,
  * else PUSH_CSR if frontier / n >= push_csr_density, else PUSH_CSC; force_dir wins
- * when not AUTO.  opt NULL = defaults. */
-int32_t tsmv_choose_dir(const tsmv_options *opt, int64_t n, int64_t frontier, int64_t m_f, int64_t m_u);
+ * when not AUTO.  alpha = pull_alpha_burst when prev_frontier > 0 and frontier >=
+ * burst_growth x prev_frontier (reading R9', r2), else pull_alpha; prev_frontier =
+ * |F| of the previous level (0 or negative: unknown).  opt NULL = defaults. */
+int32_t tsmv_choose_dir(const tsmv_options *opt, int64_t n, int64_t frontier, int64_t m_f, int64_t m_u,
+                        int64_t prev_frontier);
 
 /* Census of the built format (host out). */
 tsmv_status tsmv_get_info(const tsmv_ctx *c, tsmv_info *info);

@@ -117,6 +117,8 @@ extern "C" tsmv_status tsmv_default_options(tsmv_options *o) {
     o->pull_alpha = 2.0;
     o->force_dir = TSMV_DIR_AUTO;
     o->row_driven_density = 0.05;  // measured crossover
+    o->pull_alpha_burst = 14.0;    // reading R9': Beamer's alpha on explosive levels
+    o->burst_growth = 4.0;
     o->rank = 0;
     o->nranks = 1;
     o->row_begin = 0;

@@ -972,10 +972,12 @@ static void owned_stats(tsmv_ctx *c, const uint32_t *F, cudaStream_t st) {
     TSMV_CUDA(cudaGetLastError());
 }
 
-int choose_dir(const tsmv_options &o, long long n, long long fsize, long long mf, long long mu) {
+int choose_dir(const tsmv_options &o, long long n, long long fsize, long long mf, long long mu, long long fprev) {
     if (o.force_dir != TSMV_DIR_AUTO) return o.force_dir;
-    // reading R9: Beamer-style edge test for pull, then the paper's 0.01 density rule
-    if ((double)mf > (double)mu / o.pull_alpha) return TSMV_DIR_PULL_CSC;
+    // reading R9: Beamer-style edge test for pull, then the paper's 0.01 density rule;
+    // R9': Beamer's alpha on explosive levels (frontier grew burst_growth x)
+    const double alpha = burst_alpha(o.pull_alpha, o.pull_alpha_burst, o.burst_growth, fsize, fprev);
+    if ((double)mf > (double)mu / alpha) return TSMV_DIR_PULL_CSC;
     if ((double)fsize / (double)n >= o.push_csr_density) return TSMV_DIR_PUSH_CSR;
     return TSMV_DIR_PUSH_CSC;
 }
@@ -1042,9 +1044,10 @@ static void bfs_distributed(tsmv_ctx *c, int64_t source, tsmv_bfs_stats *stats, 
         mu -= id;
     }
     long long reached = 0, edges = 0;
-    long long L = 0;
+    long long L = 0, fprev = 0;
     while (fsize > 0) {
-        const int dir = choose_dir(c->opt, c->n, fsize, mf, mu);
+        const int dir = choose_dir(c->opt, c->n, fsize, mf, mu, fprev);
+        fprev = fsize;
         if (L < TSMV_MAX_LEVELS) {
             if (stats) {
                 stats->dir_per_level[L] = dir;
@@ -1127,6 +1130,7 @@ extern "C" tsmv_status tsmv_bfs(tsmv_ctx *c, int64_t source, int32_t *levels, ts
             TSMV_CUDA(cudaEventRecord(c->ev0, st));
             uint32_t *Fa = c->F0.as<uint32_t>(), *Fb = c->F1.as<uint32_t>();
             long long level = 0, mu = c->nnz, reached = 0, edges = 0;
+            long long fprev = 0;  // |F| of the level before `level` (R9')
             bool resume = false;
             BfsRunner R{c, st, (long long)(c->V.bytes / 4)};
             const long long maxlv = getenv("TSMV_BFS_MAXLV") ? atoll(getenv("TSMV_BFS_MAXLV")) : (1ll << 40);
@@ -1134,8 +1138,9 @@ extern "C" tsmv_status tsmv_bfs(tsmv_ctx *c, int64_t source, int32_t *levels, ts
             while (true) {
                 long long L, mu2, r2, e2;
                 int cur;
+                long long fexp = 0;  // stopped: |F| of the level the host expands next
                 const bool stopped = bfs_fused_launch(c, source, st, resume, level, Fa, Fb, mu, reached, edges,
-                                                      stop_on_pull, maxlv, L, mu2, r2, e2, cur);
+                                                      stop_on_pull, maxlv, L, mu2, r2, e2, cur, fprev, fexp);
                 if (getenv("TSMV_BFS_PHASES")) {
                     long long fl = 0;
                     if (c->lslots.p) {
@@ -1164,13 +1169,15 @@ extern "C" tsmv_status tsmv_bfs(tsmv_ctx *c, int64_t source, int32_t *levels, ts
                     std::swap(Fa, Fb);
                     ++level;
                     if (fsize == 0 || level >= maxlv) break;
-                    const int dir = choose_dir(c->opt, c->n, fsize, mf, mu - din);
+                    const int dir = choose_dir(c->opt, c->n, fsize, mf, mu - din, fexp);
+                    fprev = fexp;  // the kernel re-decides `level` from here when it resumes
                     // resume the fused kernel at `level` for push levels and for the late
                     // (wide) pull levels, which it runs in place without host round trips
                     if (dir != TSMV_DIR_PULL_CSC || (!getenv("TSMV_BFS_HOST_WIDE") && (mu - din) * 4 < c->nnz)) break;
                     mu -= din;
                     reached += fsize;
                     edges += mf;
+                    fexp = fsize;
                     if (level < TSMV_MAX_LEVELS) {
                         int dd = dir;
                         long long ff = fsize;
@@ -1213,12 +1220,13 @@ extern "C" tsmv_status tsmv_bfs(tsmv_ctx *c, int64_t source, int32_t *levels, ts
         volatile Counters *h = c->hcnt;
         long long fsize = h->fsize, mf = h->mf;
         long long mu = c->nnz - h->din;
-        long long reached = 0, edges = 0;
+        long long reached = 0, edges = 0, fprev = 0;
         int L = 0;
         if (stats) stats->nlevels = 0;
         unsigned long long *tlv = c->bfs_tlv.as<unsigned long long>();
         while (fsize > 0) {
-            int dir = choose_dir(c->opt, c->n, fsize, mf, mu);
+            int dir = choose_dir(c->opt, c->n, fsize, mf, mu, fprev);
+            fprev = fsize;
             if (stats && L < TSMV_MAX_LEVELS) {
                 stats->dir_per_level[L] = dir;
                 stats->frontier_per_level[L] = fsize;
@@ -1482,11 +1490,12 @@ extern "C" tsmv_status tsmv_bfs_dist_merge(tsmv_ctx *c, const uint32_t *gathered
     }
 }
 
-extern "C" int32_t tsmv_choose_dir(const tsmv_options *o, int64_t n, int64_t frontier, int64_t m_f, int64_t m_u) {
+extern "C" int32_t tsmv_choose_dir(const tsmv_options *o, int64_t n, int64_t frontier, int64_t m_f, int64_t m_u,
+                                   int64_t prev_frontier) {
     tsmv_options d;
     if (!o) {
         tsmv_default_options(&d);
         o = &d;
     }
-    return choose_dir(*o, n, frontier, m_f, m_u);
+    return choose_dir(*o, n, frontier, m_f, m_u, prev_frontier);
 }

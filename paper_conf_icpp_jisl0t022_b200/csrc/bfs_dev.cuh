@@ -233,9 +233,10 @@ __device__ __forceinline__ void pull_side_word(const BfsTiles &Q, const BfsView 
 
 // Device copy of the direction rule (reading R9); host: tsmv::choose_dir.
 __device__ __forceinline__ int choose_dir_dev(int force, double alpha, double dens, long long n, long long f,
-                                              long long mf, long long mu) {
+                                              long long mf, long long mu, double alpha_burst = 0,
+                                              double growth = 0, long long fprev = 0) {
     if (force) return force;
-    if ((double)mf > (double)mu / alpha) return TSMV_DIR_PULL_CSC;
+    if ((double)mf > (double)mu / burst_alpha(alpha, alpha_burst, growth, f, fprev)) return TSMV_DIR_PULL_CSC;
     if ((double)f / (double)n >= dens) return TSMV_DIR_PUSH_CSR;
     return TSMV_DIR_PUSH_CSC;
 }

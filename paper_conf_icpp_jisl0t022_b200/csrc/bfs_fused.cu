@@ -57,6 +57,8 @@ struct BfsFusedArgs {
     unsigned long long *tlv_out;  // [TSMV_MAX_LEVELS + 1] %globaltimer when level L's expansion is decided
     long long source, nnz, nseg, NW, nTR_local, max_levels;
     double alpha, dens;
+    double alpha_burst, growth;   // reading R9' (explosive levels)
+    long long fprev0;             // |F| of the level before level0 (resume), 0 = none
     int force;
     unsigned long long bar_base;
     // resume / hand-off: the kernel stops before expanding a
@@ -390,7 +392,8 @@ __device__ void solo_records(const BfsFusedArgs &a, const int *ids, bool ids_glo
 
 template <int NT>
 __device__ void solo_levels(const BfsFusedArgs &a, BfsView &B, int &level, long long &mu, long long &reached,
-                            long long &edges, long long fsize, SoloBuf &sb, SoloShared &ss, int tid) {
+                            long long &edges, long long fsize, long long &fprev, SoloBuf &sb, SoloShared &ss,
+                            int tid) {
     using word_t = typename Tr<NT>::word_t;
     const word_t *planes = (const word_t *)a.P.planes;
     long long mf2, din2, mx2;
@@ -492,7 +495,8 @@ __device__ void solo_levels(const BfsFusedArgs &a, BfsView &B, int &level, long 
             din2 = (long long)ss.din;
             mx2 = ss.maxw;
         }
-        const int dir2 = n2 > 0 ? choose_dir_dev(a.force, a.alpha, a.dens, B.n, n2, mf2, mu - din2) : 0;
+        const int dir2 =
+            n2 > 0 ? choose_dir_dev(a.force, a.alpha, a.dens, B.n, n2, mf2, mu - din2, a.alpha_burst, a.growth, n) : 0;
         const bool cont = n2 > 0 && dir2 == TSMV_DIR_PUSH_CSC && mx2 <= LIST_MAXW && n2 <= SOLO_QS &&
                           ss.W <= SOLO_ITEMS && level < a.max_levels;
         SOLO_T(3);
@@ -503,6 +507,7 @@ __device__ void solo_levels(const BfsFusedArgs &a, BfsView &B, int &level, long 
                        nlev, pc[0] / nlev, pc[1] / nlev, pc[2] / nlev, pc[3] / nlev, pc[4] / nlev);
 #endif
             // leave frontier `level` in the global list + its slot, slot level+1 zeroed
+            fprev = n;
             int *Qg = (level & 1) ? a.bq1 : a.bq0;
             for (long long i = tid; i < min(n2, (long long)SOLO_QS); i += BFB) Qg[i] = sb.nq[i];
             if (tid == 0) {
@@ -601,6 +606,7 @@ __global__ void __launch_bounds__(BFB, TSMV_BFS_MINB) k_bfs_fused(BfsFusedArgs a
     const long long per = (S + BFB - 1) / BFB;
     const long long tj0 = min(js1, js0 + tid * per), tj1 = min(js1, tj0 + per);
     int level = (int)a.level0;
+    long long fprev = a.fprev0;  // |F| of the previous level (R9')
     unsigned long long t_s1 = 0, t_s2 = 0, t_e = 0, tq = b == 0 && tid == 0 ? globaltimer_ns() : 0;
     bool redo = false;  // scan pass over a level already counted in list mode
     for (; level < a.max_levels; ++level) {
@@ -616,7 +622,8 @@ __global__ void __launch_bounds__(BFB, TSMV_BFS_MINB) k_bfs_fused(BfsFusedArgs a
             if (fsize == 0) break;
             reached += fsize;
             edges += mf;
-            const int dir = choose_dir_dev(a.force, a.alpha, a.dens, B.n, fsize, mf, mu);
+            const int dir = choose_dir_dev(a.force, a.alpha, a.dens, B.n, fsize, mf, mu, a.alpha_burst, a.growth,
+                                           fprev);
             if (b == 0 && tid == 0 && level < TSMV_MAX_LEVELS) {
                 a.dir_out[level] = dir;
                 a.front_out[level] = fsize;
@@ -643,12 +650,14 @@ __global__ void __launch_bounds__(BFB, TSMV_BFS_MINB) k_bfs_fused(BfsFusedArgs a
                 // small frontier: CTA 0 runs the next levels alone (solo_levels)
                 ++solo_n;
                 if (b == 0) {
-                    solo_levels<NT>(a, B, level, mu, reached, edges, fsize, s_solo_buf, s_solo, tid);
+                    fprev = fsize;
+                    solo_levels<NT>(a, B, level, mu, reached, edges, fsize, fprev, s_solo_buf, s_solo, tid);
                     if (tid == 0) {
                         a.lslots[17] = level;
                         a.lslots[18] = mu;
                         a.lslots[19] = reached;
                         a.lslots[20] = edges;
+                        a.lslots[21] = fprev;
                         __threadfence();
                         atomicExch((unsigned long long *)&a.lslots[16], solo_n);
                     }
@@ -663,6 +672,7 @@ __global__ void __launch_bounds__(BFB, TSMV_BFS_MINB) k_bfs_fused(BfsFusedArgs a
                     mu = __ldcg(&a.lslots[18]);
                     reached = __ldcg(&a.lslots[19]);
                     edges = __ldcg(&a.lslots[20]);
+                    fprev = __ldcg(&a.lslots[21]);
                 }
                 if (b == 0 && tid == 0) {
                     const unsigned long long t = globaltimer_ns();
@@ -676,6 +686,7 @@ __global__ void __launch_bounds__(BFB, TSMV_BFS_MINB) k_bfs_fused(BfsFusedArgs a
             unsigned long long tl0 = 0, tl1 = 0, tl2 = 0;
             if (b == 0 && tid == 0) tl0 = globaltimer_ns();
 #endif
+            fprev = fsize;
             list_level<NT>(a, B, Qc, fsize, G, gtid, gthreads, sh, Qn, slot_n);
 #ifdef TSMV_LIST_PROF
             __syncthreads();
@@ -770,7 +781,7 @@ __global__ void __launch_bounds__(BFB, TSMV_BFS_MINB) k_bfs_fused(BfsFusedArgs a
             edges += mf;
         }
         redo = false;
-        const int dir = choose_dir_dev(a.force, a.alpha, a.dens, B.n, fsize, mf, mu);
+        const int dir = choose_dir_dev(a.force, a.alpha, a.dens, B.n, fsize, mf, mu, a.alpha_burst, a.growth, fprev);
         if (b == 0 && tid == 0 && level < TSMV_MAX_LEVELS) {
             a.dir_out[level] = dir;
             a.front_out[level] = fsize;
@@ -782,8 +793,10 @@ __global__ void __launch_bounds__(BFB, TSMV_BFS_MINB) k_bfs_fused(BfsFusedArgs a
         // high-diameter traversal) run here with the wide row-tile test
         if (dir == TSMV_DIR_PULL_CSC && a.stop_on_pull && mu > 16 * gthreads && (!a.wide_in_kernel || mu * 4 >= a.nnz)) {
             stopped = 1;  // uniform across CTAs: same totals, same decision
+            fprev = fsize;  // handed to the host: |F| of the level it expands
             break;
         }
+        fprev = fsize;
         // lists (Push-CSC needs both, Push-CSR the side list; pull none)
         if (dir != TSMV_DIR_PULL_CSC) {
             long long oLt = s_pre[0] + ex[0], oWt = s_pre[1] + ex[1];
@@ -894,6 +907,7 @@ __global__ void __launch_bounds__(BFB, TSMV_BFS_MINB) k_bfs_fused(BfsFusedArgs a
         a.hm->edges = edges;
         a.hm->mf = mu;
         a.hm->din = stopped;
+        a.hm->nCt = fprev;  // |F| of the last level decided (the stopped one when stopped)
         a.hm->nLt = (Fa == a.B.F) ? 0 : 1;  // which bitmap holds the current frontier
         a.hm->Wt = (long long)t_s1;  // phase times (ns, CTA 0): count, lists, expand
         a.hm->nLs = (long long)t_s2;
@@ -946,7 +960,7 @@ int bfs_fused_occupancy(int nt) {
 bool bfs_fused_launch(tsmv_ctx *c, long long source, cudaStream_t st, bool resume, long long level0, uint32_t *Fa,
                       uint32_t *Fb, long long mu, long long reached, long long edges, bool stop_on_pull,
                       long long max_levels, long long &level_out, long long &mu_out, long long &reached_out,
-                      long long &edges_out, int &cur_out) {
+                      long long &edges_out, int &cur_out, long long fprev0, long long &fprev_out) {
     BfsFusedArgs a;
     a.P = bfs_tiles(c->P);
     a.Q = bfs_tiles(*c->Q);
@@ -976,6 +990,9 @@ bool bfs_fused_launch(tsmv_ctx *c, long long source, cudaStream_t st, bool resum
     a.alpha = c->opt.pull_alpha;
     a.dens = c->opt.push_csr_density;
     a.force = c->opt.force_dir;
+    a.alpha_burst = c->opt.pull_alpha_burst;
+    a.growth = c->opt.burst_growth;
+    a.fprev0 = fprev0;
     a.bar_base = c->bar_base;
     a.resume = resume ? 1 : 0;
     a.stop_on_pull = stop_on_pull ? 1 : 0;
@@ -1025,6 +1042,7 @@ bool bfs_fused_launch(tsmv_ctx *c, long long source, cudaStream_t st, bool resum
     edges_out = h->edges;
     mu_out = h->mf;
     cur_out = (int)h->nLt;
+    fprev_out = h->nCt;
     c->bar_base += h->bfs_bars;
     return stopped;
 }

@@ -392,7 +392,7 @@ void heavy_side_chunks(tsmv_ctx *c, cudaStream_t st);  // bfs.cu: chunks of side
 bool bfs_fused_launch(tsmv_ctx *c, long long source, cudaStream_t st, bool resume, long long level0, uint32_t *Fa,
                       uint32_t *Fb, long long mu, long long reached, long long edges, bool stop_on_pull,
                       long long max_levels, long long &level_out, long long &mu_out, long long &reached_out,
-                      long long &edges_out, int &cur_out);
+                      long long &edges_out, int &cur_out, long long fprev0, long long &fprev_out);
 // comm.cu
 bool has_comm(const tsmv_ctx *c);
 void comm_init(tsmv_ctx *c, const void *unique_id, cudaStream_t st);
@@ -402,7 +402,12 @@ void comm_exchange_frontier(tsmv_ctx *c, uint32_t *F, uint32_t *V, long long nwo
 long long comm_gather_x(tsmv_ctx *c, long long k_local, const int32_t *x_idx, const void *x_val, size_t vb,
                         const int32_t **xi_out, const void **xv_out, cudaStream_t st);
 // bfs.cu
-int choose_dir(const tsmv_options &o, long long n, long long fsize, long long mf, long long mu);
+int choose_dir(const tsmv_options &o, long long n, long long fsize, long long mf, long long mu, long long fprev);
+// reading R9': alpha of a level from the frontier's growth
+__host__ __device__ __forceinline__ double burst_alpha(double alpha, double alpha_burst, double growth, long long f,
+                                                       long long fprev) {
+    return (alpha_burst > 0 && fprev > 0 && (double)f >= growth * (double)fprev) ? alpha_burst : alpha;
+}
 // pointer classification
 bool is_device_ptr(const void *p);
 // device address of page-locked, mapped host memory (cudaHostAlloc / torch

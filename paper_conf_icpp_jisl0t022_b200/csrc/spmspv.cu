@@ -1218,6 +1218,22 @@ extern "C" tsmv_status tsmv_set_trace(tsmv_ctx *c, void *device_buffer) {
     return TSMV_OK;
 }
 
+extern "C" tsmv_status tsmv_set_direction_rule(tsmv_ctx *c, double push_csr_density, double pull_alpha,
+                                               int32_t force_dir) {
+    try {
+        TSMV_REQUIRE(c, "tsmv_set_direction_rule: NULL ctx");
+        TSMV_REQUIRE(push_csr_density > 0 && pull_alpha > 0, "tsmv_set_direction_rule: thresholds must be > 0");
+        TSMV_REQUIRE(force_dir >= TSMV_DIR_AUTO && force_dir <= TSMV_DIR_PULL_CSC,
+                     "tsmv_set_direction_rule: force_dir out of range");
+        c->opt.push_csr_density = push_csr_density;
+        c->opt.pull_alpha = pull_alpha;
+        c->opt.force_dir = force_dir;
+        return TSMV_OK;
+    } catch (const Err &e) {
+        return e.st;
+    }
+}
+
 extern "C" tsmv_status tsmv_set_timing(tsmv_ctx *c, int32_t enable) {
     try {
         TSMV_REQUIRE(c, "tsmv_set_timing: NULL ctx");

@@ -164,8 +164,10 @@ def bfs_loop(engine, source: int, group=None) -> int:
     dist.all_reduce(red, group=group)
     f, gmf, gmu = (int(x) for x in red.tolist())
     levels = 0
+    fprev = 0   # |F| of the previous level (direction rule R9')
     while f > 0:
-        d = engine.choose(engine.n, f, gmf, gmu)
+        d = engine.choose(engine.n, f, gmf, gmu, fprev)
+        fprev = f
         # late pull levels (few unvisited edges) take the wide row-tile test
         wide = getattr(engine, "nnz_total", 0) > 0 and gmu * 4 < engine.nnz_total
         owned = engine.expand(d, wide=wide)
@@ -251,8 +253,8 @@ class DistTiledMatrix:
         self.M.spmspv_async(xi, xv, y_idx, y_val, y_nnz, semiring=semiring)
 
     # ---- BFS engine interface
-    def choose(self, n, f, mf, mu):
-        return self.tsmv.choose_dir(n, f, mf, mu, self.M.opts)
+    def choose(self, n, f, mf, mu, fprev=0):
+        return self.tsmv.choose_dir(n, f, mf, mu, self.M.opts, fprev)
 
     def begin(self, source):
         import ctypes

@@ -193,8 +193,8 @@ class Dist2DBFS:
     def _st(self):
         return torch.cuda.current_stream(self.device).cuda_stream
 
-    def choose(self, f, mf, mu):
-        return self.tsmv.choose_dir(self.grid.n, f, mf, mu, self.M.opts)
+    def choose(self, f, mf, mu, fprev=0):
+        return self.tsmv.choose_dir(self.grid.n, f, mf, mu, self.M.opts, fprev)
 
     def begin(self, source: int) -> torch.Tensor:
         """Reset the state; the owner of `source` marks it (level 0) in its frontier
@@ -323,10 +323,12 @@ def bfs2d_loop(engine, source: int, comm) -> int:
     f, mf, dmu = comm.allreduce(engine.stats)
     mu = engine.nnz_total - dmu
     level = 0
+    fprev = 0
     while True:
         x = comm.col_allgather(front)
         rn = comm.row_allgather(front) if engine.needs_rows else None
-        d = engine.choose(f, mf, mu)
+        d = engine.choose(f, mf, mu, fprev)
+        fprev = f
         if engine.nnz_total > 0 and mu * 4 < engine.nnz_total:
             d |= DIST_WIDE
         y = engine.expand(x, d, rn, level)
@@ -362,11 +364,13 @@ def sim_bfs2d(engines: Sequence[Dist2DBFS], source: int, trace: Optional[list] =
     nnz_total = engines[0].nnz_total
     mu = nnz_total - dmu
     level = 0
+    fprev = 0
     while True:
         xs = [torch.cat([fronts[g.rank_of(i, j)] for i in range(Pr)]) for j in range(Pc)]
         rows = [torch.cat([fronts[g.rank_of(i, j)] for j in range(Pc)]) for i in range(Pr)] \
             if engines[0].needs_rows else [None] * Pr
-        d = engines[0].choose(f, mf, mu)
+        d = engines[0].choose(f, mf, mu, fprev)
+        fprev = f
         if nnz_total > 0 and mu * 4 < nnz_total:
             d |= DIST_WIDE
         te, tm, ys = [], [], []

@@ -42,7 +42,8 @@ class tsmv_options(ctypes.Structure):
                 ("push_csr_density", ctypes.c_double), ("pull_alpha", ctypes.c_double),
                 ("force_dir", ctypes.c_int32), ("rank", ctypes.c_int32), ("nranks", ctypes.c_int32),
                 ("row_begin", ctypes.c_int64), ("row_splits", ctypes.POINTER(ctypes.c_int64)),
-                ("nccl_unique_id", ctypes.c_void_p), ("row_driven_density", ctypes.c_double)]
+                ("nccl_unique_id", ctypes.c_void_p), ("row_driven_density", ctypes.c_double),
+                ("pull_alpha_burst", ctypes.c_double), ("burst_growth", ctypes.c_double)]
 
 
 class tsmv_call_stats(ctypes.Structure):
@@ -80,6 +81,7 @@ _SIGS = {
     "tsmv_spmspv": (ctypes.c_int, [_vp, ctypes.c_int, _i64, _vp, _vp, _i64, _vp, _vp, ctypes.POINTER(_i64), _vp]),
     "tsmv_spmspv_async": (ctypes.c_int, [_vp, ctypes.c_int, _i64, _vp, _vp, _i64, _vp, _vp, _vp, _vp]),
     "tsmv_set_timing": (ctypes.c_int, [_vp, _i32]),
+    "tsmv_set_direction_rule": (ctypes.c_int, [_vp, ctypes.c_double, ctypes.c_double, _i32]),
     "tsmv_set_trace": (ctypes.c_int, [_vp, _vp]),
     "tsmv_trace_words": (_i64, [_vp]),
     "tsmv_get_timing": (ctypes.c_int, [_vp, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(_i64)]),
@@ -96,7 +98,7 @@ _SIGS = {
     "tsmv_bfs_dist_expand": (ctypes.c_int, [_vp, _i32, _vp, _vp]),
     "tsmv_bfs_dist_merge": (ctypes.c_int, [_vp, _vp, _i64, ctypes.POINTER(_i64), _vp]),
     "tsmv_owned_words": (_i64, [_vp]),
-    "tsmv_choose_dir": (_i32, [ctypes.POINTER(tsmv_options), _i64, _i64, _i64, _i64]),
+    "tsmv_choose_dir": (_i32, [ctypes.POINTER(tsmv_options), _i64, _i64, _i64, _i64, _i64]),
     "tsmv_get_info": (ctypes.c_int, [_vp, ctypes.POINTER(tsmv_info)]),
     "tsmv_export_csr": (ctypes.c_int, [_vp, _vp, _vp, _vp]),
     "tsmv_export_bitmask_tiles": (ctypes.c_int, [_vp, _i32, _i64, _vp, _vp, _vp, ctypes.POINTER(_i64)]),
@@ -233,6 +235,19 @@ class TiledMatrix:
                                 _ptr(y_val) if sr != OR_AND else None, _ptr(y_nnz), _stream(stream)),
               "tsmv_spmspv_async")
 
+    def set_direction_rule(self, push_csr_density: Optional[float] = None, pull_alpha: Optional[float] = None,
+                           force_dir: Optional[int] = None):
+        """Retune the TileBFS direction rule (R9) for the next traversals."""
+        o = self.opts
+        if push_csr_density is not None:
+            o.push_csr_density = float(push_csr_density)
+        if pull_alpha is not None:
+            o.pull_alpha = float(pull_alpha)
+        if force_dir is not None:
+            o.force_dir = int(force_dir)
+        check(tsmv_set_direction_rule(self.ctx, o.push_csr_density, o.pull_alpha, o.force_dir),
+              "tsmv_set_direction_rule")
+
     def set_timing(self, enable: bool = True):
         check(tsmv_set_timing(self.ctx, 1 if enable else 0), "tsmv_set_timing")
 
@@ -335,5 +350,6 @@ def nccl_unique_id() -> bytes:
     return buf.raw
 
 
-def choose_dir(n, frontier, m_f, m_u, opts: Optional[tsmv_options] = None) -> int:
-    return int(tsmv_choose_dir(ctypes.byref(opts) if opts is not None else None, n, frontier, m_f, m_u))
+def choose_dir(n, frontier, m_f, m_u, opts: Optional[tsmv_options] = None, prev_frontier: int = 0) -> int:
+    return int(tsmv_choose_dir(ctypes.byref(opts) if opts is not None else None, n, frontier, m_f, m_u,
+                               prev_frontier))

@@ -27,10 +27,11 @@ gathered = torch.zeros(P * stride, dtype=torch.int32, device=dev)
 for rep in range(2):
     torch.cuda.nvtx.range_push(f"traversal{rep}")
     st = [e.begin(src) for e in engines]
-    lv = 0
+    lv, fprev = 0, 0
     while sum(x[0] for x in st) > 0:
         f, mf, mu = (sum(x[i] for x in st) for i in range(3))
-        d = engines[0].choose(engines[0].n, f, mf, mu)
+        d = engines[0].choose(engines[0].n, f, mf, mu, fprev)
+        fprev = f
         ts = []
         for p, e in enumerate(engines):
             a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)

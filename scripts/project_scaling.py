@@ -74,13 +74,14 @@ for P in [int(p) for p in args.ranks.split(",")]:
     for s in srcs:
         for rep in range(2):  # warm-up traversal, then the measured one
             st = [e.begin(s) for e in engines]
-            lv_proj, nlev, edges = [], 0, 0
+            lv_proj, nlev, edges, fprev = [], 0, 0, 0
             while sum(x[0] for x in st) > 0:
                 f = sum(x[0] for x in st)
                 mf = sum(x[1] for x in st)
                 mu = sum(x[2] for x in st)
                 edges += mf
-                d = engines[0].choose(engines[0].n, f, mf, mu)
+                d = engines[0].choose(engines[0].n, f, mf, mu, fprev)
+                fprev = f
                 te, tm = [], []
                 for p, e in enumerate(engines):
                     a, b = ev(), ev()

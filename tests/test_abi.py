@@ -51,6 +51,13 @@ def test_host_only_calls():
     assert tsmv.choose_dir(1000, 50, 10, 10_000) == tsmv.DIR_PUSH_CSR
     assert tsmv.choose_dir(1000, 10, 1000, 10_000) == tsmv.DIR_PUSH_CSC
     assert tsmv.choose_dir(1000, 10, 6000, 10_000) == tsmv.DIR_PULL_CSC
+    # reading R9': Beamer's 14 on a level whose frontier grew >= 4x (defaults 14, 4)
+    assert o.pull_alpha_burst == 14.0 and o.burst_growth == 4.0
+    assert tsmv.choose_dir(1000, 10, 1000, 10_000, None, 2) == tsmv.DIR_PULL_CSC    # 10 >= 4 x 2: 1000 > 10000/14
+    assert tsmv.choose_dir(1000, 10, 1000, 10_000, None, 3) == tsmv.DIR_PUSH_CSC    # 10 < 4 x 3: alpha 2
+    assert tsmv.choose_dir(1000, 10, 1000, 10_000, None, 0) == tsmv.DIR_PUSH_CSC    # unknown previous level
+    off = tsmv.default_options(pull_alpha_burst=0.0)
+    assert tsmv.choose_dir(1000, 10, 1000, 10_000, off, 1) == tsmv.DIR_PUSH_CSC     # R9' off: alpha 2
     o.force_dir = tsmv.DIR_PUSH_CSR
     assert tsmv.choose_dir(1000, 1, 1000, 10, o) == tsmv.DIR_PUSH_CSR
     assert tsmv.tsmv_destroy(None) == tsmv.OK

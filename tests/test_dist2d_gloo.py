@@ -98,7 +98,7 @@ class NumpyEngine2D:
         self.outdeg, self.indeg = od.numpy(), idg.numpy()
         self.seen = []
 
-    def choose(self, f, mf, mu):
+    def choose(self, f, mf, mu, fprev=0):
         self.seen.append((f, mf, mu))
         return 1
 

@@ -82,8 +82,8 @@ class NumpyEngine:
         from paper_conf_icpp_jisl0t022_b200 import tsmv
         self.tsmv = tsmv
 
-    def choose(self, n, f, mf, mu):
-        return self.tsmv.choose_dir(n, f, mf, mu)
+    def choose(self, n, f, mf, mu, fprev=0):
+        return self.tsmv.choose_dir(n, f, mf, mu, None, fprev)
 
     def _stats(self):
         # this rank's shares over its own rows (the libtsmv r2 semantics); bfs_loop sums them

@@ -46,6 +46,7 @@ def _level_stats(A, lv):
 def _sim_bfs(engines, source, dev_stats=False, expect=None):
     st = [e.begin(source) for e in engines]
     level = 0
+    fprev = 0
     while sum(s[0] for s in st) > 0:
         # every rank returns its shares over its own rows; the sums are the global numbers
         f = sum(s[0] for s in st)
@@ -54,7 +55,8 @@ def _sim_bfs(engines, source, dev_stats=False, expect=None):
         if expect is not None:
             assert (f, mf, mu) == expect[level], level
         level += 1
-        d = engines[0].choose(engines[0].n, f, mf, mu)
+        d = engines[0].choose(engines[0].n, f, mf, mu, fprev)
+        fprev = f
         nnz = sum(e.M.nnz for e in engines)
         owned = [e.expand(d, wide=mu * 4 < nnz).clone() for e in engines]   # late-pull hint as bfs_loop
         stride = engines[0].stride

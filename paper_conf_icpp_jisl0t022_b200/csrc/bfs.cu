@@ -1173,7 +1173,9 @@ extern "C" tsmv_status tsmv_bfs(tsmv_ctx *c, int64_t source, int32_t *levels, ts
                     fprev = fexp;  // the kernel re-decides `level` from here when it resumes
                     // resume the fused kernel at `level` for push levels and for the late
                     // (wide) pull levels, which it runs in place without host round trips
-                    if (dir != TSMV_DIR_PULL_CSC || (!getenv("TSMV_BFS_HOST_WIDE") && (mu - din) * 4 < c->nnz)) break;
+                    if (dir != TSMV_DIR_PULL_CSC || (!getenv("TSMV_BFS_HOST_WIDE") && (mu - din) * 4 < c->nnz &&
+                                                     mu - din <= bfs_wide_cap(c, true)))
+                        break;
                     mu -= din;
                     reached += fsize;
                     edges += mf;

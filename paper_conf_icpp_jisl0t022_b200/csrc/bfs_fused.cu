@@ -73,6 +73,7 @@ struct BfsFusedArgs {
     int use_list, use_solo;
     int qcap;                 // usable entries of the shared-memory queue (<= QCAP; TSMV_BFS_QCAP tests the overflow path)
     int wide_in_kernel;       // pull levels with m_u < nnz / 4 stay in the kernel (wide pull)
+    long long wide_cap;       // ... unless m_u > wide_cap (r2: large graphs)
     // r2: L2 warm-up of the push structures + degrees (graphs whose structures fit
     // in half the L2): bulk L2 prefetches by every CTA before the first level, so the
     // latency-bound list / solo levels of high-diameter graphs hit L2, not HBM
@@ -791,7 +792,11 @@ __global__ void __launch_bounds__(BFB, TSMV_BFS_MINB) k_bfs_fused(BfsFusedArgs a
         // levels with few unvisited edges (m_u <= 16 per thread of this grid, or
         // m_u < nnz / 4: late R-MAT levels, small graphs, the tail of a
         // high-diameter traversal) run here with the wide row-tile test
-        if (dir == TSMV_DIR_PULL_CSC && a.stop_on_pull && mu > 16 * gthreads && (!a.wide_in_kernel || mu * 4 >= a.nnz)) {
+        // (r2) and late pull levels that are still large in absolute terms (> wide_cap
+        // unvisited edges: s26) go to the host kernels too, whose occupancy the
+        // latency-bound wide pull needs more than it needs the saved round trip
+        if (dir == TSMV_DIR_PULL_CSC && a.stop_on_pull && mu > 16 * gthreads &&
+            (!a.wide_in_kernel || mu * 4 >= a.nnz || mu > a.wide_cap)) {
             stopped = 1;  // uniform across CTAs: same totals, same decision
             fprev = fsize;  // handed to the host: |F| of the level it expands
             break;
@@ -955,6 +960,18 @@ int bfs_fused_occupancy(int nt) {
     return bps;
 }
 
+// in-kernel wide pull only while m_u <= 16 edges per thread of the persistent grid
+// (measured: R-MAT s22 / s26); resume = the host's test for handing a
+// late pull level back to the fused kernel, which also needs the kernel's bitmap
+// scan to be short: <= 4 nt-segments per thread (s22 yes, s26 no)
+long long bfs_wide_cap(const tsmv_ctx *c, bool resume) {
+    const char *e = getenv(resume ? "TSMV_BFS_RESUME_CAP" : "TSMV_BFS_WIDE_CAP");
+    const double mult = e ? atof(e) : 16.0;
+    const long long threads = (long long)c->bfs_blocks * BFB;
+    if (resume && !e && c->nTC > 4 * threads) return -1;
+    return (long long)(mult * (double)threads);
+}
+
 // Launch the fused kernel from `level0` (resume) on bitmaps (Fa, Fb).  Returns
 // true if it stopped before a Pull-CSC level.
 bool bfs_fused_launch(tsmv_ctx *c, long long source, cudaStream_t st, bool resume, long long level0, uint32_t *Fa,
@@ -1009,6 +1026,7 @@ bool bfs_fused_launch(tsmv_ctx *c, long long source, cudaStream_t st, bool resum
     a.use_solo = a.use_list && !getenv("TSMV_BFS_NO_SOLO") && c->P.T < (1LL << 32) && c->P.side_nnz < (1LL << 32)
                      ? 1 : 0;
     a.wide_in_kernel = getenv("TSMV_BFS_HOST_WIDE") ? 0 : 1;
+    a.wide_cap = bfs_wide_cap(c, false);
     a.qcap = getenv("TSMV_BFS_QCAP") ? std::max(1, std::min(QCAP, atoi(getenv("TSMV_BFS_QCAP")))) : QCAP;
     if (a.use_solo) TSMV_CUDA(cudaMemsetAsync(c->lslots.as<long long>() + 16, 0, 8, st));  // release flag
     a.pf_n = 0;

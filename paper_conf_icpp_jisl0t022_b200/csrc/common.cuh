@@ -387,6 +387,7 @@ void enqueue_spmspv_rows(tsmv_ctx *c, int sr, long long k, const int32_t *xi, co
 bool use_rows_kernel(const tsmv_ctx *c, long long k);
 // bfs_fused.cu
 int bfs_fused_occupancy(int nt);
+long long bfs_wide_cap(const tsmv_ctx *c, bool resume);  // m_u above which a wide pull level leaves the fused kernel
 void bfs_list_init(tsmv_ctx *c, cudaStream_t st);
 void heavy_side_chunks(tsmv_ctx *c, cudaStream_t st);  // bfs.cu: chunks of side rows > 32 entries
 bool bfs_fused_launch(tsmv_ctx *c, long long source, cudaStream_t st, bool resume, long long level0, uint32_t *Fa,

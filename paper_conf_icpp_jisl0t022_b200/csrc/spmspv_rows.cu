@@ -413,6 +413,7 @@ __global__ void __launch_bounds__(RT, 1) k_spmspv_rows(RowArgs a) {
         for (int w = 0; w < RNW; ++w) sum += s_acct[w][tid];
         a.acct[b * 4 + tid] = sum;
     }
+    __syncthreads();  // the sums above have read s_acct (compute-sanitizer racecheck, r2)
     if (lane == 0) {
         s_acct[wid][0] = q4[0];
         s_acct[wid][1] = q4[1];

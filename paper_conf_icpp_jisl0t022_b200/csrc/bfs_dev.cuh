@@ -61,10 +61,20 @@ inline BfsTiles bfs_tiles(const TileSet &S) {
 
 // ---- one item of each level kernel -------------------------------------------
 
+// Bulk push (r2): the rows reached are only ORed into the next-frontier bitmap
+// with fire-and-forget reductions; a pass over the words afterwards takes new =
+// Fn & ~V, sets V and the levels (heavy Push-CSC levels: one returning atomic per
+// edge was the bound).
+template <int NT>
+__device__ __forceinline__ void reach(const BfsView &B, long long gseg, typename Tr<NT>::word_t bits, bool bulk) {
+    if (bulk) (void)seg_or<NT>(B.Fn, gseg, bits);
+    else discover<NT>(B, gseg, bits);
+}
+
 // Push-CSC tile item (Alg 5): OR the bit planes of the frontier's columns of tile t.
 template <int NT>
 __device__ __forceinline__ void push_tile_item(const BfsTiles &P, const BfsView &B, long long t,
-                                               typename Tr<NT>::word_t xm) {
+                                               typename Tr<NT>::word_t xm, bool bulk = false) {
     using word_t = typename Tr<NT>::word_t;
     word_t hit = ((const word_t *)P.mask)[t] & xm;
     if (hit) {
@@ -75,16 +85,16 @@ __device__ __forceinline__ void push_tile_item(const BfsTiles &P, const BfsView 
             hit &= hit - 1;
             w |= planes[(long long)c * P.T + t];
         }
-        discover<NT>(B, B.row_begin / NT + P.trow[t], w);
+        reach<NT>(B, B.row_begin / NT + P.trow[t], w, bulk);
     }
 }
 
 // Push over the side matrix: one side nonzero p of a frontier vertex's column.
 template <int NT>
-__device__ __forceinline__ void push_side_item(const BfsTiles &P, const BfsView &B, long long p) {
+__device__ __forceinline__ void push_side_item(const BfsTiles &P, const BfsView &B, long long p, bool bulk = false) {
     using word_t = typename Tr<NT>::word_t;
     long long v = B.row_begin + decode_row<NT>(P.srow[p], P.hot_list);
-    discover<NT>(B, v / NT, (word_t)1 << (v % NT));
+    reach<NT>(B, v / NT, (word_t)1 << (v % NT), bulk);
 }
 
 // Rows r of `um` whose row word in tile t meets the frontier word f.  nt = 16:

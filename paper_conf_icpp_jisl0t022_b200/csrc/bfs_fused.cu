@@ -74,6 +74,7 @@ struct BfsFusedArgs {
     int qcap;                 // usable entries of the shared-memory queue (<= QCAP; TSMV_BFS_QCAP tests the overflow path)
     int wide_in_kernel;       // pull levels with m_u < nnz / 4 stay in the kernel (wide pull)
     long long wide_cap;       // ... unless m_u > wide_cap (r2: large graphs)
+    int bulk_push;            // heavy Push-CSC levels in bulk mode (r2)
     // r2: L2 warm-up of the push structures + degrees (graphs whose structures fit
     // in half the L2): bulk L2 prefetches by every CTA before the first level, so the
     // latency-bound list / solo levels of high-diameter graphs hit L2, not HBM
@@ -847,6 +848,7 @@ __global__ void __launch_bounds__(BFB, TSMV_BFS_MINB) k_bfs_fused(BfsFusedArgs a
         }
 
         // ---- E: expand
+        bool bulk = false;
         if (dir == TSMV_DIR_PULL_CSC) {
             for (long long I0 = gwarp * 32; I0 < a.nTR_local; I0 += gwarps * 32)
                 pull_rowtiles32<NT>(a.Q, B, I0, a.nTR_local, lane);
@@ -857,6 +859,9 @@ __global__ void __launch_bounds__(BFB, TSMV_BFS_MINB) k_bfs_fused(BfsFusedArgs a
             const long long nLt = s_tot[0], Wt = s_tot[1], nLs = s_tot[2], Ws = s_tot[3];
             const long long nCt = dir == TSMV_DIR_PUSH_CSC ? (Wt + CHUNK - 1) >> CHUNK_LOG : 0;
             const long long nCs = (Ws + CHUNK - 1) >> CHUNK_LOG;
+            // heavy Push-CSC level (push items > n / 8): bulk mode, reductions into Fn
+            // then one pass over the words (below)
+            bulk = a.bulk_push && dir == TSMV_DIR_PUSH_CSC && (Wt + Ws) * 8 > B.n;
             long long *win = win_all[wid];
             unsigned ch = (unsigned)gwarp;
             while (true) {
@@ -873,7 +878,7 @@ __global__ void __launch_bounds__(BFB, TSMV_BFS_MINB) k_bfs_fused(BfsFusedArgs a
                             const int q = window_find(win, i);
                             const long long s = s0 + q;
                             push_tile_item<NT>(a.P, B, __ldcg(&a.Lv.Lt_tbeg[s]) + (i - win[q]),
-                                               (word_t)__ldcg(&a.Lv.Lt_mask[s]));
+                                               (word_t)__ldcg(&a.Lv.Lt_mask[s]), bulk);
                         }
                     }
                 } else if (ch < nCt + nCs) {
@@ -886,7 +891,7 @@ __global__ void __launch_bounds__(BFB, TSMV_BFS_MINB) k_bfs_fused(BfsFusedArgs a
                         const long long i = base + lane + 32 * u;
                         if (i < Ws) {
                             const int q = window_find(win, i);
-                            push_side_item<NT>(a.P, B, __ldcg(&a.Lv.Ls_beg[s0 + q]) + (i - win[q]));
+                            push_side_item<NT>(a.P, B, __ldcg(&a.Lv.Ls_beg[s0 + q]) + (i - win[q]), bulk);
                         }
                     }
                 } else {
@@ -897,6 +902,26 @@ __global__ void __launch_bounds__(BFB, TSMV_BFS_MINB) k_bfs_fused(BfsFusedArgs a
             }
         }
         grid_sync(&a.cnt->bar, target);
+        if (bulk) {
+            // new = Fn & ~V over all words (every reduction of the level has landed)
+            for (long long w = gtid; w < a.NW; w += gthreads) {
+                const uint32_t f = Fb[w];
+                if (!f) continue;
+                const uint32_t v = B.V[w];
+                const uint32_t nw = f & ~v;
+                Fb[w] = nw;
+                if (nw) {
+                    B.V[w] = v | nw;
+                    uint32_t bb = nw;
+                    while (bb) {
+                        const int r = __ffs(bb) - 1;
+                        bb &= bb - 1;
+                        B.levels[w * 32 + r] = level + 1;
+                    }
+                }
+            }
+            grid_sync(&a.cnt->bar, target);
+        }
         if (b == 0 && tid == 0) {
             const unsigned long long t = globaltimer_ns();
             t_e += t - tq;
@@ -1027,6 +1052,7 @@ bool bfs_fused_launch(tsmv_ctx *c, long long source, cudaStream_t st, bool resum
                      ? 1 : 0;
     a.wide_in_kernel = getenv("TSMV_BFS_HOST_WIDE") ? 0 : 1;
     a.wide_cap = bfs_wide_cap(c, false);
+    a.bulk_push = getenv("TSMV_BFS_NO_BULK") ? 0 : 1;
     a.qcap = getenv("TSMV_BFS_QCAP") ? std::max(1, std::min(QCAP, atoi(getenv("TSMV_BFS_QCAP")))) : QCAP;
     if (a.use_solo) TSMV_CUDA(cudaMemsetAsync(c->lslots.as<long long>() + 16, 0, 8, st));  // release flag
     a.pf_n = 0;

@@ -199,3 +199,23 @@ def test_level_times(tsmv):
         assert len(t) == st["nlevels"] and all(x >= 0 for x in t)
         assert 0.5 * st["ms"] <= sum(t) <= 1.05 * st["ms"] + 0.01, (sum(t), st["ms"])
     M.close()
+
+
+@pytest.mark.parametrize("sym", [True, False])
+def test_bulk_push_levels(tsmv, monkeypatch, sym):
+    """Heavy Push-CSC levels (push items > n / 8) run in bulk mode (reductions into
+    the next frontier, then one pass new = Fn & ~V): forced push on R-MAT makes
+    every middle level heavy; levels equal the oracle's with and without it."""
+    A = synth.rmat(14, 16, seed=21, symmetrize=sym)
+    C = oracle.csc_of(A)
+    M = tsmv.TiledMatrix.from_csr(A.to(DEV), dtype="pattern", force_dir=tsmv.DIR_PUSH_CSC, sparse_tile_max_nnz=8)
+    for s in [0] + synth.sample_sources(A, 3, seed=6):
+        ref = oracle.bfs_queue(C, s)
+        lv, st = M.bfs(s)
+        assert np.array_equal(lv.cpu().numpy(), ref)
+        assert st["reached"] == int((ref >= 0).sum())
+        monkeypatch.setenv("TSMV_BFS_NO_BULK", "1")
+        lv2, _ = M.bfs(s)
+        monkeypatch.delenv("TSMV_BFS_NO_BULK")
+        assert np.array_equal(lv2.cpu().numpy(), ref)
+    M.close()

@@ -203,15 +203,19 @@ __device__ __forceinline__ void pull_side_vertex(const BfsTiles &Q, const BfsVie
     if ((B.V[g >> 5] >> (g & 31)) & 1u) return;
     if (!((Q.smask[v >> 5] >> (v & 31)) & 1u)) return;  // no side in-edges
     long long p0 = Q.sptr[v], p1 = Q.sptr[v + 1];
-    // four in-neighbours per round: their ids, then their frontier bits, each
+    // PR in-neighbours per round: their ids, then their frontier bits, each
     // step as independent loads (early exit between rounds)
-    for (long long p = p0; p < p1; p += 4) {
-        int sr[4];
+#ifndef TSMV_PULL_ROUND
+#define TSMV_PULL_ROUND 2  // r2: 2 beats 4 and 8 (R-MAT s26 480 -> 493 GTEPS, s22 314 -> 319)
+#endif
+    constexpr int PR = TSMV_PULL_ROUND;
+    for (long long p = p0; p < p1; p += PR) {
+        int sr[PR];
 #pragma unroll
-        for (int j = 0; j < 4; ++j) sr[j] = p + j < p1 ? Q.srow[p + j] : 0;
+        for (int j = 0; j < PR; ++j) sr[j] = p + j < p1 ? Q.srow[p + j] : 0;
         bool hit = false;
 #pragma unroll
-        for (int j = 0; j < 4; ++j) {
+        for (int j = 0; j < PR; ++j) {
             if (p + j < p1) {
                 const long long u = decode_row<NT>(sr[j], Q.hot_list);
                 hit |= ((B.F[u >> 5] >> (u & 31)) & 1u) != 0;

@@ -442,12 +442,13 @@ __global__ void __launch_bounds__(256) k_fstats16(const uint32_t *__restrict__ F
 // Push (vector-driven): tile chunks (Push-CSC, Alg 5) and side chunks.
 template <int NT, bool DO_TILES>
 __global__ void __launch_bounds__(256)
-k_push(BfsTiles P, ListsView Lv, Counters *__restrict__ cnt, BfsView B) {
+k_push(BfsTiles P, ListsView Lv, Counters *__restrict__ cnt, BfsView B, int bulk_ok) {
     __shared__ long long win_all[8][CHUNK + 1];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     long long *win = win_all[wid];
     const long long nCt = DO_TILES ? cnt->nCt : 0, nCs = cnt->nCs;
     const long long nLt = cnt->nLt, nLs = cnt->nLs, Wt = cnt->Wt, Ws = cnt->Ws;
+    const bool bulk = bulk_ok && push_bulk(DO_TILES, Wt, Ws, B.m_local);  // k_bulk_fix finishes the level
     while (true) {
         unsigned ch = 0;
         if (lane == 0) ch = atomicAdd(&cnt->chunk_next, 1u);
@@ -462,7 +463,8 @@ k_push(BfsTiles P, ListsView Lv, Counters *__restrict__ cnt, BfsView B) {
                 if (i >= Wt) break;
                 int q = window_find(win, i);
                 long long s = s0 + q;
-                push_tile_item<NT>(P, B, Lv.Lt_tbeg[s] + (i - win[q]), (typename Tr<NT>::word_t)Lv.Lt_mask[s]);
+                push_tile_item<NT>(P, B, Lv.Lt_tbeg[s] + (i - win[q]), (typename Tr<NT>::word_t)Lv.Lt_mask[s],
+                                   bulk);
             }
             __syncwarp();
         } else if (ch < nCt + nCs) {
@@ -475,11 +477,36 @@ k_push(BfsTiles P, ListsView Lv, Counters *__restrict__ cnt, BfsView B) {
                 long long i = base + lane + 32 * u;
                 if (i >= Ws) break;
                 int q = window_find(win, i);
-                push_side_item<NT>(P, B, Lv.Ls_beg[s0 + q] + (i - win[q]));
+                push_side_item<NT>(P, B, Lv.Ls_beg[s0 + q] + (i - win[q]), bulk);
             }
             __syncwarp();
         } else {
             break;
+        }
+    }
+}
+
+// Bulk Push-CSC level (r2, as the fused kernel's): k_push only ORed the reached
+// rows into Fn; over this rank's words new = Fn & ~V, V |= new, levels (a no-op
+// when the level was not bulk: same test on the same counters)
+__global__ void k_bulk_fix(const Counters *__restrict__ cnt, BfsView B) {
+    if (!push_bulk(true, cnt->Wt, cnt->Ws, B.m_local)) return;
+    const long long w0 = B.row_begin >> 5, w1 = (B.row_begin + B.m_local + 31) >> 5;
+    for (long long w = w0 + blockIdx.x * (long long)blockDim.x + threadIdx.x; w < w1;
+         w += (long long)gridDim.x * blockDim.x) {
+        const uint32_t f = B.Fn[w];
+        if (!f) continue;
+        const uint32_t v = B.V[w];
+        const uint32_t nw = f & ~v;
+        B.Fn[w] = nw;
+        if (nw) {
+            B.V[w] = v | nw;
+            uint32_t bb = nw;
+            while (bb) {
+                const int r = __ffs(bb) - 1;
+                bb &= bb - 1;
+                B.levels[w * 32 + r - B.row_begin] = B.level + 1;
+            }
         }
     }
 }
@@ -901,9 +928,12 @@ struct BfsRunner {
         BfsView B = view();
         BfsTiles P = bfs_tiles(c->P), Q = bfs_tiles(*c->Q);
         if (dir == TSMV_DIR_PUSH_CSC) {
-            k_push<NT, true><<<c->expand_blocks, 256, 0, st>>>(P, lists_view(c), c->counters.as<Counters>(), B);
+            const int bulk_ok = getenv("TSMV_BFS_NO_BULK") ? 0 : 1;
+            k_push<NT, true><<<c->expand_blocks, 256, 0, st>>>(P, lists_view(c), c->counters.as<Counters>(), B,
+                                                               bulk_ok);
+            if (bulk_ok) k_bulk_fix<<<grid_for((c->m + 31) / 32), 256, 0, st>>>(c->counters.as<Counters>(), B);
         } else if (dir == TSMV_DIR_PUSH_CSR) {
-            k_push<NT, false><<<c->expand_blocks, 256, 0, st>>>(P, lists_view(c), c->counters.as<Counters>(), B);
+            k_push<NT, false><<<c->expand_blocks, 256, 0, st>>>(P, lists_view(c), c->counters.as<Counters>(), B, 0);
             if (Q.T) k_push_csr<NT><<<grid_for(Q.T), 256, 0, st>>>(Q, B);
         } else {
             long long nTRl = (c->m + NT - 1) / NT;

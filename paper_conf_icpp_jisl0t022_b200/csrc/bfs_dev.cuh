@@ -61,6 +61,11 @@ inline BfsTiles bfs_tiles(const TileSet &S) {
 
 // ---- one item of each level kernel -------------------------------------------
 
+// heavy Push-CSC level of the per-level kernels (push items > rows / 8): bulk mode
+__host__ __device__ __forceinline__ bool push_bulk(bool csc, long long Wt, long long Ws, long long rows) {
+    return csc && (Wt + Ws) * 8 > rows;
+}
+
 // Bulk push (r2): the rows reached are only ORed into the next-frontier bitmap
 // with fire-and-forget reductions; a pass over the words afterwards takes new =
 // Fn & ~V, sets V and the levels (heavy Push-CSC levels: one returning atomic per

@@ -155,3 +155,18 @@ def test_sim_ranks_dist_spmspv_owned_x(P, monkeypatch):
     for I, V in ((gi, gv), (ai, av)):
         assert np.array_equal(np.concatenate(I), ri)
         assert np.allclose(np.concatenate(V), rv, rtol=1e-12, atol=0)
+
+
+def test_sim_ranks_bulk_push(monkeypatch):
+    """Heavy Push-CSC levels of the per-level kernels in bulk mode (k_push ORs into
+    the next frontier, k_bulk_fix takes new = Fn & ~V over the owned words):
+    forced push on simulated ranks, with and without it."""
+    A = synth.rmat(13, 16, seed=17, symmetrize=True)
+    C = oracle.csc_of(A)
+    _, engines = _ranks(A, 3, force_dir=1)
+    for s in [0] + synth.sample_sources(A, 2, seed=9):
+        ref = oracle.bfs_queue(C, s)
+        assert np.array_equal(_sim_bfs(engines, s, expect=_level_stats(A, ref)), ref)
+        monkeypatch.setenv("TSMV_BFS_NO_BULK", "1")
+        assert np.array_equal(_sim_bfs(engines, s), ref)
+        monkeypatch.delenv("TSMV_BFS_NO_BULK")

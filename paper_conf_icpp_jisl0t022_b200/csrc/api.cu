@@ -386,7 +386,9 @@ extern "C" tsmv_status tsmv_get_info(const tsmv_ctx *c, tsmv_info *info) {
     info->bytes_bfs = (int64_t)(c->P.planes.bytes + (c->Q == &c->Qown ? c->Qown.bytes() : 0));
     info->bytes_workspace = (int64_t)(c->acc.bytes + c->rowbits.bytes + c->desc_compact.bytes + c->L.bytes() +
                                       c->V.bytes + c->F0.bytes + c->F1.bytes + c->desc_bfs.bytes +
-                                      c->outdeg.bytes + c->indeg.bytes);
+                                      c->outdeg.bytes + c->indeg.bytes + c->pb_rs.bytes + c->pb_row.bytes +
+                                      c->pb_val.bytes + c->pb_cnt.bytes + c->pb_agg.bytes +
+                                      c->pb_hp.bytes + c->pb_hr.bytes + c->pb_hs.bytes + c->pb_hso.bytes);
     info->build_ms = c->build_ms;
     return TSMV_OK;
 }

@@ -324,6 +324,17 @@ struct tsmv_ctx {
     long long flat_calls = 0;      // flat SpMSpV launches so far (piece-count buffer parity)
     int last_blocks = 0;           // CTAs of the last SpMSpV launch (partials / acct rows)
     tsmv::DevBuf partials;         // long long[fused_blocks][8]
+    // bucketed flat SpMSpV (propagation blocking, spmspv_flat.cu), set up on first use
+    int pb_state = 0;              // 0 = not yet, 1 = ready, -1 = unavailable (too many buckets)
+    int pb_bl = 0, pb_nb = 0, pb_cap = 0;
+    long long pb_calls = 0;        // bucketed launches so far (counter parity, look-back epoch)
+    tsmv::DevBuf pb_rs;            // int64[NB + 1]: staging region of bucket q (nonzeros of its rows)
+    tsmv::DevBuf pb_row, pb_val;   // u32[nnz], u64[nnz]: staged products / compacted output rows
+    tsmv::DevBuf pb_cnt;           // u32[2][NB]: staged products per bucket, double-buffered by call parity
+    tsmv::DevBuf pb_agg;           // u64[2][MAXG]: look-back aggregates, contributed list lengths
+    tsmv::DevBuf pb_hp;            // u64[MAXG][hot slots]: per-CTA hot-row partials
+    tsmv::DevBuf pb_hr;            // u64[hot slots] reduced values + u32[hot slots] their epochs
+    tsmv::DevBuf pb_hs, pb_hso;    // int32: hot slots by bucket, and their offsets [NB + 1]
     long long last_x_nnz = 0;
     int bfs_blocks = 0;            // CTAs of the fused BFS kernel
     long long bfs_last_levels = 0;

@@ -1135,25 +1135,33 @@ extern "C" tsmv_status tsmv_spmspv(tsmv_ctx *c, tsmv_semiring sr, int64_t x_nnz,
         int32_t *yi = y_idx;
         void *yv = (sr == TSMV_OR_AND) ? nullptr : y_val;
         int64_t ycap_dev = y_cap;
-        if (host_y || host_yv) ycap_dev = std::min<int64_t>(y_cap, c->m);
-        if (host_y) {
-            c->stage_y_idx.ensure(std::max<int64_t>(ycap_dev, 1) * 4);
-            yi = c->stage_y_idx.as<int32_t>();
-        }
-        if (host_yv) {
-            c->stage_y_val.ensure(std::max<int64_t>(ycap_dev, 1) * vb);
-            yv = c->stage_y_val.p;
-        }
-        // pinned (mapped) host y: copied by a kernel sized on the device, right
-        // behind the multiply, then ONE synchronisation for the whole call
+        // pinned (mapped) host y: the kernel's compaction phase writes y straight
+        // into the caller's host buffers (zero copy: the PCIe writes overlap the
+        // compaction, no copy kernel), then ONE synchronisation for the whole call.
+        // Pageable host y is staged on the device and copied after the sync.
         void *myi = host_y ? mapped_device_ptr(y_idx) : nullptr;
         void *myv = host_yv ? mapped_device_ptr(y_val) : nullptr;
         const bool direct = (!host_y || myi) && (!host_yv || myv) && (host_y || host_yv);
+        const bool copy_kernel = direct && getenv("TSMV_Y_COPY_KERNEL");  // r2 path, A/B only
+        if (direct && !copy_kernel) {
+            if (host_y) yi = static_cast<int32_t *>(myi);
+            if (host_yv) yv = myv;
+        } else if (host_y || host_yv) {
+            ycap_dev = std::min<int64_t>(y_cap, c->m);
+            if (host_y) {
+                c->stage_y_idx.ensure(std::max<int64_t>(ycap_dev, 1) * 4);
+                yi = c->stage_y_idx.as<int32_t>();
+            }
+            if (host_yv) {
+                c->stage_y_val.ensure(std::max<int64_t>(ycap_dev, 1) * vb);
+                yv = c->stage_y_val.p;
+            }
+        }
         volatile Counters *h = c->hcnt;
         int err = 0;
         for (int attempt = 0; attempt < 2; ++attempt) {
             enqueue_spmspv(c, sr, x_nnz, xi, xv, ycap_dev, yi, yv, nullptr, st);
-            if (direct) {
+            if (copy_kernel) {
                 k_copy_y<<<c->sm_count * 4, 256, 0, st>>>(yi, yv, &c->counters.as<Counters>()->y_nnz, y_cap,
                                                            static_cast<int32_t *>(myi), myv, (int)vb);
                 TSMV_CUDA(cudaGetLastError());

@@ -26,6 +26,7 @@
 #include "spmspv_common.cuh"
 #include <algorithm>
 #include <cstdlib>
+#include <vector>
 
 namespace tsmv {
 
@@ -93,20 +94,110 @@ struct FlatArgs {
     const int32_t *hot_list;
     int n_hot;
     unsigned long long *trace;  // tsmv_set_trace: per CTA 8 globaltimer stamps (dev aid)
+    // row buckets (propagation blocking, r2 session 5): products are
+    // staged per CTA in shared memory, written to the staging region of their row
+    // bucket (2^pb_bl rows) and merged bucket by bucket in shared memory in phase C
+    const long long *pb_rs;      // int64[NB + 1]: staging region of bucket q = nonzeros of its rows
+    unsigned *pb_row;            // staging: row inside the bucket; phase C output: local row
+    unsigned long long *pb_val;  // staging: the product in accumulator encoding
+    unsigned *pb_cnt;            // u32[NB]: staged products of bucket q | flags (PB_CNT)
+    unsigned *pb_cnt_next;       // the other parity's counters: zeroed here for the next call
+    unsigned long long *pb_agg;  // u64[G]: (epoch << 32) | output rows of CTA b (look-back)
+    unsigned long long *pb_pu;   // u64[G]: (epoch << 32) | length of CTA b's contributed partial list
+    unsigned long long *pb_hp;   // u64[G][n_slots]: hot-row partials of CTA b (EMPTY = untouched)
+    unsigned long long *pb_hr;   // u64[n_slots]: reduced hot-row values of this call
+    unsigned *pb_hre;            // u32[n_slots]: epoch of pb_hr[slot] (published)
+    const int *pb_hs;            // hot slots grouped by bucket: slots of bucket q = pb_hs[pb_hso[q] .. pb_hso[q+1])
+    const int *pb_hso;
+    unsigned pb_epoch;
+    int pb_bl, pb_nb, pb_cap;    // bucket width log2, bucket count, staged products per CTA in shared memory
+    long long pb_ovh;            // phase-C weight of a non-empty bucket (its bitmap work), in products
 };
+
+// A contribution a*x in accumulator encoding (spmspv_common.cuh): the fp64
+// product (-0.0 -> +0.0), the min-second key of x, or nothing (Boolean).
+template <int SR> __device__ __forceinline__ unsigned long long enc_prod(double av, double xv) {
+    if constexpr (SR == TSMV_PLUS_TIMES) return (unsigned long long)__double_as_longlong(prod_nz(av, xv));
+    else if constexpr (SR == TSMV_MIN_SECOND) return ~ord_key(xv) ^ EMPTY;
+    else return 0ull;
+}
+// Combine an encoded partial value into the global accumulator; true if the row
+// was untouched (EMPTY) before.
+template <int SR> __device__ __forceinline__ bool acc_combine_first(double *acc, long long row, unsigned long long v) {
+    if constexpr (SR == TSMV_PLUS_TIMES)
+        return (unsigned long long)__double_as_longlong(atomicAdd(&acc[row], __longlong_as_double((long long)v))) == EMPTY;
+    else if constexpr (SR == TSMV_MIN_SECOND)
+        return (unsigned long long)atomicMax((long long *)&acc[row], (long long)v) == EMPTY;
+    else
+        return atomicExch((unsigned long long *)&acc[row], 0ull) == EMPTY;
+}
+// Combine into a shared-memory accumulator slot (several threads: atomics).
+template <int SR> __device__ __forceinline__ void sacc_combine(double *s, int r, unsigned long long v) {
+    if constexpr (SR == TSMV_PLUS_TIMES) atomicAdd(&s[r], __longlong_as_double((long long)v));
+    else if constexpr (SR == TSMV_MIN_SECOND) atomicMax((long long *)&s[r], (long long)v);
+}
+// The same for a slot owned by the calling thread.
+template <int SR> __device__ __forceinline__ void sacc_combine_own(double *s, int r, unsigned long long v) {
+    if constexpr (SR == TSMV_PLUS_TIMES) s[r] = s[r] + __longlong_as_double((long long)v);
+    else if constexpr (SR == TSMV_MIN_SECOND) {
+        const long long o = __double_as_longlong(s[r]);
+        if ((long long)v > o) s[r] = __longlong_as_double((long long)v);
+    }
+}
+
+// Bucket counter: staged products (bits 0-29), a hot row touched (bit 30), rows
+// in the global accumulator from a staging-buffer overflow (bit 31).
+constexpr unsigned PB_CNT = 0x3fffffffu;
+
+// Per-CTA product staging buffer in shared memory (bucketed variant).
+struct PBS {
+    unsigned *cur;             // products staged so far by the CTA
+    unsigned *row;             // [cap] local row
+    unsigned long long *val;   // [cap] encoded value
+    int cap;
+};
+// Stage one product (row >= 0, encoded value v).  Slots are reserved with one
+// shared-memory atomic per warp (the lanes that stage together).  Beyond the
+// buffer's capacity the product goes to the global accumulator instead; its
+// row's touched bit is set and its bucket flagged, and phase C merges it.
+template <int SR>
+__device__ __forceinline__ void stage(const FlatArgs &a, const PBS &s, long long row, unsigned long long v) {
+    const unsigned am = __activemask();
+    const int lane = threadIdx.x & 31;
+    const int leader = __ffs(am) - 1;
+    unsigned base = 0;
+    if (lane == leader) base = atomicAdd(s.cur, (unsigned)__popc(am));
+    base = __shfl_sync(am, base, leader);
+    const unsigned slot = base + (unsigned)__popc(am & ((1u << lane) - 1u));
+    if (slot < (unsigned)s.cap) {
+        s.row[slot] = (unsigned)row;
+        s.val[slot] = v;
+        return;
+    }
+    if (acc_combine_first<SR>(a.acc, row, v)) {
+        atomicOr(&a.rowbits[row >> 5], 1u << (row & 31));
+        atomicOr(&a.pb_cnt[row >> a.pb_bl], 0x80000000u);
+    }
+}
 
 // One contribution a*x to row code `rc` (>= 0: local row; < 0: ~hot slot).
 // Returns the row whose touched bit must be set (first contribution), or -1.
-template <int SR>
-__device__ __forceinline__ long long contribute(const FlatArgs &a, double *s_hacc, uint32_t *s_hbits, long long rc,
-                                                double av, double xv) {
+// Bucketed variant (PB): the product is staged and -1 returned.
+template <int SR, bool PB>
+__device__ __forceinline__ long long contribute(const FlatArgs &a, double *s_hacc, uint32_t *s_hbits, const PBS &ps,
+                                                long long rc, double av, double xv) {
     if (rc < 0) {
         const int sl = (int)~rc;
         acc_shared<SR>(s_hacc, sl, av, xv);
         atomicOr(&s_hbits[sl >> 5], 1u << (sl & 31));
         return -1;
     }
-    return acc_first<SR>(a.acc, rc, av, xv) ? rc : -1;
+    if constexpr (PB) {
+        stage<SR>(a, ps, rc, enc_prod<SR>(av, xv));
+        return -1;
+    } else {
+        return acc_first<SR>(a.acc, rc, av, xv) ? rc : -1;
+    }
 }
 // first touch of `row` (>= 0; -1 = none): its bit, and its piece's count in the
 // CTA's shared-memory counters (added to the global ones once, at the end of B)
@@ -148,7 +239,407 @@ __device__ __forceinline__ ColInfo load_colinfo(const ColInfo *p) {
     return c;
 }
 
-template <class AV, class XV, int SR>
+__device__ __forceinline__ unsigned ld_acquire_u32(const unsigned *p) {
+    unsigned v;
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ unsigned ld_relaxed_u32(const unsigned *p) {
+    unsigned v;
+    asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ unsigned long long ld_relaxed_u64(const unsigned long long *p) {
+    unsigned long long v;
+    asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_release_u32(unsigned *p, unsigned v) {
+    asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ void st_release_u64(unsigned long long *p, unsigned long long v) {
+    asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+
+// Bucketed variant, end of phase B.  The CTA's privatised hot-row partials go
+// to its row of pb_hp (coalesced, EMPTY where untouched; phase C reduces them
+// over the CTAs).  The staged products are counting-sorted by bucket in shared
+// memory (rank per product, bucket starts by a block scan, permutation), one
+// global reservation per (CTA, non-empty bucket) places the CTA's run in the
+// bucket's staging region, and the sorted products are stored with consecutive
+// threads writing consecutive positions of each run.
+template <int SR>
+__device__ void pb_flush(const FlatArgs &a, const PBS &ps, const double *s_hacc, const uint32_t *s_hbits,
+                         int n_slots, unsigned *s_bhist, long long *s_bbase, unsigned short *s_brank,
+                         unsigned short *s_perm, bool err, long long (*s_acct)[4], long long (*s_scan)[NWF],
+                         unsigned long long *tr) {
+    const int tid = threadIdx.x, b = blockIdx.x;
+    if (tid < 4) {
+        long long sum = 0;
+        for (int w = 0; w < NWF; ++w) sum += s_acct[w][tid];
+        a.acct[b * 4 + tid] = sum;
+    }
+    if (err) return;
+    const int BL = a.pb_bl, NB = a.pb_nb;
+    for (int q = tid; q < n_slots; q += FT) {
+        const bool t = (s_hbits[q >> 5] >> (q & 31)) & 1u;
+        a.pb_hp[(long long)b * n_slots + q] =
+            !t ? EMPTY : (SR == TSMV_OR_AND ? 0ull : (unsigned long long)__double_as_longlong(s_hacc[q]));
+    }
+    if (tr && tid == 0) tr[12] = globaltimer_ns();
+    const int nb = (int)min(*ps.cur, (unsigned)ps.cap);
+    for (int i = tid; i < nb; i += FT) s_brank[i] = (unsigned short)atomicAdd(&s_bhist[ps.row[i] >> BL], 1u);
+    __syncthreads();
+    if (tr && tid == 0) tr[13] = globaltimer_ns();
+    {
+        constexpr int PPT = 4;  // NB <= 4 * FT (host)
+        long long h[PPT], run = 0;
+#pragma unroll
+        for (int i = 0; i < PPT; ++i) {
+            const int q = tid * PPT + i;
+            h[i] = q < NB ? (long long)s_bhist[q] : 0;
+            run += h[i];
+        }
+        long long ex, tot;
+        block_scan<1, FT>(&run, &ex, &tot, s_scan);
+#pragma unroll
+        for (int i = 0; i < PPT; ++i) {
+            const int q = tid * PPT + i;
+            if (q < NB) {
+                s_bhist[q] = (unsigned)ex;  // now the bucket's first sorted slot
+                if (h[i])
+                    s_bbase[q] = __ldg(&a.pb_rs[q]) + (long long)(atomicAdd(&a.pb_cnt[q], (unsigned)h[i]) & PB_CNT) - ex;
+            }
+            ex += h[i];
+        }
+    }
+    __syncthreads();
+    if (tr && tid == 0) tr[14] = globaltimer_ns();
+    for (int i = tid; i < nb; i += FT) s_perm[s_bhist[ps.row[i] >> BL] + s_brank[i]] = (unsigned short)i;
+    __syncthreads();
+    const unsigned lm = (1u << BL) - 1u;
+    for (int j = tid; j < nb; j += FT) {
+        const int i = s_perm[j];
+        const unsigned r = ps.row[i];
+        const long long pos = s_bbase[r >> BL] + j;
+        a.pb_row[pos] = r & lm;
+        a.pb_val[pos] = ps.val[i];
+    }
+}
+
+// CTA of weight position `pos`: the largest c with floor(W c / G) <= pos.
+__device__ __forceinline__ int pb_cta_of(long long pos, long long W, int G) {
+    int lo = 0, hi = G - 1;
+    while (lo < hi) {
+        const int mid = (lo + hi + 1) >> 1;
+        if (W * mid / G <= pos) lo = mid;
+        else hi = mid - 1;
+    }
+    return lo;
+}
+
+// Semiring join of two encoded partial values (EMPTY is the identity).
+template <int SR> __device__ __forceinline__ unsigned long long pb_join(unsigned long long x, unsigned long long y) {
+    if constexpr (SR == TSMV_PLUS_TIMES)
+        return (unsigned long long)__double_as_longlong(__longlong_as_double((long long)x) +
+                                                       __longlong_as_double((long long)y));
+    else if constexpr (SR == TSMV_MIN_SECOND)
+        return (long long)x > (long long)y ? x : y;
+    else
+        return (x == EMPTY && y == EMPTY) ? EMPTY : 0ull;
+}
+
+// Accumulate a list of (row inside the bucket, encoded value) pairs into the
+// CTA's shared-memory bucket (UN loads in flight per thread).
+template <int SR>
+__device__ __forceinline__ void pb_accumulate(const unsigned *rows, const unsigned long long *vals, long long n,
+                                              double *c_acc, unsigned *c_bits) {
+    constexpr int UN = 4;
+    const int tid = threadIdx.x;
+    for (long long i0 = 0; i0 < n; i0 += (long long)UN * FT) {
+        unsigned r[UN];
+        unsigned long long v[UN];
+#pragma unroll
+        for (int u = 0; u < UN; ++u) {
+            const long long i = i0 + tid + (long long)u * FT;
+            r[u] = 0xffffffffu;
+            if (i < n) {
+                r[u] = __ldcg(&rows[i]);
+                v[u] = __ldcg(&vals[i]);
+            }
+        }
+#pragma unroll
+        for (int u = 0; u < UN; ++u) {
+            if (r[u] != 0xffffffffu) {
+                sacc_combine<SR>(c_acc, (int)r[u], v[u]);
+                atomicOr(&c_bits[r[u] >> 5], 1u << (r[u] & 31));
+            }
+        }
+    }
+}
+
+// Write the CTA's shared-memory bucket as a compact list (rows ascending, row
+// code = row0 + row inside the bucket) and clear it; returns the list length
+// (all threads).
+__device__ __forceinline__ long long pb_compact(double *c_acc, unsigned *c_bits, unsigned *c_wex, int WB,
+                                                long long (*s_scan)[NWF], unsigned *dst_row,
+                                                unsigned long long *dst_val, long long row0) {
+    const int tid = threadIdx.x, NWB = WB >> 5;
+    long long pc = tid < NWB ? __popc(c_bits[tid]) : 0, wex, ub;
+    block_scan<1, FT>(&pc, &wex, &ub, s_scan);
+    if (tid < NWB) c_wex[tid] = (unsigned)wex;
+    __syncthreads();
+    for (int r = tid; r < WB; r += FT) {
+        const unsigned wb = c_bits[r >> 5];
+        if ((wb >> (r & 31)) & 1u) {
+            const long long pos = c_wex[r >> 5] + __popc(wb & ((1u << (r & 31)) - 1u));
+            dst_row[pos] = (unsigned)(row0 + r);
+            dst_val[pos] = (unsigned long long)__double_as_longlong(c_acc[r]);
+            c_acc[r] = __longlong_as_double((long long)EMPTY);
+        }
+    }
+    __syncthreads();
+    if (tid < NWB) c_bits[tid] = 0u;
+    return ub;
+}
+
+// Bucketed variant, phase C (a6).  Bucket q weighs its staged products plus
+// pb_ovh (if non-empty); the weight line is cut into G equal ranges and CTA b
+// takes the products in its range.  A bucket wholly inside one range is merged
+// by that CTA alone in shared memory (dense 2^BL-row accumulator + bitmap).  A
+// bucket spanning several ranges is "shared": each CTA after its first one
+// (a contributor; a CTA contributes to at most one bucket, its first) merges
+// its share, writes it back compacted in place over that share and publishes
+// the length (pb_pu[c], epoch-tagged); the first CTA (the emitter) merges its
+// own share and the contributors' lists.  Rows in the global accumulator (hot
+// rows, staging-buffer overflow: the bucket's bit 31) are merged by the emitter
+// from the touched bitmap.  Every CTA compacts its emitted buckets, in bucket
+// order, into the staging region from its first emitted bucket on (in place: a
+// bucket has at most as many output rows as nonzeros), then finds its y offset
+// by look-back over the CTAs before it and copies its rows to y.
+template <int SR, class XV>
+__device__ void pb_emit(const FlatArgs &a, bool err, long long (*s_scan)[NWF], unsigned char *s_dyn,
+                        int n_slots, unsigned long long *tr) {
+    __shared__ int s_qlo, s_qhi;
+    __shared__ long long s_off, s_u, s_pl;
+    const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+    const int G = gridDim.x, b = blockIdx.x;
+    const int BL = a.pb_bl, NB = a.pb_nb;
+    const int WB = 1 << BL, NWB = WB >> 5;
+    double *c_acc = reinterpret_cast<double *>(s_dyn);             // [WB]
+    unsigned *c_bits = reinterpret_cast<unsigned *>(c_acc + WB);    // [NWB]
+    unsigned *c_wex = c_bits + NWB;                                 // [NWB]
+    long long *s_S = reinterpret_cast<long long *>(c_wex + NWB);    // [NB]: weight prefix of bucket q
+    long long U = 0, out0 = -1;
+    if (!err) {
+        for (int i = tid; i < WB; i += FT) c_acc[i] = __longlong_as_double((long long)EMPTY);
+        for (int i = tid; i < NWB; i += FT) c_bits[i] = 0u;
+        constexpr int PPT = 4;  // NB <= 4 * FT (host)
+        long long wv[PPT], run = 0;
+#pragma unroll
+        for (int i = 0; i < PPT; ++i) {
+            const int q = tid * PPT + i;
+            wv[i] = 0;
+            if (q < NB) {
+                const unsigned cv = __ldcg(&a.pb_cnt[q]);
+                const long long c = cv & PB_CNT;
+                const bool hot = n_slots && __ldg(&a.pb_hso[q + 1]) > __ldg(&a.pb_hso[q]);
+                wv[i] = (cv || hot) ? c + a.pb_ovh : 0;
+            }
+            run += wv[i];
+        }
+        long long ex, Wt;
+        block_scan<1, FT>(&run, &ex, &Wt, s_scan);
+        const long long lo = Wt * b / G, hi = Wt * (b + 1) / G;
+        if (tid == 0) {
+            s_qlo = NB;
+            s_qhi = -1;
+        }
+        __syncthreads();
+#pragma unroll
+        for (int i = 0; i < PPT; ++i) {
+            const int q = tid * PPT + i;
+            if (q < NB) {
+                s_S[q] = ex;
+                if (wv[i] > 0 && ex < hi && ex + wv[i] > lo) {
+                    atomicMin(&s_qlo, q);
+                    atomicMax(&s_qhi, q);
+                }
+            }
+            ex += wv[i];
+        }
+        __syncthreads();
+        // hot rows: warp w of the grid reduces the CTAs' partials of hot slot w and
+        // publishes the result (epoch-tagged) for the bucket's emitter
+        for (int sl = b * NWF + wid; sl < n_slots; sl += G * NWF) {
+            constexpr int NP = MAXG / 32;
+            unsigned long long v[NP];
+#pragma unroll
+            for (int i = 0; i < NP; ++i)
+                v[i] = lane + 32 * i < G ? __ldcg(&a.pb_hp[(long long)(lane + 32 * i) * n_slots + sl]) : EMPTY;
+            unsigned long long t = EMPTY;
+#pragma unroll
+            for (int i = 0; i < NP; ++i) t = pb_join<SR>(t, v[i]);
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1) t = pb_join<SR>(t, __shfl_xor_sync(0xffffffffu, t, o));
+            if (lane == 0) {
+                a.pb_hr[sl] = t;
+                st_release_u32(&a.pb_hre[sl], a.pb_epoch);
+            }
+        }
+        const int q0 = s_qlo, q1 = s_qhi;
+        if (tr && tid == 0) tr[15] = (unsigned long long)(q1 - q0 + 1) * 1000ull;  // dev aid: buckets met (x1000 for the us print)
+        for (int q = q0; q <= q1; ++q) {
+            const unsigned cv = __ldcg(&a.pb_cnt[q]);
+            const long long cq = cv & PB_CNT;
+            const bool ovf = (cv >> 31) != 0u;
+            const int h0 = n_slots ? __ldg(&a.pb_hso[q]) : 0, h1 = n_slots ? __ldg(&a.pb_hso[q + 1]) : 0;
+            if (!cv && h1 == h0) continue;
+            const long long Sq = s_S[q];
+            const long long p0 = max(lo, Sq) - Sq, p1 = min(hi, Sq + cq) - Sq;
+            const bool emit = Sq >= lo && Sq < hi;
+            if (!emit && p1 <= p0) continue;
+            const long long rs = __ldg(&a.pb_rs[q]);
+            if (p1 > p0) pb_accumulate<SR>(a.pb_row + rs + p0, a.pb_val + rs + p0, p1 - p0, c_acc, c_bits);
+            const long long grow0 = (long long)q << BL;
+            if (emit) {
+                // hot rows of the bucket: the reduced partials published above
+                for (int h = h0 + tid; h < h1; h += FT) {
+                    const int sl = __ldg(&a.pb_hs[h]);
+                    while (ld_relaxed_u32(&a.pb_hre[sl]) != a.pb_epoch) {
+                    }
+                    (void)ld_acquire_u32(&a.pb_hre[sl]);
+                    const unsigned long long t = __ldcg(&a.pb_hr[sl]);
+                    if (t != EMPTY) {
+                        const long long row = (long long)__ldg(&a.hot_list[sl / 16]) * 16 + sl % 16;
+                        const int r = (int)(row - grow0);
+                        sacc_combine<SR>(c_acc, r, t);
+                        atomicOr(&c_bits[r >> 5], 1u << (r & 31));
+                    }
+                }
+            }
+            __syncthreads();
+            if (!emit) {
+                // a later share of a shared bucket: compacted in place, length published
+                const long long u = pb_compact(c_acc, c_bits, c_wex, WB, s_scan, a.pb_row + rs + p0,
+                                               a.pb_val + rs + p0, 0);
+                __threadfence();
+                __syncthreads();
+                if (tid == 0)
+                    st_release_u64(&a.pb_pu[b], ((unsigned long long)a.pb_epoch << 32) | (unsigned long long)u);
+                continue;
+            }
+            if (cq > 0 && p1 < cq) {
+                // the contributors: the CTAs after b whose (non-empty) range meets the
+                // bucket (every range is non-empty once Wt >= G)
+                const int last = pb_cta_of(Sq + cq - 1, Wt, G);
+                for (int c = b + 1; c <= last; ++c) {
+                    const long long loc = Wt * c / G;
+                    if (loc >= Wt * (c + 1) / G) continue;
+                    if (tid == 0) {
+                        unsigned long long v;
+                        do {
+                            v = ld_acquire_u64(&a.pb_pu[c]);
+                        } while ((unsigned)(v >> 32) != a.pb_epoch);
+                        s_pl = (long long)(v & 0xffffffffull);
+                    }
+                    __syncthreads();
+                    const long long off = rs + (loc - Sq);
+                    pb_accumulate<SR>(a.pb_row + off, a.pb_val + off, s_pl, c_acc, c_bits);
+                    __syncthreads();
+                }
+            }
+            if (ovf) {
+                // the bucket's rows in the global accumulator (clear on read); 4 rows
+                // per thread in flight
+                const int IT = WB / FT;
+                for (int i0 = 0; i0 < IT; i0 += 4) {
+                    unsigned wb[4];
+                    unsigned long long v[4];
+#pragma unroll
+                    for (int u = 0; u < 4; ++u) {
+                        const long long row = grow0 + tid + (long long)(i0 + u) * FT;
+                        wb[u] = (i0 + u < IT && row < a.m) ? __ldcg(&a.rowbits[row >> 5]) : 0u;
+                    }
+#pragma unroll
+                    for (int u = 0; u < 4; ++u) {
+                        const long long row = grow0 + tid + (long long)(i0 + u) * FT;
+                        if ((wb[u] >> lane) & 1u) v[u] = (unsigned long long)__ldcg((const long long *)&a.acc[row]);
+                    }
+#pragma unroll
+                    for (int u = 0; u < 4; ++u) {
+                        const int r = tid + (i0 + u) * FT;
+                        const bool set = (wb[u] >> lane) & 1u;
+                        if (set) {
+                            a.acc[grow0 + r] = __longlong_as_double((long long)EMPTY);
+                            sacc_combine_own<SR>(c_acc, r, v[u]);
+                        }
+                        const unsigned bal = __ballot_sync(0xffffffffu, set);
+                        if (lane == 0 && bal) {
+                            c_bits[r >> 5] |= bal;
+                            a.rowbits[(grow0 + r) >> 5] = 0u;
+                        }
+                    }
+                }
+                __syncthreads();
+            }
+            if (out0 < 0) out0 = rs;
+            U += pb_compact(c_acc, c_bits, c_wex, WB, s_scan, a.pb_row + out0 + U, a.pb_val + out0 + U, grow0);
+            __syncthreads();
+        }
+    }
+    // look-back: y offset of this CTA = output rows of the CTAs before it
+    if (tid == 0) st_release_u64(&a.pb_agg[b], ((unsigned long long)a.pb_epoch << 32) | (unsigned long long)U);
+    if (tr && tid == 0) tr[10] = globaltimer_ns();
+    if (wid == 0) {
+        // all predecessors' aggregates polled at once (relaxed: only the counts are used)
+        constexpr int NP = MAXG / 32;
+        unsigned long long v[NP];
+        const unsigned long long ready = (unsigned long long)a.pb_epoch << 32;
+#pragma unroll
+        for (int i = 0; i < NP; ++i) v[i] = lane + 32 * i < b ? ld_relaxed_u64(&a.pb_agg[lane + 32 * i]) : ready;
+        long long s = 0;
+#pragma unroll
+        for (int i = 0; i < NP; ++i) {
+            while ((unsigned)(v[i] >> 32) != a.pb_epoch) v[i] = ld_relaxed_u64(&a.pb_agg[lane + 32 * i]);
+            s += (long long)(v[i] & 0xffffffffull);
+        }
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+        if (lane == 0) {
+            s_off = s;
+            s_u = U;
+        }
+    }
+    __syncthreads();
+    if (tr && tid == 0) tr[11] = globaltimer_ns();
+    const long long off = s_off;
+    for (long long i = tid; i < U; i += FT) {
+        const long long pos = off + i;
+        if (pos < a.y_cap) {
+            const unsigned row = __ldcg(&a.pb_row[out0 + i]);
+            a.y_idx[pos] = (int32_t)((long long)row + a.row_begin);
+            if (a.y_val) {
+                const unsigned long long v = __ldcg(&a.pb_val[out0 + i]);
+                double x = __longlong_as_double((long long)v);
+                if constexpr (SR == TSMV_MIN_SECOND) x = ord_val(~(v ^ EMPTY));
+                ((XV *)a.y_val)[pos] = (XV)x;
+            }
+        }
+    }
+    if (b == G - 1 && tid == 0) {
+        const long long yt = off + U;
+        a.cnt->y_nnz = yt;
+        a.hm->y_nnz = yt;
+        if (a.ynnz_dev) *a.ynnz_dev = err ? -1 : yt;
+    }
+}
+
+// dynamic shared memory of phase B before the bucketed variant's staging buffer
+constexpr size_t FLAT_DYN_B0 = HOT_SLOTS * 8 + (size_t)NWF * ((1 << WL) + 1) * 24 + HOT_SLOTS / 8;
+constexpr size_t pb_align(size_t x) { return (x + 15) & ~(size_t)15; }
+
+template <class AV, class XV, int SR, bool PB>
 __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
     constexpr int NT = 16, LOG = 4;
     constexpr int WN = (1 << WL) + 1;
@@ -159,7 +650,31 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
     long long *s_winb = s_win + NWF * WN;                                         // [NWF][WN]
     double *s_winx = reinterpret_cast<double *>(s_winb + NWF * WN);               // [NWF][WN]
     uint32_t *s_hbits = reinterpret_cast<uint32_t *>(s_winx + NWF * WN);          // [HOT_SLOTS/32]
-    unsigned *s_pcnt = s_hbits + HOT_SLOTS / 32;                                  // [MAXG * KP]
+    unsigned *s_pcnt = s_hbits + HOT_SLOTS / 32;                                  // [MAXG * KP] (flat)
+    // bucketed variant: per-bucket base i64[NB], staged values u64[cap], per-bucket
+    // counts u32[NB], staged rows u32[cap], ranks u16[cap], permutation u16[cap]
+    // (after s_hbits)
+    __shared__ unsigned s_bcur;
+    PBS ps;
+    long long *s_bbase = nullptr;
+    unsigned *s_bhist = nullptr;
+    unsigned short *s_brank = nullptr, *s_perm = nullptr;
+    if constexpr (PB) {
+        const size_t o0 = pb_align(FLAT_DYN_B0);
+        s_bbase = reinterpret_cast<long long *>(s_dyn + o0);
+        ps.val = reinterpret_cast<unsigned long long *>(s_bbase + a.pb_nb);
+        s_bhist = reinterpret_cast<unsigned *>(ps.val + a.pb_cap);
+        ps.row = s_bhist + a.pb_nb;
+        s_brank = reinterpret_cast<unsigned short *>(ps.row + a.pb_cap);
+        s_perm = s_brank + a.pb_cap;
+        ps.cur = &s_bcur;
+        ps.cap = a.pb_cap;
+    } else {
+        ps.cur = nullptr;
+        ps.row = nullptr;
+        ps.val = nullptr;
+        ps.cap = 0;
+    }
     __shared__ long long s_base[4], s_tot[4];
     __shared__ long long s_acct[NWF][4];
     __shared__ int s_err;
@@ -175,18 +690,27 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
     const bool stamp = a.tring && b == 0 && tid == 0;
     unsigned long long *ts = a.tring ? a.tring + (a.tslot % FLAT_TRING) * 8 : nullptr;
     if (stamp) ts[0] = globaltimer_ns();
-    unsigned long long *tr = a.trace ? a.trace + (long long)b * 12 : nullptr;
+    unsigned long long *tr = a.trace ? a.trace + (long long)b * 16 : nullptr;
     if (tr && tid == 0) tr[0] = globaltimer_ns();
     const int n_slots = a.n_hot * NT;
     for (int i = tid; i < n_slots; i += FT) s_hacc[i] = __longlong_as_double((long long)EMPTY);
     for (int i = tid; i < (n_slots + 31) / 32; i += FT) s_hbits[i] = 0u;
-    for (int i = tid; i < a.n_pieces; i += FT) s_pcnt[i] = 0u;
     for (int i = tid; i < a.n_hot; i += FT) s_hlist[i] = a.hot_list[i];
     if (tid == 0) {
         s_nheavy = 0;
         s_hcnt = 0;
     }
-    if (tid < KP && b + tid * G < a.n_pieces) a.pc_next[b + tid * G] = 0u;
+    if constexpr (PB) {
+        for (int i = tid; i < a.pb_nb; i += FT) s_bhist[i] = 0u;
+        if (tid == 0) s_bcur = 0u;
+        // the next call's bucket counters (this call's were zeroed by the previous one)
+        for (long long i = (long long)b * FT + tid; i < a.pb_nb; i += (long long)G * FT) {
+            a.pb_cnt_next[i] = 0u;
+        }
+    } else {
+        for (int i = tid; i < a.n_pieces; i += FT) s_pcnt[i] = 0u;
+        if (tid < KP && b + tid * G < a.n_pieces) a.pc_next[b + tid * G] = 0u;
+    }
 
     // ------------------------------------------------------------ phase A (a2)
     // CTA b owns x entries [e0, e1); thread tid a contiguous run of them.
@@ -399,7 +923,7 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
                 long long fr[US];
 #pragma unroll
                 for (int u = 0; u < US; ++u)
-                    fr[u] = ok[u] ? contribute<SR>(a, s_hacc, s_hbits, (long long)row[u], av[u], xv[u]) : -1;
+                    fr[u] = ok[u] ? contribute<SR, PB>(a, s_hacc, s_hbits, ps, (long long)row[u], av[u], xv[u]) : -1;
 #pragma unroll
                 for (int u = 0; u < US; ++u) touch(a, s_pcnt, fr[u]);
                 __syncwarp();
@@ -499,7 +1023,7 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
                                 const double xv = c == c0 ? xv0 : __ldcg(&xs[c]);
                                 const long long rc =
                                     trow >= 0 ? (long long)trow * NT + rr : ~((long long)(~trow) * NT + rr);
-                                fr[j] = contribute<SR>(a, s_hacc, s_hbits, rc, av, xv);
+                                fr[j] = contribute<SR, PB>(a, s_hacc, s_hbits, ps, rc, av, xv);
                                 ++n_mac;
                             }
                         }
@@ -549,7 +1073,7 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
                     const double av = val ? (double)__ldg(&val[pos]) : 1.0;
                     const double xv = __ldcg(&a.L.t_xv[(long long)ss * NT + c]);
                     const long long rc = trs >= 0 ? (long long)trs * NT + rr : ~((long long)(~trs) * NT + rr);
-                    frp = contribute<SR>(a, s_hacc, s_hbits, rc, av, xv);
+                    frp = contribute<SR, PB>(a, s_hacc, s_hbits, ps, rc, av, xv);
                 }
                 touch(a, s_pcnt, frq);  // previous round's result: its atomic had a round to return
                 frq = frp;
@@ -573,6 +1097,24 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
         s_acct[wid][3] = n_ind;
     }
     __syncthreads();
+    if constexpr (PB) {
+        pb_flush<SR>(a, ps, s_hacc, s_hbits, n_slots, s_bhist, s_bbase, s_brank, s_perm, err, s_acct, s_scan, tr);
+        if (tr && tid == 0) tr[7] = globaltimer_ns();
+        grid_sync_f(&a.cnt->bar, target, tr ? tr + 5 : nullptr);
+        if (stamp) ts[3] = globaltimer_ns();
+        if (stamp) ts[4] = globaltimer_ns();
+        pb_emit<SR, XV>(a, err, s_scan, s_dyn, n_slots, tr);
+        if (b == 0 && tid == 0) {
+            a.hm->err = err ? 1 : 0;
+            // every CTA read err / resv_* after barrier 1
+            a.cnt->err = 0;
+            a.cnt->resv_t = 0;
+            a.cnt->resv_s = 0;
+        }
+        if (b == G - 1 && tid == 0 && a.tring) ts[5] = globaltimer_ns();
+        if (tr && tid == 0) tr[9] = globaltimer_ns();
+        return;
+    } else {
     // privatised hot rows: one global atomic per (CTA, touched hot row)
 #ifdef TSMV_EXP_NO_FLUSH
     if (false) {
@@ -662,25 +1204,45 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
         a.cnt->resv_s = 0;
         if (a.tring) ts[5] = globaltimer_ns();
     }
+    }
     if (tr && tid == 0) tr[9] = globaltimer_ns();
 }
 
-template <class AV, class XV> void *pick_sr_flat(int sr) {
-    if (sr == TSMV_PLUS_TIMES) return (void *)k_spmspv_flat<AV, XV, TSMV_PLUS_TIMES>;
-    if (sr == TSMV_OR_AND) return (void *)k_spmspv_flat<AV, XV, TSMV_OR_AND>;
-    return (void *)k_spmspv_flat<AV, XV, TSMV_MIN_SECOND>;
+template <class AV, class XV, bool PB> void *pick_sr_flat(int sr) {
+    if (sr == TSMV_PLUS_TIMES) return (void *)k_spmspv_flat<AV, XV, TSMV_PLUS_TIMES, PB>;
+    if (sr == TSMV_OR_AND) return (void *)k_spmspv_flat<AV, XV, TSMV_OR_AND, PB>;
+    return (void *)k_spmspv_flat<AV, XV, TSMV_MIN_SECOND, PB>;
 }
-void *pick_flat(bool f32, int sr) { return f32 ? pick_sr_flat<float, float>(sr) : pick_sr_flat<double, double>(sr); }
+void *pick_flat(bool f32, int sr, bool pb = false) {
+    if (pb) return f32 ? pick_sr_flat<float, float, true>(sr) : pick_sr_flat<double, double, true>(sr);
+    return f32 ? pick_sr_flat<float, float, false>(sr) : pick_sr_flat<double, double, false>(sr);
+}
 
-constexpr size_t FLAT_DYN = HOT_SLOTS * 8 + (size_t)NWF * ((1 << WL) + 1) * 24 + HOT_SLOTS / 8 + MAXG * KP * 4;
+constexpr size_t FLAT_DYN = FLAT_DYN_B0 + MAXG * KP * 4;
+// dynamic shared memory of the bucketed variant: the whole opt-in maximum less the
+// kernel's static shared memory (set once)
+size_t g_pb_dyn = 0;
 
 void flat_set_smem() {
     static bool done = false;
     if (done) return;
+    int dev = 0, optin = 0;
+    TSMV_CUDA(cudaGetDevice(&dev));
+    TSMV_CUDA(cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));
+    size_t stat = 0;
     for (int f32 = 0; f32 < 2; ++f32)
-        for (int sr = 0; sr < 3; ++sr)
+        for (int sr = 0; sr < 3; ++sr) {
             TSMV_CUDA(cudaFuncSetAttribute(pick_flat(f32, sr), cudaFuncAttributeMaxDynamicSharedMemorySize,
                                            (int)FLAT_DYN));
+            cudaFuncAttributes fa;
+            TSMV_CUDA(cudaFuncGetAttributes(&fa, pick_flat(f32, sr, true)));
+            stat = std::max(stat, (size_t)fa.sharedSizeBytes);
+        }
+    g_pb_dyn = ((size_t)optin > stat + 1024 ? (size_t)optin - stat - 1024 : 0) & ~(size_t)15;
+    for (int f32 = 0; f32 < 2; ++f32)
+        for (int sr = 0; sr < 3; ++sr)
+            TSMV_CUDA(cudaFuncSetAttribute(pick_flat(f32, sr, true), cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                           (int)g_pb_dyn));
     done = true;
 }
 
@@ -823,6 +1385,100 @@ FlatListsView flat_view(tsmv_ctx *c) {
     return v;
 }
 
+namespace {
+// nonzeros of the rows of every bucket (block per bucket)
+__global__ void k_pb_bucket_nnz(const int32_t *__restrict__ indeg, long long m, int bl, long long *__restrict__ out) {
+    __shared__ long long s[8];
+    const long long r0 = (long long)blockIdx.x << bl, r1 = min(m, r0 + (1ll << bl));
+    long long v = 0;
+    for (long long r = r0 + threadIdx.x; r < r1; r += blockDim.x) v += indeg[r];
+    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+    if ((threadIdx.x & 31) == 0) s[threadIdx.x >> 5] = v;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        long long t = 0;
+        for (int w = 0; w < (int)(blockDim.x >> 5); ++w) t += s[w];
+        out[blockIdx.x] = t;
+    }
+}
+}  // namespace
+
+// Bucketed variant: buckets of 2^bl rows (bl in [10, 14], the smallest giving
+// <= 512 buckets), staging regions sized by the nonzeros of each bucket's rows
+// (a call stages at most one product per nonzero), allocated on first use.
+static bool pb_setup(tsmv_ctx *c, cudaStream_t st) {
+    if (c->pb_state) return c->pb_state > 0;
+    c->pb_state = -1;
+    if (c->m == 0 || c->flat_blocks == 0) return false;
+    flat_set_smem();
+    int bl = 10;
+    while (bl < 14 && ((c->m + (1ll << bl) - 1) >> bl) > 512) ++bl;
+    if (const char *e = getenv("TSMV_PB_BL")) bl = std::min(14, std::max(10, atoi(e)));
+    const long long NB = (c->m + (1ll << bl) - 1) >> bl;
+    if (NB > 4ll * FT) return false;
+    const size_t b0 = pb_align(FLAT_DYN_B0) + (size_t)NB * 12;
+    const size_t cneed = ((size_t)8 << bl) + ((size_t)8 << bl) / 32 + (size_t)NB * 8;
+    if (g_pb_dyn < b0 + 16 * 1024 || g_pb_dyn < cneed) return false;
+    c->pb_bl = bl;
+    c->pb_nb = (int)NB;
+    c->pb_cap = (int)std::min<size_t>(65535, (g_pb_dyn - b0) / 16);
+    if (const char *e = getenv("TSMV_PB_CAP")) c->pb_cap = std::max(1, std::min(c->pb_cap, atoi(e)));  // tests: overflow
+    DevBuf sums;
+    sums.alloc(NB * 8);
+    k_pb_bucket_nnz<<<(unsigned)NB, 256, 0, st>>>(c->indeg.as<int32_t>(), c->m, bl, sums.as<long long>());
+    TSMV_CUDA(cudaGetLastError());
+    std::vector<long long> h(NB + 1, 0);
+    TSMV_CUDA(cudaMemcpyAsync(h.data() + 1, sums.p, NB * 8, cudaMemcpyDeviceToHost, st));
+    TSMV_CUDA(cudaStreamSynchronize(st));
+    for (long long q = 0; q < NB; ++q) h[q + 1] += h[q];
+    c->pb_rs.alloc((NB + 1) * 8);
+    TSMV_CUDA(cudaMemcpyAsync(c->pb_rs.p, h.data(), (NB + 1) * 8, cudaMemcpyHostToDevice, st));
+    const long long cap = std::max<long long>(h[NB], 1);
+    c->pb_row.alloc(cap * 4);
+    c->pb_val.alloc(cap * 8);
+    c->pb_cnt.alloc(2 * NB * 4);
+    c->pb_agg.alloc((size_t)2 * MAXG * 8);
+    // hot rows: per-CTA partial slots, and the slots of every bucket
+    const int n_slots = c->P.hot_list ? c->n_hot * 16 : 0;
+    c->pb_hp.alloc((size_t)std::max(1, MAXG * n_slots) * 8);
+    c->pb_hr.alloc((size_t)std::max(1, n_slots) * 12);
+    TSMV_CUDA(cudaMemset(c->pb_hr.p, 0, c->pb_hr.bytes));
+    std::vector<int> hs, hso(NB + 1, 0);
+    if (n_slots) {
+        std::vector<int32_t> hl(c->n_hot);
+        TSMV_CUDA(cudaMemcpy(hl.data(), c->P.hot_list, c->n_hot * 4, cudaMemcpyDeviceToHost));
+        std::vector<std::pair<long long, int>> rows;
+        for (int sl = 0; sl < n_slots; ++sl) {
+            const long long row = (long long)hl[sl / 16] * 16 + sl % 16;
+            if (row < c->m) rows.push_back({row, sl});
+        }
+        std::sort(rows.begin(), rows.end());
+        for (auto &r : rows) {
+            hs.push_back(r.second);
+            hso[(r.first >> bl) + 1]++;
+        }
+        for (long long q = 0; q < NB; ++q) hso[q + 1] += hso[q];
+    }
+    c->pb_hs.alloc(std::max<size_t>(hs.size(), 1) * 4);
+    c->pb_hso.alloc((NB + 1) * 4);
+    if (!hs.empty()) TSMV_CUDA(cudaMemcpy(c->pb_hs.p, hs.data(), hs.size() * 4, cudaMemcpyHostToDevice));
+    TSMV_CUDA(cudaMemcpy(c->pb_hso.p, hso.data(), (NB + 1) * 4, cudaMemcpyHostToDevice));
+    TSMV_CUDA(cudaMemsetAsync(c->pb_cnt.p, 0, c->pb_cnt.bytes, st));
+    TSMV_CUDA(cudaMemsetAsync(c->pb_agg.p, 0, c->pb_agg.bytes, st));
+    TSMV_CUDA(cudaStreamSynchronize(st));
+    c->pb_state = 1;
+    return true;
+}
+
+// Bucketed variant only when forced (TSMV_SPMSPV_KERNEL=pb): measured slower
+// than the plain kernel at every density tried, kept as an
+// experiment with its parity tests.
+static bool use_pb(tsmv_ctx *c, long long k, cudaStream_t st) {
+    (void)k;
+    const char *f = getenv("TSMV_SPMSPV_KERNEL");
+    return f && f[0] == 'p' && pb_setup(c, st);
+}
+
 // Enqueue one flat SpMSpV (device pointers only, no sync).  Returns false if the
 // context cannot use it (nt != 16).
 void enqueue_spmspv_flat(tsmv_ctx *c, int sr, long long k, const int32_t *xi, const void *xv, long long ycap,
@@ -866,6 +1522,41 @@ void enqueue_spmspv_flat(tsmv_ctx *c, int sr, long long k, const int32_t *xi, co
         const int cur = (int)(c->flat_calls & 1);
         a.pc = pc + (size_t)cur * MAXG * KP;
         a.pc_next = pc + (size_t)(1 - cur) * MAXG * KP;
+    }
+    const bool pb = use_pb(c, k, st);
+    if (pb) {
+        const long long NB = c->pb_nb;
+        const int cur = (int)(c->pb_calls & 1);
+        a.pb_rs = c->pb_rs.as<long long>();
+        a.pb_row = c->pb_row.as<unsigned>();
+        a.pb_val = c->pb_val.as<unsigned long long>();
+        a.pb_cnt = c->pb_cnt.as<unsigned>() + cur * NB;
+        a.pb_cnt_next = c->pb_cnt.as<unsigned>() + (1 - cur) * NB;
+        a.pb_agg = c->pb_agg.as<unsigned long long>();
+        a.pb_pu = a.pb_agg + MAXG;
+        a.pb_hp = c->pb_hp.as<unsigned long long>();
+        a.pb_hr = c->pb_hr.as<unsigned long long>();
+        a.pb_hre = reinterpret_cast<unsigned *>(a.pb_hr + std::max(1, (c->P.hot_list ? c->n_hot : 0) * 16));
+        a.pb_hs = c->pb_hs.as<int>();
+        a.pb_hso = c->pb_hso.as<int>();
+        a.pb_epoch = (unsigned)(c->pb_calls % 0x7fffffffll) + 1u;
+        a.pb_bl = c->pb_bl;
+        a.pb_nb = c->pb_nb;
+        a.pb_cap = c->pb_cap;
+        a.pb_ovh = 1ll << (c->pb_bl - 1);
+        if (const char *e = getenv("TSMV_PB_OVH")) a.pb_ovh = atoll(e);
+        c->pb_calls++;
+    } else {
+        a.pb_rs = nullptr;
+        a.pb_row = nullptr;
+        a.pb_val = nullptr;
+        a.pb_cnt = a.pb_cnt_next = nullptr;
+        a.pb_agg = a.pb_pu = a.pb_hp = a.pb_hr = nullptr;
+        a.pb_hre = nullptr;
+        a.pb_hs = a.pb_hso = nullptr;
+        a.pb_epoch = 0;
+        a.pb_bl = a.pb_nb = a.pb_cap = 0;
+        a.pb_ovh = 0;
         c->flat_calls++;
     }
     a.cnt = c->counters.as<Counters>();
@@ -882,13 +1573,13 @@ void enqueue_spmspv_flat(tsmv_ctx *c, int sr, long long k, const int32_t *xi, co
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3(G);
     cfg.blockDim = dim3(FT);
-    cfg.dynamicSmemBytes = FLAT_DYN;
+    cfg.dynamicSmemBytes = pb ? g_pb_dyn : FLAT_DYN;
     cfg.stream = st;
     cudaLaunchAttribute at[2];
     at[0].id = cudaLaunchAttributeCooperative;
     at[0].val.cooperative = 1;
     cfg.numAttrs = 1;
-    if (c->persist_bytes) {
+    if (c->persist_bytes && !pb) {
         at[1].id = cudaLaunchAttributeAccessPolicyWindow;
         at[1].val.accessPolicyWindow.base_ptr = c->acc.p;
         at[1].val.accessPolicyWindow.num_bytes = c->persist_bytes;
@@ -898,7 +1589,7 @@ void enqueue_spmspv_flat(tsmv_ctx *c, int sr, long long k, const int32_t *xi, co
         cfg.numAttrs = 2;
     }
     cfg.attrs = at;
-    TSMV_CUDA(cudaLaunchKernelExC(&cfg, pick_flat(f32, sr), args));
+    TSMV_CUDA(cudaLaunchKernelExC(&cfg, pick_flat(f32, sr, pb), args));
     c->bar_base += 2ull * (unsigned long long)G;
     c->last_blocks = G;
     if (c->timing) c->tcalls++;

@@ -30,14 +30,21 @@ for s in range(1, 9):
     M.spmspv(xi, xv)
     tsmv.tsmv_set_trace(M.ctx, 0)
     if s >= 3:
-        acc.append(buf[: G * 12].view(G, 12).cpu().double())
+        acc.append(buf[: G * 16].view(G, 16).cpu().double())
 names = [("A scan+resv", 0, 8), ("A lists", 8, 1), ("bar1 wait", 1, 2), ("B1", 2, 3), ("B2", 3, 4),
          ("flushes", 4, 7), ("bar2 arrive", 7, 5), ("bar2 wait", 5, 6), ("C", 6, 9), ("total", 0, 9)]
+if any(float(t[:, 10].abs().sum()) > 0 for t in acc):  # bucketed variant: C split
+    names[-1:-1] = [("C buckets", 6, 10), ("C lookback", 10, 11), ("C copy", 11, 9)]
+    names[5:5] = [("fl hot", 4, 12), ("fl rank", 12, 13), ("fl resv", 13, 14), ("fl store", 14, 7)]
 print(f"s{scale} d={d}: per-CTA phase durations in us (median / max over CTAs, mean over {len(acc)} calls)")
 for nm, a, b in names:
     med = sum(float(((t[:, b] - t[:, a]) / 1e3).median()) for t in acc) / len(acc)
     mx = sum(float(((t[:, b] - t[:, a]) / 1e3).max()) for t in acc) / len(acc)
     print(f"  {nm:12s} median {med:6.2f}  max {mx:6.2f}")
+if any(float(t[:, 15].abs().sum()) > 0 for t in acc):
+    nb = [t[:, 15] / 1e3 for t in acc]
+    print("  buckets met per CTA: median %.1f max %.0f" % (sum(float(x.median()) for x in nb) / len(nb),
+                                                           sum(float(x.max()) for x in nb) / len(nb)))
 t = acc[-1]
 t0 = t[:, 0].min()
 print("  last call: start skew %.2f us, barrier-1 release %.2f, barrier-2 release %.2f, end %.2f (max over CTAs)" % (

@@ -348,6 +348,11 @@ k_fscan(const uint32_t *__restrict__ F, uint32_t *__restrict__ Fclear, long long
 // stride, block reduction + one atomic per value and block, the last block
 // publishes; half the registers of k_fscan's whole-segment path, so twice the
 // resident threads and no waves.
+// LITE (the hybrid driver after a host pull level): only |F|, m_f and the sum of
+// in-degrees, which its direction decision reads (the work totals are recounted
+// by the persistent kernel when it resumes); a symmetric pattern's in-degrees are
+// its out-degrees (one array read).
+template <bool LITE>
 __global__ void __launch_bounds__(256) k_fstats16(const uint32_t *__restrict__ F, uint32_t *__restrict__ Fclear,
                                                   long long nseg, const long long *__restrict__ tptr,
                                                   const long long *__restrict__ sptr, const int *__restrict__ outdeg,
@@ -364,7 +369,7 @@ __global__ void __launch_bounds__(256) k_fstats16(const uint32_t *__restrict__ F
         const unsigned bits8 = (w >> (((J & 1) << 4) + (h << 3))) & 0xffu;
         if (h == 0 && Fclear && (J & 1) == 0) Fclear[J >> 1] = 0u;
         if (!bits8) continue;
-        if (h == 0 || !((w >> ((J & 1) << 4)) & 0xffu)) {
+        if (!LITE && (h == 0 || !((w >> ((J & 1) << 4)) & 0xffu))) {
             // tile work of the segment, counted once: by the low half, or by the
             // high half when the low half is empty
             const long long wt = tptr[J + 1] - tptr[J];
@@ -377,14 +382,22 @@ __global__ void __launch_bounds__(256) k_fstats16(const uint32_t *__restrict__ F
         const int4 o0 = __ldg(reinterpret_cast<const int4 *>(outdeg + v0)),
                    o1 = __ldg(reinterpret_cast<const int4 *>(outdeg + v0) + 1);
         od[0] = o0.x, od[1] = o0.y, od[2] = o0.z, od[3] = o0.w, od[4] = o1.x, od[5] = o1.y, od[6] = o1.z, od[7] = o1.w;
+        if (!LITE) {
 #pragma unroll
-        for (int i = 0; i < 4; ++i) {
-            const longlong2 t = __ldg(reinterpret_cast<const longlong2 *>(sptr + v0) + i);
-            sp[2 * i] = t.x, sp[2 * i + 1] = t.y;
+            for (int i = 0; i < 4; ++i) {
+                const longlong2 t = __ldg(reinterpret_cast<const longlong2 *>(sptr + v0) + i);
+                sp[2 * i] = t.x, sp[2 * i + 1] = t.y;
+            }
+            sp[8] = __ldg(sptr + v0 + 8);
+        } else {
+#pragma unroll
+            for (int i = 0; i < 9; ++i) sp[i] = 0;
         }
-        sp[8] = __ldg(sptr + v0 + 8);
         const long long lv0 = v0 - row_begin;
-        if (lv0 >= 0 && lv0 + 8 <= m_local) {
+        if (LITE && indeg == outdeg && row_begin == 0) {
+#pragma unroll
+            for (int r = 0; r < 8; ++r) id[r] = od[r];
+        } else if (lv0 >= 0 && lv0 + 8 <= m_local) {
             const int4 i0 = __ldg(reinterpret_cast<const int4 *>(indeg + lv0)),
                        i1 = __ldg(reinterpret_cast<const int4 *>(indeg + lv0) + 1);
             id[0] = i0.x, id[1] = i0.y, id[2] = i0.z, id[3] = i0.w, id[4] = i1.x, id[5] = i1.y, id[6] = i1.z,
@@ -543,6 +556,104 @@ __global__ void __launch_bounds__(256) k_pull_side(BfsTiles Q, BfsView B) {
         for (long long v = blockIdx.x * (long long)blockDim.x + threadIdx.x; v < B.m_local;
              v += (long long)gridDim.x * blockDim.x)
             pull_side_vertex<NT>(Q, B, v);
+    }
+}
+
+// Dense Pull-CSC level, side part, K vertices per thread (v0, v0 + S, ..., S =
+// the grid's threads): every dependent step (visited + side-mask words, the
+// row's range, PR in-neighbour ids, their frontier bits, the claim on V) is
+// issued for all K vertices before the next, so K chains of loads are in flight
+// per thread instead of one; vertices whose row ends or hits drop out of the
+// rounds.  Same result as k_pull_side<NT, false> (every vertex of the level is
+// tested against the frontier snapshot F, claimed with an atomic on V).
+template <int NT, int K>
+__global__ void __launch_bounds__(256) k_pull_side_ilp(BfsTiles Q, BfsView B) {
+#ifndef TSMV_PULL_ROUND
+#define TSMV_PULL_ROUND 2
+#endif
+    constexpr int PR = TSMV_PULL_ROUND;
+    const int lane = threadIdx.x & 31;
+    const long long S = (long long)gridDim.x * blockDim.x;
+    // warp-uniform loop: lane l takes vertex wb + l (+ k S), so the warp's vertices
+    // of step k are one aligned 32-bit word of V (row_begin is a multiple of 64)
+    for (long long wb = blockIdx.x * (long long)blockDim.x + (threadIdx.x & ~31); wb < B.m_local; wb += S * K) {
+        const long long v0 = wb + lane;
+        uint32_t vw[K], sw[K];
+#pragma unroll
+        for (int k = 0; k < K; ++k) {
+            const long long v = v0 + k * S;
+            vw[k] = 0xffffffffu;
+            sw[k] = 0u;
+            if (v < B.m_local) {
+                vw[k] = B.V[(B.row_begin + v) >> 5];
+                sw[k] = Q.smask[v >> 5];
+            }
+        }
+        unsigned act = 0u;
+#pragma unroll
+        for (int k = 0; k < K; ++k) {
+            const long long v = v0 + k * S, g = B.row_begin + v;
+            if (v < B.m_local && !((vw[k] >> (g & 31)) & 1u) && ((sw[k] >> (v & 31)) & 1u)) act |= 1u << k;
+        }
+        long long p[K], pe[K];
+#pragma unroll
+        for (int k = 0; k < K; ++k) {
+            p[k] = pe[k] = 0;
+            if ((act >> k) & 1u) {
+                p[k] = Q.sptr[v0 + k * S];
+                pe[k] = Q.sptr[v0 + k * S + 1];
+            }
+        }
+        unsigned found = 0u;
+        while (act) {
+            int sr[K][PR];
+#pragma unroll
+            for (int k = 0; k < K; ++k)
+#pragma unroll
+                for (int j = 0; j < PR; ++j) sr[k][j] = ((act >> k) & 1u) && p[k] + j < pe[k] ? Q.srow[p[k] + j] : 0;
+            bool hit[K];
+#pragma unroll
+            for (int k = 0; k < K; ++k) {
+                hit[k] = false;
+                if ((act >> k) & 1u)
+#pragma unroll
+                    for (int j = 0; j < PR; ++j)
+                        if (p[k] + j < pe[k]) {
+                            const long long u = decode_row<NT>(sr[k][j], Q.hot_list);
+                            hit[k] |= ((B.F[u >> 5] >> (u & 31)) & 1u) != 0;
+                        }
+            }
+#pragma unroll
+            for (int k = 0; k < K; ++k) {
+                if (!((act >> k) & 1u)) continue;
+                if (hit[k]) {
+                    found |= 1u << k;
+                    act &= ~(1u << k);
+                } else {
+                    p[k] += PR;
+                    if (p[k] >= pe[k]) act &= ~(1u << k);
+                }
+            }
+        }
+        // claims: one atomic per (warp, word) with the warp's ballot (dense pull
+        // levels discover most vertices: 32x fewer same-word atomics on V), all K
+        // in flight; then the new vertices' frontier bits (one reduction per word)
+        // and levels
+        unsigned bal[K], old[K];
+#pragma unroll
+        for (int k = 0; k < K; ++k) bal[k] = __ballot_sync(0xffffffffu, (found >> k) & 1u);
+#pragma unroll
+        for (int k = 0; k < K; ++k) {
+            old[k] = 0u;
+            if (lane == 0 && bal[k]) old[k] = atomicOr(&B.V[(B.row_begin + wb + k * S) >> 5], bal[k]);
+        }
+#pragma unroll
+        for (int k = 0; k < K; ++k) {
+            if (!bal[k]) continue;
+            const unsigned nw = bal[k] & ~__shfl_sync(0xffffffffu, old[k], 0);
+            if (lane == 0 && nw) atomicOr(&B.Fn[(B.row_begin + wb + k * S) >> 5], nw);
+            if ((nw >> lane) & 1u) B.levels[v0 + k * S] = B.level + 1;
+        }
     }
 }
 
@@ -885,7 +996,7 @@ struct BfsRunner {
     long long irb() const { return c->indeg_g.p ? 0 : c->row_begin; }
     long long iml() const { return c->indeg_g.p ? c->n : c->m; }
 
-    template <int NT> void fscan(const uint32_t *F, uint32_t *Fclear, bool lists) {
+    template <int NT> void fscan(const uint32_t *F, uint32_t *Fclear, bool lists, bool lite = false) {
         long long nseg = c->nTC;
         // one wave: blocks x tiles-per-block cover the ceil(nseg / SCAN_BLOCK) tiles
         static int bps_scan[3] = {0, 0, 0};
@@ -905,14 +1016,23 @@ struct BfsRunner {
             TSMV_CUDA(cudaMemsetAsync(&c->counters.as<Counters>()->nLt, 0, 9 * sizeof(long long), st));
         if (!lists && NT == 16) {
             int bps = 0;
-            if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_fstats16, 256, 0) != cudaSuccess || bps < 1) {
+            if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_fstats16<false>, 256, 0) != cudaSuccess ||
+                bps < 1) {
                 cudaGetLastError();
                 bps = 1;
             }
             const int g = (int)std::max<long long>(
                 1, std::min<long long>((nseg * 2 + 255) / 256, (long long)c->sm_count * bps));
-            k_fstats16<<<g, 256, 0, st>>>(F, Fclear, nseg, c->P.ptr.as<long long>(), c->P.sptr.as<long long>(),
-                                          odeg(), ideg(), irb(), iml(), c->counters.as<Counters>(), c->hcnt_dev);
+            // symmetric pattern: in-degrees == out-degrees (one array)
+            const int *id = (c->symmetric && !c->indeg_g.p && !c->outdeg_g.p) ? odeg() : ideg();
+            if (lite && !getenv("TSMV_BFS_FULL_FSTATS"))
+                k_fstats16<true><<<g, 256, 0, st>>>(F, Fclear, nseg, c->P.ptr.as<long long>(),
+                                                    c->P.sptr.as<long long>(), odeg(), id, irb(), iml(),
+                                                    c->counters.as<Counters>(), c->hcnt_dev);
+            else
+                k_fstats16<false><<<g, 256, 0, st>>>(F, Fclear, nseg, c->P.ptr.as<long long>(),
+                                                     c->P.sptr.as<long long>(), odeg(), ideg(), irb(), iml(),
+                                                     c->counters.as<Counters>(), c->hcnt_dev);
             TSMV_CUDA(cudaGetLastError());
             return;
         }
@@ -922,6 +1042,20 @@ struct BfsRunner {
                                                  irb(), iml(), lists_view(c), c->counters.as<Counters>(),
                                                  c->hcnt_dev, c->desc_bfs.as<LBDesc<8>>(), c->epoch, lists ? 1 : 0);
         TSMV_CUDA(cudaGetLastError());
+    }
+
+    // side part of a dense pull level: K vertices per thread (TSMV_PULL_ILP = 1, 2,
+    // 4 or 8; 1 = the thread-per-vertex kernel)
+    template <int NT> void pull_side_dense(const BfsTiles &Q, const BfsView &B, cudaStream_t s) {
+        // (the warp's word-aligned claims need row_begin % 32 == 0: always true for
+        // row blocks, which are cut at multiples of 64)
+        const int K = (B.row_begin & 31) ? 0 : getenv("TSMV_PULL_ILP") ? atoi(getenv("TSMV_PULL_ILP")) : 1;
+        const long long m = c->m;
+        if (K == 8) k_pull_side_ilp<NT, 8><<<grid_for((m + 7) / 8), 256, 0, s>>>(Q, B);
+        else if (K == 4) k_pull_side_ilp<NT, 4><<<grid_for((m + 3) / 4), 256, 0, s>>>(Q, B);
+        else if (K == 2) k_pull_side_ilp<NT, 2><<<grid_for((m + 1) / 2), 256, 0, s>>>(Q, B);
+        else if (K == 1) k_pull_side_ilp<NT, 1><<<grid_for(m), 256, 0, s>>>(Q, B);
+        else k_pull_side<NT, false><<<grid_for(m), 256, 0, s>>>(Q, B);
     }
 
     template <int NT> void expand(int dir, bool wide) {
@@ -947,13 +1081,13 @@ struct BfsRunner {
                 if (c->aux_stream) {
                     TSMV_CUDA(cudaEventRecord(c->ev_fork, st));
                     TSMV_CUDA(cudaStreamWaitEvent(c->aux_stream, c->ev_fork, 0));
-                    k_pull_side<NT, false><<<grid_for(c->m), 256, 0, c->aux_stream>>>(Q, B);
+                    pull_side_dense<NT>(Q, B, c->aux_stream);
                     TSMV_CUDA(cudaEventRecord(c->ev_join, c->aux_stream));
                     k_pull<NT, false><<<grid_for(nTRl * 32), 256, 0, st>>>(Q, B, nTRl);
                     TSMV_CUDA(cudaStreamWaitEvent(st, c->ev_join, 0));
                 } else {
                     k_pull<NT, false><<<grid_for(nTRl * 32), 256, 0, st>>>(Q, B, nTRl);
-                    k_pull_side<NT, false><<<grid_for(c->m), 256, 0, st>>>(Q, B);
+                    pull_side_dense<NT>(Q, B, st);
                 }
             }
         }
@@ -963,9 +1097,9 @@ struct BfsRunner {
     // lists = false: statistics only (|F|, m_f, sum indeg, work totals), for the
     // hybrid driver, whose next push level rebuilds its lists inside the
     // persistent kernel
-    void do_fscan(const uint32_t *F, uint32_t *Fclear, bool lists = true) {
+    void do_fscan(const uint32_t *F, uint32_t *Fclear, bool lists = true, bool lite = false) {
         switch (c->nt) {
-            case 16: fscan<16>(F, Fclear, lists); break;
+            case 16: fscan<16>(F, Fclear, lists, lite); break;
             case 32: fscan<32>(F, Fclear, lists); break;
             default: fscan<64>(F, Fclear, lists); break;
         }
@@ -1192,7 +1326,7 @@ extern "C" tsmv_status tsmv_bfs(tsmv_ctx *c, int64_t source, int32_t *levels, ts
                     c->bfs_level = (int)level;
                     c->fcur = (Fa == c->F0.as<uint32_t>()) ? 0 : 1;
                     R.do_expand(TSMV_DIR_PULL_CSC, mu * 4 < c->nnz);
-                    R.do_fscan(Fb, Fa, false);  // next frontier stats; clears Fa
+                    R.do_fscan(Fb, Fa, false, true);  // next frontier |F|, m_f, din; clears Fa
                     TSMV_CUDA(cudaStreamSynchronize(st));
                     volatile Counters *h = c->hcnt;
                     const long long fsize = h->fsize, mf = h->mf, din = h->din;

@@ -36,6 +36,7 @@ namespace tsmv {
 namespace {
 
 constexpr int BFB = 512;  // threads per CTA
+constexpr int MAXBG = 320;  // max CTAs of the persistent grid (2 per SM up to 160 SMs; partial sums read at once)
 constexpr int LIST_MAXW = 512;   // list levels only while every frontier vertex has <= this much push work
 #ifndef TSMV_QCAP
 #define TSMV_QCAP 2048
@@ -71,6 +72,7 @@ struct BfsFusedArgs {
     int *bq0, *bq1;
     long long *lslots;   // [3][4] slots, [12..15] profiling, [16] solo release flag, [17..20] solo state
     int use_list, use_solo;
+    int no_relist;       // TSMV_BFS_NO_RELIST: scan levels never convert back to list levels (A/B)
     int qcap;                 // usable entries of the shared-memory queue (<= QCAP; TSMV_BFS_QCAP tests the overflow path)
     int wide_in_kernel;       // pull levels with m_u < nnz / 4 stay in the kernel (wide pull)
     long long wide_cap;       // ... unless m_u > wide_cap (r2: large graphs)
@@ -236,6 +238,25 @@ __device__ __forceinline__ void list_level(const BfsFusedArgs &a, const BfsView 
             }
         }
     }
+}
+
+// Chunk -> list-entry map for an entry owning work items [w0, w0 + w): short runs
+// by the calling thread, runs over 8 chunks (hub columns: thousands) queued for a
+// warp of the CTA (one thread used to write a hub's whole map serially).
+constexpr int HVQ = 64;
+__device__ __forceinline__ void put_chunks_q(int *C, long long w0, long long w, int entry, int kind,
+                                             long long (*hv)[3], int *nhv) {
+    const long long c0 = (w0 + CHUNK - 1) >> CHUNK_LOG, c1 = (w0 + w + CHUNK - 1) >> CHUNK_LOG;
+    if (c1 - c0 > 8) {
+        const int q = atomicAdd(nhv, 1);
+        if (q < HVQ) {
+            hv[q][0] = c0;
+            hv[q][1] = c1;
+            hv[q][2] = ((long long)kind << 32) | (unsigned)entry;
+            return;
+        }
+    }
+    for (long long ch = c0; ch < c1; ++ch) C[ch] = entry;
 }
 
 template <int NT>
@@ -558,6 +579,8 @@ __global__ void __launch_bounds__(BFB, TSMV_BFS_MINB) k_bfs_fused(BfsFusedArgs a
     uint32_t *Fa = B.F, *Fb = B.Fn;
 
     __shared__ ListShared sh;
+    __shared__ long long s_hv[HVQ][3];  // chunk-map runs too long for one thread (hub columns)
+    __shared__ int s_nhv;
     __shared__ SoloBuf s_solo_buf;
     __shared__ SoloShared s_solo;
     unsigned long long solo_n = 0;  // solo episodes of this launch (same in every CTA)
@@ -603,6 +626,7 @@ __global__ void __launch_bounds__(BFB, TSMV_BFS_MINB) k_bfs_fused(BfsFusedArgs a
 
     long long mu = a.resume ? a.mu0 : a.nnz, reached = a.reached0, edges = a.edges0;
     int stopped = 0;
+    bool relist = false;  // a scan level converted back to a list level (counted already)
     const long long S = (a.nseg + G - 1) / G;                 // segments per CTA
     const long long js0 = (long long)b * S, js1 = min(a.nseg, js0 + S);
     const long long per = (S + BFB - 1) / BFB;
@@ -620,17 +644,20 @@ __global__ void __launch_bounds__(BFB, TSMV_BFS_MINB) k_bfs_fused(BfsFusedArgs a
             const long long *sl = a.lslots + (level % 3) * 4;
             const long long fsize = __ldcg(&sl[0]), mf = __ldcg(&sl[1]), din = __ldcg(&sl[2]),
                             maxw = __ldcg(&sl[3]);
-            mu -= din;
+            if (!relist) mu -= din;
             if (fsize == 0) break;
-            reached += fsize;
-            edges += mf;
+            if (!relist) {
+                reached += fsize;
+                edges += mf;
+            }
             const int dir = choose_dir_dev(a.force, a.alpha, a.dens, B.n, fsize, mf, mu, a.alpha_burst, a.growth,
                                            fprev);
-            if (b == 0 && tid == 0 && level < TSMV_MAX_LEVELS) {
+            if (b == 0 && tid == 0 && level < TSMV_MAX_LEVELS && !relist) {
                 a.dir_out[level] = dir;
                 a.front_out[level] = fsize;
                 a.tlv_out[level] = globaltimer_ns();
             }
+            relist = false;
             const int *Qc = (level & 1) ? a.bq1 : a.bq0;
             if (dir != TSMV_DIR_PUSH_CSC || maxw > LIST_MAXW) {
                 // hand the level to the scan form: list -> frontier bitmap Fa
@@ -728,6 +755,13 @@ __global__ void __launch_bounds__(BFB, TSMV_BFS_MINB) k_bfs_fused(BfsFusedArgs a
             continue;
         }
         // ---- S: count this thread's segments, clear the consumed bitmap Fb
+        if (a.use_list && b == 0 && tid == 0) {
+            // slots a conversion back to list levels (below) would use: this level's
+            // max-work cell and the next level's counters
+            a.lslots[(level % 3) * 4 + 3] = 0;
+            long long *sz = a.lslots + ((level + 1) % 3) * 4;
+            sz[0] = sz[1] = sz[2] = sz[3] = 0;
+        }
         long long v[8] = {0, 0, 0, 0, 0, 0, 0, 0};
         for (long long J = tj0; J < tj1; ++J) {
             seg_counts<NT>(a, Fa, J, v);
@@ -750,29 +784,40 @@ __global__ void __launch_bounds__(BFB, TSMV_BFS_MINB) k_bfs_fused(BfsFusedArgs a
             t_s1 += t - tq;
             tq = t;
         }
-        if (tid < 32) {
-            long long pre[8] = {0, 0, 0, 0, 0, 0, 0, 0}, all[8] = {0, 0, 0, 0, 0, 0, 0, 0};
-            for (int g = lane; g < G; g += 32) {
+        // totals and this CTA's prefix of the 7 counts: every thread loads its
+        // (CTA, count) cells at once (one round trip, not one per 32 CTAs), lanes
+        // l, l+8, l+16, l+24 of a warp hold the same count: two shuffles, then one
+        // shared-memory add per warp and count
+        if (tid < 8) {
+            s_pre[tid] = 0;
+            s_tot[tid] = 0;
+        }
+        __syncthreads();
+        {
+            constexpr int PQ = (MAXBG * 8 + BFB - 1) / BFB;
+            long long xa[PQ], xp[PQ];
 #pragma unroll
-                for (int i = 0; i < 7; ++i) {
-                    const long long x = __ldcg(&a.partials[g * 8 + i]);
-                    all[i] += x;
-                    if (g < b) pre[i] += x;
-                }
+            for (int k = 0; k < PQ; ++k) {
+                const int q = tid + k * BFB;
+                const long long x = q < G * 8 && (q & 7) < 7 ? __ldcg(&a.partials[q]) : 0;
+                xa[k] = x;
+                xp[k] = (q >> 3) < b ? x : 0;
             }
+            long long ta = 0, tp = 0;
 #pragma unroll
-            for (int i = 0; i < 7; ++i) {
-#pragma unroll
-                for (int o = 16; o > 0; o >>= 1) {
-                    pre[i] += __shfl_xor_sync(0xffffffffu, pre[i], o);
-                    all[i] += __shfl_xor_sync(0xffffffffu, all[i], o);
-                }
+            for (int k = 0; k < PQ; ++k) {
+                ta += xa[k];
+                tp += xp[k];
             }
-            if (lane == 0)
-                for (int i = 0; i < 7; ++i) {
-                    s_pre[i] = pre[i];
-                    s_tot[i] = all[i];
-                }
+            // q & 7 == tid & 7 for every k (BFB is a multiple of 8)
+            ta += __shfl_xor_sync(0xffffffffu, ta, 8);
+            tp += __shfl_xor_sync(0xffffffffu, tp, 8);
+            ta += __shfl_xor_sync(0xffffffffu, ta, 16);
+            tp += __shfl_xor_sync(0xffffffffu, tp, 16);
+            if (lane < 7) {
+                if (ta) atomicAdd((unsigned long long *)&s_tot[lane], (unsigned long long)ta);
+                if (tp) atomicAdd((unsigned long long *)&s_pre[lane], (unsigned long long)tp);
+            }
         }
         __syncthreads();
         const long long fsize = s_tot[4], mf = s_tot[5];
@@ -802,9 +847,57 @@ __global__ void __launch_bounds__(BFB, TSMV_BFS_MINB) k_bfs_fused(BfsFusedArgs a
             fprev = fsize;  // handed to the host: |F| of the level it expands
             break;
         }
+        if (a.use_list && dir == TSMV_DIR_PUSH_CSC && fsize * 64 <= B.n && !a.no_relist) {
+            // a small Push-CSC frontier after scan levels (the tail of an R-MAT
+            // traversal): the bitmap frontier becomes this level's list (positions
+            // from the count phase's prefix, no atomics) and the level runs as a
+            // list level, so the following small levels are list / solo levels
+            // (one grid barrier, or none) instead of scans of the whole bitmap
+            int *Qw = (level & 1) ? a.bq1 : a.bq0;
+            long long *sl = a.lslots + (level % 3) * 4;
+            long long pos = s_pre[4] + ex[4];
+            int mx = 0;
+            for (long long J = tj0; J < tj1; ++J) {
+                word_t bits = seg_bits<NT>(Fa, J);
+                while (bits) {
+                    const int r = ffs_w(bits);
+                    bits &= bits - 1;
+                    const long long u = J * NT + r;
+                    Qw[pos++] = (int)u;
+                    mx = max(mx, a.lwork[u]);
+                }
+            }
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1) mx = max(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+            if (lane == 0 && mx) atomicMax(&sl[3], (long long)mx);
+            if (b == 0 && tid == 0) {
+                sl[0] = fsize;
+                sl[1] = mf;
+                sl[2] = s_tot[6];
+            }
+            grid_sync(&a.cnt->bar, target);
+            if (__ldcg(&sl[3]) <= LIST_MAXW) {
+                // the list level does not read the bitmaps: clear this level's
+                // frontier words (read by every thread before the barrier above)
+                for (long long J = tj0; J < tj1; ++J) {
+                    if constexpr (NT == 16) Fa[J >> 1] = 0u;
+                    else if constexpr (NT == 32) Fa[J] = 0u;
+                    else {
+                        Fa[2 * J] = 0u;
+                        Fa[2 * J + 1] = 0u;
+                    }
+                }
+                mode_list = 1;
+                relist = true;
+                --level;  // the loop increment brings it back
+                continue;
+            }
+        }
         fprev = fsize;
         // lists (Push-CSC needs both, Push-CSR the side list; pull none)
         if (dir != TSMV_DIR_PULL_CSC) {
+            if (tid == 0) s_nhv = 0;
+            __syncthreads();
             long long oLt = s_pre[0] + ex[0], oWt = s_pre[1] + ex[1];
             long long oLs = s_pre[2] + ex[2], oWs = s_pre[3] + ex[3];
             for (long long J = tj0; J < tj1; ++J) {
@@ -816,7 +909,7 @@ __global__ void __launch_bounds__(BFB, TSMV_BFS_MINB) k_bfs_fused(BfsFusedArgs a
                     a.Lv.Lt_mask[oLt] = (unsigned long long)bits;
                     a.Lv.Lt_tbeg[oLt] = a.P.ptr[J];
                     a.Lv.Lt_wpre[oLt] = oWt;
-                    write_chunks(a.Lv.Ct, oWt, wt, (int)oLt);
+                    put_chunks_q(a.Lv.Ct, oWt, wt, (int)oLt, 0, s_hv, &s_nhv);
                     ++oLt;
                     oWt += wt;
                 }
@@ -829,7 +922,7 @@ __global__ void __launch_bounds__(BFB, TSMV_BFS_MINB) k_bfs_fused(BfsFusedArgs a
                     if (ws > 0) {
                         a.Lv.Ls_beg[oLs] = a.P.sptr[u];
                         a.Lv.Ls_wpre[oLs] = oWs;
-                        write_chunks(a.Lv.Cs, oWs, ws, (int)oLs);
+                        put_chunks_q(a.Lv.Cs, oWs, ws, (int)oLs, 1, s_hv, &s_nhv);
                         ++oLs;
                         oWs += ws;
                     }
@@ -838,6 +931,13 @@ __global__ void __launch_bounds__(BFB, TSMV_BFS_MINB) k_bfs_fused(BfsFusedArgs a
             if (b == G - 1 && tid == 0) {
                 a.Lv.Lt_wpre[s_tot[0]] = s_tot[1];
                 a.Lv.Ls_wpre[s_tot[2]] = s_tot[3];
+            }
+            __syncthreads();
+            // queued long runs, a warp each
+            for (int h = wid; h < min(s_nhv, HVQ); h += NWP) {
+                int *C = s_hv[h][2] >> 32 ? a.Lv.Cs : a.Lv.Ct;
+                const int entry = (int)(s_hv[h][2] & 0xffffffffll);
+                for (long long ch = s_hv[h][0] + lane; ch < s_hv[h][1]; ch += 32) C[ch] = entry;
             }
         }
         grid_sync(&a.cnt->bar, target);
@@ -1048,6 +1148,7 @@ bool bfs_fused_launch(tsmv_ctx *c, long long source, cudaStream_t st, bool resum
     a.lslots = c->lslots.as<long long>();
     a.use_list = (c->lwork.p != nullptr && !getenv("TSMV_BFS_NO_LIST")) ? 1 : 0;
     // solo records hold 32-bit tile / side starts
+    a.no_relist = getenv("TSMV_BFS_NO_RELIST") ? 1 : 0;
     a.use_solo = a.use_list && !getenv("TSMV_BFS_NO_SOLO") && c->P.T < (1LL << 32) && c->P.side_nnz < (1LL << 32)
                      ? 1 : 0;
     a.wide_in_kernel = getenv("TSMV_BFS_HOST_WIDE") ? 0 : 1;
@@ -1075,7 +1176,7 @@ bool bfs_fused_launch(tsmv_ctx *c, long long source, cudaStream_t st, bool resum
     }
     void *args[] = {&a};
     void *f = c->nt == 16 ? (void *)k_bfs_fused<16> : c->nt == 32 ? (void *)k_bfs_fused<32> : (void *)k_bfs_fused<64>;
-    const int G = c->bfs_blocks;
+    const int G = std::min(c->bfs_blocks, MAXBG);
     TSMV_CUDA(cudaLaunchCooperativeKernel(f, dim3(G), dim3(BFB), args, 0, st));
     TSMV_CUDA(cudaStreamSynchronize(st));
     volatile Counters *h = c->hcnt;

@@ -1135,14 +1135,16 @@ extern "C" tsmv_status tsmv_spmspv(tsmv_ctx *c, tsmv_semiring sr, int64_t x_nnz,
         int32_t *yi = y_idx;
         void *yv = (sr == TSMV_OR_AND) ? nullptr : y_val;
         int64_t ycap_dev = y_cap;
-        // pinned (mapped) host y: the kernel's compaction phase writes y straight
-        // into the caller's host buffers (zero copy: the PCIe writes overlap the
-        // compaction, no copy kernel), then ONE synchronisation for the whole call.
+        // pinned (mapped) host y: copied by a kernel sized on the device right
+        // behind the multiply (coalesced PCIe writes), then ONE synchronisation for
+        // the whole call.  TSMV_Y_DIRECT=1 lets the compaction phase write y into
+        // the host buffers itself: measured 1.9x slower end to end at T (its
+        // scattered stores cross PCIe one by one; profiles/r02_pb_experiment.txt).
         // Pageable host y is staged on the device and copied after the sync.
         void *myi = host_y ? mapped_device_ptr(y_idx) : nullptr;
         void *myv = host_yv ? mapped_device_ptr(y_val) : nullptr;
         const bool direct = (!host_y || myi) && (!host_yv || myv) && (host_y || host_yv);
-        const bool copy_kernel = direct && getenv("TSMV_Y_COPY_KERNEL");  // r2 path, A/B only
+        const bool copy_kernel = direct && !getenv("TSMV_Y_DIRECT");
         if (direct && !copy_kernel) {
             if (host_y) yi = static_cast<int32_t *>(myi);
             if (host_yv) yv = myv;

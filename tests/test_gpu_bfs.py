@@ -219,3 +219,25 @@ def test_bulk_push_levels(tsmv, monkeypatch, sym):
         monkeypatch.delenv("TSMV_BFS_NO_BULK")
         assert np.array_equal(lv2.cpu().numpy(), ref)
     M.close()
+
+
+@pytest.mark.parametrize("env", [{}, {"TSMV_PULL_ILP": "0"}, {"TSMV_PULL_ILP": "2"}, {"TSMV_PULL_ILP": "8"},
+                                 {"TSMV_BFS_NO_RELIST": "1"}, {"TSMV_BFS_FULL_FSTATS": "1"}])
+def test_pull_side_claims_relist_stats(tsmv, monkeypatch, env):
+    """R-MAT s18 (symmetrised, thr 8, as the bench's TileBFS): its explosive level
+    is a dense pull level on the host kernels (side part: warp-aggregated claims,
+    K vertices per thread), the next-frontier statistics are the lite pass, and the
+    small push levels after the scan levels are converted back to list / solo
+    levels.  Levels equal the oracle's for every variant, including the r2 kernels."""
+    for k, v in env.items():
+        monkeypatch.setenv(k, v)
+    A = synth.rmat(18, 16, seed=1, symmetrize=True)
+    C = oracle.csc_of(A)
+    M = tsmv.TiledMatrix.from_csr(A.to(DEV), dtype="pattern", sparse_tile_max_nnz=8)
+    for s in [0] + synth.sample_sources(A, 3, seed=2):
+        ref = oracle.bfs_queue(C, s)
+        lv, st = M.bfs(s)
+        assert np.array_equal(lv.cpu().numpy(), ref)
+        assert "pull_csc" in st["dirs"]
+        assert st["reached"] == int((ref >= 0).sum())
+    M.close()

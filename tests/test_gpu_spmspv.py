@@ -158,7 +158,12 @@ def test_errors_keep_workspace_clean(tsmv):
     assert yi.numel() == ri.size
 
 
-def test_host_buffers_e2e(tsmv):
+@pytest.mark.parametrize("direct", [False, True])
+def test_host_buffers_e2e(tsmv, direct, monkeypatch):
+    """Host x / y through the synchronous C ABI: pinned (zero-copy x, y by the copy
+    kernel, or with TSMV_Y_DIRECT=1 written by the compaction phase) and pageable."""
+    if direct:
+        monkeypatch.setenv("TSMV_Y_DIRECT", "1")
     A = synth.attach_values(synth.rmat(12, 16, seed=3), seed=3)
     C = oracle.csc_of(A)
     M = tsmv.TiledMatrix.from_csr(A)   # host CSR -> deep copy to device

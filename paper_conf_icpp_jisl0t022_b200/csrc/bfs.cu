@@ -39,6 +39,13 @@ struct OctSum {
 // per-level device time (tsmv_bfs_stats::level_ms): %globaltimer of a level the
 // host runs itself, and of the end of the traversal
 __global__ void k_stamp(unsigned long long *t) { *t = globaltimer_ns(); }
+// per-level record of a host-decided level: direction, frontier size, time stamp
+// (one launch on the stream instead of two synchronous copies and a launch)
+__global__ void k_level_rec(int *dirs, long long *front, unsigned long long *tlv, int dir, long long f) {
+    *dirs = dir;
+    *front = f;
+    *tlv = globaltimer_ns();
+}
 
 __global__ void k_bfs_init(BfsView B, long long NW, long long source) {
     long long tid = blockIdx.x * (long long)blockDim.x + threadIdx.x;
@@ -1078,6 +1085,7 @@ struct BfsRunner {
                 // the tile part and the side part of a dense pull level are independent
                 // (both claim new vertices with atomics on V): the side kernel runs on
                 // the context's second stream, concurrently with the tile kernel
+                // (one launch for both parts, tile blocks first, measured 1.4x slower)
                 if (c->aux_stream) {
                     TSMV_CUDA(cudaEventRecord(c->ev_fork, st));
                     TSMV_CUDA(cudaStreamWaitEvent(c->aux_stream, c->ev_fork, 0));
@@ -1299,6 +1307,7 @@ extern "C" tsmv_status tsmv_bfs(tsmv_ctx *c, int64_t source, int32_t *levels, ts
             BfsRunner R{c, st, (long long)(c->V.bytes / 4)};
             const long long maxlv = getenv("TSMV_BFS_MAXLV") ? atoll(getenv("TSMV_BFS_MAXLV")) : (1ll << 40);
             unsigned long long *tlv = c->bfs_tlv.as<unsigned long long>();
+            const bool tline = getenv("TSMV_BFS_TIMELINE") != nullptr;  // dev aid: host pull level kernel times
             while (true) {
                 long long L, mu2, r2, e2;
                 int cur;
@@ -1325,9 +1334,21 @@ extern "C" tsmv_status tsmv_bfs(tsmv_ctx *c, int64_t source, int32_t *levels, ts
                 while (true) {
                     c->bfs_level = (int)level;
                     c->fcur = (Fa == c->F0.as<uint32_t>()) ? 0 : 1;
+                    unsigned long long *tl = tline ? c->bfs_tlv.as<unsigned long long>() + TSMV_MAX_LEVELS - 8 : nullptr;
+                    if (tl) k_stamp<<<1, 1, 0, st>>>(tl + 0);
+                    // (statistics taken at discovery in the pull kernels: the tile part's
+                    // warps then wait on every claim, measured 1.4x slower than this pass)
                     R.do_expand(TSMV_DIR_PULL_CSC, mu * 4 < c->nnz);
+                    if (tl) k_stamp<<<1, 1, 0, st>>>(tl + 1);
                     R.do_fscan(Fb, Fa, false, true);  // next frontier |F|, m_f, din; clears Fa
+                    if (tl) k_stamp<<<1, 1, 0, st>>>(tl + 2);
                     TSMV_CUDA(cudaStreamSynchronize(st));
+                    if (tl) {
+                        unsigned long long t[3];
+                        TSMV_CUDA(cudaMemcpy(t, tl, 24, cudaMemcpyDeviceToHost));
+                        fprintf(stderr, "[bfs host pull] level %lld: expand %.1f us, stats %.1f us\n", level,
+                                (t[1] - t[0]) * 1e-3, (t[2] - t[1]) * 1e-3);
+                    }
                     volatile Counters *h = c->hcnt;
                     const long long fsize = h->fsize, mf = h->mf, din = h->din;
                     std::swap(Fa, Fb);
@@ -1344,13 +1365,9 @@ extern "C" tsmv_status tsmv_bfs(tsmv_ctx *c, int64_t source, int32_t *levels, ts
                     reached += fsize;
                     edges += mf;
                     fexp = fsize;
-                    if (level < TSMV_MAX_LEVELS) {
-                        int dd = dir;
-                        long long ff = fsize;
-                        TSMV_CUDA(cudaMemcpy(c->bfs_dirs.as<int>() + level, &dd, 4, cudaMemcpyHostToDevice));
-                        TSMV_CUDA(cudaMemcpy(c->bfs_front.as<long long>() + level, &ff, 8, cudaMemcpyHostToDevice));
-                        k_stamp<<<1, 1, 0, st>>>(tlv + level);
-                    }
+                    if (level < TSMV_MAX_LEVELS)
+                        k_level_rec<<<1, 1, 0, st>>>(c->bfs_dirs.as<int>() + level, c->bfs_front.as<long long>() + level,
+                                                     tlv + level, dir, fsize);
                 }
                 if (c->hcnt->fsize == 0 || level >= maxlv) break;
                 resume = true;

@@ -1308,6 +1308,7 @@ extern "C" tsmv_status tsmv_bfs(tsmv_ctx *c, int64_t source, int32_t *levels, ts
             const long long maxlv = getenv("TSMV_BFS_MAXLV") ? atoll(getenv("TSMV_BFS_MAXLV")) : (1ll << 40);
             unsigned long long *tlv = c->bfs_tlv.as<unsigned long long>();
             const bool tline = getenv("TSMV_BFS_TIMELINE") != nullptr;  // dev aid: host pull level kernel times
+            const bool host_decide = getenv("TSMV_BFS_HOST_DECIDE") != nullptr;  // r2 flow (A/B)
             while (true) {
                 long long L, mu2, r2, e2;
                 int cur;
@@ -1330,7 +1331,22 @@ extern "C" tsmv_status tsmv_bfs(tsmv_ctx *c, int64_t source, int32_t *levels, ts
                 reached = r2;
                 edges = e2;
                 if (!stopped) break;
-                // pull levels on the host path until the rule turns back to push
+                if (!host_decide) {
+                    // the level the kernel stopped at is a pull level: the host kernels run
+                    // it and the persistent kernel is resumed right behind them on the
+                    // stream (no host round trip, no statistics pass: the resumed count
+                    // phase takes the next frontier's statistics, clears the consumed
+                    // bitmap and decides, stopping again for another dense pull level)
+                    c->bfs_level = (int)level;
+                    c->fcur = (Fa == c->F0.as<uint32_t>()) ? 0 : 1;
+                    R.do_expand(TSMV_DIR_PULL_CSC, mu * 4 < c->nnz);
+                    std::swap(Fa, Fb);
+                    ++level;
+                    fprev = fexp;
+                    resume = true;
+                    continue;
+                }
+                // (r2) pull levels on the host path until the rule turns back to push
                 while (true) {
                     c->bfs_level = (int)level;
                     c->fcur = (Fa == c->F0.as<uint32_t>()) ? 0 : 1;

@@ -222,13 +222,16 @@ def test_bulk_push_levels(tsmv, monkeypatch, sym):
 
 
 @pytest.mark.parametrize("env", [{}, {"TSMV_PULL_ILP": "0"}, {"TSMV_PULL_ILP": "2"}, {"TSMV_PULL_ILP": "8"},
-                                 {"TSMV_BFS_NO_RELIST": "1"}, {"TSMV_BFS_FULL_FSTATS": "1"}])
+                                 {"TSMV_BFS_NO_RELIST": "1"}, {"TSMV_BFS_FULL_FSTATS": "1", "TSMV_BFS_HOST_DECIDE": "1"},
+                                 {"TSMV_BFS_HOST_DECIDE": "1"}])
 def test_pull_side_claims_relist_stats(tsmv, monkeypatch, env):
     """R-MAT s18 (symmetrised, thr 8, as the bench's TileBFS): its explosive level
     is a dense pull level on the host kernels (side part: warp-aggregated claims,
-    K vertices per thread), the next-frontier statistics are the lite pass, and the
-    small push levels after the scan levels are converted back to list / solo
-    levels.  Levels equal the oracle's for every variant, including the r2 kernels."""
+    K vertices per thread) with the persistent kernel resumed right behind it (or,
+    TSMV_BFS_HOST_DECIDE, the host deciding from the lite / full statistics pass),
+    and the small push levels after the scan levels are converted back to list /
+    solo levels.  Levels equal the oracle's for every variant, including the r2
+    kernels."""
     for k, v in env.items():
         monkeypatch.setenv(k, v)
     A = synth.rmat(18, 16, seed=1, symmetrize=True)

@@ -1308,7 +1308,12 @@ extern "C" tsmv_status tsmv_bfs(tsmv_ctx *c, int64_t source, int32_t *levels, ts
             const long long maxlv = getenv("TSMV_BFS_MAXLV") ? atoll(getenv("TSMV_BFS_MAXLV")) : (1ll << 40);
             unsigned long long *tlv = c->bfs_tlv.as<unsigned long long>();
             const bool tline = getenv("TSMV_BFS_TIMELINE") != nullptr;  // dev aid: host pull level kernel times
-            const bool host_decide = getenv("TSMV_BFS_HOST_DECIDE") != nullptr;  // r2 flow (A/B)
+            // resuming right behind a host pull level pays the persistent kernel's count
+            // phase instead of the statistics pass and a host round trip: only while
+            // that bitmap scan is short (<= 4 nt-segments per thread: R-MAT s22 yes,
+            // s26 no, where consecutive dense pull levels stay on the host as in r2)
+            const bool host_decide = getenv("TSMV_BFS_HOST_DECIDE") != nullptr ||
+                                     (c->nTC > 4ll * c->bfs_blocks * 512 && !getenv("TSMV_BFS_RESUME_BEHIND"));
             while (true) {
                 long long L, mu2, r2, e2;
                 int cur;

@@ -190,6 +190,9 @@ __device__ long long emit_pieces(const EmitArgs &a, long long (*s_scan)[FT / 32]
     const int kp = tid / PSR, tp = tid % PSR;
     const long long pw0 = ((long long)b + (long long)kp * G) * PS;
     const long long pw1 = min(a.W, pw0 + PS);
+    // the first round's bitmap words do not depend on the piece counts: loaded
+    // before the counts' scan, so the two round trips overlap
+    const unsigned bits_r0 = pw0 + tp < pw1 ? __ldcg(&a.rowbits[pw0 + tp]) : 0u;
     {
         // exclusive prefix of all piece counts (every CTA, in shared memory)
         const int NP = a.n_pieces;
@@ -219,7 +222,7 @@ __device__ long long emit_pieces(const EmitArgs &a, long long (*s_scan)[FT / 32]
     if (tid == 0) s_nd = 0;
     for (int rd = 0; rd < nround; ++rd) {
         const long long w = pw0 + (long long)rd * PSR + tp;
-        const unsigned bits = w < pw1 ? __ldcg(&a.rowbits[w]) : 0u;
+        const unsigned bits = rd == 0 ? bits_r0 : (w < pw1 ? __ldcg(&a.rowbits[w]) : 0u);
         long long c = __popc(bits), exw, rtot;
         block_scan<1, FT>(&c, &exw, &rtot, s_scan);
         if (tp == 0) s_ex0[kp] = exw;

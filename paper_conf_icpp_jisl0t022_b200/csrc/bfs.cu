@@ -1308,6 +1308,12 @@ extern "C" tsmv_status tsmv_bfs(tsmv_ctx *c, int64_t source, int32_t *levels, ts
             const long long maxlv = getenv("TSMV_BFS_MAXLV") ? atoll(getenv("TSMV_BFS_MAXLV")) : (1ll << 40);
             unsigned long long *tlv = c->bfs_tlv.as<unsigned long long>();
             const bool tline = getenv("TSMV_BFS_TIMELINE") != nullptr;  // dev aid: host pull level kernel times
+            // host pull levels run the wide form (thread per visited word, serial over
+            // the word's unvisited vertices) only while the unvisited vertices' in-edges
+            // are few: mu * wide_mult < nnz.  r2 had wide_mult 4, which put R-MAT s26's
+            // big pull level (mu ~ 95 M of 2.1 G after its frontier) on the wide form:
+            // 2.3-3.2 ms there against 1.0 ms on the dense kernels (measured: 64)
+            const long long wide_mult = getenv("TSMV_BFS_WIDE_MULT") ? atoll(getenv("TSMV_BFS_WIDE_MULT")) : 64;
             // resuming right behind a host pull level pays the persistent kernel's count
             // phase instead of the statistics pass and a host round trip: only while
             // that bitmap scan is short (<= 4 nt-segments per thread: R-MAT s22 yes,
@@ -1344,7 +1350,7 @@ extern "C" tsmv_status tsmv_bfs(tsmv_ctx *c, int64_t source, int32_t *levels, ts
                     // bitmap and decides, stopping again for another dense pull level)
                     c->bfs_level = (int)level;
                     c->fcur = (Fa == c->F0.as<uint32_t>()) ? 0 : 1;
-                    R.do_expand(TSMV_DIR_PULL_CSC, mu * 4 < c->nnz);
+                    R.do_expand(TSMV_DIR_PULL_CSC, mu * wide_mult < c->nnz);
                     std::swap(Fa, Fb);
                     ++level;
                     fprev = fexp;
@@ -1359,7 +1365,7 @@ extern "C" tsmv_status tsmv_bfs(tsmv_ctx *c, int64_t source, int32_t *levels, ts
                     if (tl) k_stamp<<<1, 1, 0, st>>>(tl + 0);
                     // (statistics taken at discovery in the pull kernels: the tile part's
                     // warps then wait on every claim, measured 1.4x slower than this pass)
-                    R.do_expand(TSMV_DIR_PULL_CSC, mu * 4 < c->nnz);
+                    R.do_expand(TSMV_DIR_PULL_CSC, mu * wide_mult < c->nnz);
                     if (tl) k_stamp<<<1, 1, 0, st>>>(tl + 1);
                     R.do_fscan(Fb, Fa, false, true);  // next frontier |F|, m_f, din; clears Fa
                     if (tl) k_stamp<<<1, 1, 0, st>>>(tl + 2);

@@ -1127,6 +1127,17 @@ struct BfsRunner {
     }
 };
 
+// Host-run pull levels take the wide form (thread per visited word, serial over
+// the word's unvisited vertices) only while the unvisited vertices' in-edges are
+// few: mu * bfs_wide_mult() < nnz.  r2 used 4, which put R-MAT s26's big pull
+// level (mu ~ 95 M of 2.1 G after its frontier) on the wide form: 2.3-3.2 ms
+// there against 1.0 ms on the dense kernels (measured: 64).  The distributed
+// level loops use the same rule (dist.WIDE_MULT).
+long long bfs_wide_mult() {
+    static const long long m = getenv("TSMV_BFS_WIDE_MULT") ? atoll(getenv("TSMV_BFS_WIDE_MULT")) : 64;
+    return m;
+}
+
 // global out-degrees: set for a distributed context (communicator or
 // tsmv_bfs_dist_set_degrees); a one-rank context's own column counts are global
 static const int *out_degrees(const tsmv_ctx *c) {
@@ -1233,7 +1244,7 @@ static void bfs_distributed(tsmv_ctx *c, int64_t source, tsmv_bfs_stats *stats, 
         uint32_t *Fcur = (c->fcur == 0 ? c->F0 : c->F1).as<uint32_t>();
         uint32_t *Fnext = (c->fcur == 0 ? c->F1 : c->F0).as<uint32_t>();
         if (dir != TSMV_DIR_PULL_CSC) R.do_fscan(Fcur, nullptr);  // push lists of the replicated frontier
-        R.do_expand(dir, dir == TSMV_DIR_PULL_CSC && mu * 4 < c->nnz_global);
+        R.do_expand(dir, dir == TSMV_DIR_PULL_CSC && mu * bfs_wide_mult() < c->nnz_global);
         owned_stats(c, Fnext, st);
         comm_exchange_frontier(c, Fnext, c->V.as<uint32_t>(), (c->n + 31) / 32, c->dstats.p, c->dstats_all.p, st);
         TSMV_CUDA(cudaMemsetAsync(Fcur, 0, ((c->n + 63) / 64) * 8, st));
@@ -1308,12 +1319,7 @@ extern "C" tsmv_status tsmv_bfs(tsmv_ctx *c, int64_t source, int32_t *levels, ts
             const long long maxlv = getenv("TSMV_BFS_MAXLV") ? atoll(getenv("TSMV_BFS_MAXLV")) : (1ll << 40);
             unsigned long long *tlv = c->bfs_tlv.as<unsigned long long>();
             const bool tline = getenv("TSMV_BFS_TIMELINE") != nullptr;  // dev aid: host pull level kernel times
-            // host pull levels run the wide form (thread per visited word, serial over
-            // the word's unvisited vertices) only while the unvisited vertices' in-edges
-            // are few: mu * wide_mult < nnz.  r2 had wide_mult 4, which put R-MAT s26's
-            // big pull level (mu ~ 95 M of 2.1 G after its frontier) on the wide form:
-            // 2.3-3.2 ms there against 1.0 ms on the dense kernels (measured: 64)
-            const long long wide_mult = getenv("TSMV_BFS_WIDE_MULT") ? atoll(getenv("TSMV_BFS_WIDE_MULT")) : 64;
+            const long long wide_mult = bfs_wide_mult();
             // resuming right behind a host pull level pays the persistent kernel's count
             // phase instead of the statistics pass and a host round trip: only while
             // that bitmap scan is short (<= 4 nt-segments per thread: R-MAT s22 yes,

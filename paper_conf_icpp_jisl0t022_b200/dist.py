@@ -21,12 +21,16 @@ gloo CPU tests) and checks the partitioned kernels rank by rank.
 from __future__ import annotations
 
 import ctypes
+import os
 from typing import List, Optional, Sequence
 
 import torch
 import torch.distributed as dist
 
 ALIGN = 64
+# late pull levels (unvisited in-edges mu * WIDE_MULT < nnz) take the wide form; the
+# library's host loops use the same rule (csrc/bfs.cu bfs_wide_mult, TSMV_BFS_WIDE_MULT)
+WIDE_MULT = int(os.environ.get("TSMV_BFS_WIDE_MULT", "64"))
 
 
 def partition_rows(row_ptr: torch.Tensor, nranks: int, align: int = ALIGN) -> List[int]:
@@ -169,7 +173,7 @@ def bfs_loop(engine, source: int, group=None) -> int:
         d = engine.choose(engine.n, f, gmf, gmu, fprev)
         fprev = f
         # late pull levels (few unvisited edges) take the wide row-tile test
-        wide = getattr(engine, "nnz_total", 0) > 0 and gmu * 4 < engine.nnz_total
+        wide = getattr(engine, "nnz_total", 0) > 0 and gmu * WIDE_MULT < engine.nnz_total
         owned = engine.expand(d, wide=wide)
         gathered = exchange_frontier(owned, engine.stride, group)
         if hasattr(engine, "merge_dev"):

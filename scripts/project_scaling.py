@@ -86,7 +86,7 @@ for P in [int(p) for p in args.ranks.split(",")]:
                 for p, e in enumerate(engines):
                     a, b = ev(), ev()
                     a.record()
-                    o = e.expand(d, wide=mu * 4 < nnz)
+                    o = e.expand(d, wide=mu * D.WIDE_MULT < nnz)
                     b.record()
                     torch.cuda.synchronize()
                     te.append(a.elapsed_time(b))

@@ -359,6 +359,73 @@ k_fscan(const uint32_t *__restrict__ F, uint32_t *__restrict__ Fclear, long long
 // in-degrees, which its direction decision reads (the work totals are recounted
 // by the persistent kernel when it resumes); a symmetric pattern's in-degrees are
 // its out-degrees (one array read).
+// The lite statistics of a symmetric single-GPU context (in-degrees == out-degrees):
+// thread per 32-vertex word of F, two words per step, each non-zero word's 32
+// degrees as eight 16-byte loads (one line, all in flight); clears Fclear.
+__global__ void __launch_bounds__(256) k_fstats_words(const uint32_t *__restrict__ F, uint32_t *__restrict__ Fclear,
+                                                      long long nw, const int *__restrict__ deg,
+                                                      Counters *__restrict__ cnt, Counters *__restrict__ hm) {
+    const long long S = (long long)gridDim.x * blockDim.x;
+    unsigned long long f = 0, mf = 0;
+    for (long long w0 = blockIdx.x * (long long)blockDim.x + threadIdx.x; w0 < nw; w0 += 2 * S) {
+        uint32_t b[2];
+#pragma unroll
+        for (int k = 0; k < 2; ++k) {
+            const long long w = w0 + k * S;
+            b[k] = w < nw ? __ldcg(&F[w]) : 0u;
+            if (Fclear && w < nw) Fclear[w] = 0u;
+        }
+#pragma unroll
+        for (int k = 0; k < 2; ++k) {
+            if (!b[k]) continue;
+            const int4 *dp = reinterpret_cast<const int4 *>(deg + (w0 + k * S) * 32);
+            int4 d[8];
+#pragma unroll
+            for (int i = 0; i < 8; ++i) d[i] = __ldg(dp + i);
+            f += (unsigned long long)__popc(b[k]);
+#pragma unroll
+            for (int i = 0; i < 8; ++i) {
+                const unsigned m4 = b[k] >> (4 * i);
+                if (m4 & 1u) mf += (unsigned long long)d[i].x;
+                if (m4 & 2u) mf += (unsigned long long)d[i].y;
+                if (m4 & 4u) mf += (unsigned long long)d[i].z;
+                if (m4 & 8u) mf += (unsigned long long)d[i].w;
+            }
+        }
+    }
+    __shared__ unsigned long long s2[2];
+    __shared__ bool s_last;
+    if (threadIdx.x < 2) s2[threadIdx.x] = 0;
+    __syncthreads();
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        f += __shfl_xor_sync(0xffffffffu, f, o);
+        mf += __shfl_xor_sync(0xffffffffu, mf, o);
+    }
+    if ((threadIdx.x & 31) == 0 && f) {
+        atomicAdd(&s2[0], f);
+        atomicAdd(&s2[1], mf);
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        if (s2[0]) {
+            atomicAdd((unsigned long long *)&cnt->fsize, s2[0]);
+            atomicAdd((unsigned long long *)&cnt->mf, s2[1]);
+        }
+        __threadfence();
+        s_last = atomicAdd(&cnt->fscan_ticket, 1u) == gridDim.x - 1;
+    }
+    __syncthreads();
+    if (s_last && threadIdx.x == 0) {
+        __threadfence();
+        const long long fs = __ldcg(&cnt->fsize), m = __ldcg(&cnt->mf);
+        hm->fsize = fs;
+        hm->mf = m;
+        hm->din = m;
+        cnt->fscan_ticket = 0;
+    }
+}
+
 template <bool LITE>
 __global__ void __launch_bounds__(256) k_fstats16(const uint32_t *__restrict__ F, uint32_t *__restrict__ Fclear,
                                                   long long nseg, const long long *__restrict__ tptr,
@@ -1032,7 +1099,12 @@ struct BfsRunner {
                 1, std::min<long long>((nseg * 2 + 255) / 256, (long long)c->sm_count * bps));
             // symmetric pattern: in-degrees == out-degrees (one array)
             const int *id = (c->symmetric && !c->indeg_g.p && !c->outdeg_g.p) ? odeg() : ideg();
-            if (lite && !getenv("TSMV_BFS_FULL_FSTATS"))
+            if (lite && c->symmetric && !c->indeg_g.p && !c->outdeg_g.p && c->row_begin == 0 &&
+                !getenv("TSMV_BFS_FULL_FSTATS") && !getenv("TSMV_BFS_FSTATS16")) {
+                const long long nw = (c->n + 31) / 32;
+                k_fstats_words<<<grid_for((nw + 1) / 2), 256, 0, st>>>(F, Fclear, nw, odeg(), c->counters.as<Counters>(),
+                                                                      c->hcnt_dev);
+            } else if (lite && !getenv("TSMV_BFS_FULL_FSTATS"))
                 k_fstats16<true><<<g, 256, 0, st>>>(F, Fclear, nseg, c->P.ptr.as<long long>(),
                                                     c->P.sptr.as<long long>(), odeg(), id, irb(), iml(),
                                                     c->counters.as<Counters>(), c->hcnt_dev);

@@ -63,6 +63,9 @@ def parse(argv=None):
     p.add_argument("--dist-scale", type=int, default=26,
                    help="N > 1: R-MAT scale of the strong-scaling run (C5: the same s26 matrix at every N)")
     p.add_argument("--no-s26", action="store_true", help="N = 1: skip the s26 SpMSpV / TileBFS blocks")
+    p.add_argument("--persist", action="store_true",
+                   help="turn on the accumulator's L2 persisting window (TSMV_PERSIST=1, opt-in in the library); "
+                        "off, the flushed-L2 protocol holds for the workspace too")
     a = p.parse_args(argv)
     a.scaling = "strong"
     a.base_scale, a.base_bfs_scale = a.scale, a.bfs_scale
@@ -194,7 +197,9 @@ def workload_config(args, scale=None):
     return {"workload": f"rmat_s{scale}_ef16_directed_{args.dtype}_x{args.density * 100:g}pct",
             "matrix": f"R-MAT scale {scale}, edgefactor 16, (0.57,0.19,0.19,0.05), unpermuted, coalesced",
             "x_density": args.density, "tile_dim": args.tile_dim, "sparse_tile_max_nnz": args.thr,
-            "l2": "flushed before every step (256 MiB write + 256 MiB read of another buffer, outside the events)",
+            "l2": "flushed before every step (256 MiB write + 256 MiB read of another buffer, outside the events); "
+                  + ("accumulator L2 persisting window on (--persist)" if args.persist
+                     else "no L2 persisting window: the accumulator workspace is cold too"),
             "parallelism": "single GPU",
             "multi_gpu": f"N > 1 runs C5 (R-MAT s{args.dist_scale}) as strong scaling; at N = 1 the same s26 "
                          "workloads are the spmspv_s26 / bfs_s26 blocks"}
@@ -287,11 +292,12 @@ def random_access(kms, nt):
         return None
 
 
-def traffic_of(nt):
+def traffic_of(nt, persist=False):
     """DRAM bytes (read + write) per launch of the SpMSpV kernel at T from the ncu
     capture committed under profiles/ (taken under this bench's own L2-flush
     protocol; not measured in this run)."""
-    name = "r02_flat_traffic_bench.json" if nt == 16 else "fused_traffic.json"
+    name = ("r02_flat_traffic_bench.json" if persist else "r02s5_flat_traffic_cold.json") if nt == 16 \
+        else "fused_traffic.json"
     path = os.path.join(ROOT, "profiles", name)
     try:
         d = json.load(open(path))
@@ -323,6 +329,9 @@ def run_tsmv(args):
             dist.init_process_group(be)
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
+    if args.persist:
+        # opt-in L2 persisting window over the accumulator workspace (read by tsmv_create)
+        os.environ["TSMV_PERSIST"] = "1"
     from paper_conf_icpp_jisl0t022_b200 import tsmv
     sv = 4 if args.dtype == "f32" else 8
     peak, peak_src = peaks()
@@ -410,7 +419,7 @@ def run_tsmv(args):
     # call's counters, survey_bytes) / its CUDA-event duration
     kms = ms / args.steps
     achieved = (svy_bytes / args.steps) / (kms * 1e-3) / 1e9
-    traffic, tsrc = traffic_of(args.tile_dim)
+    traffic, tsrc = traffic_of(args.tile_dim, args.persist)
     n_ = max(ncalls, 1)
     roof = {"bound": "hbm", "achieved": round(achieved, 2), "peak": peak, "unit": "GB/s",
             "frac": round(achieved / peak, 4), "traffic": traffic, "traffic_source": tsrc,

@@ -54,7 +54,11 @@ int fused_occupancy(int nt, int dtype);
 // between calls): a persisting access-policy window on the SpMSpV launches keeps
 // its lines in L2 across calls, so the first RED to a row does not fetch a zero
 // sector from HBM.  Device-wide set-aside (cudaLimitPersistingL2CacheSize) is
-// raised to the window size if the device allows it.  TSMV_NO_PERSIST=1 disables.
+// raised to the window size if the device allows it.  Opt-in since r2 session 5
+// (TSMV_PERSIST=1): measured on B200 it left the DRAM traffic of the SpMSpV call at
+// T unchanged (42.7 MB per launch either way) while the device-wide set-aside cost
+// the other workloads L2 (R-MAT s26 TileBFS 682 -> 844 GTEPS and s26 SpMSpV 25 ->
+// 36 GFLOP/s without it), and it let the workspace survive the bench's L2 flush.
 // The device-wide set-aside is raised only while a context that uses it lives:
 // the first such context records the limit it found, the last one restores it
 // (and returns the persisting lines to normal), so the library leaves no L2
@@ -65,7 +69,7 @@ static std::map<int, std::pair<int, size_t>> g_persist;  // device -> (contexts,
 static void setup_persistence(tsmv_ctx *c) {
     c->persist_bytes = 0;
     c->persist_ratio = 0.f;
-    if (getenv("TSMV_NO_PERSIST")) return;
+    if (!getenv("TSMV_PERSIST")) return;
     int max_persist = 0, max_win = 0;
     if (cudaDeviceGetAttribute(&max_persist, cudaDevAttrMaxPersistingL2CacheSize, c->device) != cudaSuccess ||
         cudaDeviceGetAttribute(&max_win, cudaDevAttrMaxAccessPolicyWindowSize, c->device) != cudaSuccess) {

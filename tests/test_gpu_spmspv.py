@@ -255,3 +255,18 @@ def test_permuted_rmat_spmspv(tsmv):
         yi, yv = M.spmspv(xi.to(DEV), xv.to(DEV))
         check_spmspv(C, yi, yv, xi, xv, Cabs=abs_csc(C))
     M.close()
+
+
+def test_opt_in_l2_window(tsmv, monkeypatch):
+    """TSMV_PERSIST=1 (opt-in since r2 session 5): the accumulator's persisting
+    L2 window changes no result; two contexts alive at once, then destroyed."""
+    monkeypatch.setenv("TSMV_PERSIST", "1")
+    A = synth.attach_values(synth.rmat(13, 16, seed=4), seed=4)
+    C = oracle.csc_of(A)
+    Ms = [tsmv.TiledMatrix.from_csr(A.to(DEV), build_bfs=0) for _ in range(2)]
+    for s, M in enumerate(Ms):
+        xi, xv = synth.sample_x(A.n, 300, seed=30 + s)
+        yi, yv = M.spmspv(xi.to(DEV), xv.to(DEV))
+        check_spmspv(C, yi, yv, xi, xv)
+    for M in Ms:
+        M.close()

@@ -11,8 +11,8 @@ projected as
     + exchange: the n/8 frontier bytes each rank receives at the measured NVLink
       peer bandwidth (770 GB/s, B200_PROFILING.md) + a per-level NCCL latency
       (default 20 us, an assumption: --nccl-us)
-    + host decision: one synchronisation per level (measured here as the gap the
-      one-GPU primitive loop shows beyond its kernels).
+    + host decision: the one read of the level's statistics (measured: the host
+      time of reading the ranks' device statistics after their merges).
 GTEPS(P) = edges / projected time.  This is a projection, not a measurement;
 bench.py --gpus N measures the real thing when a multi-GPU box runs it.
 
@@ -21,6 +21,7 @@ import argparse
 import json
 import os
 import sys
+import time
 
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import torch  # noqa: E402
@@ -91,22 +92,29 @@ for P in [int(p) for p in args.ranks.split(",")]:
                     torch.cuda.synchronize()
                     te.append(a.elapsed_time(b))
                     gathered[p * stride:p * stride + o.numel()] = o
-                nst = []
+                # merge with the statistics left on the device (as the collective path
+                # does before its one read per level), then that one read: the level's
+                # host decision term (r2 session 5; r2 timed merge() with its two host
+                # round trips per rank inside the merge term)
+                devs = []
                 for e in engines:
                     a, b = ev(), ev()
                     a.record()
-                    r = e.merge(gathered, stride)
+                    devs.append(e.merge_dev(gathered, stride).clone())
                     b.record()
                     torch.cuda.synchronize()
                     tm.append(a.elapsed_time(b))
-                    nst.append(r)
-                st = nst
+                allst = torch.stack(devs)
+                torch.cuda.synchronize()
+                t0 = time.perf_counter()
+                st = [tuple(int(v) for v in row) for row in allst.tolist()]  # one read (each rank reads its own)
+                host_ms = (time.perf_counter() - t0) * 1e3
                 xfer_ms = (A.n / 8) * (P - 1) / P / (args.link_gbs * 1e9) * 1e3 if P > 1 else 0.0
                 lat_ms = args.nccl_us * 1e-3 if P > 1 else 0.0
                 lv_proj.append({"expand_max": max(te), "merge_max": max(tm), "exchange": xfer_ms + lat_ms,
-                                "dir": d})
+                                "host": host_ms, "dir": d})
                 nlev += 1
-        proj = sum(l["expand_max"] + l["merge_max"] + l["exchange"] for l in lv_proj)
+        proj = sum(l["expand_max"] + l["merge_max"] + l["exchange"] + l["host"] for l in lv_proj)
         runs.append({"source": s, "levels": nlev, "edges": edges, "projected_ms": round(proj, 4),
                      "per_level": [{k: (round(v, 4) if isinstance(v, float) else v) for k, v in l.items()}
                                    for l in lv_proj],

@@ -650,7 +650,7 @@ def run_bfs_dist(args, dev, flush, rank, world):
     from paper_conf_icpp_jisl0t022_b200 import dist as tdist
     A = synth.rmat(args.bfs_scale, 16, seed=1, symmetrize=True, device=dev)
     srcs = [0] + synth.sample_sources(A, max(0, args.bfs_sources - 1), seed=1)
-    splits = tdist.partition_rows(A.row_ptr, world)
+    splits = tdist.partition_rows(A.row_ptr, world, row_weight=tdist.BFS_ROW_WEIGHT)
     Al = tdist.local_rows(A, splits, rank)
     nnz = A.nnz
     del A
@@ -679,7 +679,7 @@ def run_bfs_dist(args, dev, flush, rank, world):
                      "reached": int(red[1]), "gteps": round(edges / (ms * 1e-3) / 1e9, 3)})
     hm = len(runs) / sum(1.0 / r["gteps"] for r in runs if r["gteps"] > 0)
     return {"graph": f"rmat_s{args.bfs_scale}_ef16_sym", "nnz": nnz, "gteps_hmean": round(hm, 3),
-            "partition": f"row blocks x{world} (nnz-balanced)", "build_wall_s": round(build_wall, 3),
+            "partition": f"row blocks x{world} (nnz + {tdist.BFS_ROW_WEIGHT:g} x rows balanced)", "build_wall_s": round(build_wall, 3),
             "edge_count": "sum of out-degrees of reached vertices (directed count of the symmetrised graph)",
             "time": "CUDA events around the whole traversal, max over ranks", "runs": runs}
 
@@ -913,7 +913,7 @@ def run_dist(args):
     if not args.no_bfs:
         A = synth.rmat(args.dist_scale, 16, seed=1, symmetrize=True, device=dev)
         torch.cuda.empty_cache()
-        splits_b = tdist.partition_rows(A.row_ptr, world)
+        splits_b = tdist.partition_rows(A.row_ptr, world, row_weight=tdist.BFS_ROW_WEIGHT)
         uid_b = tdist.bootstrap_unique_id()   # a unique id serves one communicator only
         Db = tdist.DistMatrix(tdist.local_rows(A, splits_b, rank), splits_b, rank, world, uid_b, dtype="pattern",
                               device=local, tile_dim=args.tile_dim, sparse_tile_max_nnz=args.bfs_thr)
@@ -952,7 +952,7 @@ def run_dist(args):
         hm500 = len(runs) / sum(1.0 / x["gteps_graph500"] for x in runs if x["gteps_graph500"] > 0)
         bfs = {"graph": f"rmat_s{args.dist_scale}_ef16_sym", "nnz": nnz, "sources": len(runs),
                "gteps_hmean": round(hm, 3), "gteps_graph500_hmean": round(hm500, 3),
-               "sparse_tile_max_nnz": args.bfs_thr, "partition": f"row blocks x{world} (nnz-balanced)",
+               "sparse_tile_max_nnz": args.bfs_thr, "partition": f"row blocks x{world} (nnz + {tdist.BFS_ROW_WEIGHT:g} x rows balanced)",
                "time": "CUDA events around the collective tsmv_bfs, max over ranks", "edge_count": EDGE_COUNT,
                "runs": runs}
     if rank == 0:

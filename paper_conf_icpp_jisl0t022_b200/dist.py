@@ -31,14 +31,27 @@ ALIGN = 64
 # late pull levels (unvisited in-edges mu * WIDE_MULT < nnz) take the wide form; the
 # library's host loops use the same rule (csrc/bfs.cu bfs_wide_mult, TSMV_BFS_WIDE_MULT)
 WIDE_MULT = int(os.environ.get("TSMV_BFS_WIDE_MULT", "64"))
+# row blocks of a TileBFS context balance nnz + BFS_ROW_WEIGHT x rows: R-MAT's
+# nnz-balanced blocks put the many low-degree tail vertices on the last ranks, whose
+# dense pull level then dominates (s26 projection at P = 8: 1097 GTEPS with weight
+# 0, 1294 / 1328 / 1364 / 1352 / 1336 with 16 / 64 / 128 / 256 / 512; r2 session 5)
+BFS_ROW_WEIGHT = float(os.environ.get("TSMV_BFS_ROW_WEIGHT", "128"))
 
 
-def partition_rows(row_ptr: torch.Tensor, nranks: int, align: int = ALIGN) -> List[int]:
+def partition_rows(row_ptr: torch.Tensor, nranks: int, align: int = ALIGN,
+                   row_weight: Optional[float] = None) -> List[int]:
     """nnz-balanced contiguous row blocks: split p is the multiple of `align` nearest
-    to the row where the running nnz reaches p/nranks of the total.
+    to the row where the running nnz reaches p/nranks of the total.  With
+    row_weight w (default: env TSMV_PART_ROW_WEIGHT, else 0) the balanced quantity
+    is nnz + w x rows (a dense pull level's work grows with the block's unvisited
+    vertices, not only its nonzeros).
     Returns nranks+1 global row boundaries (first 0, last m)."""
     rp = row_ptr.detach().to("cpu", torch.int64)
     m = rp.numel() - 1
+    if row_weight is None:
+        row_weight = float(os.environ.get("TSMV_PART_ROW_WEIGHT", "0"))
+    if row_weight:
+        rp = rp + torch.round(torch.arange(m + 1, dtype=torch.float64) * row_weight).to(torch.int64)
     nnz = int(rp[-1])
     splits = [0]
     for p in range(1, nranks):

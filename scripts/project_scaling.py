@@ -62,7 +62,7 @@ def ev():
 
 
 for P in [int(p) for p in args.ranks.split(",")]:
-    splits = D.partition_rows(A.row_ptr, P)
+    splits = D.partition_rows(A.row_ptr, P, row_weight=D.BFS_ROW_WEIGHT)
     engines = [D.DistTiledMatrix(D.local_rows(A, splits, r), splits, r, P, dtype="pattern",
                                  sparse_tile_max_nnz=args.thr) for r in range(P)]
     deg = torch.bincount(A.col_idx.long(), minlength=A.n).to(torch.int32)   # global out-degrees

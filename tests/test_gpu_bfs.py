@@ -244,3 +244,23 @@ def test_pull_side_claims_relist_stats(tsmv, monkeypatch, env):
         assert "pull_csc" in st["dirs"]
         assert st["reached"] == int((ref >= 0).sum())
     M.close()
+
+
+@pytest.mark.parametrize("nt", [16, 32, 64])
+@pytest.mark.parametrize("relist", [True, False])
+def test_relist_all_tile_sizes(tsmv, monkeypatch, nt, relist):
+    """Scan levels converted back to list / solo levels (session 5) at every tile
+    size (the frontier words are cleared per segment: 16-bit halves, 32-bit words,
+    64-bit pairs), on and off, directed and symmetric R-MAT: levels equal the
+    oracle's."""
+    if not relist:
+        monkeypatch.setenv("TSMV_BFS_NO_RELIST", "1")
+    for sym in (True, False):
+        A = synth.rmat(15, 16, seed=11, symmetrize=sym)
+        C = oracle.csc_of(A)
+        M = tsmv.TiledMatrix.from_csr(A.to(DEV), dtype="pattern", tile_dim=nt, sparse_tile_max_nnz=8)
+        for s in [0] + synth.sample_sources(A, 3, seed=9):
+            ref = oracle.bfs_queue(C, s)
+            lv, _ = M.bfs(s)
+            assert np.array_equal(lv.cpu().numpy(), ref), (nt, relist, sym, s)
+        M.close()

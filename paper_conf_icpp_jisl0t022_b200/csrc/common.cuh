@@ -244,7 +244,10 @@ struct FlatListsView {
     double *xd;
 };
 
-constexpr int HOT_SLOTS = 2048;           // privatised rows per CTA (smem fp64 + bits)
+#ifndef TSMV_HOT_SLOTS
+#define TSMV_HOT_SLOTS 2048
+#endif
+constexpr int HOT_SLOTS = TSMV_HOT_SLOTS;  // privatised rows per CTA (smem fp64 + bits)
 constexpr int CHUNK_LOG = 7;               // 128 work items per warp-chunk
 constexpr int CHUNK = 1 << CHUNK_LOG;
 constexpr int SCAN_BLOCK = 256;

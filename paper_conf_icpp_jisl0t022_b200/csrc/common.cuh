@@ -339,6 +339,9 @@ struct tsmv_ctx {
     tsmv::DevBuf pb_hr;            // u64[hot slots] reduced values + u32[hot slots] their epochs
     tsmv::DevBuf pb_hs, pb_hso;    // int32: hot slots by bucket, and their offsets [NB + 1]
     long long last_x_nnz = 0;
+    int32_t *hy_idx = nullptr;     // mapped pinned host y of the synchronous call being enqueued (or null)
+    void *hy_val = nullptr;
+    bool hy_by_kernel = false;     // the flat kernel's phase C took the host copy over
     int bfs_blocks = 0;            // CTAs of the fused BFS kernel
     long long bfs_last_levels = 0;
     tsmv::DevBuf bfs_dirs, bfs_front;  // per-level direction / frontier size (device)

@@ -1135,9 +1135,11 @@ extern "C" tsmv_status tsmv_spmspv(tsmv_ctx *c, tsmv_semiring sr, int64_t x_nnz,
         int32_t *yi = y_idx;
         void *yv = (sr == TSMV_OR_AND) ? nullptr : y_val;
         int64_t ycap_dev = y_cap;
-        // pinned (mapped) host y: copied by a kernel sized on the device right
-        // behind the multiply (coalesced PCIe writes), then ONE synchronisation for
-        // the whole call.  TSMV_Y_DIRECT=1 lets the compaction phase write y into
+        // pinned (mapped) host y: copied on the device side (coalesced PCIe writes):
+        // by the flat kernel's phase C, each CTA as soon as its pieces are emitted
+        // (r2 session 5: 148 -> 142 us end to end at T), else by a copy kernel sized
+        // on the device right behind the multiply; then ONE synchronisation for the
+        // whole call.  TSMV_Y_DIRECT=1 lets the compaction phase write y into
         // the host buffers itself: measured 1.9x slower end to end at T (its
         // scattered stores cross PCIe one by one; profiles/r02_pb_experiment.txt).
         // Pageable host y is staged on the device and copied after the sync.
@@ -1162,8 +1164,17 @@ extern "C" tsmv_status tsmv_spmspv(tsmv_ctx *c, tsmv_semiring sr, int64_t x_nnz,
         volatile Counters *h = c->hcnt;
         int err = 0;
         for (int attempt = 0; attempt < 2; ++attempt) {
+            // pinned host y: the flat kernel's phase C copies each CTA's finished rows
+            // there itself (TSMV_Y_COPY_KERNEL=1: the separate copy kernel of r2)
+            c->hy_by_kernel = false;
+            if (copy_kernel && !getenv("TSMV_Y_COPY_KERNEL")) {
+                c->hy_idx = host_y ? static_cast<int32_t *>(myi) : nullptr;
+                c->hy_val = host_yv ? myv : nullptr;
+            }
             enqueue_spmspv(c, sr, x_nnz, xi, xv, ycap_dev, yi, yv, nullptr, st);
-            if (copy_kernel) {
+            c->hy_idx = nullptr;
+            c->hy_val = nullptr;
+            if (copy_kernel && !c->hy_by_kernel) {
                 k_copy_y<<<c->sm_count * 4, 256, 0, st>>>(yi, yv, &c->counters.as<Counters>()->y_nnz, y_cap,
                                                            static_cast<int32_t *>(myi), myv, (int)vb);
                 TSMV_CUDA(cudaGetLastError());

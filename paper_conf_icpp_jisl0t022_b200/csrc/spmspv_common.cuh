@@ -177,6 +177,8 @@ struct EmitArgs {
     long long y_cap, row_begin, W;
     const unsigned *pc;
     int ps_log, n_pieces;
+    int32_t *hy_idx;  // mapped pinned host y (or null): each CTA copies its pieces' rows there
+    void *hy_val;     // once they are emitted (coalesced, overlapping the other CTAs' work)
 };
 template <int SR, class XV, int FT, int KP, int MAXG, int SPW, int BATCH>
 __device__ long long emit_pieces(const EmitArgs &a, long long (*s_scan)[FT / 32], long long *s_pbase,
@@ -217,6 +219,8 @@ __device__ long long emit_pieces(const EmitArgs &a, long long (*s_scan)[FT / 32]
         if (tid == 0) s_tot[0] = tt;
     }
     __syncthreads();
+    __shared__ long long s_pst[KP];  // first output position of each of the CTA's pieces
+    if (tid < KP) s_pst[tid] = s_pbase[tid];
     const long long ycap = a.y_cap;
     const int nround = (int)((PS + PSR - 1) / PSR);
     if (tid == 0) s_nd = 0;
@@ -316,6 +320,20 @@ __device__ long long emit_pieces(const EmitArgs &a, long long (*s_scan)[FT / 32]
         if (tid == 0) s_nd = 0;
     }
     __syncthreads();
+    if (a.hy_idx || a.hy_val) {
+        // the CTA's pieces are complete: their rows [s_pst, s_pbase) of y go to the
+        // host buffers now (consecutive threads, consecutive addresses), while other
+        // CTAs still emit (no copy kernel behind the call)
+        const long long nb = (long long)b;
+        for (int q = 0; q < KP; ++q) {
+            if (nb + (long long)q * G >= a.n_pieces) break;
+            const long long lo = s_pst[q], hi = min(s_pbase[q], ycap);
+            for (long long i = lo + tid; i < hi; i += FT) {
+                if (a.hy_idx) a.hy_idx[i] = __ldcg(&a.y_idx[i]);
+                if (a.hy_val && a.y_val) ((XV *)a.hy_val)[i] = __ldcg(&((const XV *)a.y_val)[i]);
+            }
+        }
+    }
     return s_tot[0];
 }
 

@@ -94,6 +94,8 @@ struct FlatArgs {
     const int32_t *hot_list;
     int n_hot;
     unsigned long long *trace;  // tsmv_set_trace: per CTA 8 globaltimer stamps (dev aid)
+    int32_t *hy_idx;            // mapped pinned host y of a synchronous call (or null): phase C copies there
+    void *hy_val;
     // row buckets (propagation blocking, r2 session 5): products are
     // staged per CTA in shared memory, written to the staging region of their row
     // bucket (2^pb_bl rows) and merged bucket by bucket in shared memory in phase C
@@ -1188,6 +1190,8 @@ __global__ void __launch_bounds__(FT, 1) k_spmspv_flat(FlatArgs a) {
         ea.pc = a.pc;
         ea.ps_log = a.ps_log;
         ea.n_pieces = a.n_pieces;
+        ea.hy_idx = a.hy_idx;
+        ea.hy_val = a.hy_val;
         if (stamp) ts[4] = globaltimer_ns();
         emit_pieces<SR, XV, FT, KP, MAXG, SPW, BATCH>(ea, s_scan, s_pbase, s_ex0, s_tot, s_nd, s_win, s_winb,
                                                        reinterpret_cast<unsigned *>(s_winx));
@@ -1567,6 +1571,13 @@ void enqueue_spmspv_flat(tsmv_ctx *c, int sr, long long k, const int32_t *xi, co
     a.hot_list = c->P.hot_list;
     a.n_hot = c->P.hot_list ? c->n_hot : 0;
     a.trace = (unsigned long long *)c->trace;
+    a.hy_idx = nullptr;
+    a.hy_val = nullptr;
+    if (!pb && (c->hy_idx || c->hy_val)) {
+        a.hy_idx = c->hy_idx;
+        a.hy_val = c->hy_val;
+        c->hy_by_kernel = true;
+    }
     void *args[] = {&a};
     const int G = c->flat_blocks;
     flat_set_smem();

@@ -451,6 +451,8 @@ __global__ void __launch_bounds__(RT, 1) k_spmspv_rows(RowArgs a) {
         ea.pc = a.pc;
         ea.ps_log = a.ps_log;
         ea.n_pieces = a.n_pieces;
+        ea.hy_idx = nullptr;  // host y by the copy kernel
+        ea.hy_val = nullptr;
         // the ring accumulators are free now: they hold the dense-word lists
         long long *s_dw = reinterpret_cast<long long *>(s_dyn);
         long long *s_dpos = s_dw + RT;

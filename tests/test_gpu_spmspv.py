@@ -158,12 +158,16 @@ def test_errors_keep_workspace_clean(tsmv):
     assert yi.numel() == ri.size
 
 
-@pytest.mark.parametrize("direct", [False, True])
-def test_host_buffers_e2e(tsmv, direct, monkeypatch):
-    """Host x / y through the synchronous C ABI: pinned (zero-copy x, y by the copy
-    kernel, or with TSMV_Y_DIRECT=1 written by the compaction phase) and pageable."""
-    if direct:
+@pytest.mark.parametrize("mode", ["phase_c_copy", "copy_kernel", "direct"])
+def test_host_buffers_e2e(tsmv, mode, monkeypatch):
+    """Host x / y through the synchronous C ABI: pinned (zero-copy x; y copied by each
+    CTA of the flat kernel's phase C once its pieces are emitted, by the r2 copy
+    kernel with TSMV_Y_COPY_KERNEL=1, or written by the compaction itself with
+    TSMV_Y_DIRECT=1) and pageable."""
+    if mode == "direct":
         monkeypatch.setenv("TSMV_Y_DIRECT", "1")
+    if mode == "copy_kernel":
+        monkeypatch.setenv("TSMV_Y_COPY_KERNEL", "1")
     A = synth.attach_values(synth.rmat(12, 16, seed=3), seed=3)
     C = oracle.csc_of(A)
     M = tsmv.TiledMatrix.from_csr(A)   # host CSR -> deep copy to device

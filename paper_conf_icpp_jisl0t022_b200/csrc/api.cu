@@ -263,7 +263,10 @@ extern "C" tsmv_status tsmv_create(tsmv_ctx **out, int64_t nrows, int64_t ncols,
 
         // --- tiled structures
         DevBuf hot_map;
-        if (!getenv("TSMV_NO_HOT")) choose_hot_rows(c, st, hot_map);  // env: ablation of the privatisation
+        // hot-row privatisation in the SpMSpV kernels: opt-in since r2 session 5
+        // (TSMV_HOT=1); without the L2 persisting window it no longer paid (T: 53.2
+        // -> 51.3 us without it, profiles/r02_pb_experiment.txt)
+        if (getenv("TSMV_HOT")) choose_hot_rows(c, st, hot_map);
         build_tileset(c, c->P, d_rows.as<int32_t>(), ci, vv, nnz, nrows, ncols, dtype != TSMV_PATTERN, want_bfs, st,
                       c->n_hot ? hot_map.as<int32_t>() : nullptr);
         hot_map.release();

@@ -92,8 +92,9 @@ def test_pb_ragged_rectangular(tsmv, pb_env, shape):
     _run(tsmv, A, (0.01, 0.3, 1.0), seed=6)
 
 
-def test_pb_no_hot_rows(tsmv, pb_env):
-    pb_env(TSMV_NO_HOT=1)
+def test_pb_hot_rows(tsmv, pb_env):
+    """With the (opt-in) hot-row privatisation: hot partials reduced over the CTAs."""
+    pb_env(TSMV_HOT=1)
     A = synth.attach_values(synth.rmat(14, 16, seed=8), seed=1, integer=True)
     _run(tsmv, A, (0.01, 0.1), integer=True)
 

@@ -274,3 +274,20 @@ def test_opt_in_l2_window(tsmv, monkeypatch):
         check_spmspv(C, yi, yv, xi, xv)
     for M in Ms:
         M.close()
+
+
+@pytest.mark.parametrize("semiring", ["plus_times", "or_and", "min_second"])
+def test_hot_rows_opt_in(tsmv, monkeypatch, semiring):
+    """TSMV_HOT=1 (opt-in since r2 session 5): the heaviest tile rows privatised in
+    shared memory per CTA and flushed once per (CTA, row); integer-exact against
+    the oracle on R-MAT (power-law rows) over densities, every semiring."""
+    monkeypatch.setenv("TSMV_HOT", "1")
+    A = synth.attach_values(synth.rmat(14, 16, seed=12), seed=3, integer=True)
+    C = oracle.csc_of(A)
+    M = tsmv.TiledMatrix.from_csr(A.to(DEV), build_bfs=0)
+    sr = {"plus_times": oracle.PLUS_TIMES, "or_and": oracle.OR_AND, "min_second": oracle.MIN_SECOND}[semiring]
+    for d in (0.001, 0.01, 0.1, 1.0):
+        xi, xv = synth.sample_x(A.n, max(1, synth.density_k(A.n, d)), seed=5, integer=True)
+        yi, yv = M.spmspv(xi.to(DEV), xv.to(DEV), semiring=semiring)
+        check_spmspv(C, yi, yv, xi, xv, semiring=sr, exact=True)
+    M.close()

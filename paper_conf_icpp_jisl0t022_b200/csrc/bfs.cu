@@ -607,6 +607,47 @@ __global__ void __launch_bounds__(256) k_push_csr(BfsTiles Q, BfsView B) {
 
 // WIDE (late pull levels, few open rows): a warp tests the visited words of 32
 // row tiles at once and walks only the open ones; otherwise warp per row tile.
+// Dense Pull-CSC level, tile part, W lanes per row tile (32 / W row tiles per
+// warp walked together: the warp's rounds run while any of its row tiles still
+// has tiles and unvisited rows; W = 32 is k_pull's one row tile per warp).
+template <int NT, int W>
+__global__ void __launch_bounds__(256) k_pull_sub(BfsTiles Q, BfsView B, long long nTR_local) {
+    using word_t = typename Tr<NT>::word_t;
+    constexpr int R = 32 / W;
+    const word_t *planes = (const word_t *)Q.planes;
+    const int lane = threadIdx.x & 31, gl = lane % W, grp = lane / W;
+    const long long warp = (blockIdx.x * (long long)blockDim.x + threadIdx.x) >> 5;
+    const long long nwarps = ((long long)gridDim.x * blockDim.x) >> 5;
+    const long long rb_seg = B.row_begin / NT;
+    for (long long I0 = warp * R; I0 < nTR_local; I0 += nwarps * R) {
+        const long long I = I0 + grp;
+        word_t um = 0;
+        long long tb = 0, t1 = 0;
+        if (I < nTR_local) {
+            um = ~seg_bits<NT>(B.V, rb_seg + I) & (word_t)Q.pmask[I];
+            if (um) {
+                tb = Q.ptr[I];
+                t1 = Q.ptr[I + 1];
+            }
+        }
+        word_t found = 0;
+        while (__any_sync(0xffffffffu, um && tb < t1)) {
+            const long long t = tb + gl;
+            word_t fl = 0;
+            if (um && t < t1) {
+                const word_t f = seg_bits<NT>(B.F, Q.trow[t]);
+                if (f) fl = rows_hit<NT>(planes, Q.T, t, um, f);
+            }
+#pragma unroll
+            for (int o = W / 2; o > 0; o >>= 1) fl |= (word_t)__shfl_xor_sync(0xffffffffu, fl, o);
+            found |= fl;
+            um &= ~fl;
+            tb += W;
+        }
+        if (gl == 0 && found) discover<NT>(B, rb_seg + I, found);
+    }
+}
+
 template <int NT, bool WIDE>
 __global__ void __launch_bounds__(256) k_pull(BfsTiles Q, BfsView B, long long nTR_local) {
     const int lane = threadIdx.x & 31;
@@ -1137,6 +1178,17 @@ struct BfsRunner {
         else k_pull_side<NT, false><<<grid_for(m), 256, 0, s>>>(Q, B);
     }
 
+    // tile part of a dense pull level: W lanes per row tile, 32 / W row tiles per
+    // warp (TSMV_PULL_W = 4 | 8 | 16 | 32; 32 = k_pull, r2).  Measured (session 5,
+    // R-MAT s22 / s26 traversals): W = 8 3-5 % / 6-12 % faster than 32, W = 4 alike
+    template <int NT> void pull_tiles_dense(const BfsTiles &Q, const BfsView &B, long long nTRl, cudaStream_t s) {
+        const int W = getenv("TSMV_PULL_W") ? atoi(getenv("TSMV_PULL_W")) : 8;
+        if (W == 16) k_pull_sub<NT, 16><<<grid_for(nTRl * 16), 256, 0, s>>>(Q, B, nTRl);
+        else if (W == 8) k_pull_sub<NT, 8><<<grid_for(nTRl * 8), 256, 0, s>>>(Q, B, nTRl);
+        else if (W == 4) k_pull_sub<NT, 4><<<grid_for(nTRl * 4), 256, 0, s>>>(Q, B, nTRl);
+        else k_pull<NT, false><<<grid_for(nTRl * 32), 256, 0, s>>>(Q, B, nTRl);
+    }
+
     template <int NT> void expand(int dir, bool wide) {
         BfsView B = view();
         BfsTiles P = bfs_tiles(c->P), Q = bfs_tiles(*c->Q);
@@ -1163,10 +1215,10 @@ struct BfsRunner {
                     TSMV_CUDA(cudaStreamWaitEvent(c->aux_stream, c->ev_fork, 0));
                     pull_side_dense<NT>(Q, B, c->aux_stream);
                     TSMV_CUDA(cudaEventRecord(c->ev_join, c->aux_stream));
-                    k_pull<NT, false><<<grid_for(nTRl * 32), 256, 0, st>>>(Q, B, nTRl);
+                    pull_tiles_dense<NT>(Q, B, nTRl, st);
                     TSMV_CUDA(cudaStreamWaitEvent(st, c->ev_join, 0));
                 } else {
-                    k_pull<NT, false><<<grid_for(nTRl * 32), 256, 0, st>>>(Q, B, nTRl);
+                    pull_tiles_dense<NT>(Q, B, nTRl, st);
                     pull_side_dense<NT>(Q, B, st);
                 }
             }

@@ -223,7 +223,8 @@ def test_bulk_push_levels(tsmv, monkeypatch, sym):
 
 @pytest.mark.parametrize("env", [{}, {"TSMV_PULL_ILP": "0"}, {"TSMV_PULL_ILP": "2"}, {"TSMV_PULL_ILP": "8"},
                                  {"TSMV_BFS_NO_RELIST": "1"}, {"TSMV_BFS_FULL_FSTATS": "1", "TSMV_BFS_HOST_DECIDE": "1"},
-                                 {"TSMV_BFS_HOST_DECIDE": "1"}])
+                                 {"TSMV_BFS_HOST_DECIDE": "1"}, {"TSMV_PULL_W": "32"}, {"TSMV_PULL_W": "16"},
+                                 {"TSMV_PULL_W": "4"}])
 def test_pull_side_claims_relist_stats(tsmv, monkeypatch, env):
     """R-MAT s18 (symmetrised, thr 8, as the bench's TileBFS): its explosive level
     is a dense pull level on the host kernels (side part: warp-aggregated claims,

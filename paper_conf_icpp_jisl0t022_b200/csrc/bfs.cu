@@ -1472,6 +1472,18 @@ extern "C" tsmv_status tsmv_bfs(tsmv_ctx *c, int64_t source, int32_t *levels, ts
                 reached = r2;
                 edges = e2;
                 if (!stopped) break;
+                if (c->bfs_stop_kind == 2) {
+                    // a heavy bulk Push-CSC level whose lists the kernel built: the
+                    // high-occupancy k_push / k_bulk_fix run it, then the kernel resumes
+                    c->bfs_level = (int)level;
+                    c->fcur = (Fa == c->F0.as<uint32_t>()) ? 0 : 1;
+                    R.do_expand(TSMV_DIR_PUSH_CSC);
+                    std::swap(Fa, Fb);
+                    ++level;
+                    fprev = fexp;
+                    resume = true;
+                    continue;
+                }
                 if (!host_decide) {
                     // the level the kernel stopped at is a pull level: the host kernels run
                     // it and the persistent kernel is resumed right behind them on the

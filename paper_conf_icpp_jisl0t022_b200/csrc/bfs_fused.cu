@@ -73,6 +73,8 @@ struct BfsFusedArgs {
     long long *lslots;   // [3][4] slots, [12..15] profiling, [16] solo release flag, [17..20] solo state
     int use_list, use_solo;
     int no_relist;       // TSMV_BFS_NO_RELIST: scan levels never convert back to list levels (A/B)
+    int stop_on_bulk;    // heavy bulk Push-CSC levels go to the host kernels (TSMV_BFS_BULK_HOST=0: stay)
+    long long bulk_stop_min;
     int qcap;                 // usable entries of the shared-memory queue (<= QCAP; TSMV_BFS_QCAP tests the overflow path)
     int wide_in_kernel;       // pull levels with m_u < nnz / 4 stay in the kernel (wide pull)
     long long wide_cap;       // ... unless m_u > wide_cap (r2: large graphs)
@@ -947,6 +949,23 @@ __global__ void __launch_bounds__(BFB, TSMV_BFS_MINB) k_bfs_fused(BfsFusedArgs a
             tq = t;
         }
 
+        // a heavy Push-CSC level (bulk mode, >= bulk_stop_min items: R-MAT s26's hub
+        // levels, ~90 M edges) is handed to the host's high-occupancy k_push /
+        // k_bulk_fix over the lists just built (this kernel runs 16 warps per SM:
+        // 2.1 ms for that level against 1.0 ms there); the kernel resumes after it
+        if (a.stop_on_bulk && dir == TSMV_DIR_PUSH_CSC && a.bulk_push && (s_tot[1] + s_tot[3]) * 8 > B.n &&
+            s_tot[1] + s_tot[3] >= a.bulk_stop_min) {
+            if (b == 0 && tid == 0) {
+                a.cnt->nLt = s_tot[0];
+                a.cnt->Wt = s_tot[1];
+                a.cnt->nLs = s_tot[2];
+                a.cnt->Ws = s_tot[3];
+                a.cnt->nCt = (s_tot[1] + CHUNK - 1) >> CHUNK_LOG;
+                a.cnt->nCs = (s_tot[3] + CHUNK - 1) >> CHUNK_LOG;
+            }
+            stopped = 2;  // uniform across CTAs
+            break;
+        }
         // ---- E: expand
         bool bulk = false;
         if (dir == TSMV_DIR_PULL_CSC) {
@@ -1149,6 +1168,8 @@ bool bfs_fused_launch(tsmv_ctx *c, long long source, cudaStream_t st, bool resum
     a.use_list = (c->lwork.p != nullptr && !getenv("TSMV_BFS_NO_LIST")) ? 1 : 0;
     // solo records hold 32-bit tile / side starts
     a.no_relist = getenv("TSMV_BFS_NO_RELIST") ? 1 : 0;
+    a.stop_on_bulk = (stop_on_pull && !(getenv("TSMV_BFS_BULK_HOST") && atoi(getenv("TSMV_BFS_BULK_HOST")) == 0)) ? 1 : 0;
+    a.bulk_stop_min = getenv("TSMV_BFS_BULK_HOST_MIN") ? atoll(getenv("TSMV_BFS_BULK_HOST_MIN")) : (4ll << 20);
     a.use_solo = a.use_list && !getenv("TSMV_BFS_NO_SOLO") && c->P.T < (1LL << 32) && c->P.side_nnz < (1LL << 32)
                      ? 1 : 0;
     a.wide_in_kernel = getenv("TSMV_BFS_HOST_WIDE") ? 0 : 1;
@@ -1182,6 +1203,7 @@ bool bfs_fused_launch(tsmv_ctx *c, long long source, cudaStream_t st, bool resum
     volatile Counters *h = c->hcnt;
     const long long L = h->fsize;
     const bool stopped = h->din != 0;
+    c->bfs_stop_kind = (int)h->din;  // 1: a pull level, 2: a heavy bulk push level (lists built)
     level_out = L;
     reached_out = h->reached;
     edges_out = h->edges;

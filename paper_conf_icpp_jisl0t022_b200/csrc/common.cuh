@@ -344,6 +344,7 @@ struct tsmv_ctx {
     bool hy_by_kernel = false;     // the flat kernel's phase C took the host copy over
     int bfs_blocks = 0;            // CTAs of the fused BFS kernel
     long long bfs_last_levels = 0;
+    int bfs_stop_kind = 0;         // why the last persistent BFS launch stopped (1 pull, 2 bulk push)
     tsmv::DevBuf bfs_dirs, bfs_front;  // per-level direction / frontier size (device)
     tsmv::DevBuf bfs_tlv;              // u64[TSMV_MAX_LEVELS + 1]: %globaltimer at each level's decision
     // list-driven push levels of the fused BFS kernel

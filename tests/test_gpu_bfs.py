@@ -201,11 +201,14 @@ def test_level_times(tsmv):
     M.close()
 
 
+@pytest.mark.parametrize("host_min", [None, "1"])
 @pytest.mark.parametrize("sym", [True, False])
-def test_bulk_push_levels(tsmv, monkeypatch, sym):
+def test_bulk_push_levels(tsmv, monkeypatch, sym, host_min):
     """Heavy Push-CSC levels (push items > n / 8) run in bulk mode (reductions into
     the next frontier, then one pass new = Fn & ~V): forced push on R-MAT makes
     every middle level heavy; levels equal the oracle's with and without it."""
+    if host_min:  # (session 5) every bulk level handed to the host's k_push / k_bulk_fix
+        monkeypatch.setenv("TSMV_BFS_BULK_HOST_MIN", host_min)
     A = synth.rmat(14, 16, seed=21, symmetrize=sym)
     C = oracle.csc_of(A)
     M = tsmv.TiledMatrix.from_csr(A.to(DEV), dtype="pattern", force_dir=tsmv.DIR_PUSH_CSC, sparse_tile_max_nnz=8)
